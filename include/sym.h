@@ -1,0 +1,218 @@
+/*
+ * sym.h -- C-ABI of the B200 symmetry-breaking library (libsym.so, sm_100a).
+ *
+ * Implements the data-parallel hot path of Nayyaroddeen, Gambhir, Kothapalli,
+ * "A Study of Graph Decomposition Algorithms for Parallel Symmetry Breaking"
+ * (IPDPS-W 2017).  Citations "P:<line>" refer to that paper's text, and
+ * "DESIGN §x" to DESIGN.md, which fixes every reading of a silent or garbled passage.
+ *
+ *   decomposition  RAND (Alg 2) and DEGk (Alg 3)
+ *   MIS            LubyMIS rounds; MIS-Rand; MIS-Deg2
+ *   MM             LMAX handshake rounds; MM-Rand (Alg 5);
+ *                  MM-Degk (Alg 6)
+ *   COLOR          Jones-Plassmann; COLOR-Rand (Alg 8);
+ *                  COLOR-Degk (Alg 9)
+ *
+ * All priorities are a counter-based hash of (vertex or edge, seed) (DESIGN §3 H),
+ * so every output is a deterministic function of (graph, params): the
+ * lexicographically-first MIS / maximal matching / first-fit colouring of each
+ * phase, bit-identical to the CPU oracle and independent of GPU scheduling.
+ *
+ * Conventions (all functions):
+ *  - Pointers inside sym_graph / sym_decomp and the output arrays are DEVICE
+ *    pointers; the sym_* structs themselves and sym_stats are HOST memory.
+ *  - The caller owns every buffer.  The library allocates no device memory: query
+ *    sym_workspace_bytes() first and pass a device workspace of at least that
+ *    size (any alignment >= 256 B recommended; the library aligns internally).
+ *  - Work is ordered on `stream` (a cudaStream_t; NULL = legacy default stream).
+ *    Round loops are host-driven in batches: a call returns after its last host
+ *    poll of a device round counter, i.e. with all its kernels complete.
+ *  - Arguments are checked on the host before any launch (SYM_EINVAL).  Graph
+ *    validity (symmetric, no self-loops, ids in range, rows sorted ascending
+ *    without duplicates) is a PRECONDITION, checked only by sym_validate() or
+ *    when params->flags has SYM_F_VALIDATE.
+ *  - n == 0 is a valid no-op.  Vertex ids must fit in int32 (n < 2^31); arc
+ *    offsets are int64 (nnz may exceed 2^31).
+ *  - On any error a thread-local message is available from sym_last_error().
+ */
+#ifndef SYM_H
+#define SYM_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *sym_stream_t; /* == cudaStream_t */
+
+/* return codes */
+enum {
+    SYM_OK = 0,
+    SYM_EINVAL = 1,     /* null pointer, n < 0, nnz < 0, RAND p == 0 or p > 65535, bad kind/problem */
+    SYM_EWORKSPACE = 2, /* ws_bytes smaller than sym_workspace_bytes() */
+    SYM_EGRAPH = 3,     /* sym_validate / SYM_F_VALIDATE found an invalid graph */
+    SYM_ECUDA = 4,      /* a CUDA runtime call or kernel launch failed */
+    SYM_ENCCL = 5,      /* reserved for the sharded path */
+    SYM_EROUNDS = 6     /* params->max_rounds reached before the phase converged */
+};
+
+/* decomposition kinds: NONE = no decomposition (the paper's baselines) */
+typedef enum { SYM_DECOMP_NONE = 0, SYM_DECOMP_RAND = 1, SYM_DECOMP_DEGK = 2 } sym_decomp_kind;
+
+/* problem ids for sym_workspace_bytes */
+typedef enum {
+    SYM_PROBLEM_DECOMPOSE = 0,
+    SYM_PROBLEM_MIS = 1,
+    SYM_PROBLEM_MM = 2,
+    SYM_PROBLEM_COLOR = 3,
+    SYM_PROBLEM_VALIDATE = 4
+} sym_problem;
+
+#define SYM_F_VALIDATE 0x1u /* run sym_validate first; SYM_EGRAPH if invalid */
+#define SYM_F_STATS 0x2u    /* fill sym_stats counters that need extra device reads */
+#define SYM_F_EXT_DECOMP 0x4u /* a sym_decompose() result will be passed in: the workspace
+                                 (query and call) then excludes the internal decomposition,
+                                 and sym_mis/mm/color require decomp != NULL */
+
+/* Symmetric simple graph in CSR (directed edges symmetrised, self-loops
+   dropped).  row_ptr int64[n+1] with row_ptr[0] = 0 and row_ptr[n] = nnz;
+   col_idx int32[nnz] holds neighbour ids; each undirected edge appears as two arcs. */
+typedef struct {
+    int64_t n, nnz;
+    const int64_t *row_ptr;
+    const int32_t *col_idx;
+} sym_graph;
+
+/* kind: sym_decomp_kind.  param: p = number of parts for RAND (1..65535; the paper's
+   "k" of Alg 2, reading G2), k = degree threshold for DEGk (deg <= k -> V_L),
+   ignored for NONE.  seed: the 64-bit method seed (priorities and RAND labels).
+   max_rounds: cap on rounds per phase (0 = unlimited). */
+typedef struct {
+    int32_t kind;
+    uint32_t param;
+    uint64_t seed;
+    uint32_t flags;
+    uint32_t max_rounds;
+} sym_params;
+
+/* Output of sym_decompose (caller-allocated device arrays, filled by the call):
+   the induced subgraphs G[V_1..V_p] (RAND) or G_L u G_H (DEGk) as ONE "intra" CSR
+   over all n rows, and the cross-edge graph G_{k+1} / G_C as a
+   "cross" CSR over all n rows.  Each row's arcs keep their input order.
+     row_ptr_in int64[n+1], col_in int32[>= nnz capacity]
+     row_ptr_x  int64[n+1], col_x  int32[>= nnz capacity]
+     label      uint16[n] optional (may be NULL): RAND part of each vertex, or
+                DEGk class (1 = V_H, 0 = V_L).
+   nnz_in / nnz_x are written (host) by sym_decompose.  kind/param/seed are
+   written too and must match the params of a later sym_mis/mm/color call. */
+typedef struct {
+    int64_t n;
+    int32_t kind;
+    uint32_t param;
+    uint64_t seed;
+    int64_t *row_ptr_in;
+    int32_t *col_in;
+    int64_t *row_ptr_x;
+    int32_t *col_x;
+    int64_t nnz_in, nnz_x;
+    uint16_t *label;
+} sym_decomp;
+
+/* Informational statistics (host struct; not part of the bit-exact result).
+   rounds[i] = productive rounds of phase i (phase 0 = the induced/first phase,
+   phase 1 = the fix-up phase); phase_vertices[i] = vertices entering phase i;
+   result_size = |I|, |M| (edges) or the number of colours; conflicts = COLOR-RAND
+   |V'|; max_color = largest colour; ms[0..3] = decompose / phase0 / fix-up /
+   phase1 milliseconds (host-measured, includes launch gaps). */
+typedef struct {
+    uint32_t rounds[3];
+    int64_t phase_vertices[3];
+    int64_t result_size;
+    int64_t conflicts;
+    uint32_t max_color;
+    float ms[4];
+} sym_stats;
+
+/* Bytes of device workspace needed by sym_decompose / sym_mis / sym_mm /
+   sym_color / sym_validate (problem = sym_problem) for this graph and params.
+   Host only; launches nothing.  The MIS/MM/COLOR sizes include room for an
+   internal decomposition (used when their `decomp` argument is NULL).
+   Returns 0 on invalid arguments. */
+size_t sym_workspace_bytes(const sym_graph *g, const sym_params *p, int problem);
+
+/* RAND (Alg 2): label(v) = floor(pv_RAND(v) * p / 2^32) (DESIGN §3 D1);
+   DEGk (Alg 3): class(v) = deg(v) > k (DESIGN §3 D2); NONE: everything
+   intra.  Splits every arc (v,w) into intra (same class) or cross, order-preserving.
+   Synchronises `stream` once at the end to fill out->nnz_in / out->nnz_x. */
+int sym_decompose(const sym_graph *g, const sym_params *p, void *ws, size_t ws_bytes, sym_decomp *out,
+                  sym_stream_t stream);
+
+/* Maximal independent set.  in_set uint8[n] (device): 1 iff v in I, else 0.
+   NONE: LubyMIS with fixed priorities (= LF-MIS(G)).
+   DEGK: MIS-Deg2 (readings G9): I_L = MIS(G_L); remove N[I_L]; I_R = MIS of
+         the remaining V_H.
+   RAND: MIS-Rand (reading G10): I_A = MIS of the partition interiors;
+         remove N[I_A]; I_B = MIS of the remaining graph.
+   decomp: a sym_decompose() result for the same graph/params, or NULL to compute
+   it inside the workspace.  stats: nullable. */
+int sym_mis(const sym_graph *g, const sym_params *p, const sym_decomp *decomp, void *ws, size_t ws_bytes,
+            uint8_t *in_set, sym_stats *stats, sym_stream_t stream);
+
+/* Maximal matching.  mate int32[n] (device): partner id, or -1 if unmatched;
+   mate[mate[v]] == v.  NONE: LMAX handshake rounds with hash edge
+   priorities (= greedy GM order).  RAND: MM-Rand (Alg 5): match inside the
+   parts, then on the cross edges among unmatched vertices.  DEGK: MM-Degk (Alg 6):
+   match G_H, then G_L u G_C among unmatched vertices. */
+int sym_mm(const sym_graph *g, const sym_params *p, const sym_decomp *decomp, void *ws, size_t ws_bytes,
+           int32_t *mate, sym_stats *stats, sym_stream_t stream);
+
+/* Vertex colouring.  color uint32[n] (device): colours >= 1, proper on G.
+   NONE: Jones-Plassmann = first-fit in priority order.
+   DEGK: COLOR-Degk (Alg 9): C_H on G_H; G_L coloured with max(C_H)+1 ..
+         max(C_H)+k+1 (reading: JP replaces the speculative 3-slot loop).
+   RAND: COLOR-Rand (Alg 8): JP on the parts with one palette; the
+         endpoints of monochromatic cross edges are re-coloured by JP against G. */
+int sym_color(const sym_graph *g, const sym_params *p, const sym_decomp *decomp, void *ws, size_t ws_bytes,
+              uint32_t *color, sym_stats *stats, sym_stream_t stream);
+
+/* Checks the CSR precondition on the device: row_ptr[0] = 0, row_ptr monotone,
+   row_ptr[n] = nnz; every id in [0,n); no self-loop; each row sorted strictly
+   ascending (so no duplicate arcs); symmetry (each arc (v,w) has (w,v), found by
+   binary search in row w).  *bad_out (host, nullable) receives the number of
+   violating rows/arcs.  Returns SYM_OK, SYM_EGRAPH, or an argument/CUDA error. */
+int sym_validate(const sym_graph *g, void *ws, size_t ws_bytes, int64_t *bad_out, sym_stream_t stream);
+
+/* Static description of a return code; and the calling thread's last error text. */
+const char *sym_error_string(int code);
+const char *sym_last_error(void);
+
+/* Library version string ("symbreak-b200 <semver> sm_100a"). */
+const char *sym_version(void);
+
+/* ---- kernel profiling hook (measurement only; off by default) ----
+   sym_profile_enable(1) makes every later call record a CUDA event pair on its
+   stream around each hot-kernel launch, grouped by kernel class ("split",
+   "mis_round", "mis_huge", "mm_round0", "mm_round", "mm_huge", "jp_init",
+   "jp_round", "jp_huge", ...).  sym_profile_collect() synchronises those events and
+   returns, per class: launches, summed device milliseconds, and the algorithmic
+   bytes those launches had to move when the library knows them exactly from host
+   sizes (split = 8 B/arc + 24 B/vertex; first MM round = 4 B/arc + 24
+   B/vertex of its phase graph), else -1.  Collect resets the accumulators.
+   Not thread-safe: profile one host thread at a time. */
+typedef struct {
+    char name[24];
+    int64_t launches;
+    double ms;
+    double alg_bytes;
+} sym_kernel_profile;
+
+int sym_profile_enable(int on);
+int sym_profile_collect(sym_kernel_profile *out, int max_entries, int *count);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* SYM_H */

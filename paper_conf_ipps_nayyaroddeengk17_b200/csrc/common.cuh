@@ -1,0 +1,106 @@
+// common.cuh -- device-side building blocks shared by the sm_100a kernels.
+//
+// Hash contract (DESIGN.md §3 H; the paper is silent on its RNG):
+//   K(seed,tag,round) = mix64(mix64(seed ^ 0x9E3779B97F4A7C15) ^ (tag<<32 | round))
+//   pv(v)       = fmix32(v ^ Klo) ^ Khi                 vertex priority
+//   pe(lo,hi)   = fmix32(lo*0x9E3779B1 ^ hi ^ Klo) ^ Khi edge priority
+//   label(v)    = (pv_RAND(v) * p) >> 32                 RAND part (Alg 2 l.3)
+// Vertices are ordered by the 64-bit key (pv(v) << 32 | v); edges at a fixed
+// endpoint u by (pe(u,w) << 32 | w), which agrees with the global (pe, lo, hi)
+// order (DESIGN §3 H).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace sym {
+
+constexpr uint32_t TAG_VERTEX = 1, TAG_EDGE = 2, TAG_RAND = 3;
+constexpr unsigned FULL = 0xffffffffu;
+
+// MIS vertex status (1 byte per vertex)
+constexpr uint8_t ST_UNDEC = 0, ST_IN = 1, ST_OUT = 2, ST_INACTIVE = 3;
+
+__host__ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
+    z ^= z >> 30;
+    z *= 0xBF58476D1CE4E5B9ULL;
+    z ^= z >> 27;
+    z *= 0x94D049BB133111EBULL;
+    z ^= z >> 31;
+    return z;
+}
+
+__host__ __device__ __forceinline__ uint32_t fmix32(uint32_t h) {
+    h ^= h >> 16;
+    h *= 0x85EBCA6Bu;
+    h ^= h >> 13;
+    h *= 0xC2B2AE35u;
+    h ^= h >> 16;
+    return h;
+}
+
+struct Key {
+    uint32_t lo, hi;
+};
+
+inline Key stream_key(uint64_t seed, uint32_t tag, uint32_t round) {
+    uint64_t k = mix64(mix64(seed ^ 0x9E3779B97F4A7C15ULL) ^ (((uint64_t)tag << 32) | round));
+    return Key{(uint32_t)k, (uint32_t)(k >> 32)};
+}
+
+__device__ __forceinline__ uint32_t pv(Key k, uint32_t v) { return fmix32(v ^ k.lo) ^ k.hi; }
+
+// 64-bit vertex order key: larger wins; unique because ids are unique
+__device__ __forceinline__ uint64_t vkey(Key k, uint32_t v) { return ((uint64_t)pv(k, v) << 32) | v; }
+
+__device__ __forceinline__ uint32_t pe(Key k, uint32_t a, uint32_t b) {
+    uint32_t lo = min(a, b), hi = max(a, b);
+    return fmix32((lo * 0x9E3779B1u) ^ hi ^ k.lo) ^ k.hi;
+}
+
+// edge key seen from endpoint u towards w: (pe << 32) | w
+__device__ __forceinline__ uint64_t ekey(Key k, uint32_t u, uint32_t w) { return ((uint64_t)pe(k, u, w) << 32) | w; }
+
+__device__ __forceinline__ uint32_t rand_label(Key k, uint32_t v, uint32_t p) {
+    return (uint32_t)(((uint64_t)pv(k, v) * (uint64_t)p) >> 32);
+}
+
+// ---------------------------------------------------------------- warp helpers
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
+// warp-aggregated append: every lane with `pred` gets a unique slot in list
+// (returns the slot; -1 for lanes without pred).  Must be called by all lanes of
+// the warp in converged control flow.
+__device__ __forceinline__ int64_t warp_append(bool pred, uint32_t *counter) {
+    unsigned m = __ballot_sync(FULL, pred);
+    if (!m) return -1;
+    int leader = __ffs(m) - 1;
+    uint32_t base = 0;
+    if (lane_id() == leader) base = atomicAdd(counter, (uint32_t)__popc(m));
+    base = __shfl_sync(FULL, base, leader);
+    if (!pred) return -1;
+    return (int64_t)base + __popc(m & ((1u << lane_id()) - 1));
+}
+
+__device__ __forceinline__ uint64_t ld_volatile_u64(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t *p) {
+    uint32_t v;
+    asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// status read that bypasses L1 (L2-coherent within a kernel): decisions taken
+// earlier in the same round become visible sooner, cutting rounds.
+__device__ __forceinline__ uint8_t ld_status(const uint8_t *p) {
+    uint16_t v;
+    asm volatile("ld.relaxed.gpu.global.u8 %0, [%1];" : "=h"(v) : "l"(p));
+    return (uint8_t)v;
+}
+
+__device__ __forceinline__ int32_t ld_stream_i32(const int32_t *p) { return __ldcs(p); }
+
+}  // namespace sym

@@ -1,0 +1,154 @@
+// internal.h -- host-side internals of libsym (not part of the C-ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stddef.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "../../include/sym.h"
+#include "common.cuh"
+
+namespace sym {
+
+// ------------------------------------------------------------------ errors
+void set_error(const std::string &msg);
+int cuda_fail(cudaError_t e, const char *what, const char *file, int line);
+
+#define SYM_CUDA(call)                                                          \
+    do {                                                                        \
+        cudaError_t e_ = (call);                                                \
+        if (e_ != cudaSuccess) return ::sym::cuda_fail(e_, #call, __FILE__, __LINE__); \
+    } while (0)
+#define SYM_LAUNCH_CHECK() SYM_CUDA(cudaGetLastError())
+#define SYM_TRY(expr)               \
+    do {                            \
+        int rc_ = (expr);           \
+        if (rc_ != SYM_OK) return rc_; \
+    } while (0)
+
+// ------------------------------------------------------------------ workspace carving
+// A bump allocator over the caller's workspace.  In "dry" mode (base == nullptr) it
+// only counts bytes, so sym_workspace_bytes and the real carving share one code path.
+struct Arena {
+    char *base = nullptr;
+    size_t cap = 0, used = 0;
+    bool dry() const { return base == nullptr; }
+    template <class T>
+    T *take(size_t count) {
+        size_t off = (used + 255) & ~(size_t)255;
+        used = off + count * sizeof(T) + 0;
+        if (dry()) return nullptr;
+        return reinterpret_cast<T *>(base + off);
+    }
+};
+
+// device control block: counters used by the round loops
+struct Ctl {
+    uint32_t ring[4];       // frontier counts (ring of 3)
+    uint32_t huge[2];       // deferred long-row counts (ring of 2)
+    uint32_t cnt_front;     // class list: front count
+    uint32_t cnt_back;      // class list: back count
+    uint32_t tile_counter;  // dynamic tile ids for the look-back split
+    uint32_t flag;          // generic flag / error word
+    uint32_t max_color;     // COLOR
+    uint32_t conflicts;     // COLOR-RAND |V'|
+    uint32_t done;          // JP: coloured count
+    uint32_t q_head, q_tail;
+    uint32_t pad[15];
+    uint64_t result;        // reductions
+    uint64_t scanned;       // SYM_F_STATS: arcs inspected
+    uint32_t hist[1 << 12]; // per-round frontier sizes (stats)
+};
+
+// decomposition view used by the flows (device pointers)
+struct Split {
+    const int64_t *rp_in = nullptr, *rp_x = nullptr;
+    const int32_t *ci_in = nullptr, *ci_x = nullptr;
+    int64_t nnz_in = -1;  // known on the host only for a caller-supplied decomposition
+};
+
+struct Graph {
+    int64_t n, nnz;
+    const int64_t *rp;
+    const int32_t *ci;
+};
+
+// ------------------------------------------------------------------ decomposition (decompose.cu)
+constexpr int SPLIT_THREADS = 256;
+constexpr int SPLIT_PER_THREAD = 8;
+constexpr int SPLIT_TILE = SPLIT_THREADS * SPLIT_PER_THREAD;  // arcs per tile
+
+struct SplitWs {
+    uint32_t *hbits = nullptr;   // DEGk V_H bitmap [ceil(n/32)]
+    int64_t *first_row = nullptr;
+    uint64_t *tile_state = nullptr;
+    int64_t ntiles = 0;
+};
+void carve_split_ws(Arena &a, int64_t n, int64_t nnz, SplitWs &w);
+
+// class bitmap (+ optional vertex lists: class-0 from the front, class-1 from the back)
+int launch_classify_degk(const Graph &g, uint32_t k, uint32_t *hbits, int32_t *vlist, Ctl *ctl,
+                         cudaStream_t s);
+// decompose into caller buffers (rp_in, ci_in, rp_x, ci_x) ; kind in {NONE,RAND,DEGK}
+int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const SplitWs &w, Ctl *ctl,
+              int64_t *rp_in, int32_t *ci_in, int64_t *rp_x, int32_t *ci_x, uint16_t *label, cudaStream_t s);
+
+// ------------------------------------------------------------------ profiling hook (profile.cu)
+bool prof_on();
+void prof_begin(const char *cls, cudaStream_t s);
+void prof_end(cudaStream_t s, double alg_bytes);  // alg_bytes < 0: unknown on the host
+
+// ------------------------------------------------------------------ helpers (api.cu)
+int read_u32(const uint32_t *dev, uint32_t *host, cudaStream_t s);
+int read_u64(const uint64_t *dev, uint64_t *host, cudaStream_t s);
+int num_sms();
+
+// ------------------------------------------------------------------ flows
+struct FlowArgs {
+    Graph g;
+    sym_params p;
+    Split split;                // valid when p.kind != NONE
+    uint32_t *hbits;            // DEGk bitmap workspace
+    Ctl *ctl;
+    sym_stats *stats;
+    cudaStream_t stream;
+};
+
+struct MisWs {
+    uint8_t *st = nullptr;
+    int32_t *vlist = nullptr;          // class lists (front / back)
+    int32_t *fr[2] = {nullptr, nullptr};  // frontier ping-pong
+    int64_t *huge = nullptr;           // deferred (v, resume) pairs
+    int64_t huge_cap = 0;
+};
+
+struct MmWs {
+    int32_t *pick[2] = {nullptr, nullptr};
+    int32_t *vlist = nullptr;
+    int32_t *fr[2] = {nullptr, nullptr};
+    int64_t *huge = nullptr;
+    unsigned long long *huge_best = nullptr;
+    int64_t huge_cap = 0;
+};
+
+struct ColorWs {
+    uint32_t *cnt = nullptr;       // pending higher-priority neighbours
+    uint32_t *bits = nullptr;      // forbidden-colour bitmaps, (deg+1) bits per vertex
+    int32_t *queue = nullptr;      // ready queue (each vertex enqueued once)
+    int32_t *vlist = nullptr;
+    uint8_t *mark = nullptr;       // COLOR-RAND V'
+    int64_t *task = nullptr;
+    int64_t queue_cap = 0;
+};
+
+void carve_mis_ws(Arena &a, int64_t n, int64_t nnz, MisWs &w);
+int run_mis(const FlowArgs &f, MisWs &w, uint8_t *in_set);
+
+void carve_mm_ws(Arena &a, int64_t n, int64_t nnz, MmWs &w);
+int run_mm(const FlowArgs &f, MmWs &w, int32_t *mate);
+
+void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w);
+int run_color(const FlowArgs &f, ColorWs &w, uint32_t *color);
+
+}  // namespace sym

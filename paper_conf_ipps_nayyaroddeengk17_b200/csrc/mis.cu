@@ -1,0 +1,364 @@
+// mis.cu -- Luby local-maximum rounds and the MIS flows.
+//
+// Round rule (P:272-274 with fixed priorities, DESIGN §3 M1): an undecided vertex v
+//   -> OUT  if some phase neighbour is IN,
+//   -> IN   if no undecided phase neighbour has a larger (pv, id) key,
+//   else stays undecided and is appended to the next frontier.
+// Status moves only UNDEC -> {IN, OUT}, and v turns IN only when every higher
+// neighbour is final-OUT, so decisions may be taken in place and read by other
+// threads of the same round: any interleaving yields the lexicographically-first
+// MIS (Blelloch et al. [6]).  Neighbours marked INACTIVE are not
+// in the current phase and are ignored.
+//
+// Load balance for power-law rows (R-MAT: max degree ~4e5 at scale 24):
+//   rows <= MIS_SMALL arcs  : one lane scans serially with early exit;
+//   longer rows             : the warp scans 4x32 arcs per step (ballot early exit)
+//                             for up to MIS_BUDGET arcs;
+//   rows still undecided    : deferred (v, resume offset) to k_mis_huge, where a
+//                             whole CTA scans the rest with __syncthreads_or exits.
+#include "internal.h"
+
+namespace sym {
+
+constexpr int MIS_SMALL = 8;
+constexpr int MIS_BUDGET = 4096;
+constexpr int MIS_THREADS = 256;
+constexpr int MIS_HUGE_THREADS = 512;
+
+enum { R_NONE = 0, R_IN = 1, R_OUT = 2, R_BLK = 3, R_DEFER = 4 };
+
+struct MisRoundArgs {
+    const int64_t *rp;
+    const int32_t *ci;
+    uint8_t *st;
+    const int32_t *in_list;  // nullptr => implicit list [0, implicit_n)
+    int in_rev;              // list stored backwards: v = in_list[-1 - i]
+    const uint32_t *in_cnt;
+    int64_t implicit_n;
+    int32_t *out_list;
+    uint32_t *out_cnt;
+    uint32_t *clear_cnt;
+    int64_t *huge;
+    uint32_t *huge_cnt;
+    uint32_t *huge_clear;
+    uint32_t *hist;
+    int round;
+    Key k;
+};
+
+__device__ __forceinline__ int mis_scan_serial(const int32_t *__restrict__ ci, const uint8_t *st, int64_t b,
+                                               int64_t e, uint64_t kv, Key k) {
+    for (int64_t x = b; x < e; x++) {
+        uint32_t w = (uint32_t)__ldg(ci + x);
+        uint8_t sw = st[w];
+        if (sw == ST_IN) return R_OUT;
+        if (sw == ST_UNDEC && vkey(k, w) > kv) return R_BLK;
+    }
+    return R_IN;
+}
+
+__global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
+    const uint32_t cnt = A.in_list ? *A.in_cnt : (uint32_t)A.implicit_n;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        *A.clear_cnt = 0;
+        *A.huge_clear = 0;
+        if (A.hist && A.round < (1 << 12)) A.hist[A.round] = cnt;
+    }
+    const int lane = lane_id();
+    const int64_t warp_g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t base = warp_g * 32; base < cnt; base += nwarps * 32) {
+        int64_t i = base + lane;
+        int32_t v = -1;
+        if (i < cnt) v = A.in_list ? (A.in_rev ? A.in_list[-1 - i] : A.in_list[i]) : (int32_t)i;
+        bool active = v >= 0 && A.st[v] == ST_UNDEC;
+        int64_t b = 0, e = 0;
+        uint64_t kv = 0;
+        if (active) {
+            b = A.rp[v];
+            e = A.rp[v + 1];
+            kv = vkey(A.k, (uint32_t)v);
+        }
+        int res = R_NONE;
+        int64_t resume = 0;
+        if (active && e - b <= MIS_SMALL) res = mis_scan_serial(A.ci, A.st, b, e, kv, A.k);
+        unsigned longm = __ballot_sync(FULL, active && e - b > MIS_SMALL);
+        while (longm) {
+            const int src = __ffs(longm) - 1;
+            longm &= longm - 1;
+            const int64_t wb = __shfl_sync(FULL, b, src), we = __shfl_sync(FULL, e, src);
+            const uint64_t wk = __shfl_sync(FULL, kv, src);
+            const int64_t lim = min(we, wb + MIS_BUDGET);
+            int r = R_IN;
+            for (int64_t x = wb; x < lim; x += 128) {
+                uint32_t w[4];
+                bool ok[4];
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    int64_t y = x + u * 32 + lane;
+                    ok[u] = y < lim;
+                    w[u] = ok[u] ? (uint32_t)__ldg(A.ci + y) : 0u;
+                }
+                bool fin = false, fblk = false;
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    if (ok[u]) {
+                        uint8_t sw = A.st[w[u]];
+                        fin |= sw == ST_IN;
+                        fblk |= (sw == ST_UNDEC) && (vkey(A.k, w[u]) > wk);
+                    }
+                }
+                if (__any_sync(FULL, fin)) { r = R_OUT; break; }
+                if (__any_sync(FULL, fblk)) { r = R_BLK; break; }
+            }
+            if (r == R_IN && lim < we) r = R_DEFER;
+            if (lane == src) {
+                res = r;
+                resume = lim;
+            }
+        }
+        if (res == R_IN) A.st[v] = ST_IN;
+        else if (res == R_OUT) A.st[v] = ST_OUT;
+        int64_t slot = warp_append(res == R_BLK, A.out_cnt);
+        if (slot >= 0) A.out_list[slot] = v;
+        int64_t hs = warp_append(res == R_DEFER, A.huge_cnt);
+        if (hs >= 0) {
+            A.huge[2 * hs] = v;
+            A.huge[2 * hs + 1] = resume;
+        }
+    }
+}
+
+// deferred long rows: one CTA per vertex, scanning the remainder of its row
+__global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
+    const uint32_t cnt = *A.huge_cnt;
+    for (uint32_t h = blockIdx.x; h < cnt; h += gridDim.x) {
+        const int32_t v = (int32_t)A.huge[2 * h];
+        const int64_t b = A.huge[2 * h + 1], e = A.rp[v + 1];
+        const uint64_t kv = vkey(A.k, (uint32_t)v);
+        int r = R_IN;
+        for (int64_t x = b; x < e; x += 4 * MIS_HUGE_THREADS) {
+            bool fin = false, fblk = false;
+            uint32_t w[4];
+            bool ok[4];
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                int64_t y = x + u * MIS_HUGE_THREADS + threadIdx.x;
+                ok[u] = y < e;
+                w[u] = ok[u] ? (uint32_t)__ldg(A.ci + y) : 0u;
+            }
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                if (ok[u]) {
+                    uint8_t sw = A.st[w[u]];
+                    fin |= sw == ST_IN;
+                    fblk |= (sw == ST_UNDEC) && (vkey(A.k, w[u]) > kv);
+                }
+            }
+            if (__syncthreads_or(fin)) { r = R_OUT; break; }
+            if (__syncthreads_or(fblk)) { r = R_BLK; break; }
+        }
+        if (threadIdx.x == 0) {
+            if (r == R_IN) A.st[v] = ST_IN;
+            else if (r == R_OUT) A.st[v] = ST_OUT;
+            else {
+                uint32_t slot = atomicAdd(A.out_cnt, 1u);
+                A.out_list[slot] = v;
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// MIS-Deg2 fix-up: every cross neighbour of I_L leaves the remaining graph
+__global__ void k_mis_kill_cross(const int64_t *__restrict__ rp_x, const int32_t *__restrict__ ci_x,
+                                 const int32_t *__restrict__ list, const uint32_t *cnt, uint8_t *st) {
+    const uint32_t c = *cnt;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < c; i += gridDim.x * blockDim.x) {
+        int32_t v = list[i];
+        if (st[v] != ST_IN) continue;
+        for (int64_t x = rp_x[v]; x < rp_x[v + 1]; x++) st[ci_x[x]] = ST_OUT;
+    }
+}
+
+// MIS-Rand: classify by cross degree: interior (front list, UNDEC) / boundary B
+// (back list, INACTIVE during phase A)
+__global__ void k_mis_classify_cross(const int64_t *__restrict__ rp_x, int64_t n, uint8_t *st, int32_t *vlist,
+                                     uint32_t *cnt_front, uint32_t *cnt_back) {
+    int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
+        int64_t v = base + threadIdx.x;
+        bool valid = v < n;
+        bool bnd = valid && (rp_x[v + 1] > rp_x[v]);
+        if (valid) st[v] = bnd ? ST_INACTIVE : ST_UNDEC;
+        int64_t sI = warp_append(valid && !bnd, cnt_front);
+        int64_t sB = warp_append(bnd, cnt_back);
+        if (sI >= 0) vlist[sI] = (int32_t)v;
+        if (sB >= 0) vlist[n - 1 - sB] = (int32_t)v;
+    }
+}
+
+// MIS-Rand fix-up: remove N(I_A) (all arcs of interior vertices are intra)
+__global__ void k_mis_kill_all(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci,
+                               const int32_t *__restrict__ list, const uint32_t *cnt, uint8_t *st) {
+    const uint32_t c = *cnt;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < c; i += gridDim.x * blockDim.x) {
+        int32_t v = list[i];
+        if (st[v] != ST_IN) continue;
+        for (int64_t x = rp[v]; x < rp[v + 1]; x++) st[ci[x]] = ST_OUT;
+    }
+}
+
+__global__ void k_mis_reactivate(const int32_t *__restrict__ list_end, const uint32_t *cnt, uint8_t *st) {
+    const uint32_t c = *cnt;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < c; i += gridDim.x * blockDim.x) {
+        int32_t v = list_end[-1 - (int64_t)i];
+        if (st[v] == ST_INACTIVE) st[v] = ST_UNDEC;
+    }
+}
+
+__global__ void k_mis_finish(uint8_t *st, int64_t n, unsigned long long *count) {
+    int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    uint32_t local = 0;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+        uint8_t s = st[v];
+        uint8_t o = (s == ST_IN) ? 1 : 0;
+        st[v] = o;
+        local += o;
+    }
+    if (count) {
+        for (int d = 16; d; d >>= 1) local += __shfl_xor_sync(FULL, local, d);
+        if (lane_id() == 0 && local) atomicAdd(count, (unsigned long long)local);
+    }
+}
+
+// ------------------------------------------------------------------ host side
+void carve_mis_ws(Arena &a, int64_t n, int64_t nnz, MisWs &w) {
+    w.vlist = a.take<int32_t>((size_t)n + 1);
+    w.fr[0] = a.take<int32_t>((size_t)n + 1);
+    w.fr[1] = a.take<int32_t>((size_t)n + 1);
+    w.huge_cap = nnz / MIS_BUDGET + 2;
+    w.huge = a.take<int64_t>((size_t)(2 * w.huge_cap));
+}
+
+static int round_grid() { return num_sms() * (2048 / MIS_THREADS); }
+
+// Run Luby rounds of one phase until the frontier is empty.  Round 0 reads
+// (list0, rev0, cnt0) -- or the implicit range [0, implicit_n) when list0 == nullptr.
+static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp, const int32_t *ci,
+                     const int32_t *list0, int rev0, const uint32_t *cnt0, int64_t implicit_n, int phase) {
+    Ctl *ctl = f.ctl;
+    cudaStream_t s = f.stream;
+    SYM_CUDA(cudaMemsetAsync(ctl->ring, 0, sizeof(ctl->ring) + sizeof(ctl->huge), s));
+    const Key k = stream_key(f.p.seed, TAG_VERTEX, 0);
+    const uint32_t maxr = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
+    const int grid = round_grid();
+    int r = 0;
+    int batch = 4;
+    for (;;) {
+        for (int b = 0; b < batch; b++, r++) {
+            MisRoundArgs A;
+            A.rp = rp;
+            A.ci = ci;
+            A.st = st;
+            if (r == 0) {
+                A.in_list = list0;
+                A.in_rev = rev0;
+                A.in_cnt = cnt0;
+            } else {
+                A.in_list = w.fr[r & 1];
+                A.in_rev = 0;
+                A.in_cnt = &ctl->ring[r % 3];
+            }
+            A.implicit_n = implicit_n;
+            A.out_list = w.fr[(r + 1) & 1];
+            A.out_cnt = &ctl->ring[(r + 1) % 3];
+            A.clear_cnt = &ctl->ring[(r + 2) % 3];
+            A.huge = w.huge;
+            A.huge_cnt = &ctl->huge[r & 1];
+            A.huge_clear = &ctl->huge[(r + 1) & 1];
+            A.hist = (phase == 0) ? ctl->hist : ctl->hist + 2048;
+            A.round = r < 2048 ? r : 2047;
+            A.k = k;
+            prof_begin("mis_round", s);
+            k_mis_round<<<grid, MIS_THREADS, 0, s>>>(A);
+            prof_end(s, -1);
+            SYM_LAUNCH_CHECK();
+            prof_begin("mis_huge", s);
+            k_mis_huge<<<num_sms() * 2, MIS_HUGE_THREADS, 0, s>>>(A);
+            prof_end(s, -1);
+            SYM_LAUNCH_CHECK();
+        }
+        uint32_t left = 0;
+        SYM_TRY(read_u32(&ctl->ring[r % 3], &left, s));
+        if (left == 0) break;
+        if ((uint32_t)r >= maxr) {
+            set_error("MIS phase did not converge within max_rounds");
+            return SYM_EROUNDS;
+        }
+        if (batch < 16) batch *= 2;
+    }
+    if (f.stats) f.stats->rounds[phase] = (uint32_t)r;  // refined from hist below
+    return SYM_OK;
+}
+
+int run_mis(const FlowArgs &f, MisWs &w, uint8_t *st) {
+    const Graph &g = f.g;
+    cudaStream_t s = f.stream;
+    Ctl *ctl = f.ctl;
+    const int kind = f.p.kind;
+    if (kind == SYM_DECOMP_NONE) {
+        SYM_CUDA(cudaMemsetAsync(st, ST_UNDEC, (size_t)g.n, s));
+        SYM_TRY(mis_phase(f, w, st, g.rp, g.ci, nullptr, 0, nullptr, g.n, 0));
+        if (f.stats) f.stats->phase_vertices[0] = g.n;
+    } else if (kind == SYM_DECOMP_DEGK) {
+        // lists V_L (front) and V_H (back); status all undecided
+        SYM_CUDA(cudaMemsetAsync(st, ST_UNDEC, (size_t)g.n, s));
+        SYM_CUDA(cudaMemsetAsync(&ctl->cnt_front, 0, 2 * sizeof(uint32_t), s));
+        SYM_TRY(launch_classify_degk(g, f.p.param, f.hbits, w.vlist, ctl, s));
+        // phase L: I_L = MIS(G_L) on the intra CSR restricted to V_L
+        SYM_TRY(mis_phase(f, w, st, f.split.rp_in, f.split.ci_in, w.vlist, 0, &ctl->cnt_front, 0, 0));
+        // fix-up: remove N(I_L) from V_H through the cross arcs G_C
+        k_mis_kill_cross<<<num_sms() * 4, 256, 0, s>>>(f.split.rp_x, f.split.ci_x, w.vlist, &ctl->cnt_front, st);
+        SYM_LAUNCH_CHECK();
+        // phase R: MIS of the remaining V_H on G_H
+        SYM_TRY(mis_phase(f, w, st, f.split.rp_in, f.split.ci_in, w.vlist + g.n, 1, &ctl->cnt_back, 0, 1));
+    } else {
+        SYM_CUDA(cudaMemsetAsync(&ctl->cnt_front, 0, 2 * sizeof(uint32_t), s));
+        k_mis_classify_cross<<<num_sms() * 8, 256, 0, s>>>(f.split.rp_x, g.n, st, w.vlist, &ctl->cnt_front,
+                                                           &ctl->cnt_back);
+        SYM_LAUNCH_CHECK();
+        // phase A: I_A = MIS of the partition interiors (boundary vertices INACTIVE)
+        SYM_TRY(mis_phase(f, w, st, f.split.rp_in, f.split.ci_in, w.vlist, 0, &ctl->cnt_front, 0, 0));
+        // R = G - N[I_A]
+        k_mis_kill_all<<<num_sms() * 4, 256, 0, s>>>(f.split.rp_in, f.split.ci_in, w.vlist, &ctl->cnt_front, st);
+        SYM_LAUNCH_CHECK();
+        k_mis_reactivate<<<num_sms() * 4, 256, 0, s>>>(w.vlist + g.n, &ctl->cnt_back, st);
+        SYM_LAUNCH_CHECK();
+        // phase B: I_B = MIS(R) on G
+        SYM_TRY(mis_phase(f, w, st, g.rp, g.ci, w.vlist + g.n, 1, &ctl->cnt_back, 0, 1));
+    }
+    unsigned long long *cnt = (f.p.flags & SYM_F_STATS) ? (unsigned long long *)&ctl->result : nullptr;
+    if (cnt) SYM_CUDA(cudaMemsetAsync(cnt, 0, sizeof(uint64_t), s));
+    k_mis_finish<<<num_sms() * 8, 256, 0, s>>>(st, g.n, cnt);
+    SYM_LAUNCH_CHECK();
+    if (f.stats) {
+        uint32_t hist[4096];
+        SYM_CUDA(cudaMemcpyAsync(hist, ctl->hist, sizeof(hist), cudaMemcpyDeviceToHost, s));
+        SYM_CUDA(cudaStreamSynchronize(s));
+        for (int ph = 0; ph < 2; ph++) {
+            uint32_t rr = 0;
+            for (int i = 0; i < 2048 && i < (int)f.stats->rounds[ph]; i++) rr += hist[ph * 2048 + i] ? 1 : 0;
+            f.stats->rounds[ph] = rr;
+            f.stats->phase_vertices[ph] = hist[ph * 2048];
+        }
+        if (cnt) {
+            uint64_t c = 0;
+            SYM_TRY(read_u64(&ctl->result, &c, s));
+            f.stats->result_size = (int64_t)c;
+        }
+    }
+    return SYM_OK;
+}
+
+}  // namespace sym

@@ -1,0 +1,402 @@
+// mm.cu -- handshake (LMAX) matching rounds and the MM flows.
+//
+// Round r, for every vertex u of the frontier (Birn et al. [5]):
+//   resolve: if u picked p in round r-1 and p picked u, the edge is matched
+//            (both endpoints write their own mate; "mutual picks are matched");
+//   pick:    otherwise u picks the heaviest edge (pe(u,w), w) to a neighbour w that is
+//            still unmatched in the phase graph; no such neighbour => u is dead.
+// Picks are double-buffered (pick[r&1] written in round r, pick[(r+1)&1] read), so the
+// mutual test always compares round r-1 picks.  A vertex that matches or dies writes
+// -1 as its current pick, so stale picks never pair with it.  mate only moves
+// -1 -> partner, so reading it in place (stale) can only add dead candidates; every
+// mutual pick is then locally heaviest among truly live edges, which is the greedy
+// (GM) order with the same fixed priorities ([6]).
+//
+// Round 0 of the first phase specialises away the mate gathers (nothing is matched
+// yet): a pure streaming pass over col_idx with the edge hash computed on the fly.
+#include "internal.h"
+
+namespace sym {
+
+constexpr int MM_SMALL = 8;
+constexpr int MM_BUDGET = 4096;  // rows longer than this go to the CTA kernel
+constexpr int MM_THREADS = 256;
+constexpr int MM_HUGE_THREADS = 512;
+
+struct MmRoundArgs {
+    const int64_t *rp, *rp2;  // dual mode: hbits[u] ? (rp2, ci2) : (rp, ci)
+    const int32_t *ci, *ci2;
+    const uint32_t *hbits;
+    int dual;
+    int32_t *mate;
+    const int32_t *pick_prev;
+    int32_t *pick_cur;
+    const int32_t *in_list;
+    int in_rev;
+    const uint32_t *in_cnt;
+    int64_t implicit_n;
+    int32_t *out_list;
+    uint32_t *out_cnt;
+    uint32_t *clear_cnt;
+    int32_t *huge;
+    uint32_t *huge_cnt;
+    uint32_t *huge_clear;
+    uint32_t *hist;
+    int round;
+    Key k;
+};
+
+__device__ __forceinline__ void mm_row(const MmRoundArgs &A, int32_t u, int64_t &b, int64_t &e, const int32_t *&ci) {
+    if (A.dual && ((A.hbits[u >> 5] >> (u & 31)) & 1u)) {
+        b = A.rp2[u];
+        e = A.rp2[u + 1];
+        ci = A.ci2;
+    } else {
+        b = A.rp[u];
+        e = A.rp[u + 1];
+        ci = A.ci;
+    }
+}
+
+template <bool RESOLVE, bool MATE>
+__global__ void __launch_bounds__(MM_THREADS) k_mm_round(MmRoundArgs A) {
+    const uint32_t cnt = A.in_list ? *A.in_cnt : (uint32_t)A.implicit_n;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        *A.clear_cnt = 0;
+        *A.huge_clear = 0;
+        if (A.hist && A.round < 2048) A.hist[A.round] = cnt;
+    }
+    const int lane = lane_id();
+    const int64_t warp_g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t base = warp_g * 32; base < cnt; base += nwarps * 32) {
+        int64_t i = base + lane;
+        int32_t u = -1;
+        if (i < cnt) u = A.in_list ? (A.in_rev ? A.in_list[-1 - i] : A.in_list[i]) : (int32_t)i;
+        bool active = u >= 0;
+        if (RESOLVE && active) {
+            int32_t p = A.pick_prev[u];
+            if (p >= 0 && A.pick_prev[p] == u) {
+                A.mate[u] = p;
+                A.pick_cur[u] = -1;
+                active = false;
+            } else if (A.mate[u] >= 0) {  // defensive: never re-pick a matched vertex
+                A.pick_cur[u] = -1;
+                active = false;
+            }
+        }
+        int64_t b = 0, e = 0;
+        const int32_t *ci = A.ci;
+        if (active) mm_row(A, u, b, e, ci);
+        const int64_t d = e - b;
+        uint64_t best = 0;
+        bool has = false;
+        if (active && d <= MM_SMALL) {
+            for (int64_t x = b; x < e; x++) {
+                uint32_t w = (uint32_t)__ldg(ci + x);
+                if (!MATE || A.mate[w] < 0) {
+                    uint64_t kk = ekey(A.k, (uint32_t)u, w);
+                    if (!has || kk > best) best = kk;
+                    has = true;
+                }
+            }
+        }
+        // warp-cooperative argmax for medium rows
+        unsigned medm = __ballot_sync(FULL, active && d > MM_SMALL && d <= MM_BUDGET);
+        while (medm) {
+            const int src = __ffs(medm) - 1;
+            medm &= medm - 1;
+            const int64_t wb = __shfl_sync(FULL, b, src), we = __shfl_sync(FULL, e, src);
+            const int32_t wu = __shfl_sync(FULL, u, src);
+            const int32_t *wci = (const int32_t *)__shfl_sync(FULL, (unsigned long long)ci, src);
+            uint64_t lb = 0;
+            bool lh = false;
+            for (int64_t x = wb; x < we; x += 128) {
+                uint32_t w[4];
+                bool ok[4];
+#pragma unroll
+                for (int q = 0; q < 4; q++) {
+                    int64_t y = x + q * 32 + lane;
+                    ok[q] = y < we;
+                    w[q] = ok[q] ? (uint32_t)__ldg(wci + y) : 0u;
+                }
+#pragma unroll
+                for (int q = 0; q < 4; q++) {
+                    if (ok[q] && (!MATE || A.mate[w[q]] < 0)) {
+                        uint64_t kk = ekey(A.k, (uint32_t)wu, w[q]);
+                        if (!lh || kk > lb) lb = kk;
+                        lh = true;
+                    }
+                }
+            }
+#pragma unroll
+            for (int dd = 16; dd; dd >>= 1) {
+                uint64_t o = __shfl_xor_sync(FULL, lb, dd);
+                lb = o > lb ? o : lb;
+            }
+            bool anyh = __any_sync(FULL, lh);
+            if (lane == src) {
+                best = lb;
+                has = anyh;
+            }
+        }
+        bool defer = active && d > MM_BUDGET;
+        if (active && !defer) A.pick_cur[u] = has ? (int32_t)(uint32_t)best : -1;
+        int64_t slot = warp_append(active && !defer && has, A.out_cnt);
+        if (slot >= 0) A.out_list[slot] = u;
+        int64_t hs = warp_append(defer, A.huge_cnt);
+        if (hs >= 0) A.huge[hs] = u;
+    }
+}
+
+// rows longer than MM_BUDGET: one CTA per vertex, block argmax
+template <bool MATE>
+__global__ void __launch_bounds__(MM_HUGE_THREADS) k_mm_huge(MmRoundArgs A) {
+    const uint32_t cnt = *A.huge_cnt;
+    __shared__ unsigned long long s_best[MM_HUGE_THREADS / 32];
+    __shared__ int s_has[MM_HUGE_THREADS / 32];
+    const int lane = lane_id(), warp = threadIdx.x >> 5;
+    for (uint32_t h = blockIdx.x; h < cnt; h += gridDim.x) {
+        const int32_t u = A.huge[h];
+        int64_t b, e;
+        const int32_t *ci;
+        mm_row(A, u, b, e, ci);
+        uint64_t lb = 0;
+        bool lh = false;
+        for (int64_t x = b; x < e; x += 4 * MM_HUGE_THREADS) {
+            uint32_t w[4];
+            bool ok[4];
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                int64_t y = x + q * MM_HUGE_THREADS + threadIdx.x;
+                ok[q] = y < e;
+                w[q] = ok[q] ? (uint32_t)__ldg(ci + y) : 0u;
+            }
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                if (ok[q] && (!MATE || A.mate[w[q]] < 0)) {
+                    uint64_t kk = ekey(A.k, (uint32_t)u, w[q]);
+                    if (!lh || kk > lb) lb = kk;
+                    lh = true;
+                }
+            }
+        }
+#pragma unroll
+        for (int dd = 16; dd; dd >>= 1) {
+            uint64_t o = __shfl_xor_sync(FULL, lb, dd);
+            lb = o > lb ? o : lb;
+        }
+        bool wh = __any_sync(FULL, lh);
+        if (lane == 0) {
+            s_best[warp] = lb;
+            s_has[warp] = wh;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            uint64_t bb = 0;
+            bool hh = false;
+            for (int q = 0; q < MM_HUGE_THREADS / 32; q++) {
+                if (s_has[q]) {
+                    bb = (!hh || s_best[q] > bb) ? s_best[q] : bb;
+                    hh = true;
+                }
+            }
+            A.pick_cur[u] = hh ? (int32_t)(uint32_t)bb : -1;
+            if (hh) {
+                uint32_t slot = atomicAdd(A.out_cnt, 1u);
+                A.out_list[slot] = u;
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// phase-2 frontier: unmatched vertices that have phase-2 arcs
+__global__ void k_mm_phase2_list(const int64_t *__restrict__ rp, const int64_t *__restrict__ rp2,
+                                 const uint32_t *__restrict__ hbits, int dual, int64_t n, const int32_t *mate,
+                                 int32_t *list, uint32_t *cnt) {
+    int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
+        int64_t v = base + threadIdx.x;
+        bool take = false;
+        if (v < n && mate[v] < 0) {
+            bool useX = dual ? ((hbits[v >> 5] >> (v & 31)) & 1u) : true;
+            const int64_t *r = useX ? rp2 : rp;
+            take = r[v + 1] > r[v];
+        }
+        int64_t s = warp_append(take, cnt);
+        if (s >= 0) list[s] = (int32_t)v;
+    }
+}
+
+__global__ void k_mm_count(const int32_t *mate, int64_t n, unsigned long long *count) {
+    int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    uint32_t local = 0;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) local += mate[v] > v;
+    for (int d = 16; d; d >>= 1) local += __shfl_xor_sync(FULL, local, d);
+    if (lane_id() == 0 && local) atomicAdd(count, (unsigned long long)local);
+}
+
+// ------------------------------------------------------------------ host side
+void carve_mm_ws(Arena &a, int64_t n, int64_t nnz, MmWs &w) {
+    w.pick[0] = a.take<int32_t>((size_t)n + 1);
+    w.pick[1] = a.take<int32_t>((size_t)n + 1);
+    w.vlist = a.take<int32_t>((size_t)n + 1);
+    w.fr[0] = a.take<int32_t>((size_t)n + 1);
+    w.fr[1] = a.take<int32_t>((size_t)n + 1);
+    w.huge_cap = nnz / MM_BUDGET + 2;
+    w.huge = reinterpret_cast<int64_t *>(a.take<int32_t>((size_t)w.huge_cap));
+}
+
+struct MmPhase {
+    const int64_t *rp, *rp2;
+    const int32_t *ci, *ci2;
+    int dual;
+    const int32_t *list0;
+    int rev0;
+    const uint32_t *cnt0;
+    int64_t implicit_n;
+    bool first;  // no vertex matched yet: round 0 skips the mate gathers
+    int64_t nnz = -1;  // arcs of the phase CSR when known on the host (profiling only)
+};
+
+static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph, int phase) {
+    Ctl *ctl = f.ctl;
+    cudaStream_t s = f.stream;
+    SYM_CUDA(cudaMemsetAsync(ctl->ring, 0, sizeof(ctl->ring) + sizeof(ctl->huge), s));
+    const Key k = stream_key(f.p.seed, TAG_EDGE, 0);
+    const uint32_t maxr = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
+    const int grid = num_sms() * (2048 / MM_THREADS);
+    int r = 0, batch = 4;
+    for (;;) {
+        for (int bb = 0; bb < batch; bb++, r++) {
+            MmRoundArgs A;
+            A.rp = ph.rp;
+            A.rp2 = ph.rp2;
+            A.ci = ph.ci;
+            A.ci2 = ph.ci2;
+            A.hbits = f.hbits;
+            A.dual = ph.dual;
+            A.mate = mate;
+            A.pick_prev = w.pick[(r + 1) & 1];
+            A.pick_cur = w.pick[r & 1];
+            if (r == 0) {
+                A.in_list = ph.list0;
+                A.in_rev = ph.rev0;
+                A.in_cnt = ph.cnt0;
+            } else {
+                A.in_list = w.fr[r & 1];
+                A.in_rev = 0;
+                A.in_cnt = &ctl->ring[r % 3];
+            }
+            A.implicit_n = ph.implicit_n;
+            A.out_list = w.fr[(r + 1) & 1];
+            A.out_cnt = &ctl->ring[(r + 1) % 3];
+            A.clear_cnt = &ctl->ring[(r + 2) % 3];
+            A.huge = reinterpret_cast<int32_t *>(w.huge);
+            A.huge_cnt = &ctl->huge[r & 1];
+            A.huge_clear = &ctl->huge[(r + 1) & 1];
+            A.hist = ctl->hist + phase * 2048;
+            A.round = r < 2048 ? r : 2047;
+            A.k = k;
+            // round 0 of a phase has nothing to resolve (its pick buffers hold stale or
+            // uninitialised values); round 0 of the first phase has nothing matched yet
+            if (r == 0 && ph.first) {
+                // first round over an implicit vertex range streams the whole phase
+                // CSR: 4 B/arc + row_ptr (8 B) + pick (4 B) per vertex
+                double bytes = (ph.list0 == nullptr && ph.nnz >= 0) ? 4.0 * ph.nnz + 12.0 * ph.implicit_n : -1.0;
+                prof_begin("mm_round0", s);
+                k_mm_round<false, false><<<grid, MM_THREADS, 0, s>>>(A);
+                prof_end(s, bytes);
+                SYM_LAUNCH_CHECK();
+                prof_begin("mm_huge", s);
+                k_mm_huge<false><<<num_sms() * 2, MM_HUGE_THREADS, 0, s>>>(A);
+                prof_end(s, -1);
+            } else if (r == 0) {
+                prof_begin("mm_round", s);
+                k_mm_round<false, true><<<grid, MM_THREADS, 0, s>>>(A);
+                prof_end(s, -1);
+                SYM_LAUNCH_CHECK();
+                prof_begin("mm_huge", s);
+                k_mm_huge<true><<<num_sms() * 2, MM_HUGE_THREADS, 0, s>>>(A);
+                prof_end(s, -1);
+            } else {
+                prof_begin("mm_round", s);
+                k_mm_round<true, true><<<grid, MM_THREADS, 0, s>>>(A);
+                prof_end(s, -1);
+                SYM_LAUNCH_CHECK();
+                prof_begin("mm_huge", s);
+                k_mm_huge<true><<<num_sms() * 2, MM_HUGE_THREADS, 0, s>>>(A);
+                prof_end(s, -1);
+            }
+            SYM_LAUNCH_CHECK();
+        }
+        uint32_t left = 0;
+        SYM_TRY(read_u32(&ctl->ring[r % 3], &left, s));
+        if (left == 0) break;
+        if ((uint32_t)r >= maxr) {
+            set_error("MM phase did not converge within max_rounds");
+            return SYM_EROUNDS;
+        }
+        if (batch < 16) batch *= 2;
+    }
+    if (f.stats) f.stats->rounds[phase] = (uint32_t)r;
+    return SYM_OK;
+}
+
+int run_mm(const FlowArgs &f, MmWs &w, int32_t *mate) {
+    const Graph &g = f.g;
+    cudaStream_t s = f.stream;
+    Ctl *ctl = f.ctl;
+    SYM_CUDA(cudaMemsetAsync(mate, 0xff, sizeof(int32_t) * (size_t)g.n, s));
+    const int kind = f.p.kind;
+    MmPhase ph{};
+    if (kind == SYM_DECOMP_NONE) {
+        ph = MmPhase{g.rp, nullptr, g.ci, nullptr, 0, nullptr, 0, nullptr, g.n, true};
+        ph.nnz = g.nnz;
+        SYM_TRY(mm_phase(f, w, mate, ph, 0));
+    } else {
+        // phase 1: M_IS = MM(union G_i) (RAND, Alg 5 l.5) / M_H = MM(G_H) (DEGk, Alg 6 l.5)
+        if (kind == SYM_DECOMP_RAND) {
+            ph = MmPhase{f.split.rp_in, nullptr, f.split.ci_in, nullptr, 0, nullptr, 0, nullptr, g.n, true};
+            ph.nnz = f.split.nnz_in;
+        } else {
+            SYM_CUDA(cudaMemsetAsync(&ctl->cnt_front, 0, 2 * sizeof(uint32_t), s));
+            SYM_TRY(launch_classify_degk(g, f.p.param, f.hbits, w.vlist, ctl, s));
+            ph = MmPhase{f.split.rp_in, nullptr, f.split.ci_in, nullptr, 0, w.vlist + g.n, 1, &ctl->cnt_back, 0,
+                         true};
+        }
+        SYM_TRY(mm_phase(f, w, mate, ph, 0));
+        // phase 2: V' = unmatched; MM(G_{k+1}[V']) (Alg 5 l.6-7) / MM(G_LC[V']) (Alg 6 l.6-7)
+        const int dual = kind == SYM_DECOMP_DEGK;
+        SYM_CUDA(cudaMemsetAsync(&ctl->cnt_front, 0, sizeof(uint32_t), s));
+        k_mm_phase2_list<<<num_sms() * 8, 256, 0, s>>>(g.rp, f.split.rp_x, f.hbits, dual, g.n, mate, w.vlist,
+                                                         &ctl->cnt_front);
+        SYM_LAUNCH_CHECK();
+        if (dual) ph = MmPhase{g.rp, f.split.rp_x, g.ci, f.split.ci_x, 1, w.vlist, 0, &ctl->cnt_front, 0, false};
+        else ph = MmPhase{f.split.rp_x, nullptr, f.split.ci_x, nullptr, 0, w.vlist, 0, &ctl->cnt_front, 0, false};
+        SYM_TRY(mm_phase(f, w, mate, ph, 1));
+    }
+    if (f.stats) {
+        uint32_t hist[4096];
+        SYM_CUDA(cudaMemcpyAsync(hist, ctl->hist, sizeof(hist), cudaMemcpyDeviceToHost, s));
+        SYM_CUDA(cudaStreamSynchronize(s));
+        for (int ph2 = 0; ph2 < 2; ph2++) {
+            uint32_t rr = 0;
+            for (int i = 0; i < 2048 && i < (int)f.stats->rounds[ph2]; i++) rr += hist[ph2 * 2048 + i] ? 1 : 0;
+            f.stats->rounds[ph2] = rr;
+            f.stats->phase_vertices[ph2] = hist[ph2 * 2048];
+        }
+        if (f.p.flags & SYM_F_STATS) {
+            SYM_CUDA(cudaMemsetAsync(&ctl->result, 0, sizeof(uint64_t), s));
+            k_mm_count<<<num_sms() * 8, 256, 0, s>>>(mate, g.n, (unsigned long long *)&ctl->result);
+            SYM_LAUNCH_CHECK();
+            uint64_t c = 0;
+            SYM_TRY(read_u64(&ctl->result, &c, s));
+            f.stats->result_size = (int64_t)c;
+        }
+    }
+    return SYM_OK;
+}
+
+}  // namespace sym

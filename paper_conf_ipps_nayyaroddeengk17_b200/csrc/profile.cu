@@ -1,0 +1,103 @@
+// profile.cu -- optional per-kernel-class device timing (sym_profile_enable/collect).
+// CUDA event pairs are recorded on the launching stream around each hot launch;
+// collection synchronises them after the caller's timed region.
+#include <cstring>
+#include <map>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+namespace sym {
+
+namespace {
+struct Rec {
+    std::string cls;
+    cudaEvent_t a, b;
+    double bytes;
+};
+bool g_on = false;
+std::vector<Rec> g_recs;
+std::vector<cudaEvent_t> g_pool;
+std::vector<std::pair<std::string, double>> g_open;  // pending begin (class, bytes)
+std::vector<cudaEvent_t> g_open_ev;
+
+cudaEvent_t get_event() {
+    if (!g_pool.empty()) {
+        cudaEvent_t e = g_pool.back();
+        g_pool.pop_back();
+        return e;
+    }
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    return e;
+}
+}  // namespace
+
+bool prof_on() { return g_on; }
+
+void prof_begin(const char *cls, cudaStream_t s) {
+    if (!g_on) return;
+    cudaEvent_t e = get_event();
+    cudaEventRecord(e, s);
+    g_open.emplace_back(cls, 0.0);
+    g_open_ev.push_back(e);
+}
+
+void prof_end(cudaStream_t s, double bytes) {
+    if (!g_on || g_open.empty()) return;
+    cudaEvent_t e = get_event();
+    cudaEventRecord(e, s);
+    Rec r{g_open.back().first, g_open_ev.back(), e, bytes};
+    g_open.pop_back();
+    g_open_ev.pop_back();
+    g_recs.push_back(r);
+}
+
+}  // namespace sym
+
+using namespace sym;
+
+extern "C" int sym_profile_enable(int on) {
+    g_on = on != 0;
+    return SYM_OK;
+}
+
+extern "C" int sym_profile_collect(sym_kernel_profile *out, int max_entries, int *count) {
+    struct Acc {
+        int64_t n = 0;
+        double ms = 0, bytes = 0;
+        bool known = true;
+    };
+    std::map<std::string, Acc> acc;
+    std::vector<std::string> order;
+    for (auto &r : g_recs) {
+        cudaError_t e = cudaEventSynchronize(r.b);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaEventSynchronize", __FILE__, __LINE__);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, r.a, r.b);
+        if (!acc.count(r.cls)) order.push_back(r.cls);
+        Acc &x = acc[r.cls];
+        x.n++;
+        x.ms += ms;
+        if (r.bytes < 0) x.known = false;
+        else x.bytes += r.bytes;
+        g_pool.push_back(r.a);
+        g_pool.push_back(r.b);
+    }
+    g_recs.clear();
+    int c = 0;
+    for (auto &name : order) {
+        if (out && c < max_entries) {
+            Acc &x = acc[name];
+            memset(&out[c], 0, sizeof(out[c]));
+            strncpy(out[c].name, name.c_str(), sizeof(out[c].name) - 1);
+            out[c].launches = x.n;
+            out[c].ms = x.ms;
+            out[c].alg_bytes = x.known ? x.bytes : -1.0;
+        }
+        c++;
+    }
+    if (count) *count = c;
+    return SYM_OK;
+}
