@@ -135,10 +135,11 @@ struct MmWs {
 struct ColorWs {
     uint32_t *cnt = nullptr;       // pending higher-priority neighbours
     uint32_t *bits = nullptr;      // forbidden-colour bitmaps, (deg+1) bits per vertex
-    int32_t *queue = nullptr;      // ready queue (each vertex enqueued once)
+    int64_t bits_words = 0;
+    int32_t *queue = nullptr;      // deferred long rows of the init pass
     int32_t *vlist = nullptr;
     uint8_t *mark = nullptr;       // COLOR-RAND V'
-    int64_t *task = nullptr;
+    int64_t *task = nullptr;       // two task lists (ping-pong), queue_cap each
     int64_t queue_cap = 0;
 };
 
