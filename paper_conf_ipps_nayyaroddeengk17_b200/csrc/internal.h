@@ -76,7 +76,7 @@ struct Graph {
 
 // ------------------------------------------------------------------ decomposition (decompose.cu)
 constexpr int SPLIT_THREADS = 256;
-constexpr int SPLIT_PER_THREAD = 8;
+constexpr int SPLIT_PER_THREAD = 16;
 constexpr int SPLIT_TILE = SPLIT_THREADS * SPLIT_PER_THREAD;  // arcs per tile
 
 struct SplitWs {

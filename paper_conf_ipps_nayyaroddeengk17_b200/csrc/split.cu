@@ -80,28 +80,48 @@ __device__ __forceinline__ T warp_incl_scan(T x, Op op) {
 // ------------------------------------------------------------------ the split
 constexpr uint64_t LB_AGG = 1ULL << 62, LB_INC = 2ULL << 62, LB_VAL = (1ULL << 62) - 1;
 
+// One tile = SPLIT_TILE consecutive arcs = SPLIT_PER_THREAD per thread (blocked).
+// Tile id = blockIdx.x: CUDA dispatches blocks in index order, so every predecessor
+// of a tile is resident or finished when the tile looks back (as CUB's single-pass
+// scans rely on).
 template <int KIND, bool VEC>
 __global__ void __launch_bounds__(SPLIT_THREADS)
     k_split(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, int64_t n, int64_t nnz,
             const int64_t *__restrict__ first_row, int64_t ntiles, const uint32_t *__restrict__ hbits, Key kr,
-            uint32_t p, uint64_t *tile_state, uint32_t *tile_counter, int64_t *__restrict__ rp_in,
-            int32_t *__restrict__ ci_in, int64_t *__restrict__ rp_x, int32_t *__restrict__ ci_x) {
+            uint32_t p, uint64_t *tile_state, int64_t *__restrict__ rp_in, int32_t *__restrict__ ci_in,
+            int64_t *__restrict__ rp_x, int32_t *__restrict__ ci_x) {
     constexpr int T = SPLIT_TILE, V = SPLIT_PER_THREAD, NT = SPLIT_THREADS, NW = NT / 32;
-    __shared__ __align__(16) int32_t s_head[T];   // head position of the row owning each arc
-    __shared__ __align__(16) uint16_t s_cls[T];   // class of the row whose head is here
+    static_assert(V % 4 == 0 && T < 32768, "tile layout");
+    __shared__ __align__(16) int16_t s_head[T];   // head position of the row owning each arc, or -1
+    __shared__ __align__(16) uint16_t s_cls[T];   // class of the row whose head is at this position
     __shared__ __align__(16) int32_t s_out[T];    // compacted tile: intra then cross
     __shared__ __align__(16) uint16_t s_excl[T + 8];
     __shared__ int32_t s_wsum[NW];
     __shared__ int64_t s_prefix;
-    __shared__ int64_t s_tile;
     __shared__ uint32_t s_cls0;
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (tid == 0) s_tile = atomicAdd(tile_counter, 1u);
-    __syncthreads();
-    const int64_t t = s_tile;
+    const int64_t t = blockIdx.x;
     const int64_t a = t * T;
     const int len = (int)min((int64_t)T, nnz - a);
+    const int j0 = tid * V;
+
+    // 1. issue this thread's column loads first (streaming, 128-bit)
+    int32_t dst[V];
+    if (VEC && j0 + V <= len) {
+        const int4 *p4 = reinterpret_cast<const int4 *>(ci + a + j0);
+#pragma unroll
+        for (int q = 0; q < V / 4; q++) {
+            int4 x = __ldcs(p4 + q);
+            dst[4 * q] = x.x;
+            dst[4 * q + 1] = x.y;
+            dst[4 * q + 2] = x.z;
+            dst[4 * q + 3] = x.w;
+        }
+    } else {
+#pragma unroll
+        for (int i = 0; i < V; i++) dst[i] = (j0 + i < len) ? __ldcs(ci + a + j0 + i) : 0;
+    }
     const int64_t r_begin = first_row[t];
     const int64_t r_end = (t + 1 < ntiles) ? first_row[t + 1] : n + 1;
 
@@ -111,8 +131,11 @@ __global__ void __launch_bounds__(SPLIT_THREADS)
         return 0u;
     };
 
-    // 1. heads of the non-empty rows starting in this tile
-    for (int j = tid; j < T; j += NT) s_head[j] = -1;
+    // 2. heads of the non-empty rows starting in this tile
+    {
+        int4 m1 = make_int4(-1, -1, -1, -1);
+        for (int j = tid * 8; j < T; j += NT * 8) *reinterpret_cast<int4 *>(s_head + j) = m1;
+    }
     if (tid == 0) s_cls0 = (r_begin > 0) ? vclass((uint32_t)(r_begin - 1)) : 0u;
     __syncthreads();
     for (int64_t r = r_begin + tid; r < r_end; r += NT) {
@@ -120,37 +143,30 @@ __global__ void __launch_bounds__(SPLIT_THREADS)
         int64_t s = rp[r], e = rp[r + 1];
         if (e > s) {
             int j = (int)(s - a);
-            s_head[j] = j;
+            s_head[j] = (int16_t)j;
             s_cls[j] = (uint16_t)vclass((uint32_t)r);
         }
     }
     __syncthreads();
 
-    // 2. this thread's V consecutive arcs: destination ids and head positions
-    int32_t dst[V];
-    int hp[V];
-    const int j0 = tid * V;
-    if (VEC && j0 + V <= len) {
-        const int4 *p4 = reinterpret_cast<const int4 *>(ci + a + j0);
-        int4 x0 = __ldcs(p4), x1 = __ldcs(p4 + 1);
-        dst[0] = x0.x; dst[1] = x0.y; dst[2] = x0.z; dst[3] = x0.w;
-        dst[4] = x1.x; dst[5] = x1.y; dst[6] = x1.z; dst[7] = x1.w;
-    } else {
+    // 3. the source row of each arc = last head at or before it: thread-local max,
+    //    block exclusive max-scan, then the intra flags
+    int hmax = -1;
 #pragma unroll
-        for (int i = 0; i < V; i++) dst[i] = (j0 + i < len) ? __ldcs(ci + a + j0 + i) : 0;
-    }
-    {
-        const int4 *h4 = reinterpret_cast<const int4 *>(s_head + j0);
-        int4 h0 = h4[0], h1 = h4[1];
-        hp[0] = h0.x; hp[1] = h0.y; hp[2] = h0.z; hp[3] = h0.w;
-        hp[4] = h1.x; hp[5] = h1.y; hp[6] = h1.z; hp[7] = h1.w;
-    }
-    // running max inside the thread, then exclusive max-scan across threads
+    for (int q = 0; q < V / 8; q++) {
+        int4 h = *reinterpret_cast<const int4 *>(s_head + j0 + 8 * q);
+        const int16_t *hh = reinterpret_cast<const int16_t *>(&h);
 #pragma unroll
-    for (int i = 1; i < V; i++) hp[i] = max(hp[i], hp[i - 1]);
+        for (int i = 0; i < 8; i++) hmax = max(hmax, (int)hh[i]);
+    }
     int carry;
     {
-        int incl = warp_incl_scan(hp[V - 1], [](int x, int y) { return max(x, y); });
+        int incl = hmax;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            int y = __shfl_up_sync(FULL, incl, d);
+            if (lane >= d) incl = max(incl, y);
+        }
         if (lane == 31) s_wsum[warp] = incl;
         int excl_w = __shfl_up_sync(FULL, incl, 1);
         if (lane == 0) excl_w = -1;
@@ -158,69 +174,95 @@ __global__ void __launch_bounds__(SPLIT_THREADS)
         int wcarry = -1;
         for (int w = 0; w < warp; w++) wcarry = max(wcarry, s_wsum[w]);
         carry = max(excl_w, wcarry);
-        __syncthreads();
     }
-    // 3. intra flags
     uint32_t flags = 0;
     int cnt = 0;
+    {
+        int h = carry;
 #pragma unroll
-    for (int i = 0; i < V; i++) {
-        int h = max(hp[i], carry);
-        if (j0 + i < len) {
-            uint32_t cs = (h >= 0) ? (uint32_t)s_cls[h] : s_cls0;
-            bool intra = (KIND == KIND_NONE) ? true : (vclass((uint32_t)dst[i]) == cs);
-            flags |= (intra ? 1u : 0u) << i;
-            cnt += intra;
+        for (int q = 0; q < V / 8; q++) {
+            int4 hv = *reinterpret_cast<const int4 *>(s_head + j0 + 8 * q);
+            const int16_t *hh = reinterpret_cast<const int16_t *>(&hv);
+#pragma unroll
+            for (int i = 0; i < 8; i++) {
+                const int k = 8 * q + i;
+                h = max(h, (int)hh[i]);
+                if (j0 + k < len) {
+                    uint32_t cs = (h >= 0) ? (uint32_t)s_cls[h] : s_cls0;
+                    bool intra = (KIND == KIND_NONE) ? true : (vclass((uint32_t)dst[k]) == cs);
+                    flags |= (intra ? 1u : 0u) << k;
+                    cnt += intra;
+                }
+            }
         }
     }
-    // 4. block exclusive sum of cnt
-    int excl;
-    int total;
+    __syncthreads();  // s_wsum reuse
+    // 4. block exclusive sum of the intra counts
+    int excl, total;
     {
-        int incl = warp_incl_scan(cnt, [](int x, int y) { return x + y; });
+        int incl = cnt;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            int y = __shfl_up_sync(FULL, incl, d);
+            if (lane >= d) incl += y;
+        }
         if (lane == 31) s_wsum[warp] = incl;
         __syncthreads();
         int wbase = 0;
         total = 0;
+#pragma unroll
         for (int w = 0; w < NW; w++) {
             int sv = s_wsum[w];
-            if (w < warp) wbase += sv;
+            wbase += (w < warp) ? sv : 0;
             total += sv;
         }
         excl = wbase + incl - cnt;
     }
-    // 5. decoupled look-back for the tile's global intra prefix
-    if (warp == 0) {
-        int64_t prefix = 0;
-        if (t == 0) {
-            if (lane == 0) atomicExch((unsigned long long *)&tile_state[0], (unsigned long long)(LB_INC | (uint64_t)total));
-        } else {
-            if (lane == 0) atomicExch((unsigned long long *)&tile_state[t], (unsigned long long)(LB_AGG | (uint64_t)total));
-            int64_t pos = t - 1;
-            for (;;) {
-                int64_t idx = pos - lane;
-                uint64_t sv = LB_INC;  // idx < 0 acts as an inclusive zero
-                if (idx >= 0) {
-                    do {
-                        sv = ld_volatile_u64(&tile_state[idx]);
-                    } while ((sv >> 62) == 0);
-                }
-                unsigned inc = __ballot_sync(FULL, (sv >> 62) == 2);
-                int64_t val = (int64_t)(sv & LB_VAL);
-                int upto = inc ? (__ffs(inc) - 1) : 31;
-                int64_t contrib = (lane <= upto) ? val : 0;
-#pragma unroll
-                for (int d = 16; d; d >>= 1) contrib += __shfl_xor_sync(FULL, contrib, d);
-                prefix += contrib;
-                if (inc) break;
-                pos -= 32;
-            }
-            if (lane == 0)
-                atomicExch((unsigned long long *)&tile_state[t], (unsigned long long)(LB_INC | (uint64_t)(prefix + total)));
+    // 5. decoupled look-back for the tile's global intra prefix, by the whole CTA:
+    //    NT predecessors per step (a one-warp look-back walks ~tiles_in_flight/32
+    //    dependent L2 reads per tile, which caps the kernel near 2 TB/s)
+    if (t == 0) {
+        if (tid == 0) {
+            atomicExch((unsigned long long *)&tile_state[0], (unsigned long long)(LB_INC | (uint64_t)total));
+            s_prefix = 0;
         }
-        if (lane == 0) s_prefix = prefix;
+    } else {
+        __shared__ int s_upto[NW];
+        __shared__ long long s_part[NW];
+        if (tid == 0) atomicExch((unsigned long long *)&tile_state[t], (unsigned long long)(LB_AGG | (uint64_t)total));
+        int64_t prefix = 0;
+        int64_t pos = t - 1;
+        for (;;) {
+            const int64_t idx = pos - tid;  // tid 0 = nearest predecessor
+            uint64_t sv = LB_INC;           // idx < 0 acts as an inclusive zero
+            if (idx >= 0) {
+                do {
+                    sv = ld_volatile_u64(&tile_state[idx]);
+                } while ((sv >> 62) == 0);
+            }
+            const unsigned inc = __ballot_sync(FULL, (sv >> 62) == 2);
+            if (lane == 0) s_upto[warp] = inc ? warp * 32 + __ffs(inc) - 1 : NT;
+            __syncthreads();
+            int upto = NT;
+#pragma unroll
+            for (int w = 0; w < NW; w++) upto = min(upto, s_upto[w]);
+            long long contrib = (tid <= upto) ? (long long)(sv & LB_VAL) : 0;
+#pragma unroll
+            for (int d = 16; d; d >>= 1) contrib += __shfl_xor_sync(FULL, contrib, d);
+            if (lane == 0) s_part[warp] = contrib;
+            __syncthreads();
+#pragma unroll
+            for (int w = 0; w < NW; w++) prefix += s_part[w];
+            __syncthreads();
+            if (upto < NT) break;
+            pos -= NT;
+        }
+        if (tid == 0) {
+            atomicExch((unsigned long long *)&tile_state[t], (unsigned long long)(LB_INC | (uint64_t)(prefix + total)));
+            s_prefix = prefix;
+        }
     }
-    // 6. stage the compacted tile in shared memory, and the per-position intra prefix
+    // 6. stage the compacted tile and the per-position intra prefix in shared memory
     {
         int o = excl;
         uint16_t ex[V];
@@ -234,16 +276,18 @@ __global__ void __launch_bounds__(SPLIT_THREADS)
             }
             o += (flags >> i) & 1u;
         }
-        uint4 pk;
-        pk.x = (uint32_t)ex[0] | ((uint32_t)ex[1] << 16);
-        pk.y = (uint32_t)ex[2] | ((uint32_t)ex[3] << 16);
-        pk.z = (uint32_t)ex[4] | ((uint32_t)ex[5] << 16);
-        pk.w = (uint32_t)ex[6] | ((uint32_t)ex[7] << 16);
-        *reinterpret_cast<uint4 *>(s_excl + j0) = pk;
-        if (tid == 0) s_excl[T] = 0;
+#pragma unroll
+        for (int q = 0; q < V / 8; q++) {
+            uint4 pk;
+            pk.x = (uint32_t)ex[8 * q + 0] | ((uint32_t)ex[8 * q + 1] << 16);
+            pk.y = (uint32_t)ex[8 * q + 2] | ((uint32_t)ex[8 * q + 3] << 16);
+            pk.z = (uint32_t)ex[8 * q + 4] | ((uint32_t)ex[8 * q + 5] << 16);
+            pk.w = (uint32_t)ex[8 * q + 6] | ((uint32_t)ex[8 * q + 7] << 16);
+            *reinterpret_cast<uint4 *>(s_excl + j0 + 8 * q) = pk;
+        }
     }
     __syncthreads();
-    if (tid == 0) s_excl[len] = (uint16_t)total;  // position len (last tile rows at nnz)
+    if (tid == 0) s_excl[len] = (uint16_t)total;  // position len (last tile: rows starting at nnz)
     __syncthreads();
     const int64_t P = s_prefix;
     // 7. coalesced stores of the two compacted streams
@@ -299,14 +343,13 @@ int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const Spl
     }
     if (kind == KIND_DEGK) SYM_TRY(launch_classify_degk(g, param, w.hbits, nullptr, ctl, s));
     SYM_CUDA(cudaMemsetAsync(w.tile_state, 0, sizeof(uint64_t) * (size_t)w.ntiles, s));
-    SYM_CUDA(cudaMemsetAsync(&ctl->tile_counter, 0, sizeof(uint32_t), s));
     k_first_row<<<(unsigned)((w.ntiles + 255) / 256), 256, 0, s>>>(g.rp, g.n, w.ntiles, w.first_row);
     SYM_LAUNCH_CHECK();
     bool vec = ((uintptr_t)g.ci & 15) == 0;
     dim3 grid((unsigned)w.ntiles);
     prof_begin("split", s);
 #define SPLIT_ARGS                                                                                          \
-    g.rp, g.ci, g.n, g.nnz, w.first_row, w.ntiles, w.hbits, kr, param, w.tile_state, &ctl->tile_counter, rp_in, \
+    g.rp, g.ci, g.n, g.nnz, w.first_row, w.ntiles, w.hbits, kr, param, w.tile_state, rp_in, \
         ci_in, rp_x, ci_x
     if (kind == KIND_RAND) {
         if (vec) k_split<KIND_RAND, true><<<grid, SPLIT_THREADS, 0, s>>>(SPLIT_ARGS);
