@@ -21,6 +21,8 @@
 // decrement) -> reservation; each arc is read twice in total (init + push).
 // Rounds = the JP dependency depth (~5e3 on R-MAT scale 24), so a round is latency-
 // bound: one kernel per round on a short grid.
+#include <cstdlib>
+
 #include "internal.h"
 
 namespace sym {
@@ -425,8 +427,290 @@ void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
 
 // JP over (rp, ci) for the vertex set S (list/implicit) with membership inS; the
 // bitmap layout follows this CSR (offset rp[v] + v, deg+1 bits).
+// ---------------------------------------------------------------- asynchronous JP
+// No global rounds: a persistent grid of warps colours vertices as soon as they are
+// ready.  A lane that makes a short-row vertex (deg <= JP_LANE) ready colours it
+// itself next (per-lane continuation stack, no queue hop); longer rows are split into
+// JP_CHUNK-arc tasks appended to one global queue that idle warps claim.  Pushes set
+// the forbidden bit, fence, then decrement; the decrement that reaches 0 is followed
+// by a fence before the bitmap is read, so every higher neighbour's colour is seen.
+// Termination: an exact count of coloured vertices (flushed before a warp waits).
+// A warp waiting on an empty queue slot also watches the count, an error flag and a
+// %globaltimer deadline, so a bug cannot hang the device.
+constexpr int JA_STACK = 16;
+constexpr uint64_t JA_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
+
+struct JaArgs {
+    const int64_t *rp;
+    const int32_t *ci;
+    const uint8_t *inS;
+    uint32_t *color;
+    uint32_t *cnt;
+    uint32_t *bits;
+    JpTask *q;
+    int64_t qcap;
+    uint32_t *head, *tail, *done, *err;
+    const uint32_t *target;  // vertices to colour by tasks
+    Key k;
+};
+
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
+__device__ __forceinline__ int32_t ld_volatile_i32(const int32_t *p) {
+    int32_t v;
+    asm volatile("ld.volatile.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void st_volatile_i32(int32_t *p, int32_t v) {
+    asm volatile("st.volatile.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// lane-level enqueue of all chunk tasks of vertex w (flag field v written last)
+__device__ __forceinline__ void ja_enqueue(const JaArgs &A, int32_t w, int64_t wb, int64_t we) {
+    const uint32_t nt = n_tasks(we - wb);
+    const uint32_t slot = atomicAdd(A.tail, nt);
+    for (uint32_t q = 0; q < nt; q++) {
+        JpTask *t = A.q + slot + q;
+        t->b = wb;
+        t->e = we;
+        t->j = q;
+    }
+    __threadfence();
+    for (uint32_t q = 0; q < nt; q++) st_volatile_i32(&A.q[slot + q].v, w);
+}
+
+struct JaStack {
+    int32_t v[JA_STACK];
+    int64_t b[JA_STACK], e[JA_STACK];
+    int sp;
+};
+
+__device__ __forceinline__ void ja_ready(const JaArgs &A, JaStack &st, int32_t w, int64_t wb, int64_t we) {
+    if (we - wb <= JP_LANE && st.sp < JA_STACK) {
+        st.v[st.sp] = w;
+        st.b[st.sp] = wb;
+        st.e[st.sp] = we;
+        st.sp++;
+    } else {
+        ja_enqueue(A, w, wb, we);
+    }
+}
+
+// colour a short-row vertex and push to its lower S-neighbours (one lane)
+__device__ __forceinline__ void ja_lane_vertex(const JaArgs &A, JaStack &st, int32_t v, int64_t b, int64_t e,
+                                               uint32_t &ncol) {
+    const uint64_t kv = vkey(A.k, (uint32_t)v);
+    __threadfence();  // acquire: the decrement that made v ready precedes these reads
+    const uint32_t c = lane_mex(A.bits, b + v, e - b + 1);
+    A.color[v] = c;
+    ncol++;
+    uint32_t w[JP_LANE];
+    bool low[JP_LANE];
+    int64_t wb[JP_LANE], we[JP_LANE];
+#pragma unroll
+    for (int u = 0; u < JP_LANE; u++) {
+        low[u] = b + u < e;
+        w[u] = low[u] ? (uint32_t)__ldg(A.ci + b + u) : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < JP_LANE; u++) {
+        low[u] = low[u] && in_set(A.inS, w[u]) && vkey(A.k, w[u]) < kv;
+        if (low[u]) {
+            wb[u] = A.rp[w[u]];
+            we[u] = A.rp[w[u] + 1];
+        }
+    }
+#pragma unroll
+    for (int u = 0; u < JP_LANE; u++)
+        if (low[u]) set_forbidden(A.bits, wb[u] + w[u], we[u] - wb[u] + 1, c);
+    __threadfence();  // release: the forbidden bits precede the decrements
+#pragma unroll
+    for (int u = 0; u < JP_LANE; u++)
+        if (low[u] && atomicSub(A.cnt + w[u], 1u) == 1u) ja_ready(A, st, (int32_t)w[u], wb[u], we[u]);
+}
+
+__global__ void __launch_bounds__(JP_THREADS) k_jp_async(JaArgs A) {
+    const int lane = lane_id();
+    JaStack st;
+    st.sp = 0;
+    uint32_t ncol = 0;
+    const uint64_t t0 = globaltimer_ns();
+    const uint32_t target = *A.target;
+    for (;;) {
+        // 1. drain the lanes' continuation stacks
+        while (__any_sync(FULL, st.sp > 0)) {
+            if (st.sp > 0) {
+                st.sp--;
+                ja_lane_vertex(A, st, st.v[st.sp], st.b[st.sp], st.e[st.sp], ncol);
+            }
+        }
+        // 2. flush the coloured count, then claim one queued task for the warp
+        uint32_t sum = ncol;
+        for (int d = 16; d; d >>= 1) sum += __shfl_xor_sync(FULL, sum, d);
+        ncol = 0;
+        int32_t tv = -1;
+        uint32_t idx = 0;
+        bool quit = false;
+        if (lane == 0) {
+            if (sum) atomicAdd(A.done, sum);
+            idx = atomicAdd(A.head, 1u);
+            uint32_t spins = 0;
+            for (;;) {
+                tv = idx < A.qcap ? ld_volatile_i32(&A.q[idx].v) : -1;
+                if (tv >= 0) break;
+                if ((++spins & 63u) == 0) {
+                    if (ld_volatile_u32(A.done) >= target || ld_volatile_u32(A.err)) {
+                        quit = true;
+                        break;
+                    }
+                    if (globaltimer_ns() - t0 > JA_TIMEOUT_NS) {
+                        atomicExch(A.err, 1u);
+                        quit = true;
+                        break;
+                    }
+                }
+                __nanosleep(64);
+            }
+        }
+        quit = __shfl_sync(FULL, quit, 0);
+        if (quit) return;
+        tv = __shfl_sync(FULL, tv, 0);
+        idx = __shfl_sync(FULL, idx, 0);
+        __threadfence();
+        const int64_t tb = __ldcg(&A.q[idx].b), te = __ldcg(&A.q[idx].e);
+        const uint32_t tj = __ldcg(&A.q[idx].j);
+        // 3. process the chunk with the whole warp
+        const uint64_t tk = vkey(A.k, (uint32_t)tv);
+        const int64_t cb = tb + (int64_t)tj * JP_CHUNK;
+        constexpr int U = JP_CHUNK / 32;
+        uint32_t w[U];
+        bool low[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            int64_t x = cb + u * 32 + lane;
+            low[u] = x < te;
+            w[u] = low[u] ? (uint32_t)__ldg(A.ci + x) : 0u;
+        }
+        const uint32_t c = warp_mex(A.bits, tb + tv, te - tb + 1);
+        if (tj == 0 && lane == 0) {
+            A.color[tv] = c;
+            ncol++;
+        }
+        int64_t wb[U], we[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            low[u] = low[u] && in_set(A.inS, w[u]) && vkey(A.k, w[u]) < tk;
+            if (low[u]) {
+                wb[u] = A.rp[w[u]];
+                we[u] = A.rp[w[u] + 1];
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++)
+            if (low[u]) set_forbidden(A.bits, wb[u] + w[u], we[u] - wb[u] + 1, c);
+        __threadfence();
+#pragma unroll
+        for (int u = 0; u < U; u++)
+            if (low[u] && atomicSub(A.cnt + w[u], 1u) == 1u) ja_ready(A, st, (int32_t)w[u], wb[u], we[u]);
+    }
+}
+
+// target = #S vertices with phase arcs (the others were coloured by the init pass)
+__global__ void k_jp_count_targets(const int64_t *__restrict__ rp, const int32_t *list, const uint32_t *list_cnt,
+                                   int64_t implicit_n, uint32_t *target) {
+    const uint32_t cnt = list ? *list_cnt : (uint32_t)implicit_n;
+    uint32_t local = 0;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
+        int64_t v = list ? list[i] : (int64_t)i;
+        local += rp[v + 1] > rp[v] ? 1u : 0u;
+    }
+    for (int d = 16; d; d >>= 1) local += __shfl_xor_sync(FULL, local, d);
+    if (lane_id() == 0 && local) atomicAdd(target, local);
+}
+
+static int jp_run_async(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
+                        const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n,
+                        int phase) {
+    Ctl *ctl = f.ctl;
+    cudaStream_t s = f.stream;
+    const Key k = stream_key(f.p.seed, TAG_VERTEX, 0);
+    JpTask *q = reinterpret_cast<JpTask *>(w.task);
+    const int64_t qcap = 2 * w.queue_cap;
+    // counters: ring[0] = tail (init writes the first ready tasks there), ring[1] =
+    // head, ring[2] = done, flag = error, q_head = target
+    SYM_CUDA(cudaMemsetAsync(ctl->ring, 0, sizeof(ctl->ring) + sizeof(ctl->huge), s));
+    SYM_CUDA(cudaMemsetAsync(&ctl->flag, 0, sizeof(uint32_t), s));
+    SYM_CUDA(cudaMemsetAsync(&ctl->q_head, 0, sizeof(uint32_t), s));
+    SYM_CUDA(cudaMemsetAsync(w.bits, 0, sizeof(uint32_t) * (size_t)w.bits_words, s));
+    SYM_CUDA(cudaMemsetAsync(q, 0xff, sizeof(JpTask) * (size_t)qcap, s));
+    prof_begin("jp_init", s);
+    JpArgs A;
+    A.rp = rp;
+    A.ci = ci;
+    A.inS = inS;
+    A.color = color;
+    A.cnt = w.cnt;
+    A.bits = w.bits;
+    A.k = k;
+    A.huge = w.queue;
+    A.hist = nullptr;
+    A.in_list = list0;
+    A.in_cnt = cnt0;
+    A.implicit_n = implicit_n;
+    A.tin = nullptr;
+    A.tout = q;
+    A.out_cnt = &ctl->ring[0];
+    A.clear_cnt = &ctl->ring[3];
+    A.huge_cnt = &ctl->huge[1];
+    A.huge_clear = &ctl->huge[0];
+    A.round = 0;
+    k_jp_init<<<num_sms() * (2048 / JP_THREADS), JP_THREADS, 0, s>>>(A);
+    SYM_LAUNCH_CHECK();
+    k_jp_init_huge<<<num_sms() * 2, JP_HUGE_THREADS, 0, s>>>(A);
+    SYM_LAUNCH_CHECK();
+    k_jp_count_targets<<<num_sms() * 4, 256, 0, s>>>(rp, list0, cnt0, implicit_n, &ctl->q_head);
+    prof_end(s, -1);
+    SYM_LAUNCH_CHECK();
+    JaArgs J;
+    J.rp = rp;
+    J.ci = ci;
+    J.inS = inS;
+    J.color = color;
+    J.cnt = w.cnt;
+    J.bits = w.bits;
+    J.q = q;
+    J.qcap = qcap;
+    J.tail = &ctl->ring[0];
+    J.head = &ctl->ring[1];
+    J.done = &ctl->ring[2];
+    J.err = &ctl->flag;
+    J.target = &ctl->q_head;
+    J.k = k;
+    int per_sm = 0;
+    SYM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_jp_async, JP_THREADS, 0));
+    if (per_sm < 1) per_sm = 1;
+    prof_begin("jp_async", s);
+    k_jp_async<<<num_sms() * per_sm, JP_THREADS, 0, s>>>(J);
+    prof_end(s, -1);
+    SYM_LAUNCH_CHECK();
+    uint32_t err = 0;
+    SYM_TRY(read_u32(&ctl->flag, &err, s));
+    if (err) {
+        set_error("asynchronous JP stalled (device timeout)");
+        return SYM_ECUDA;
+    }
+    if (f.stats) f.stats->rounds[phase] = 0;
+    return SYM_OK;
+}
+
 static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
                   const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n, int phase) {
+    if (!getenv("SYM_JP_ROUNDS")) return jp_run_async(f, w, color, rp, ci, inS, list0, cnt0, implicit_n, phase);
     Ctl *ctl = f.ctl;
     cudaStream_t s = f.stream;
     const Key k = stream_key(f.p.seed, TAG_VERTEX, 0);

@@ -1,4 +1,5 @@
-"""Diagnostic: JP task count per round (first 2048 rounds) read from the Ctl block."""
+"""Diagnostic: JP tasks and lower-neighbour pushes per round (first 2048 rounds),
+read from the control block (needs SYM_DEBUG_JP=1 for pushes)."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch, graphgen, paper_conf_ipps_nayyaroddeengk17_b200 as sb
@@ -8,11 +9,7 @@ rp, ci = graphgen.rmat(scale, 16, seed=1, device=dev)
 d = sb.sym_decompose(rp, ci, "degk", 2, 42)
 C, st = sb.sym_color(rp, ci, "degk", 2, 42, decomp=d, stats=True)
 ws = sb._WS[0]
-base = (ws.data_ptr() + 255) & ~255
-off = base - ws.data_ptr()
-hist = ws[off + 136: off + 136 + 8192].cpu().numpy().view(np.uint32)
-print("rounds", st["rounds"], "colours", int(C.max()))
-h = hist[:2048]
-print("first 40:", h[:40].tolist())
-print("percentiles tasks/round (rounds 0..2047):", np.percentile(h[h > 0], [10, 50, 90, 99]).tolist(), "sum", int(h.sum()))
-print("rounds 1000..1040:", h[1000:1040].tolist())
+off = ((ws.data_ptr() + 255) & ~255) - ws.data_ptr()
+hist = ws[off + 136: off + 136 + 16384].cpu().numpy().view(np.uint32)
+np.save(os.path.join(os.environ.get("GRAFT_REPO_ROOT", "."), "gpurun_out", "jp_hist.npy"), hist)
+print("rounds", st["rounds"], "tasks[:10]", hist[:10].tolist(), "pushes[:10]", hist[2048:2058].tolist())
