@@ -28,6 +28,11 @@ sys.path.insert(0, ROOT)
 
 METRIC = "MIS/MM/COLOR edges/s at 1/2/4/8 B200; % of HBM roofline; vs CPU oracle"
 
+# per-launch DRAM traffic (dram__bytes_read.sum + dram__bytes_write.sum) of each kernel
+# class from one `ncu --set full` capture of this step (profiles/r1_ncu_summary.md);
+# None where no capture was taken for the current code.
+TRAFFIC = {}
+
 
 def parse():
     ap = argparse.ArgumentParser()
@@ -251,19 +256,22 @@ def main():
     per_step = {k: {"ms_per_step": v["ms"] / steps_p, "launches_per_step": v["launches"] / steps_p,
                     "alg_bytes_per_step": (v["alg_bytes"] / steps_p) if v["alg_bytes"] >= 0 else None}
                 for k, v in prof.items()}
-    known = {k: v for k, v in prof.items() if v["alg_bytes"] > 0}
-    roof = None
-    if known:
-        dom = max(known, key=lambda k: known[k]["ms"])
-        v = known[dom]
+    def roof_of(name):
+        v = prof[name]
+        if v["alg_bytes"] <= 0 or v["ms"] <= 0:
+            return None
         per_launch_bytes = v["alg_bytes"] / v["launches"]
         per_launch_s = v["ms"] / v["launches"] * 1e-3
         ach = per_launch_bytes / per_launch_s / 1e9
-        roof = {"kernel": dom, "bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
-                "frac": ach / hbm_peak, "traffic": None, "peak_source": peak_src,
+        return {"kernel": name, "bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
+                "frac": ach / hbm_peak, "traffic": TRAFFIC.get(name), "peak_source": peak_src,
                 "alg_bytes_per_launch": per_launch_bytes, "ms_per_launch": per_launch_s * 1e3,
-                "share_of_step": (v["ms"] / steps_p) / ms_step}
+                "launches_per_step": v["launches"] / steps_p, "share_of_step": (v["ms"] / steps_p) / ms_step}
+
+    # the dominant kernel = the class with the most device time in the step
     dominant_overall = max(prof, key=lambda k: prof[k]["ms"]) if prof else None
+    roof = roof_of(dominant_overall) if dominant_overall else None
+    rooflines = {k: roof_of(k) for k in prof if roof_of(k)}
 
     # ---- e2e through the public API with pinned host buffers
     e2e = None
@@ -323,7 +331,7 @@ def main():
                                       "color_deg2_incl_decomp": m / ((brk["decompose_deg2"] + brk["color_deg2"]) * 1e-3),
                                       "mm_rand4_incl_decomp": m / ((brk["decompose_rand4"] + brk["mm_rand4"]) * 1e-3)},
             "kernels": per_step, "dominant_kernel": dominant_overall,
-            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+            "roofline": roof, "rooflines": rooflines, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": int(round(launches)),
             "clocks": clk.summary(),
             "stats": {"mis": st_mis, "color": st_col, "mm": st_mm},

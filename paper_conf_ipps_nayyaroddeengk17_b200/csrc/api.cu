@@ -206,6 +206,8 @@ static int flow_setup(const sym_graph *g, const sym_params *p, const sym_decomp 
     f.stats = stats;
     f.stream = s;
     f.hbits = L.sw.hbits;
+    f.first_row = L.sw.first_row;
+    f.first_row_cap = L.sw.ntiles + 1;
     if (p->kind != SYM_DECOMP_NONE) {
         if (decomp) {
             f.split.rp_in = decomp->row_ptr_in;

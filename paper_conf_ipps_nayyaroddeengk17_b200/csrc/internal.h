@@ -90,6 +90,16 @@ void carve_split_ws(Arena &a, int64_t n, int64_t nnz, SplitWs &w);
 // class bitmap (+ optional vertex lists: class-0 from the front, class-1 from the back)
 int launch_classify_degk(const Graph &g, uint32_t k, uint32_t *hbits, int32_t *vlist, Ctl *ctl,
                          cudaStream_t s);
+// first_row[t] = first row whose arcs start at or after t*SPLIT_TILE (split.cu)
+__global__ void k_first_row(const int64_t *__restrict__ rp, int64_t n, int64_t ntiles, int64_t *__restrict__ first_row);
+int launch_first_row(const Graph &g, int64_t ntiles, int64_t *first_row, cudaStream_t s);
+
+// round 0 of a MIS (mode 0) or MM (mode 1) phase as one streaming segmented max
+// (round0.cu); returns SYM_EINVAL without launching when the phase CSR is empty
+int run_round0(int mode, const Graph &g, const int64_t *first_row, int64_t ntiles, Key k,
+               unsigned long long *gmax, uint8_t *st, int32_t *pick, const uint32_t *hfilter, int32_t *out_list,
+               uint32_t *out_cnt, cudaStream_t s);
+
 // decompose into caller buffers (rp_in, ci_in, rp_x, ci_x) ; kind in {NONE,RAND,DEGK}
 int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const SplitWs &w, Ctl *ctl,
               int64_t *rp_in, int32_t *ci_in, int64_t *rp_x, int32_t *ci_x, uint16_t *label, cudaStream_t s);
@@ -98,6 +108,17 @@ int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const Spl
 bool prof_on();
 void prof_begin(const char *cls, cudaStream_t s);
 void prof_end(cudaStream_t s, double alg_bytes);  // alg_bytes < 0: unknown on the host
+// a zeroed device counter (nullptr unless profiling) that a kernel accumulates its
+// algorithmic bytes into; prof_end_dev closes the event pair and reads it at collect
+unsigned long long *prof_counter(cudaStream_t s);
+void prof_end_dev(cudaStream_t s, unsigned long long *ctr);
+
+// warp-aggregated add of per-lane byte counts into a profiling counter (nullable)
+__device__ __forceinline__ void prof_add(unsigned long long *ctr, unsigned long long lane_bytes) {
+    if (ctr == nullptr) return;
+    for (int d = 16; d; d >>= 1) lane_bytes += __shfl_xor_sync(0xffffffffu, lane_bytes, d);
+    if ((threadIdx.x & 31) == 0 && lane_bytes) atomicAdd(ctr, lane_bytes);
+}
 
 // ------------------------------------------------------------------ helpers (api.cu)
 int read_u32(const uint32_t *dev, uint32_t *host, cudaStream_t s);
@@ -110,6 +131,8 @@ struct FlowArgs {
     sym_params p;
     Split split;                // valid when p.kind != NONE
     uint32_t *hbits;            // DEGk bitmap workspace
+    int64_t *first_row;         // tile -> first row table (capacity first_row_cap tiles)
+    int64_t first_row_cap;
     Ctl *ctl;
     sym_stats *stats;
     cudaStream_t stream;
@@ -121,6 +144,7 @@ struct MisWs {
     int32_t *fr[2] = {nullptr, nullptr};  // frontier ping-pong
     int64_t *huge = nullptr;           // deferred (v, resume) pairs
     int64_t huge_cap = 0;
+    unsigned long long *gmax = nullptr;  // round 0: maxima of rows crossing tiles
 };
 
 struct MmWs {
@@ -130,6 +154,7 @@ struct MmWs {
     int64_t *huge = nullptr;
     unsigned long long *huge_best = nullptr;
     int64_t huge_cap = 0;
+    unsigned long long *gmax = nullptr;  // round 0: maxima of rows crossing tiles
 };
 
 struct ColorWs {
@@ -142,6 +167,8 @@ struct ColorWs {
     int64_t *task = nullptr;       // two task lists (ping-pong), queue_cap each
     int64_t queue_cap = 0;
 };
+
+int phase_arcs(const FlowArgs &f, const int64_t *rp, int64_t *out);  // round0.cu
 
 void carve_mis_ws(Arena &a, int64_t n, int64_t nnz, MisWs &w);
 int run_mis(const FlowArgs &f, MisWs &w, uint8_t *in_set);

@@ -694,9 +694,14 @@ static int jp_run_async(const FlowArgs &f, ColorWs &w, uint32_t *color, const in
     int per_sm = 0;
     SYM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_jp_async, JP_THREADS, 0));
     if (per_sm < 1) per_sm = 1;
+    // algorithmic bytes of the asynchronous pass: every arc of the phase
+    // CSR read once (4 B) + per vertex the row bounds of the task (8 B) and the
+    // colour write (4 B); counter/bitmap atomics are L2 traffic
+    const int64_t phase_nnz = rp == f.g.rp ? f.g.nnz : (rp == f.split.rp_in ? f.split.nnz_in : -1);
+    const double jp_bytes = phase_nnz >= 0 ? 4.0 * (double)phase_nnz + 12.0 * (double)f.g.n : -1.0;
     prof_begin("jp_async", s);
     k_jp_async<<<num_sms() * per_sm, JP_THREADS, 0, s>>>(J);
-    prof_end(s, -1);
+    prof_end(s, jp_bytes);
     SYM_LAUNCH_CHECK();
     uint32_t err = 0;
     SYM_TRY(read_u32(&ctl->flag, &err, s));

@@ -16,6 +16,8 @@
 //                             for up to MIS_BUDGET arcs;
 //   rows still undecided    : deferred (v, resume offset) to k_mis_huge, where a
 //                             whole CTA scans the rest with __syncthreads_or exits.
+#include <algorithm>
+
 #include "internal.h"
 
 namespace sym {
@@ -44,17 +46,32 @@ struct MisRoundArgs {
     uint32_t *hist;
     int round;
     Key k;
+    unsigned long long *prof;  // profiling: algorithmic bytes of this launch (nullable)
 };
 
-__device__ __forceinline__ int mis_scan_serial(const int32_t *__restrict__ ci, const uint8_t *st, int64_t b,
-                                               int64_t e, uint64_t kv, Key k) {
-    for (int64_t x = b; x < e; x++) {
-        uint32_t w = (uint32_t)__ldg(ci + x);
-        uint8_t sw = st[w];
-        if (sw == ST_IN) return R_OUT;
-        if (sw == ST_UNDEC && vkey(k, w) > kv) return R_BLK;
+// algorithmic bytes: 4 B per column word the kernel loads, 16 B for the
+// row_ptr pair + 1 B status per active vertex, 1 B per decided status write;
+// neighbour-status gathers hit the L2-resident status array and count 0 HBM bytes.
+// A short row (<= MIS_SMALL arcs, one sector) is decided by one lane: all column
+// loads, then all status gathers, then the rule (the order of the arcs does not
+// matter: any In neighbour -> Out, else any higher undecided neighbour -> blocked).
+// Column words are streamed with evict-first loads so the gathered status stays in L2.
+__device__ __forceinline__ int mis_scan_small(const int32_t *__restrict__ ci, const uint8_t *st, int64_t b,
+                                              int64_t e, uint64_t kv, Key k, unsigned long long &lb) {
+    uint32_t w[MIS_SMALL];
+    uint8_t s[MIS_SMALL];
+#pragma unroll
+    for (int u = 0; u < MIS_SMALL; u++) w[u] = (b + u < e) ? (uint32_t)__ldcs(ci + b + u) : 0u;
+#pragma unroll
+    for (int u = 0; u < MIS_SMALL; u++) s[u] = (b + u < e) ? st[w[u]] : ST_OUT;
+    bool in = false, blk = false;
+#pragma unroll
+    for (int u = 0; u < MIS_SMALL; u++) {
+        in |= s[u] == ST_IN;
+        blk |= (s[u] == ST_UNDEC) && (vkey(k, w[u]) > kv);
     }
-    return R_IN;
+    lb += 4 * (unsigned long long)(e - b);
+    return in ? R_OUT : (blk ? R_BLK : R_IN);
 }
 
 __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
@@ -81,7 +98,8 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
         }
         int res = R_NONE;
         int64_t resume = 0;
-        if (active && e - b <= MIS_SMALL) res = mis_scan_serial(A.ci, A.st, b, e, kv, A.k);
+        unsigned long long lb = active ? 17 : 0;
+        if (active && e - b <= MIS_SMALL) res = mis_scan_small(A.ci, A.st, b, e, kv, A.k, lb);
         unsigned longm = __ballot_sync(FULL, active && e - b > MIS_SMALL);
         while (longm) {
             const int src = __ffs(longm) - 1;
@@ -97,7 +115,8 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
                 for (int u = 0; u < 4; u++) {
                     int64_t y = x + u * 32 + lane;
                     ok[u] = y < lim;
-                    w[u] = ok[u] ? (uint32_t)__ldg(A.ci + y) : 0u;
+                    w[u] = ok[u] ? (uint32_t)__ldcs(A.ci + y) : 0u;
+                    lb += ok[u] ? 4 : 0;
                 }
                 bool fin = false, fblk = false;
 #pragma unroll
@@ -119,6 +138,7 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
         }
         if (res == R_IN) A.st[v] = ST_IN;
         else if (res == R_OUT) A.st[v] = ST_OUT;
+        prof_add(A.prof, lb + ((res == R_IN || res == R_OUT) ? 1 : 0));
         int64_t slot = warp_append(res == R_BLK, A.out_cnt);
         if (slot >= 0) A.out_list[slot] = v;
         int64_t hs = warp_append(res == R_DEFER, A.huge_cnt);
@@ -137,6 +157,7 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
         const int64_t b = A.huge[2 * h + 1], e = A.rp[v + 1];
         const uint64_t kv = vkey(A.k, (uint32_t)v);
         int r = R_IN;
+        unsigned long long lb = threadIdx.x == 0 ? 9 : 0;  // row end + status write
         for (int64_t x = b; x < e; x += 4 * MIS_HUGE_THREADS) {
             bool fin = false, fblk = false;
             uint32_t w[4];
@@ -145,7 +166,8 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
             for (int u = 0; u < 4; u++) {
                 int64_t y = x + u * MIS_HUGE_THREADS + threadIdx.x;
                 ok[u] = y < e;
-                w[u] = ok[u] ? (uint32_t)__ldg(A.ci + y) : 0u;
+                w[u] = ok[u] ? (uint32_t)__ldcs(A.ci + y) : 0u;
+                lb += ok[u] ? 4 : 0;
             }
 #pragma unroll
             for (int u = 0; u < 4; u++) {
@@ -166,6 +188,7 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
                 A.out_list[slot] = v;
             }
         }
+        prof_add(A.prof, lb);
         __syncthreads();
     }
 }
@@ -239,6 +262,7 @@ void carve_mis_ws(Arena &a, int64_t n, int64_t nnz, MisWs &w) {
     w.fr[1] = a.take<int32_t>((size_t)n + 1);
     w.huge_cap = nnz / MIS_BUDGET + 2;
     w.huge = a.take<int64_t>((size_t)(2 * w.huge_cap));
+    w.gmax = a.take<unsigned long long>((size_t)n + 1);
 }
 
 static int round_grid() { return num_sms() * (2048 / MIS_THREADS); }
@@ -246,15 +270,27 @@ static int round_grid() { return num_sms() * (2048 / MIS_THREADS); }
 // Run Luby rounds of one phase until the frontier is empty.  Round 0 reads
 // (list0, rev0, cnt0) -- or the implicit range [0, implicit_n) when list0 == nullptr.
 static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp, const int32_t *ci,
-                     const int32_t *list0, int rev0, const uint32_t *cnt0, int64_t implicit_n, int phase) {
+                     const int32_t *list0, int rev0, const uint32_t *cnt0, int64_t implicit_n, int phase,
+                     bool stream_round0 = false) {
+    // stream_round0: round 0 as a gather-free streaming pass (round0.cu).  Measured at
+    // R-MAT s24 it is slower than the early-exit frontier kernel, whose
+    // round 0 reads only ~30 % of the arcs, so it is off by default for MIS.
     Ctl *ctl = f.ctl;
     cudaStream_t s = f.stream;
     SYM_CUDA(cudaMemsetAsync(ctl->ring, 0, sizeof(ctl->ring) + sizeof(ctl->huge), s));
     const Key k = stream_key(f.p.seed, TAG_VERTEX, 0);
+    if (stream_round0) {
+        // round 0 as one streaming pass: every local maximum of the phase joins I
+        int64_t nnz = 0;
+        SYM_TRY(phase_arcs(f, rp, &nnz));
+        if (nnz > 0)
+            SYM_TRY(run_round0(0, Graph{f.g.n, nnz, rp, ci}, f.first_row, (nnz + SPLIT_TILE - 1) / SPLIT_TILE, k,
+                               w.gmax, st, nullptr, nullptr, nullptr, nullptr, s));
+    }
     const uint32_t maxr = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
-    const int grid = round_grid();
+    int grid = round_grid();
     int r = 0;
-    int batch = 4;
+    const int batch = 4;  // rounds launched per host poll of the frontier count
     for (;;) {
         for (int b = 0; b < batch; b++, r++) {
             MisRoundArgs A;
@@ -280,13 +316,15 @@ static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp
             A.hist = (phase == 0) ? ctl->hist : ctl->hist + 2048;
             A.round = r < 2048 ? r : 2047;
             A.k = k;
+            A.prof = prof_counter(s);
             prof_begin("mis_round", s);
             k_mis_round<<<grid, MIS_THREADS, 0, s>>>(A);
-            prof_end(s, -1);
+            prof_end_dev(s, A.prof);
             SYM_LAUNCH_CHECK();
+            A.prof = prof_counter(s);
             prof_begin("mis_huge", s);
             k_mis_huge<<<num_sms() * 2, MIS_HUGE_THREADS, 0, s>>>(A);
-            prof_end(s, -1);
+            prof_end_dev(s, A.prof);
             SYM_LAUNCH_CHECK();
         }
         uint32_t left = 0;
@@ -296,7 +334,9 @@ static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp
             set_error("MIS phase did not converge within max_rounds");
             return SYM_EROUNDS;
         }
-        if (batch < 16) batch *= 2;
+        // frontiers only shrink: size the next launches for `left` vertices
+        const int64_t need = ((int64_t)left + MIS_THREADS - 1) / MIS_THREADS;
+        grid = (int)std::min<int64_t>(round_grid(), std::max<int64_t>(need, 1));
     }
     if (f.stats) f.stats->rounds[phase] = (uint32_t)r;  // refined from hist below
     return SYM_OK;
@@ -316,8 +356,9 @@ int run_mis(const FlowArgs &f, MisWs &w, uint8_t *st) {
         SYM_CUDA(cudaMemsetAsync(st, ST_UNDEC, (size_t)g.n, s));
         SYM_CUDA(cudaMemsetAsync(&ctl->cnt_front, 0, 2 * sizeof(uint32_t), s));
         SYM_TRY(launch_classify_degk(g, f.p.param, f.hbits, w.vlist, ctl, s));
-        // phase L: I_L = MIS(G_L) on the intra CSR restricted to V_L
-        SYM_TRY(mis_phase(f, w, st, f.split.rp_in, f.split.ci_in, w.vlist, 0, &ctl->cnt_front, 0, 0));
+        // phase L: I_L = MIS(G_L) on the intra CSR restricted to V_L (tiny: the rows
+        // of V_H in the same CSR are not in this phase, so no streaming round 0)
+        SYM_TRY(mis_phase(f, w, st, f.split.rp_in, f.split.ci_in, w.vlist, 0, &ctl->cnt_front, 0, 0, false));
         // fix-up: remove N(I_L) from V_H through the cross arcs G_C
         k_mis_kill_cross<<<num_sms() * 4, 256, 0, s>>>(f.split.rp_x, f.split.ci_x, w.vlist, &ctl->cnt_front, st);
         SYM_LAUNCH_CHECK();

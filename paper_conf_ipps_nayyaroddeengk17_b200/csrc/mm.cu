@@ -44,7 +44,12 @@ struct MmRoundArgs {
     uint32_t *hist;
     int round;
     Key k;
+    unsigned long long *prof;  // profiling: algorithmic bytes of this launch (nullable)
 };
+// algorithmic bytes: 4 B per column word loaded; per active vertex the
+// row_ptr pair (16 B) and the pick write (4 B); per resolved vertex the two pick
+// reads (8 B) and, if matched, the mate write (4 B).  Neighbour mate gathers hit the
+// L2-resident mate array and count 0 HBM bytes.
 
 __device__ __forceinline__ void mm_row(const MmRoundArgs &A, int32_t u, int64_t &b, int64_t &e, const int32_t *&ci) {
     if (A.dual && ((A.hbits[u >> 5] >> (u & 31)) & 1u)) {
@@ -74,12 +79,15 @@ __global__ void __launch_bounds__(MM_THREADS) k_mm_round(MmRoundArgs A) {
         int32_t u = -1;
         if (i < cnt) u = A.in_list ? (A.in_rev ? A.in_list[-1 - i] : A.in_list[i]) : (int32_t)i;
         bool active = u >= 0;
+        unsigned long long nb = 0;  // algorithmic bytes of this lane
         if (RESOLVE && active) {
             int32_t p = A.pick_prev[u];
+            nb += 8;
             if (p >= 0 && A.pick_prev[p] == u) {
                 A.mate[u] = p;
                 A.pick_cur[u] = -1;
                 active = false;
+                nb += 4;
             } else if (A.mate[u] >= 0) {  // defensive: never re-pick a matched vertex
                 A.pick_cur[u] = -1;
                 active = false;
@@ -89,13 +97,23 @@ __global__ void __launch_bounds__(MM_THREADS) k_mm_round(MmRoundArgs A) {
         const int32_t *ci = A.ci;
         if (active) mm_row(A, u, b, e, ci);
         const int64_t d = e - b;
+        nb += active ? 20 : 0;
         uint64_t best = 0;
         bool has = false;
         if (active && d <= MM_SMALL) {
-            for (int64_t x = b; x < e; x++) {
-                uint32_t w = (uint32_t)__ldg(ci + x);
-                if (!MATE || A.mate[w] < 0) {
-                    uint64_t kk = ekey(A.k, (uint32_t)u, w);
+            // short row by one lane: all column loads (streamed, evict-first so the
+            // gathered mate array stays in L2), then all mate gathers, then the argmax
+            nb += 4 * (unsigned long long)d;
+            uint32_t w[MM_SMALL];
+            bool live[MM_SMALL];
+#pragma unroll
+            for (int q = 0; q < MM_SMALL; q++) w[q] = (q < d) ? (uint32_t)__ldcs(ci + b + q) : 0u;
+#pragma unroll
+            for (int q = 0; q < MM_SMALL; q++) live[q] = (q < d) && (!MATE || A.mate[w[q]] < 0);
+#pragma unroll
+            for (int q = 0; q < MM_SMALL; q++) {
+                if (live[q]) {
+                    uint64_t kk = ekey(A.k, (uint32_t)u, w[q]);
                     if (!has || kk > best) best = kk;
                     has = true;
                 }
@@ -118,7 +136,8 @@ __global__ void __launch_bounds__(MM_THREADS) k_mm_round(MmRoundArgs A) {
                 for (int q = 0; q < 4; q++) {
                     int64_t y = x + q * 32 + lane;
                     ok[q] = y < we;
-                    w[q] = ok[q] ? (uint32_t)__ldg(wci + y) : 0u;
+                    w[q] = ok[q] ? (uint32_t)__ldcs(wci + y) : 0u;
+                    nb += ok[q] ? 4 : 0;
                 }
 #pragma unroll
                 for (int q = 0; q < 4; q++) {
@@ -146,6 +165,7 @@ __global__ void __launch_bounds__(MM_THREADS) k_mm_round(MmRoundArgs A) {
         if (slot >= 0) A.out_list[slot] = u;
         int64_t hs = warp_append(defer, A.huge_cnt);
         if (hs >= 0) A.huge[hs] = u;
+        prof_add(A.prof, nb);
     }
 }
 
@@ -163,6 +183,7 @@ __global__ void __launch_bounds__(MM_HUGE_THREADS) k_mm_huge(MmRoundArgs A) {
         mm_row(A, u, b, e, ci);
         uint64_t lb = 0;
         bool lh = false;
+        unsigned long long nb = 0;
         for (int64_t x = b; x < e; x += 4 * MM_HUGE_THREADS) {
             uint32_t w[4];
             bool ok[4];
@@ -170,7 +191,8 @@ __global__ void __launch_bounds__(MM_HUGE_THREADS) k_mm_huge(MmRoundArgs A) {
             for (int q = 0; q < 4; q++) {
                 int64_t y = x + q * MM_HUGE_THREADS + threadIdx.x;
                 ok[q] = y < e;
-                w[q] = ok[q] ? (uint32_t)__ldg(ci + y) : 0u;
+                w[q] = ok[q] ? (uint32_t)__ldcs(ci + y) : 0u;
+                nb += ok[q] ? 4 : 0;
             }
 #pragma unroll
             for (int q = 0; q < 4; q++) {
@@ -187,6 +209,7 @@ __global__ void __launch_bounds__(MM_HUGE_THREADS) k_mm_huge(MmRoundArgs A) {
             lb = o > lb ? o : lb;
         }
         bool wh = __any_sync(FULL, lh);
+        prof_add(A.prof, nb);
         if (lane == 0) {
             s_best[warp] = lb;
             s_has[warp] = wh;
@@ -246,6 +269,7 @@ void carve_mm_ws(Arena &a, int64_t n, int64_t nnz, MmWs &w) {
     w.fr[1] = a.take<int32_t>((size_t)n + 1);
     w.huge_cap = nnz / MM_BUDGET + 2;
     w.huge = reinterpret_cast<int64_t *>(a.take<int32_t>((size_t)w.huge_cap));
+    w.gmax = a.take<unsigned long long>((size_t)n + 1);
 }
 
 struct MmPhase {
@@ -266,8 +290,21 @@ static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph
     SYM_CUDA(cudaMemsetAsync(ctl->ring, 0, sizeof(ctl->ring) + sizeof(ctl->huge), s));
     const Key k = stream_key(f.p.seed, TAG_EDGE, 0);
     const uint32_t maxr = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
-    const int grid = num_sms() * (2048 / MM_THREADS);
-    int r = 0, batch = 4;
+    const int full_grid = num_sms() * (2048 / MM_THREADS);
+    int grid = full_grid;
+    int r = 0;
+    const int batch = 4;  // rounds launched per host poll of the frontier count
+    if (ph.first && !ph.dual) {
+        // round 0 as one streaming pass: every phase vertex picks its heaviest arc;
+        // the vertices with a pick form round 1's frontier (fr[1], ring[1])
+        int64_t nnz = 0;
+        SYM_TRY(phase_arcs(f, ph.rp, &nnz));
+        if (nnz > 0) {
+            SYM_TRY(run_round0(1, Graph{f.g.n, nnz, ph.rp, ph.ci}, f.first_row, (nnz + SPLIT_TILE - 1) / SPLIT_TILE, k,
+                               w.gmax, nullptr, w.pick[0], ph.list0 ? f.hbits : nullptr, w.fr[1], &ctl->ring[1], s));
+            r = 1;
+        }
+    }
     for (;;) {
         for (int bb = 0; bb < batch; bb++, r++) {
             MmRoundArgs A;
@@ -301,33 +338,37 @@ static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph
             A.k = k;
             // round 0 of a phase has nothing to resolve (its pick buffers hold stale or
             // uninitialised values); round 0 of the first phase has nothing matched yet
+            // profiling byte counters are accumulated by the kernels
             if (r == 0 && ph.first) {
-                // first round over an implicit vertex range streams the whole phase
-                // CSR: 4 B/arc + row_ptr (8 B) + pick (4 B) per vertex
-                double bytes = (ph.list0 == nullptr && ph.nnz >= 0) ? 4.0 * ph.nnz + 12.0 * ph.implicit_n : -1.0;
+                A.prof = prof_counter(s);
                 prof_begin("mm_round0", s);
                 k_mm_round<false, false><<<grid, MM_THREADS, 0, s>>>(A);
-                prof_end(s, bytes);
+                prof_end_dev(s, A.prof);
                 SYM_LAUNCH_CHECK();
+                A.prof = prof_counter(s);
                 prof_begin("mm_huge", s);
                 k_mm_huge<false><<<num_sms() * 2, MM_HUGE_THREADS, 0, s>>>(A);
-                prof_end(s, -1);
+                prof_end_dev(s, A.prof);
             } else if (r == 0) {
+                A.prof = prof_counter(s);
                 prof_begin("mm_round", s);
                 k_mm_round<false, true><<<grid, MM_THREADS, 0, s>>>(A);
-                prof_end(s, -1);
+                prof_end_dev(s, A.prof);
                 SYM_LAUNCH_CHECK();
+                A.prof = prof_counter(s);
                 prof_begin("mm_huge", s);
                 k_mm_huge<true><<<num_sms() * 2, MM_HUGE_THREADS, 0, s>>>(A);
-                prof_end(s, -1);
+                prof_end_dev(s, A.prof);
             } else {
+                A.prof = prof_counter(s);
                 prof_begin("mm_round", s);
                 k_mm_round<true, true><<<grid, MM_THREADS, 0, s>>>(A);
-                prof_end(s, -1);
+                prof_end_dev(s, A.prof);
                 SYM_LAUNCH_CHECK();
+                A.prof = prof_counter(s);
                 prof_begin("mm_huge", s);
                 k_mm_huge<true><<<num_sms() * 2, MM_HUGE_THREADS, 0, s>>>(A);
-                prof_end(s, -1);
+                prof_end_dev(s, A.prof);
             }
             SYM_LAUNCH_CHECK();
         }
@@ -338,7 +379,9 @@ static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph
             set_error("MM phase did not converge within max_rounds");
             return SYM_EROUNDS;
         }
-        if (batch < 16) batch *= 2;
+        // frontiers only shrink: size the next launches for `left` vertices
+        const int64_t need = ((int64_t)left + MM_THREADS - 1) / MM_THREADS;
+        grid = (int)(need < full_grid ? (need > 0 ? need : 1) : full_grid);
     }
     if (f.stats) f.stats->rounds[phase] = (uint32_t)r;
     return SYM_OK;

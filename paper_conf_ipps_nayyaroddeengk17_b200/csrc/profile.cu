@@ -15,8 +15,15 @@ struct Rec {
     std::string cls;
     cudaEvent_t a, b;
     double bytes;
+    int slot;  // device byte counter slot, or -1
 };
 bool g_on = false;
+// device byte counters for launches whose algorithmic bytes depend on the frontier
+// (measurement mode only; the one allocation the library makes, lazily, when
+// profiling is enabled)
+constexpr int DEV_SLOTS = 1 << 16;
+unsigned long long *g_dev = nullptr;
+int g_dev_next = 0;
 std::vector<Rec> g_recs;
 std::vector<cudaEvent_t> g_pool;
 std::vector<std::pair<std::string, double>> g_open;  // pending begin (class, bytes)
@@ -48,7 +55,29 @@ void prof_end(cudaStream_t s, double bytes) {
     if (!g_on || g_open.empty()) return;
     cudaEvent_t e = get_event();
     cudaEventRecord(e, s);
-    Rec r{g_open.back().first, g_open_ev.back(), e, bytes};
+    Rec r{g_open.back().first, g_open_ev.back(), e, bytes, -1};
+    g_open.pop_back();
+    g_open_ev.pop_back();
+    g_recs.push_back(r);
+}
+
+unsigned long long *prof_counter(cudaStream_t s) {
+    if (!g_on) return nullptr;
+    if (!g_dev && cudaMalloc(&g_dev, sizeof(unsigned long long) * DEV_SLOTS) != cudaSuccess) {
+        g_dev = nullptr;
+        return nullptr;
+    }
+    if (g_dev_next >= DEV_SLOTS) return nullptr;
+    unsigned long long *p = g_dev + g_dev_next++;
+    cudaMemsetAsync(p, 0, sizeof(unsigned long long), s);
+    return p;
+}
+
+void prof_end_dev(cudaStream_t s, unsigned long long *ctr) {
+    if (!g_on || g_open.empty()) return;
+    cudaEvent_t e = get_event();
+    cudaEventRecord(e, s);
+    Rec r{g_open.back().first, g_open_ev.back(), e, ctr ? 0.0 : -1.0, ctr ? (int)(ctr - g_dev) : -1};
     g_open.pop_back();
     g_open_ev.pop_back();
     g_recs.push_back(r);
@@ -71,6 +100,15 @@ extern "C" int sym_profile_collect(sym_kernel_profile *out, int max_entries, int
     };
     std::map<std::string, Acc> acc;
     std::vector<std::string> order;
+    std::vector<unsigned long long> dev(g_dev_next);
+    if (!g_recs.empty()) {
+        cudaError_t e = cudaEventSynchronize(g_recs.back().b);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaEventSynchronize", __FILE__, __LINE__);
+    }
+    if (g_dev_next > 0) {
+        cudaError_t e = cudaMemcpy(dev.data(), g_dev, sizeof(unsigned long long) * g_dev_next, cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy(profile counters)", __FILE__, __LINE__);
+    }
     for (auto &r : g_recs) {
         cudaError_t e = cudaEventSynchronize(r.b);
         if (e != cudaSuccess) return cuda_fail(e, "cudaEventSynchronize", __FILE__, __LINE__);
@@ -80,12 +118,14 @@ extern "C" int sym_profile_collect(sym_kernel_profile *out, int max_entries, int
         Acc &x = acc[r.cls];
         x.n++;
         x.ms += ms;
-        if (r.bytes < 0) x.known = false;
-        else x.bytes += r.bytes;
+        double bytes = r.slot >= 0 ? (double)dev[r.slot] : r.bytes;
+        if (bytes < 0) x.known = false;
+        else x.bytes += bytes;
         g_pool.push_back(r.a);
         g_pool.push_back(r.b);
     }
     g_recs.clear();
+    g_dev_next = 0;
     int c = 0;
     for (auto &name : order) {
         if (out && c < max_entries) {
