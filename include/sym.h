@@ -191,6 +191,46 @@ const char *sym_last_error(void);
 /* Library version string ("symbreak-b200 <semver> sm_100a"). */
 const char *sym_version(void);
 
+/* ---- sharded MIS (multi-GPU; one process per GPU) ----
+   A rank owns the contiguous vertex range [v_begin, v_end) (v_begin a multiple of
+   32) and holds those rows as a local CSR with GLOBAL column ids:
+     row_ptr int64[v_end - v_begin + 1] (row_ptr[0] = 0, local arc offsets),
+     col_idx int32[nnz] (global ids).
+   Every rank keeps a full replica of the MIS status array, uint8[n_global] (0 =
+   undecided, 1 = In, 2 = Out), zero-initialised by the caller.  The exchange is the
+   caller's (bindings: torch.distributed all_gather over NCCL/NVLink): after each round
+   and after the fix-up, the owned segments of the status replicas are all-gathered
+   and the next-frontier counts all-reduced; the phase ends when the global count is
+   0.  Priorities are the single-GPU ones, so the result equals sym_mis() bit for bit
+   (FIXED mode is schedule-independent).  MIS-Deg2: phase L =
+   rounds on V_L with cls = 0, sym_shard_mis_kill, phase R = rounds on V_H with
+   cls = 1.  MIS-NONE: rounds with cls = -1.  All pointers are device pointers. */
+typedef struct {
+    int64_t n_global, v_begin, v_end, nnz;
+    const int64_t *row_ptr;
+    const int32_t *col_idx;
+} sym_graph_shard;
+
+/* workspace for sym_shard_mis_round (host only; 0 on invalid arguments) */
+size_t sym_shard_workspace_bytes(const sym_graph_shard *g);
+/* DEGk class bits (deg > k, Alg 3) of the owned rows into hbits (uint32
+   words, n_global bits; words v_begin/32 .. written, the rest untouched) */
+int sym_shard_classify(const sym_graph_shard *g, uint32_t k, uint32_t *hbits, sym_stream_t stream);
+/* owned undecided vertices of class cls (-1: any) -> list (int32), *count (device u32) */
+int sym_shard_frontier(const sym_graph_shard *g, const uint32_t *hbits, int cls, const uint8_t *status,
+                       int32_t *list, uint32_t *count, sym_stream_t stream);
+/* one Luby round over the owned frontier (list, *count on the device);
+   neighbours whose class differs from cls are outside the phase (cls = -1: none);
+   still-undecided vertices -> next, *next_count (device u32, set by the call) */
+int sym_shard_mis_round(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits, int cls,
+                        uint8_t *status, const int32_t *frontier, const uint32_t *count, int32_t *next,
+                        uint32_t *next_count, void *ws, size_t ws_bytes, sym_stream_t stream);
+/* MIS-Deg2 fix-up: owned undecided V_H vertices with an In V_L neighbour -> Out */
+int sym_shard_mis_kill(const sym_graph_shard *g, const uint32_t *hbits, uint8_t *status, sym_stream_t stream);
+/* in_set_owned[v - v_begin] = (status[v] == In) for the owned range */
+int sym_shard_mis_finish(const sym_graph_shard *g, const uint8_t *status, uint8_t *in_set_owned,
+                         sym_stream_t stream);
+
 /* ---- kernel profiling hook (measurement only; off by default) ----
    sym_profile_enable(1) makes every later call record a CUDA event pair on its
    stream around each hot-kernel launch, grouped by kernel class ("split",

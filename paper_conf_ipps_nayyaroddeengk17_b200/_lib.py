@@ -19,7 +19,14 @@ F_VALIDATE, F_STATS, F_EXT_DECOMP = 0x1, 0x2, 0x4
 EXPORTS = (
     "sym_workspace_bytes", "sym_decompose", "sym_mis", "sym_mm", "sym_color", "sym_validate",
     "sym_error_string", "sym_last_error", "sym_version", "sym_profile_enable", "sym_profile_collect",
+    "sym_shard_workspace_bytes", "sym_shard_classify", "sym_shard_frontier", "sym_shard_mis_round",
+    "sym_shard_mis_kill", "sym_shard_mis_finish",
 )
+
+
+class SymGraphShard(ctypes.Structure):
+    _fields_ = [("n_global", ctypes.c_int64), ("v_begin", ctypes.c_int64), ("v_end", ctypes.c_int64),
+                ("nnz", ctypes.c_int64), ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p)]
 
 
 class SymKernelProfile(ctypes.Structure):
@@ -87,6 +94,13 @@ def load(build_if_missing: bool = False):
         "sym_error_string": (ctypes.c_char_p, [ctypes.c_int]),
         "sym_last_error": (ctypes.c_char_p, []),
         "sym_version": (ctypes.c_char_p, []),
+        "sym_shard_workspace_bytes": (ctypes.c_size_t, [ctypes.POINTER(SymGraphShard)]),
+        "sym_shard_classify": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), ctypes.c_uint32, P, P]),
+        "sym_shard_frontier": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, ctypes.c_int, P, P, P, P]),
+        "sym_shard_mis_round": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, ctypes.c_int, P, P, P, P, P,
+                                               P, ctypes.c_size_t, P]),
+        "sym_shard_mis_kill": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P]),
+        "sym_shard_mis_finish": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P]),
         "sym_profile_enable": (ctypes.c_int, [ctypes.c_int]),
         "sym_profile_collect": (ctypes.c_int, [ctypes.POINTER(SymKernelProfile), ctypes.c_int,
                                                ctypes.POINTER(ctypes.c_int)]),

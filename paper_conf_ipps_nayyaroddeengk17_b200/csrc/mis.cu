@@ -47,7 +47,16 @@ struct MisRoundArgs {
     int round;
     Key k;
     unsigned long long *prof;  // profiling: algorithmic bytes of this launch (nullable)
+    // sharded mode: rows are local (row of vertex v is v - row_base); neighbours whose
+    // class bit in `nfilter` differs from `ncls` are not in the phase (ncls < 0: none)
+    int64_t row_base;
+    const uint32_t *nfilter;
+    int ncls;
 };
+
+__device__ __forceinline__ bool mis_in_phase(const MisRoundArgs &A, uint32_t w) {
+    return A.ncls < 0 || (int)((A.nfilter[w >> 5] >> (w & 31)) & 1u) == A.ncls;
+}
 
 // algorithmic bytes: 4 B per column word the kernel loads, 16 B for the
 // row_ptr pair + 1 B status per active vertex, 1 B per decided status write;
@@ -56,19 +65,19 @@ struct MisRoundArgs {
 // loads, then all status gathers, then the rule (the order of the arcs does not
 // matter: any In neighbour -> Out, else any higher undecided neighbour -> blocked).
 // Column words are streamed with evict-first loads so the gathered status stays in L2.
-__device__ __forceinline__ int mis_scan_small(const int32_t *__restrict__ ci, const uint8_t *st, int64_t b,
-                                              int64_t e, uint64_t kv, Key k, unsigned long long &lb) {
+__device__ __forceinline__ int mis_scan_small(const MisRoundArgs &A, int64_t b, int64_t e, uint64_t kv,
+                                              unsigned long long &lb) {
     uint32_t w[MIS_SMALL];
     uint8_t s[MIS_SMALL];
 #pragma unroll
-    for (int u = 0; u < MIS_SMALL; u++) w[u] = (b + u < e) ? (uint32_t)__ldcs(ci + b + u) : 0u;
+    for (int u = 0; u < MIS_SMALL; u++) w[u] = (b + u < e) ? (uint32_t)__ldcs(A.ci + b + u) : 0u;
 #pragma unroll
-    for (int u = 0; u < MIS_SMALL; u++) s[u] = (b + u < e) ? st[w[u]] : ST_OUT;
+    for (int u = 0; u < MIS_SMALL; u++) s[u] = (b + u < e && mis_in_phase(A, w[u])) ? A.st[w[u]] : ST_OUT;
     bool in = false, blk = false;
 #pragma unroll
     for (int u = 0; u < MIS_SMALL; u++) {
         in |= s[u] == ST_IN;
-        blk |= (s[u] == ST_UNDEC) && (vkey(k, w[u]) > kv);
+        blk |= (s[u] == ST_UNDEC) && (vkey(A.k, w[u]) > kv);
     }
     lb += 4 * (unsigned long long)(e - b);
     return in ? R_OUT : (blk ? R_BLK : R_IN);
@@ -92,14 +101,14 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
         int64_t b = 0, e = 0;
         uint64_t kv = 0;
         if (active) {
-            b = A.rp[v];
-            e = A.rp[v + 1];
+            b = A.rp[v - A.row_base];
+            e = A.rp[v - A.row_base + 1];
             kv = vkey(A.k, (uint32_t)v);
         }
         int res = R_NONE;
         int64_t resume = 0;
         unsigned long long lb = active ? 17 : 0;
-        if (active && e - b <= MIS_SMALL) res = mis_scan_small(A.ci, A.st, b, e, kv, A.k, lb);
+        if (active && e - b <= MIS_SMALL) res = mis_scan_small(A, b, e, kv, lb);
         unsigned longm = __ballot_sync(FULL, active && e - b > MIS_SMALL);
         while (longm) {
             const int src = __ffs(longm) - 1;
@@ -121,7 +130,7 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
                 bool fin = false, fblk = false;
 #pragma unroll
                 for (int u = 0; u < 4; u++) {
-                    if (ok[u]) {
+                    if (ok[u] && mis_in_phase(A, w[u])) {
                         uint8_t sw = A.st[w[u]];
                         fin |= sw == ST_IN;
                         fblk |= (sw == ST_UNDEC) && (vkey(A.k, w[u]) > wk);
@@ -154,7 +163,7 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
     const uint32_t cnt = *A.huge_cnt;
     for (uint32_t h = blockIdx.x; h < cnt; h += gridDim.x) {
         const int32_t v = (int32_t)A.huge[2 * h];
-        const int64_t b = A.huge[2 * h + 1], e = A.rp[v + 1];
+        const int64_t b = A.huge[2 * h + 1], e = A.rp[v - A.row_base + 1];
         const uint64_t kv = vkey(A.k, (uint32_t)v);
         int r = R_IN;
         unsigned long long lb = threadIdx.x == 0 ? 9 : 0;  // row end + status write
@@ -171,7 +180,7 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
             }
 #pragma unroll
             for (int u = 0; u < 4; u++) {
-                if (ok[u]) {
+                if (ok[u] && mis_in_phase(A, w[u])) {
                     uint8_t sw = A.st[w[u]];
                     fin |= sw == ST_IN;
                     fblk |= (sw == ST_UNDEC) && (vkey(A.k, w[u]) > kv);
@@ -316,6 +325,9 @@ static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp
             A.hist = (phase == 0) ? ctl->hist : ctl->hist + 2048;
             A.round = r < 2048 ? r : 2047;
             A.k = k;
+            A.row_base = 0;
+            A.nfilter = nullptr;
+            A.ncls = -1;
             A.prof = prof_counter(s);
             prof_begin("mis_round", s);
             k_mis_round<<<grid, MIS_THREADS, 0, s>>>(A);
@@ -402,4 +414,181 @@ int run_mis(const FlowArgs &f, MisWs &w, uint8_t *st) {
     return SYM_OK;
 }
 
+// ------------------------------------------------------------------ sharded MIS
+// A rank owns rows [v_begin, v_end) (global ids, v_begin % 32 == 0) stored with global
+// column ids and keeps a full replica of the status array; after every round the
+// caller all-gathers the owned status segments (torch.distributed / NCCL over NVLink)
+// and all-reduces the frontier counts.  DEGk is applied as a class predicate on the
+// owned rows (the global class bitmap is all-gathered once): phase L runs on V_L with
+// V_H neighbours ignored, the fix-up turns every owned V_H vertex with an In V_L
+// neighbour Out, phase R runs on V_H with V_L neighbours ignored.
+
+__global__ void k_shard_classify(const int64_t *__restrict__ rp, int64_t v0, int64_t v1, uint32_t k,
+                                 uint32_t *__restrict__ hbits) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = v0 + (int64_t)blockIdx.x * blockDim.x; base < v1; base += stride) {
+        const int64_t v = base + threadIdx.x;  // base is a multiple of 32 (v0 % 32 == 0)
+        const bool h = v < v1 && (rp[v - v0 + 1] - rp[v - v0]) > (int64_t)k;
+        const unsigned word = __ballot_sync(FULL, h);
+        if (lane_id() == 0 && base + (threadIdx.x & ~31) < v1) hbits[v >> 5] = word;
+    }
+}
+
+__global__ void k_shard_frontier(const uint32_t *__restrict__ hbits, int cls, const uint8_t *__restrict__ st,
+                                 int64_t v0, int64_t v1, int32_t *list, uint32_t *count) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = v0 + (int64_t)blockIdx.x * blockDim.x; base < v1; base += stride) {
+        const int64_t v = base + threadIdx.x;
+        bool take = v < v1 && st[v] == ST_UNDEC && (cls < 0 || (int)((hbits[v >> 5] >> (v & 31)) & 1u) == cls);
+        int64_t slot = warp_append(take, count);
+        if (slot >= 0) list[slot] = (int32_t)v;
+    }
+}
+
+// MIS-Deg2 fix-up, pull form: an owned undecided V_H vertex with an In V_L neighbour
+// leaves the remaining graph (warp per vertex, ballot early exit)
+__global__ void k_shard_kill(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci,
+                             const uint32_t *__restrict__ hbits, uint8_t *st, int64_t v0, int64_t v1) {
+    const int lane = lane_id();
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = v0 + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); v < v1; v += nw) {
+        if (!((hbits[v >> 5] >> (v & 31)) & 1u) || st[v] != ST_UNDEC) continue;
+        const int64_t b = rp[v - v0], e = rp[v - v0 + 1];
+        bool hit = false;
+        for (int64_t x = b; x < e && !hit; x += 32) {
+            bool h = false;
+            if (x + lane < e) {
+                const uint32_t w = (uint32_t)__ldcs(ci + x + lane);
+                h = !((hbits[w >> 5] >> (w & 31)) & 1u) && st[w] == ST_IN;
+            }
+            hit = __any_sync(FULL, h);
+        }
+        if (hit && lane == 0) st[v] = ST_OUT;
+    }
+}
+
+__global__ void k_shard_finish(const uint8_t *__restrict__ st, int64_t v0, int64_t v1, uint8_t *__restrict__ out) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = v0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < v1; v += stride)
+        out[v - v0] = st[v] == ST_IN ? 1 : 0;
+}
+
 }  // namespace sym
+
+using namespace sym;
+
+static int check_shard(const sym_graph_shard *g) {
+    if (!g) { set_error("shard is NULL"); return SYM_EINVAL; }
+    if (g->n_global < 0 || g->n_global >= ((int64_t)1 << 31) - 1 || g->v_begin < 0 || g->v_end < g->v_begin ||
+        g->v_end > g->n_global || g->nnz < 0) {
+        set_error("bad shard range: need 0 <= v_begin <= v_end <= n_global < 2^31 - 1, nnz >= 0");
+        return SYM_EINVAL;
+    }
+    if (g->v_begin % 32 && g->v_end > g->v_begin) {
+        set_error("v_begin must be a multiple of 32");
+        return SYM_EINVAL;
+    }
+    if (g->v_end > g->v_begin && !g->row_ptr) { set_error("row_ptr is NULL"); return SYM_EINVAL; }
+    if (g->nnz > 0 && !g->col_idx) { set_error("col_idx is NULL"); return SYM_EINVAL; }
+    return SYM_OK;
+}
+
+static int shard_grid(int64_t items) {
+    int64_t want = (items + 255) / 256;
+    int64_t cap = (int64_t)num_sms() * 8;
+    return (int)(want < 1 ? 1 : (want < cap ? want : cap));
+}
+
+extern "C" size_t sym_shard_workspace_bytes(const sym_graph_shard *g) {
+    if (check_shard(g) != SYM_OK) return 0;
+    return 256 + 64 + sizeof(int64_t) * 2 * (size_t)(g->nnz / MIS_BUDGET + 2) + 256;
+}
+
+extern "C" int sym_shard_classify(const sym_graph_shard *g, uint32_t k, uint32_t *hbits, sym_stream_t stream) {
+    SYM_TRY(check_shard(g));
+    if (g->v_end == g->v_begin) return SYM_OK;
+    if (!hbits) { set_error("hbits is NULL"); return SYM_EINVAL; }
+    k_shard_classify<<<shard_grid(g->v_end - g->v_begin), 256, 0, (cudaStream_t)stream>>>(g->row_ptr, g->v_begin,
+                                                                                           g->v_end, k, hbits);
+    SYM_LAUNCH_CHECK();
+    return SYM_OK;
+}
+
+extern "C" int sym_shard_frontier(const sym_graph_shard *g, const uint32_t *hbits, int cls, const uint8_t *status,
+                                  int32_t *list, uint32_t *count, sym_stream_t stream) {
+    SYM_TRY(check_shard(g));
+    if (!status || !list || !count || (cls >= 0 && !hbits)) { set_error("NULL argument"); return SYM_EINVAL; }
+    cudaStream_t s = (cudaStream_t)stream;
+    SYM_CUDA(cudaMemsetAsync(count, 0, sizeof(uint32_t), s));
+    if (g->v_end == g->v_begin) return SYM_OK;
+    k_shard_frontier<<<shard_grid(g->v_end - g->v_begin), 256, 0, s>>>(hbits, cls, status, g->v_begin, g->v_end, list,
+                                                                       count);
+    SYM_LAUNCH_CHECK();
+    return SYM_OK;
+}
+
+extern "C" int sym_shard_mis_round(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits, int cls,
+                                   uint8_t *status, const int32_t *frontier, const uint32_t *count, int32_t *next,
+                                   uint32_t *next_count, void *ws, size_t ws_bytes, sym_stream_t stream) {
+    SYM_TRY(check_shard(g));
+    if (!p || !status || !frontier || !count || !next || !next_count || (cls >= 0 && !hbits)) {
+        set_error("NULL argument");
+        return SYM_EINVAL;
+    }
+    const size_t need = sym_shard_workspace_bytes(g);
+    if (!ws || ws_bytes < need) { set_error("shard workspace too small"); return SYM_EWORKSPACE; }
+    cudaStream_t s = (cudaStream_t)stream;
+    char *base = (char *)(((uintptr_t)ws + 255) & ~(uintptr_t)255);
+    uint32_t *ctr = reinterpret_cast<uint32_t *>(base);               // [0] huge count, [1..3] scratch
+    int64_t *huge = reinterpret_cast<int64_t *>(base + 64);
+    SYM_CUDA(cudaMemsetAsync(ctr, 0, 64, s));
+    SYM_CUDA(cudaMemsetAsync(next_count, 0, sizeof(uint32_t), s));
+    MisRoundArgs A;
+    A.rp = g->row_ptr;
+    A.ci = g->col_idx;
+    A.st = status;
+    A.in_list = frontier;
+    A.in_rev = 0;
+    A.in_cnt = count;
+    A.implicit_n = 0;
+    A.out_list = next;
+    A.out_cnt = next_count;
+    A.clear_cnt = ctr + 1;
+    A.huge = huge;
+    A.huge_cnt = ctr;
+    A.huge_clear = ctr + 2;
+    A.hist = nullptr;
+    A.round = 0;
+    A.k = stream_key(p->seed, TAG_VERTEX, 0);
+    A.prof = nullptr;
+    A.row_base = g->v_begin;
+    A.nfilter = hbits;
+    A.ncls = cls;
+    k_mis_round<<<round_grid(), MIS_THREADS, 0, s>>>(A);
+    SYM_LAUNCH_CHECK();
+    k_mis_huge<<<num_sms() * 2, MIS_HUGE_THREADS, 0, s>>>(A);
+    SYM_LAUNCH_CHECK();
+    return SYM_OK;
+}
+
+extern "C" int sym_shard_mis_kill(const sym_graph_shard *g, const uint32_t *hbits, uint8_t *status,
+                                  sym_stream_t stream) {
+    SYM_TRY(check_shard(g));
+    if (!hbits || !status) { set_error("NULL argument"); return SYM_EINVAL; }
+    if (g->v_end == g->v_begin) return SYM_OK;
+    k_shard_kill<<<num_sms() * 8, 256, 0, (cudaStream_t)stream>>>(g->row_ptr, g->col_idx, hbits, status, g->v_begin,
+                                                                   g->v_end);
+    SYM_LAUNCH_CHECK();
+    return SYM_OK;
+}
+
+extern "C" int sym_shard_mis_finish(const sym_graph_shard *g, const uint8_t *status, uint8_t *in_set_owned,
+                                    sym_stream_t stream) {
+    SYM_TRY(check_shard(g));
+    if (!status || (g->v_end > g->v_begin && !in_set_owned)) { set_error("NULL argument"); return SYM_EINVAL; }
+    if (g->v_end == g->v_begin) return SYM_OK;
+    k_shard_finish<<<shard_grid(g->v_end - g->v_begin), 256, 0, (cudaStream_t)stream>>>(status, g->v_begin, g->v_end,
+                                                                                        in_set_owned);
+    SYM_LAUNCH_CHECK();
+    return SYM_OK;
+}
