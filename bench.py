@@ -31,7 +31,12 @@ METRIC = "MIS/MM/COLOR edges/s at 1/2/4/8 B200; % of HBM roofline; vs CPU oracle
 # per-launch DRAM traffic (dram__bytes_read.sum + dram__bytes_write.sum) of each kernel
 # class from one `ncu --set full` capture of this step (profiles/r1_ncu_summary.md);
 # None where no capture was taken for the current code.
-TRAFFIC = {}
+TRAFFIC = {
+    "split": 4.51e9,       # k_split<DEGK> at R-MAT s24 (profiles/r1_ncu.md): 2.22 GB read + 2.29 GB written
+    "mm_round0": 0.717e9,  # k_round0<MM> on the RAND-4 intra CSR
+    "jp_init": 1.90e9,
+    "jp_async": 25.04e9,   # 20.0 GB read + 5.04 GB written: random record/bitmap traffic
+}
 
 
 def parse():
@@ -304,6 +309,34 @@ def main():
                "h2d_bytes_per_step": rp_h.numel() * 8 + ci_h.numel() * 4, "d2h_bytes_per_step": outs_bytes,
                "ms_per_step": e_ms, "steps": args.e2e_steps}
 
+    # ---- sharded MIS-Deg2 of ONE graph across the N ranks (the exchange path,
+    #      SURVEY §8(e)): per round, NCCL all-gather of the owned 1-byte status segments
+    from paper_conf_ipps_nayyaroddeengk17_b200 import sharded as S
+    shards = S.make_shards(rp, ci, world, ranks=[rank])
+    tr = S.DistTransport() if world > 1 else S.LocalTransport()
+    sst = {}
+    S.sym_mis_sharded(shards, "degk", 2, args.seed, tr, None, sst)  # warm-up
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    reps = 3
+    s0.record(stream)
+    for _ in range(reps):
+        S.sym_mis_sharded(shards, "degk", 2, args.seed, tr, None, sst)
+    s1.record(stream)
+    torch.cuda.synchronize()
+    sh_ms = s0.elapsed_time(s1) / reps
+    if world > 1:
+        t = torch.tensor([sh_ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        sh_ms = float(t.item())
+    sharded = {"problem": "MIS-Deg2 (no decomposition materialised; DEGk as a class predicate)",
+               "ranks": world, "ms": sh_ms, "edges_per_s": m / (sh_ms * 1e-3), "rounds": sst.get("rounds"),
+               "exchange": "all_gather_into_tensor of owned status segments + all_reduce of frontier counts per round",
+               "scaling": "strong (one graph)"}
+    del shards
+
     # ---- CPU oracle (rank 0, N = 1 only), bounded sample
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
@@ -331,7 +364,7 @@ def main():
                                       "color_deg2_incl_decomp": m / ((brk["decompose_deg2"] + brk["color_deg2"]) * 1e-3),
                                       "mm_rand4_incl_decomp": m / ((brk["decompose_rand4"] + brk["mm_rand4"]) * 1e-3)},
             "kernels": per_step, "dominant_kernel": dominant_overall,
-            "roofline": roof, "rooflines": rooflines, "cpu_baseline": cpu, "e2e": e2e,
+            "roofline": roof, "rooflines": rooflines, "cpu_baseline": cpu, "e2e": e2e, "sharded_mis": sharded,
             "gpu_launches": int(round(launches)),
             "clocks": clk.summary(),
             "stats": {"mis": st_mis, "color": st_col, "mm": st_mm},
