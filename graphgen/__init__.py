@@ -98,6 +98,40 @@ def csr_from_edges(n: int, src: torch.Tensor, dst: torch.Tensor):
     return row_ptr, col
 
 
+def csr_from_edges_bucketed(n: int, src: torch.Tensor, dst: torch.Tensor, nbuckets: int):
+    """csr_from_edges for graphs whose arc list does not fit a global sort in memory:
+    the arcs are grouped by source-vertex bucket, each bucket is deduplicated and
+    sorted on its own.  The result is identical (same canonical CSR)."""
+    dev = src.device
+    keep = src != dst
+    src, dst = src[keep], dst[keep]
+    B = (n + nbuckets - 1) // nbuckets
+    deg = torch.zeros(n + 1, dtype=torch.int64, device=dev)
+    parts = []
+    for b in range(nbuckets):
+        lo, hi = b * B, min(n, (b + 1) * B)
+        if lo >= hi:
+            break
+        m1 = (src >= lo) & (src < hi)
+        m2 = (dst >= lo) & (dst < hi)
+        a = torch.cat([src[m1], dst[m2]]).to(torch.int64)
+        c = torch.cat([dst[m1], src[m2]]).to(torch.int64)
+        del m1, m2
+        key = torch.unique((a - lo) * n + c, sorted=True)
+        del a, c
+        s = key // n
+        parts.append((key - s * n).to(torch.int32))
+        deg[lo + 1:hi + 1] = torch.bincount(s, minlength=hi - lo)
+        del key, s
+    row_ptr = torch.cumsum(deg, 0)
+    col = torch.empty(int(row_ptr[-1]), dtype=torch.int32, device=dev)
+    off = 0
+    for p in parts:
+        col[off:off + p.numel()] = p
+        off += p.numel()
+    return row_ptr, col
+
+
 def _perm_bits(x: torch.Tensor, scale: int, seed: int) -> torch.Tensor:
     """A bijection on [0, 2^scale): two rounds of (odd multiply mod 2^s, xorshift)."""
     if scale == 0:
@@ -121,9 +155,14 @@ _T2 = int((RMAT_A + RMAT_B) * 2**32)
 _T3 = int((RMAT_A + RMAT_B + RMAT_C) * 2**32)
 
 
-def rmat(scale: int, ef: int, seed: int = 1, device="cpu", chunk: int = 1 << 26):
+def rmat(scale: int, ef: int, seed: int = 1, device="cpu", chunk: int = 1 << 26, buckets: int | None = None):
+    """buckets: assemble the CSR in source buckets (default: 1 below scale 26, else 16)
+    so that scale 27 (2^31 edges) fits in one GPU's memory; same output either way."""
     n = 1 << scale
     ne = ef << scale
+    if buckets is None:
+        buckets = 1 if scale < 26 else 16
+    small_ids = buckets > 1 and n < 2**31
     srcs, dsts = [], []
     for c0 in range(0, ne, chunk):
         i = torch.arange(c0, min(ne, c0 + chunk), dtype=torch.int64, device=device)
@@ -135,12 +174,16 @@ def rmat(scale: int, ef: int, seed: int = 1, device="cpu", chunk: int = 1 << 26)
             db = ((r >= _T1) & (r < _T2)) | (r >= _T3)            # quadrants b,d
             s = (s << 1) | sb
             d = (d << 1) | db.to(torch.int64)
-        srcs.append(_perm_bits(s, scale, seed))
-        dsts.append(_perm_bits(d, scale, seed))
-        del i, s, d
+        ps, pd = _perm_bits(s, scale, seed), _perm_bits(d, scale, seed)
+        srcs.append(ps.to(torch.int32) if small_ids else ps)
+        dsts.append(pd.to(torch.int32) if small_ids else pd)
+        del i, s, d, ps, pd
     src = torch.cat(srcs)
+    del srcs
     dst = torch.cat(dsts)
-    del srcs, dsts
+    del dsts
+    if buckets > 1:
+        return csr_from_edges_bucketed(n, src, dst, buckets)
     return csr_from_edges(n, src, dst)
 
 
