@@ -231,6 +231,39 @@ int sym_shard_mis_kill(const sym_graph_shard *g, const uint32_t *hbits, uint8_t 
 int sym_shard_mis_finish(const sym_graph_shard *g, const uint8_t *status, uint8_t *in_set_owned,
                          sym_stream_t stream);
 
+/* ---- sharded MM (MM-NONE / MM-Rand, Alg 5; handshake rounds P:152-154) ----
+   Same shard layout as above (v_begin need not be 32-aligned here).  Every rank keeps
+   full replicas of mate int32[n_global] (caller-initialised to -1) and of two pick
+   buffers int32[n_global] (contents arbitrary before round 0).  Round r writes
+   pick_cur = picks[r & 1] and reads pick_prev = picks[(r + 1) & 1] (round 0 reads no
+   picks).  After each round the caller all-gathers the owned segments of pick_cur
+   and mate and all-reduces *next_count; the phase ends when the global count is 0.
+   MM-Rand: decompose the owned rows with sym_shard_decompose (labels hash the GLOBAL
+   id, so the parts equal the single-GPU ones), phase 1 = rounds on the local intra
+   CSR, phase 2 = rounds on the local cross CSR starting from the vertices still
+   unmatched.  Priorities are the single-GPU ones, so the result equals sym_mm() bit
+   for bit.  All pointers are device pointers. */
+
+/* workspace for sym_shard_decompose (host only; 0 on invalid arguments) */
+size_t sym_shard_decompose_workspace_bytes(const sym_graph_shard *g);
+/* RAND decomposition (Alg 2) of the owned rows: local intra / cross CSRs
+   row_ptr_* int64[v_end - v_begin + 1], col_idx_* int32[nnz] (capacity; global ids),
+   the intra arcs first in the same order as sym_decompose.  p->kind RAND or NONE. */
+int sym_shard_decompose(const sym_graph_shard *g, const sym_params *p, void *ws, size_t ws_bytes,
+                        int64_t *row_ptr_in, int32_t *col_idx_in, int64_t *row_ptr_x, int32_t *col_idx_x,
+                        sym_stream_t stream);
+/* workspace for sym_shard_mm_round (host only; 0 on invalid arguments) */
+size_t sym_shard_mm_workspace_bytes(const sym_graph_shard *g);
+/* owned vertices with mate < 0 and at least one arc in g -> list, *count (device u32) */
+int sym_shard_mm_frontier(const sym_graph_shard *g, const int32_t *mate, int32_t *list, uint32_t *count,
+                          sym_stream_t stream);
+/* one handshake round over the owned frontier: resolve round-(r-1) mutual picks
+   (r > 0), then pick the heaviest edge to a neighbour with mate < 0; vertices with a
+   pick -> next, *next_count (device u32, set by the call) */
+int sym_shard_mm_round(const sym_graph_shard *g, const sym_params *p, int round, int32_t *mate,
+                       const int32_t *pick_prev, int32_t *pick_cur, const int32_t *frontier, const uint32_t *count,
+                       int32_t *next, uint32_t *next_count, void *ws, size_t ws_bytes, sym_stream_t stream);
+
 /* ---- kernel profiling hook (measurement only; off by default) ----
    sym_profile_enable(1) makes every later call record a CUDA event pair on its
    stream around each hot-kernel launch, grouped by kernel class ("split",

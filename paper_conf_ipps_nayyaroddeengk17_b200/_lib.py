@@ -21,6 +21,8 @@ EXPORTS = (
     "sym_error_string", "sym_last_error", "sym_version", "sym_profile_enable", "sym_profile_collect",
     "sym_shard_workspace_bytes", "sym_shard_classify", "sym_shard_frontier", "sym_shard_mis_round",
     "sym_shard_mis_kill", "sym_shard_mis_finish",
+    "sym_shard_decompose_workspace_bytes", "sym_shard_decompose", "sym_shard_mm_workspace_bytes",
+    "sym_shard_mm_frontier", "sym_shard_mm_round",
 )
 
 
@@ -101,6 +103,13 @@ def load(build_if_missing: bool = False):
                                                P, ctypes.c_size_t, P]),
         "sym_shard_mis_kill": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P]),
         "sym_shard_mis_finish": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P]),
+        "sym_shard_decompose_workspace_bytes": (ctypes.c_size_t, [ctypes.POINTER(SymGraphShard)]),
+        "sym_shard_decompose": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, ctypes.c_size_t, P, P, P, P,
+                                               P]),
+        "sym_shard_mm_workspace_bytes": (ctypes.c_size_t, [ctypes.POINTER(SymGraphShard)]),
+        "sym_shard_mm_frontier": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P, P]),
+        "sym_shard_mm_round": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, ctypes.c_int, P, P, P, P, P, P,
+                                              P, P, ctypes.c_size_t, P]),
         "sym_profile_enable": (ctypes.c_int, [ctypes.c_int]),
         "sym_profile_collect": (ctypes.c_int, [ctypes.POINTER(SymKernelProfile), ctypes.c_int,
                                                ctypes.POINTER(ctypes.c_int)]),

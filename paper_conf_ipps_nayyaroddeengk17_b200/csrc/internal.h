@@ -100,9 +100,12 @@ int run_round0(int mode, const Graph &g, const int64_t *first_row, int64_t ntile
                unsigned long long *gmax, uint8_t *st, int32_t *pick, const uint32_t *hfilter, int32_t *out_list,
                uint32_t *out_cnt, cudaStream_t s);
 
-// decompose into caller buffers (rp_in, ci_in, rp_x, ci_x) ; kind in {NONE,RAND,DEGK}
+// decompose into caller buffers (rp_in, ci_in, rp_x, ci_x) ; kind in {NONE,RAND,DEGK}.
+// row_base = global id of local row 0 (a shard's row block; RAND/NONE only, since the
+// DEGk bitmap is indexed by local row)
 int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const SplitWs &w, Ctl *ctl,
-              int64_t *rp_in, int32_t *ci_in, int64_t *rp_x, int32_t *ci_x, uint16_t *label, cudaStream_t s);
+              int64_t *rp_in, int32_t *ci_in, int64_t *rp_x, int32_t *ci_x, uint16_t *label, cudaStream_t s,
+              int64_t row_base = 0);
 
 // ------------------------------------------------------------------ profiling hook (profile.cu)
 bool prof_on();

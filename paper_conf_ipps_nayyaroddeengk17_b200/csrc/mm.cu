@@ -45,6 +45,7 @@ struct MmRoundArgs {
     int round;
     Key k;
     unsigned long long *prof;  // profiling: algorithmic bytes of this launch (nullable)
+    int64_t row_base;          // global id of local row 0 (sharded path; 0 otherwise)
 };
 // algorithmic bytes: 4 B per column word loaded; per active vertex the
 // row_ptr pair (16 B) and the pick write (4 B); per resolved vertex the two pick
@@ -53,12 +54,12 @@ struct MmRoundArgs {
 
 __device__ __forceinline__ void mm_row(const MmRoundArgs &A, int32_t u, int64_t &b, int64_t &e, const int32_t *&ci) {
     if (A.dual && ((A.hbits[u >> 5] >> (u & 31)) & 1u)) {
-        b = A.rp2[u];
-        e = A.rp2[u + 1];
+        b = A.rp2[u - A.row_base];
+        e = A.rp2[u - A.row_base + 1];
         ci = A.ci2;
     } else {
-        b = A.rp[u];
-        e = A.rp[u + 1];
+        b = A.rp[u - A.row_base];
+        e = A.rp[u - A.row_base + 1];
         ci = A.ci;
     }
 }
@@ -336,6 +337,7 @@ static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph
             A.hist = ctl->hist + phase * 2048;
             A.round = r < 2048 ? r : 2047;
             A.k = k;
+            A.row_base = 0;
             // round 0 of a phase has nothing to resolve (its pick buffers hold stale or
             // uninitialised values); round 0 of the first phase has nothing matched yet
             // profiling byte counters are accumulated by the kernels
@@ -442,4 +444,102 @@ int run_mm(const FlowArgs &f, MmWs &w, int32_t *mate) {
     return SYM_OK;
 }
 
+// ------------------------------------------------------------------ sharded MM (C-ABI below)
+// owned vertices [v0, v1) with mate[v] < 0 and at least one arc in the local phase CSR
+__global__ void k_shard_mm_frontier(const int64_t *__restrict__ rp, int64_t v0, int64_t v1, const int32_t *mate,
+                                    int32_t *list, uint32_t *cnt) {
+    const int64_t n = v1 - v0, stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
+        const int64_t i = base + threadIdx.x;
+        const bool take = i < n && mate[v0 + i] < 0 && rp[i + 1] > rp[i];
+        const int64_t s = warp_append(take, cnt);
+        if (s >= 0) list[s] = (int32_t)(v0 + i);
+    }
+}
+
 }  // namespace sym
+
+using namespace sym;
+
+static int check_mm_shard(const sym_graph_shard *g) {
+    if (!g) { set_error("shard is NULL"); return SYM_EINVAL; }
+    if (g->n_global < 0 || g->n_global >= ((int64_t)1 << 31) - 1 || g->v_begin < 0 || g->v_end < g->v_begin ||
+        g->v_end > g->n_global || g->nnz < 0) {
+        set_error("bad shard range: need 0 <= v_begin <= v_end <= n_global < 2^31 - 1, nnz >= 0");
+        return SYM_EINVAL;
+    }
+    if (g->v_end > g->v_begin && !g->row_ptr) { set_error("row_ptr is NULL"); return SYM_EINVAL; }
+    if (g->nnz > 0 && !g->col_idx) { set_error("col_idx is NULL"); return SYM_EINVAL; }
+    return SYM_OK;
+}
+
+extern "C" size_t sym_shard_mm_workspace_bytes(const sym_graph_shard *g) {
+    if (check_mm_shard(g) != SYM_OK) return 0;
+    return 256 + 64 + sizeof(int32_t) * (size_t)(g->nnz / MM_BUDGET + 2) + 256;
+}
+
+extern "C" int sym_shard_mm_frontier(const sym_graph_shard *g, const int32_t *mate, int32_t *list, uint32_t *count,
+                                     sym_stream_t stream) {
+    SYM_TRY(check_mm_shard(g));
+    if (!mate || !list || !count) { set_error("NULL argument"); return SYM_EINVAL; }
+    cudaStream_t s = (cudaStream_t)stream;
+    SYM_CUDA(cudaMemsetAsync(count, 0, sizeof(uint32_t), s));
+    const int64_t nl = g->v_end - g->v_begin;
+    if (nl == 0) return SYM_OK;
+    int64_t want = (nl + 255) / 256, cap = (int64_t)num_sms() * 8;
+    k_shard_mm_frontier<<<(int)(want < cap ? want : cap), 256, 0, s>>>(g->row_ptr, g->v_begin, g->v_end, mate, list,
+                                                                       count);
+    SYM_LAUNCH_CHECK();
+    return SYM_OK;
+}
+
+extern "C" int sym_shard_mm_round(const sym_graph_shard *g, const sym_params *p, int round, int32_t *mate,
+                                  const int32_t *pick_prev, int32_t *pick_cur, const int32_t *frontier,
+                                  const uint32_t *count, int32_t *next, uint32_t *next_count, void *ws,
+                                  size_t ws_bytes, sym_stream_t stream) {
+    SYM_TRY(check_mm_shard(g));
+    if (!p || !mate || !pick_cur || (round > 0 && !pick_prev) || !frontier || !count || !next || !next_count) {
+        set_error("NULL argument");
+        return SYM_EINVAL;
+    }
+    if (round < 0) { set_error("round must be >= 0"); return SYM_EINVAL; }
+    const size_t need = sym_shard_mm_workspace_bytes(g);
+    if (!ws || ws_bytes < need) { set_error("shard workspace too small"); return SYM_EWORKSPACE; }
+    cudaStream_t s = (cudaStream_t)stream;
+    char *base = (char *)(((uintptr_t)ws + 255) & ~(uintptr_t)255);
+    uint32_t *ctr = reinterpret_cast<uint32_t *>(base);  // [0] huge count, [1..3] scratch
+    SYM_CUDA(cudaMemsetAsync(ctr, 0, 64, s));
+    SYM_CUDA(cudaMemsetAsync(next_count, 0, sizeof(uint32_t), s));
+    MmRoundArgs A;
+    A.rp = g->row_ptr;
+    A.rp2 = nullptr;
+    A.ci = g->col_idx;
+    A.ci2 = nullptr;
+    A.hbits = nullptr;
+    A.dual = 0;
+    A.mate = mate;
+    A.pick_prev = pick_prev;
+    A.pick_cur = pick_cur;
+    A.in_list = frontier;
+    A.in_rev = 0;
+    A.in_cnt = count;
+    A.implicit_n = 0;
+    A.out_list = next;
+    A.out_cnt = next_count;
+    A.clear_cnt = ctr + 1;
+    A.huge = reinterpret_cast<int32_t *>(base + 64);
+    A.huge_cnt = ctr;
+    A.huge_clear = ctr + 2;
+    A.hist = nullptr;
+    A.round = 0;
+    A.k = stream_key(p->seed, TAG_EDGE, 0);
+    A.prof = nullptr;
+    A.row_base = g->v_begin;
+    const int grid = num_sms() * (2048 / MM_THREADS);
+    if (round == 0) k_mm_round<false, true><<<grid, MM_THREADS, 0, s>>>(A);
+    else k_mm_round<true, true><<<grid, MM_THREADS, 0, s>>>(A);
+    SYM_LAUNCH_CHECK();
+    k_mm_huge<true><<<num_sms() * 2, MM_HUGE_THREADS, 0, s>>>(A);
+    SYM_LAUNCH_CHECK();
+    return SYM_OK;
+}

@@ -89,7 +89,7 @@ __global__ void __launch_bounds__(SPLIT_THREADS)
     k_split(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, int64_t n, int64_t nnz,
             const int64_t *__restrict__ first_row, int64_t ntiles, const uint32_t *__restrict__ hbits, Key kr,
             uint32_t p, uint64_t *tile_state, int64_t *__restrict__ rp_in, int32_t *__restrict__ ci_in,
-            int64_t *__restrict__ rp_x, int32_t *__restrict__ ci_x) {
+            int64_t *__restrict__ rp_x, int32_t *__restrict__ ci_x, int64_t row_base) {
     constexpr int T = SPLIT_TILE, V = SPLIT_PER_THREAD, NT = SPLIT_THREADS, NW = NT / 32;
     static_assert(V % 4 == 0 && T < 32768, "tile layout");
     __shared__ __align__(16) int16_t s_head[T];   // head position of the row owning each arc, or -1
@@ -136,7 +136,7 @@ __global__ void __launch_bounds__(SPLIT_THREADS)
         int4 m1 = make_int4(-1, -1, -1, -1);
         for (int j = tid * 8; j < T; j += NT * 8) *reinterpret_cast<int4 *>(s_head + j) = m1;
     }
-    if (tid == 0) s_cls0 = (r_begin > 0) ? vclass((uint32_t)(r_begin - 1)) : 0u;
+    if (tid == 0) s_cls0 = (r_begin > 0) ? vclass((uint32_t)(row_base + r_begin - 1)) : 0u;
     __syncthreads();
     for (int64_t r = r_begin + tid; r < r_end; r += NT) {
         if (r >= n) continue;
@@ -144,7 +144,7 @@ __global__ void __launch_bounds__(SPLIT_THREADS)
         if (e > s) {
             int j = (int)(s - a);
             s_head[j] = (int16_t)j;
-            s_cls[j] = (uint16_t)vclass((uint32_t)r);
+            s_cls[j] = (uint16_t)vclass((uint32_t)(row_base + r));
         }
     }
     __syncthreads();
@@ -330,7 +330,7 @@ int launch_classify_degk(const Graph &g, uint32_t k, uint32_t *hbits, int32_t *v
 }
 
 int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const SplitWs &w, Ctl *ctl, int64_t *rp_in,
-              int32_t *ci_in, int64_t *rp_x, int32_t *ci_x, uint16_t *label, cudaStream_t s) {
+              int32_t *ci_in, int64_t *rp_x, int32_t *ci_x, uint16_t *label, cudaStream_t s, int64_t row_base) {
     Key kr = stream_key(seed, TAG_RAND, 0);
     if (label && g.n > 0) {
         k_labels<<<grid_for(g.n, 256), 256, 0, s>>>(g.rp, g.n, kind, param, kr, label);
@@ -350,7 +350,7 @@ int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const Spl
     prof_begin("split", s);
 #define SPLIT_ARGS                                                                                          \
     g.rp, g.ci, g.n, g.nnz, w.first_row, w.ntiles, w.hbits, kr, param, w.tile_state, rp_in, \
-        ci_in, rp_x, ci_x
+        ci_in, rp_x, ci_x, row_base
     if (kind == KIND_RAND) {
         if (vec) k_split<KIND_RAND, true><<<grid, SPLIT_THREADS, 0, s>>>(SPLIT_ARGS);
         else k_split<KIND_RAND, false><<<grid, SPLIT_THREADS, 0, s>>>(SPLIT_ARGS);
@@ -370,3 +370,55 @@ int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const Spl
 }
 
 }  // namespace sym
+
+// ------------------------------------------------------------------ sharded decomposition (C-ABI)
+using namespace sym;
+
+static int check_split_shard(const sym_graph_shard *g) {
+    if (!g) { set_error("shard is NULL"); return SYM_EINVAL; }
+    if (g->n_global < 0 || g->n_global >= ((int64_t)1 << 31) - 1 || g->v_begin < 0 || g->v_end < g->v_begin ||
+        g->v_end > g->n_global || g->nnz < 0) {
+        set_error("bad shard range: need 0 <= v_begin <= v_end <= n_global < 2^31 - 1, nnz >= 0");
+        return SYM_EINVAL;
+    }
+    if (g->v_end > g->v_begin && !g->row_ptr) { set_error("row_ptr is NULL"); return SYM_EINVAL; }
+    if (g->nnz > 0 && !g->col_idx) { set_error("col_idx is NULL"); return SYM_EINVAL; }
+    return SYM_OK;
+}
+
+extern "C" size_t sym_shard_decompose_workspace_bytes(const sym_graph_shard *g) {
+    if (check_split_shard(g) != SYM_OK) return 0;
+    Arena a;
+    SplitWs w;
+    carve_split_ws(a, g->v_end - g->v_begin, g->nnz, w);
+    return a.used + 256;
+}
+
+extern "C" int sym_shard_decompose(const sym_graph_shard *g, const sym_params *p, void *ws, size_t ws_bytes,
+                                   int64_t *row_ptr_in, int32_t *col_idx_in, int64_t *row_ptr_x, int32_t *col_idx_x,
+                                   sym_stream_t stream) {
+    SYM_TRY(check_split_shard(g));
+    if (!p) { set_error("params is NULL"); return SYM_EINVAL; }
+    if (p->kind != SYM_DECOMP_RAND && p->kind != SYM_DECOMP_NONE) {
+        set_error("sharded decomposition supports RAND (and NONE) only");
+        return SYM_EINVAL;
+    }
+    if (p->kind == SYM_DECOMP_RAND && (p->param < 1 || p->param > 65535)) {
+        set_error("RAND needs 1 <= p <= 65535");
+        return SYM_EINVAL;
+    }
+    if (!row_ptr_in || !row_ptr_x || (g->nnz > 0 && (!col_idx_in || !col_idx_x))) {
+        set_error("NULL output buffer");
+        return SYM_EINVAL;
+    }
+    const size_t need = sym_shard_decompose_workspace_bytes(g);
+    if (!ws || ws_bytes < need) { set_error("shard workspace too small"); return SYM_EWORKSPACE; }
+    Arena a;
+    a.base = (char *)(((uintptr_t)ws + 255) & ~(uintptr_t)255);
+    a.cap = ws_bytes - 256;
+    SplitWs w;
+    const int64_t nl = g->v_end - g->v_begin;
+    carve_split_ws(a, nl, g->nnz, w);
+    return run_split(Graph{nl, g->nnz, g->row_ptr, g->col_idx}, p->kind, p->param, p->seed, w, nullptr, row_ptr_in,
+                     col_idx_in, row_ptr_x, col_idx_x, nullptr, (cudaStream_t)stream, g->v_begin);
+}

@@ -1,4 +1,4 @@
-"""Sharded MIS over several GPUs (C-ABI: include/sym.h `sym_shard_*`).
+"""Sharded MIS and MM over several GPUs (C-ABI: include/sym.h `sym_shard_*`).
 
 One process per GPU.  Rank r owns the 32-aligned vertex block [r*B, min(n, (r+1)*B))
 and holds those rows with global column ids; every rank keeps a full replica of the
@@ -10,6 +10,12 @@ MIS-Deg2 applies the DEGk decomposition as a class predicate on the owne
 rows: the global V_H bitmap is all-gathered once; phase L on V_L, the fix-up
 `sym_shard_mis_kill`, phase R on V_H.  Results equal the single-GPU sym_mis() bit
 for bit (fixed priorities make every schedule give the lexicographically-first MIS).
+
+MM-NONE / MM-Rand (Alg 5) keep replicas of `mate` and of the two pick
+buffers; per handshake round (`sym_shard_mm_round`) the owned segments of
+the current picks and of mate are all-gathered.  MM-Rand decomposes the owned rows
+locally (`sym_shard_decompose`; labels hash the global id): phase 1 on the local
+intra CSR, phase 2 on the local cross CSR.  Results equal sym_mm() bit for bit.
 
 This module is orchestration only: every step of the method runs in libsym.so
 kernels (`GpuBackend`); the exchange is a `Transport`:
@@ -64,6 +70,9 @@ class Shard:
     cur_cnt: torch.Tensor = None
     nxt_cnt: torch.Tensor = None
     ws: torch.Tensor = None
+    mate: torch.Tensor = None    # MM: replica, int32[nranks * block]
+    picks: list = None           # MM: two pick replicas (round r writes picks[r & 1])
+    pick_cur: torch.Tensor = None
     extra: dict = field(default_factory=dict)
 
     def __post_init__(self):
@@ -83,8 +92,34 @@ class Shard:
     def owned(self) -> slice:
         return slice(self.rank * self.block, (self.rank + 1) * self.block)
 
+    def segment(self, attr) -> slice:
+        """Owned part of a replica: per-vertex arrays by vertex, the bitmap by word."""
+        if attr == "hbits":
+            return slice(self.owned.start // 32, self.owned.stop // 32)
+        return self.owned
+
     def c_struct(self) -> L.SymGraphShard:
         return L.SymGraphShard(self.n_global, self.v0, self.v1, self.col_idx.numel(), self.row_ptr.data_ptr(),
+                               self.col_idx.data_ptr() if self.col_idx.numel() else 0)
+
+    def init_mm(self):
+        dev = self.row_ptr.device
+        pad = self.nranks * self.block
+        self.mate = torch.full((pad,), -1, dtype=torch.int32, device=dev)
+        self.picks = [torch.full((pad,), -1, dtype=torch.int32, device=dev) for _ in range(2)]
+
+
+@dataclass
+class PhaseView:
+    """A local phase CSR over the shard's owned rows (global column ids)."""
+    shard: Shard
+    row_ptr: torch.Tensor
+    col_idx: torch.Tensor
+    nnz: int
+
+    def c_struct(self) -> L.SymGraphShard:
+        sh = self.shard
+        return L.SymGraphShard(sh.n_global, sh.v0, sh.v1, self.nnz, self.row_ptr.data_ptr(),
                                self.col_idx.data_ptr() if self.col_idx.numel() else 0)
 
 
@@ -95,7 +130,7 @@ class LocalTransport:
     def allgather(self, shards, attr):
         for s in shards:
             src = getattr(s, attr)
-            seg = s.owned if attr == "status" else slice(s.owned.start // 32, s.owned.stop // 32)
+            seg = s.segment(attr)
             for o in shards:
                 if o is not s:
                     getattr(o, attr)[seg].copy_(src[seg])
@@ -114,7 +149,7 @@ class DistTransport:
         import torch.distributed as dist
         (s,) = shards
         full = getattr(s, attr)
-        seg = s.owned if attr == "status" else slice(s.owned.start // 32, s.owned.stop // 32)
+        seg = s.segment(attr)
         mine = full[seg].clone()
         dist.all_gather_into_tensor(full, mine, group=self.group)
 
@@ -171,6 +206,45 @@ class GpuBackend:
                   "finish")
         return out[: sh.v1 - sh.v0]
 
+    # ---- MM
+    def decompose(self, sh: Shard, param: int, seed: int):
+        """Local RAND decomposition of the owned rows -> (intra, cross) PhaseViews."""
+        g = sh.c_struct()
+        dev = sh.row_ptr.device
+        nl, nnz = sh.v1 - sh.v0, sh.col_idx.numel()
+        nbytes = self.lib.sym_shard_decompose_workspace_bytes(ctypes.byref(g))
+        ws = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=dev)
+        rp_in = torch.empty(nl + 1, dtype=torch.int64, device=dev)
+        rp_x = torch.empty(nl + 1, dtype=torch.int64, device=dev)
+        ci_in = torch.empty(max(nnz, 1), dtype=torch.int32, device=dev)
+        ci_x = torch.empty(max(nnz, 1), dtype=torch.int32, device=dev)
+        p = L.SymParams(L.RAND, int(param), seed & (2**64 - 1), 0, 0)
+        self._chk(self.lib.sym_shard_decompose(ctypes.byref(g), ctypes.byref(p), ws.data_ptr(), ws.numel(),
+                                               rp_in.data_ptr(), ci_in.data_ptr(), rp_x.data_ptr(), ci_x.data_ptr(),
+                                               self._s(sh)), "decompose")
+        n_in = int(rp_in[-1])
+        return PhaseView(sh, rp_in, ci_in, n_in), PhaseView(sh, rp_x, ci_x, nnz - n_in)
+
+    def mm_frontier(self, view: PhaseView):
+        sh = view.shard
+        g = view.c_struct()
+        self._chk(self.lib.sym_shard_mm_frontier(ctypes.byref(g), sh.mate.data_ptr(), sh.cur.data_ptr(),
+                                                 sh.cur_cnt.data_ptr(), self._s(sh)), "mm_frontier")
+
+    def mm_round(self, view: PhaseView, seed: int, r: int):
+        sh = view.shard
+        g = view.c_struct()
+        if sh.extra.get("mm_ws") is None:
+            nbytes = self.lib.sym_shard_mm_workspace_bytes(ctypes.byref(sh.c_struct()))
+            sh.extra["mm_ws"] = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=sh.row_ptr.device)
+        ws = sh.extra["mm_ws"]
+        p = L.SymParams(L.NONE, 0, seed & (2**64 - 1), 0, 0)
+        self._chk(self.lib.sym_shard_mm_round(ctypes.byref(g), ctypes.byref(p), r, sh.mate.data_ptr(),
+                                              sh.picks[(r + 1) & 1].data_ptr(), sh.picks[r & 1].data_ptr(),
+                                              sh.cur.data_ptr(), sh.cur_cnt.data_ptr(), sh.nxt.data_ptr(),
+                                              sh.nxt_cnt.data_ptr(), ws.data_ptr(), ws.numel(), self._s(sh)),
+                  "mm_round")
+
 
 # ------------------------------------------------------------------ the flow
 def sym_mis_sharded(shards, kind="none", param=0, seed=42, transport=None, backend=None, stats=None):
@@ -216,6 +290,46 @@ def sym_mis_sharded(shards, kind="none", param=0, seed=42, transport=None, backe
     if stats is not None:
         stats["rounds"] = rounds
     return [backend.finish(s) for s in shards]
+
+
+def sym_mm_sharded(shards, kind="none", param=0, seed=42, transport=None, backend=None, stats=None):
+    """MM-NONE / MM-Rand over the given shards.  Returns the owned mate (int32, -1 =
+    unmatched) of every shard, in the order given."""
+    kind = {"none": L.NONE, "rand": L.RAND}.get(kind, kind) if isinstance(kind, str) else int(kind)
+    if kind not in (L.NONE, L.RAND):
+        raise ValueError("sharded MM supports the NONE and RAND decompositions")
+    transport = transport or LocalTransport()
+    backend = backend or GpuBackend()
+    for s in shards:
+        s.init_mm()
+    if kind == L.RAND:
+        views = [backend.decompose(s, int(param), seed) for s in shards]  # per shard: (intra, cross)
+        phases = [[v[0] for v in views], [v[1] for v in views]]
+    else:
+        phases = [[PhaseView(s, s.row_ptr, s.col_idx, s.col_idx.numel()) for s in shards]]
+    rounds = []
+    for pv in phases:
+        for v in pv:
+            backend.mm_frontier(v)
+        r = 0
+        while True:
+            for v in pv:
+                backend.mm_round(v, seed, r)
+            for s in shards:
+                s.pick_cur = s.picks[r & 1]
+            transport.allgather(shards, "pick_cur")
+            transport.allgather(shards, "mate")
+            r += 1
+            left = transport.allreduce_sum(shards, "nxt_cnt")
+            for s in shards:
+                s.cur, s.nxt = s.nxt, s.cur
+                s.cur_cnt, s.nxt_cnt = s.nxt_cnt, s.cur_cnt
+            if left == 0:
+                break
+        rounds.append(r)
+    if stats is not None:
+        stats["rounds"] = rounds
+    return [s.mate[s.v0:s.v1].clone() for s in shards]
 
 
 def make_shards(row_ptr, col_idx, nranks, ranks=None):
