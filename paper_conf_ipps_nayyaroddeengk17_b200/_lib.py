@@ -8,7 +8,7 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libsym.so")
+LIB_PATH = os.environ.get("SYM_LIB") or os.path.join(HERE, "libsym.so")  # SYM_LIB: diagnostic builds
 
 SYM_OK, SYM_EINVAL, SYM_EWORKSPACE, SYM_EGRAPH, SYM_ECUDA, SYM_ENCCL, SYM_EROUNDS = range(7)
 NONE, RAND, DEGK = 0, 1, 2

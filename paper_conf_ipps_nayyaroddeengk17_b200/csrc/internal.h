@@ -161,14 +161,15 @@ struct MmWs {
 };
 
 struct ColorWs {
-    uint32_t *cnt = nullptr;       // pending higher-priority neighbours
-    uint32_t *bits = nullptr;      // forbidden-colour bitmaps, (deg+1) bits per vertex
+    uint8_t *rec = nullptr;        // 32-B per-vertex records (count, degree, row, colours 1..128)
+    uint32_t *bits = nullptr;      // overflow forbidden-colour bitmaps, (deg+1) bits per vertex
     int64_t bits_words = 0;
-    int32_t *queue = nullptr;      // deferred long rows of the init pass
+    int64_t *queue = nullptr;      // init pass: (piece << 32 | v) items of the huge rows
     int32_t *vlist = nullptr;
     uint8_t *mark = nullptr;       // COLOR-RAND V'
     int64_t *task = nullptr;       // two task lists (ping-pong), queue_cap each
     int64_t queue_cap = 0;
+    uint32_t *sync = nullptr;      // levels kernel: barrier / error / level-count words
 };
 
 int phase_arcs(const FlowArgs &f, const int64_t *rp, int64_t *out);  // round0.cu

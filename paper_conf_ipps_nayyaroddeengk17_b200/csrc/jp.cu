@@ -1,38 +1,58 @@
-// color.cu -- Jones-Plassmann colouring and the COLOR flows.
+// jp.cu -- Jones-Plassmann colouring and the COLOR flows.
 //
 // JP ([18]) with fixed priorities colours v once every higher-(pv,id)
 // neighbour of its phase set S is coloured, with the smallest colour >= 1 not held by
 // any coloured neighbour: exactly first-fit greedy in priority order (DESIGN §3 C1).
 //
-// Push form with forbidden-colour bitmaps (the FORBIDDEN array of P:214/P:234, sized
-// deg(v)+1 bits per vertex since mex <= deg+1; bit offset row_ptr[v] + v):
-//   init   cnt[v] = #higher S-neighbours; fixed colours of neighbours outside S
-//          (COLOR-Rand recolouring) are pre-set in v's bitmap; cnt == 0 -> ready
-//          (a ready vertex without phase arcs takes colour 1 at once).
-//   round  every ready vertex v is split into tasks of <= JP_CHUNK arcs that carry
-//          v's row bounds.  A task computes colour(v) = first zero bit of v's bitmap
-//          (complete: all higher neighbours pushed in earlier rounds), and for each
-//          lower S-neighbour w of its chunk sets bit colour(v) in w's bitmap and
-//          decrements cnt[w]; the decrement reaching 0 appends w's tasks for the
-//          next round.  Rows <= JP_LANE arcs are handled by one lane, longer chunks
-//          by a warp; consecutive task indices go to different warps so the chunks
-//          of one hub run in parallel.
-// The dependent chain per round is: task -> (arcs | bitmap) -> (row bounds of w |
-// decrement) -> reservation; each arc is read twice in total (init + push).
-// Rounds = the JP dependency depth (~5e3 on R-MAT scale 24), so a round is latency-
-// bound: one kernel per round on a short grid.
+// Push form with forbidden-colour sets (the FORBIDDEN array of P:214/P:234):
+//   record  every S vertex owns one 32-byte record {cnt, deg, row start, bits of the
+//           colours 1..JP_WIN}: a push to w touches ONE sector and needs no row-pointer
+//           load.  Colours > JP_WIN (the dense core only: ~1 % of pushes at R-MAT s24)
+//           go to an overflow bitmap addressed by the row (bit offset row_ptr[w] + w,
+//           deg+1 bits, since mex <= deg+1).
+//   init    cnt[v] = #higher S-neighbours; fixed colours of neighbours outside S
+//           (COLOR-Rand recolouring) are pre-set; cnt == 0 -> ready (a ready vertex
+//           without phase arcs takes colour 1 at once).
+//   level   every ready vertex v is split into tasks of <= JP_CHUNK arcs that carry
+//           v's row bounds.  A task computes colour(v) = mex of v's forbidden set
+//           (complete: every higher neighbour pushed in an earlier level) and, for
+//           each lower S-neighbour w of its chunk, decrements cnt[w] and sets bit
+//           colour(v) of w; the decrement reaching 0 appends w's tasks for the next
+//           level.  Rows <= JP_LANE arcs are one lane's task, longer chunks a warp's.
+// Levels = the JP dependency depth (~5e3 on R-MAT scale 24); each level is a burst of
+// ~5e4 scattered pushes, so the cost per level is the latency of that burst plus one
+// grid barrier: all levels run inside ONE persistent cooperative kernel (k_jp_levels)
+// with a software grid barrier between levels.
+#include <cstdio>
 #include <cstdlib>
 
 #include "internal.h"
 
 namespace sym {
 
-constexpr int JP_SMALL = 32;
-constexpr int JP_BUDGET = 4096;
+constexpr int JP_SMALL = 32;     // init: rows <= JP_SMALL arcs are counted by one lane
+constexpr int JP_BUDGET = 4096;  // init: rows > JP_BUDGET arcs are split into pieces
 constexpr int JP_THREADS = 256;
 constexpr int JP_HUGE_THREADS = 512;
-constexpr int JP_CHUNK = 256;  // arcs per warp task (8 per lane)
-constexpr int JP_LANE = 8;     // rows with <= JP_LANE arcs are a lane task
+#ifndef SYM_JP_CHUNK
+#define SYM_JP_CHUNK 64
+#endif
+constexpr int JP_CHUNK = SYM_JP_CHUNK;  // arcs per warp task (2 per lane: few pushes in flight per warp)
+constexpr int JP_LANE = 8;              // rows with <= JP_LANE arcs are a lane task
+constexpr int JP_PIECE = 8192;          // arcs per CTA piece of a huge row in the init pass
+constexpr uint32_t JP_WIN = 128;        // colours held in the record
+#ifndef JP_LDCI
+#define JP_LDCI __ldcs  // column loads: streaming, so the hot records stay in L2
+#endif
+
+// per-vertex record (one 32-byte sector)
+struct __align__(32) JpRec {
+    uint32_t cnt;       // higher S-neighbours not yet coloured
+    uint32_t deg;       // phase degree
+    int64_t b;          // row_ptr[v] of the phase CSR
+    uint32_t win[4];    // forbidden colours 1..JP_WIN
+};
+static_assert(sizeof(JpRec) == 32, "JpRec layout");
 
 // a task: one chunk of a ready vertex's row, with the row bounds
 struct __align__(16) JpTask {
@@ -48,8 +68,8 @@ struct JpArgs {
     const int32_t *ci;
     const uint8_t *inS;  // nullable: S = all vertices
     uint32_t *color;
-    uint32_t *cnt;
-    uint32_t *bits;      // forbidden-colour bitmaps
+    JpRec *rec;
+    uint32_t *bits;      // overflow bitmaps (colours > JP_WIN)
     const int32_t *in_list;    // init: vertex list (nullable = implicit)
     const uint32_t *in_cnt;
     int64_t implicit_n;
@@ -57,13 +77,18 @@ struct JpArgs {
     JpTask *tout;
     uint32_t *out_cnt;
     uint32_t *clear_cnt;
-    int32_t *huge;
+    int64_t *huge;        // init: (piece << 32 | v) items of the huge rows
     uint32_t *huge_cnt;
-    uint32_t *huge_clear;
     uint32_t *hist;
     int round;
     Key k;
 };
+
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
 
 __device__ __forceinline__ bool in_set(const uint8_t *inS, uint32_t w) { return inS == nullptr || inS[w] != 0; }
 
@@ -101,65 +126,88 @@ __device__ __forceinline__ int64_t warp_reserve(uint32_t k_lane, uint32_t *count
     return (int64_t)base + incl - k_lane;
 }
 
-__device__ __forceinline__ void set_forbidden(uint32_t *bits, int64_t B, int64_t nbits, uint32_t c) {
-    if (c >= 1 && (int64_t)c <= nbits) {
-        int64_t pos = B + c - 1;
+// overflow bit of colour c (> JP_WIN) in the bitmap of a vertex with row start b, degree d
+__device__ __forceinline__ void set_overflow(uint32_t *bits, int64_t b, int32_t v, uint32_t d, uint32_t c) {
+    if (c <= d + 1) {
+        const int64_t pos = b + v + c - 1;
         atomicOr(bits + (pos >> 5), 1u << (pos & 31));
     }
 }
 
-// first zero bit of bits[B, B+nbits) -> mex (1-based); warp-cooperative
-__device__ __forceinline__ uint32_t warp_mex(const uint32_t *bits, int64_t B, int64_t nbits) {
+// colour c is forbidden for v (window bits accumulated by the caller; overflow direct)
+__device__ __forceinline__ void note_colour(uint32_t (&win)[4], uint32_t *bits, int64_t b, int32_t v, uint32_t d,
+                                            uint32_t c) {
+    if (c == 0) return;
+    if (c <= JP_WIN) win[(c - 1) >> 5] |= 1u << ((c - 1) & 31);
+    else set_overflow(bits, b, v, d, c);
+}
+
+__device__ __forceinline__ void store_rec(JpRec *r, uint32_t cnt, uint32_t deg, int64_t b, const uint32_t (&win)[4]) {
+    uint4 *p = reinterpret_cast<uint4 *>(r);
+    p[0] = make_uint4(cnt, deg, (uint32_t)(uint64_t)b, (uint32_t)((uint64_t)b >> 32));
+    p[1] = make_uint4(win[0], win[1], win[2], win[3]);
+}
+
+// mex of v's forbidden set (colours 1..deg+1), warp-cooperative: window first, then
+// the overflow bitmap from colour JP_WIN+1
+__device__ __forceinline__ uint32_t warp_mex(const JpRec *r, const uint32_t *bits, int64_t B, uint32_t deg) {
     const int lane = lane_id();
+    const uint32_t nbits = deg + 1;
+    {
+        const uint4 wv = __ldcg(reinterpret_cast<const uint4 *>(r) + 1);
+        const uint32_t wd[4] = {wv.x, wv.y, wv.z, wv.w};
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            const uint32_t lo = 32u * q;
+            if (lo >= nbits) break;
+            const uint32_t width = min(32u, nbits - lo);
+            const uint32_t z = ~wd[q] & (width >= 32 ? 0xffffffffu : ((1u << width) - 1u));
+            if (z) return lo + __ffs(z);
+        }
+    }
+    // overflow: bit positions B + JP_WIN .. B + nbits - 1 (colour = position - B + 1)
     const int64_t end = B + nbits;
-    const int64_t w0 = B >> 5, w1 = (end - 1) >> 5;
+    const int64_t w0 = (B + JP_WIN) >> 5, w1 = (end - 1) >> 5;
     for (int64_t k0 = w0; k0 <= w1; k0 += 32) {
-        int64_t wi = k0 + lane;
+        const int64_t wi = k0 + lane;
         uint32_t zeros = 0;
         if (wi <= w1) {
-            uint32_t word = __ldcg(bits + wi);
-            int64_t lo = max(B, wi * 32) - wi * 32, hi = min(end, wi * 32 + 32) - wi * 32;
-            uint32_t width = (uint32_t)(hi - lo);
-            uint32_t mask = (width >= 32 ? 0xffffffffu : ((1u << width) - 1u)) << lo;
+            const uint32_t word = __ldcg(bits + wi);
+            const int64_t lo = max(B + (int64_t)JP_WIN, wi * 32) - wi * 32, hi = min(end, wi * 32 + 32) - wi * 32;
+            const uint32_t width = (uint32_t)(hi - lo);
+            const uint32_t mask = (width >= 32 ? 0xffffffffu : ((1u << width) - 1u)) << lo;
             zeros = ~word & mask;
         }
-        unsigned bal = __ballot_sync(FULL, zeros != 0);
+        const unsigned bal = __ballot_sync(FULL, zeros != 0);
         if (bal) {
-            int src = __ffs(bal) - 1;
-            uint32_t z = __shfl_sync(FULL, zeros, src);
-            int64_t pos = (k0 + src) * 32 + __ffs(z) - 1;
+            const int src = __ffs(bal) - 1;
+            const uint32_t z = __shfl_sync(FULL, zeros, src);
+            const int64_t pos = (k0 + src) * 32 + __ffs(z) - 1;
             return (uint32_t)(pos - B + 1);
         }
     }
-    return (uint32_t)nbits;  // unreachable: at most nbits-1 bits can be set
+    return nbits;  // unreachable: at most deg bits can be set
 }
 
-// mex of a short bitmap (nbits <= 33) by one lane
-__device__ __forceinline__ uint32_t lane_mex(const uint32_t *bits, int64_t B, int64_t nbits) {
-    const int64_t w0 = B >> 5;
-    const uint64_t lo = __ldcg(bits + w0), hi = __ldcg(bits + w0 + 1);
-    const uint64_t word = (lo | (hi << 32)) >> (B & 31);
-    const uint64_t valid = nbits >= 64 ? ~0ULL : ((1ULL << nbits) - 1ULL);
-    return (uint32_t)__ffsll((long long)(~word & valid));
+// mex of a short row (deg <= JP_LANE < 32): window word 0 only
+__device__ __forceinline__ uint32_t lane_mex(const JpRec *r, uint32_t deg) {
+    const uint32_t w0 = __ldcg(&r->win[0]);
+    return (uint32_t)__ffs(~w0 & ((1u << (deg + 1)) - 1u));
 }
 
 // ---------------------------------------------------------------- init
-// cnt[v] = #higher S-neighbours; pre-set fixed colours of non-S neighbours; ready
-// vertices enqueue their tasks for round 0.
+// record of every S vertex: cnt = #higher S-neighbours, fixed colours of non-S
+// neighbours; ready vertices enqueue their level-0 tasks; huge rows are deferred
 __global__ void __launch_bounds__(JP_THREADS) k_jp_init(JpArgs A) {
     const uint32_t cnt = A.in_list ? *A.in_cnt : (uint32_t)A.implicit_n;
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        *A.clear_cnt = 0;
-        *A.huge_clear = 0;
-    }
     const int lane = lane_id();
     const int64_t warp_g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t base = warp_g * 32; base < cnt; base += nwarps * 32) {
-        int64_t i = base + lane;
+        const int64_t i = base + lane;
         int32_t v = -1;
         if (i < cnt) v = A.in_list ? A.in_list[i] : (int32_t)i;
-        bool active = v >= 0;
+        const bool active = v >= 0;
         int64_t b = 0, e = 0;
         uint64_t kv = 0;
         if (active) {
@@ -167,12 +215,14 @@ __global__ void __launch_bounds__(JP_THREADS) k_jp_init(JpArgs A) {
             e = A.rp[v + 1];
             kv = vkey(A.k, (uint32_t)v);
         }
+        const uint32_t deg = (uint32_t)(e - b);
         uint32_t c = 0;
+        uint32_t win[4] = {0u, 0u, 0u, 0u};
         if (active && e - b <= JP_SMALL) {
             for (int64_t x = b; x < e; x++) {
-                uint32_t w = (uint32_t)__ldg(A.ci + x);
+                const uint32_t w = (uint32_t)__ldg(A.ci + x);
                 if (in_set(A.inS, w)) c += vkey(A.k, w) > kv ? 1u : 0u;
-                else set_forbidden(A.bits, b + v, e - b + 1, A.color[w]);
+                else note_colour(win, A.bits, b, v, deg, A.color[w]);
             }
         }
         unsigned medm = __ballot_sync(FULL, active && e - b > JP_SMALL && e - b <= JP_BUDGET);
@@ -183,121 +233,216 @@ __global__ void __launch_bounds__(JP_THREADS) k_jp_init(JpArgs A) {
             const uint64_t wk = __shfl_sync(FULL, kv, src);
             const int32_t wv = __shfl_sync(FULL, v, src);
             uint32_t lc = 0;
+            uint32_t lw[4] = {0u, 0u, 0u, 0u};
             for (int64_t x = wb + lane; x < we; x += 32) {
-                uint32_t w = (uint32_t)__ldg(A.ci + x);
+                const uint32_t w = (uint32_t)__ldg(A.ci + x);
                 if (in_set(A.inS, w)) lc += vkey(A.k, w) > wk ? 1u : 0u;
-                else set_forbidden(A.bits, wb + wv, we - wb + 1, A.color[w]);
+                else note_colour(lw, A.bits, wb, wv, (uint32_t)(we - wb), A.color[w]);
             }
-            for (int d = 16; d; d >>= 1) lc += __shfl_xor_sync(FULL, lc, d);
-            if (lane == src) c = lc;
+            lc = __reduce_add_sync(FULL, lc);
+#pragma unroll
+            for (int q = 0; q < 4; q++) lw[q] = __reduce_or_sync(FULL, lw[q]);
+            if (lane == src) {
+                c = lc;
+#pragma unroll
+                for (int q = 0; q < 4; q++) win[q] = lw[q];
+            }
         }
-        bool huge = active && e - b > JP_BUDGET;
-        if (active && !huge) A.cnt[v] = c;
+        const bool huge = active && e - b > JP_BUDGET;
+        if (active) store_rec(A.rec + v, huge ? 0u : c, deg, b, win);
         bool ready = active && !huge && c == 0;
         if (ready && e == b) {  // no phase neighbour: colour 1 now, no task
             A.color[v] = 1u;
             ready = false;
         }
-        uint32_t nt = ready ? n_tasks(e - b) : 0u;
-        int64_t slot = warp_reserve(nt, A.out_cnt);
+        const uint32_t nt = ready ? n_tasks(e - b) : 0u;
+        const int64_t slot = warp_reserve(nt, A.out_cnt);
         put_tasks(A.tout, slot, v, b, e, nt);
-        int64_t hs = warp_append(huge, A.huge_cnt);
-        if (hs >= 0) A.huge[hs] = v;
+        // huge rows: one (v, piece) entry per JP_PIECE arcs, counted by k_jp_init_huge
+        const uint32_t np = huge ? (uint32_t)((e - b + JP_PIECE - 1) / JP_PIECE) : 0u;
+        const int64_t ps = warp_reserve(np, A.huge_cnt);
+        for (uint32_t q = 0; q < np; q++) A.huge[ps + q] = ((int64_t)q << 32) | (uint32_t)v;
     }
 }
 
+// counts of the huge rows, one CTA per JP_PIECE-arc piece (a 4e5-arc hub is spread
+// over ~50 CTAs instead of serialising one CTA)
 __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jp_init_huge(JpArgs A) {
     const uint32_t cnt = *A.huge_cnt;
-    __shared__ uint32_t s_sum;
-    __shared__ int64_t s_slot;
     for (uint32_t h = blockIdx.x; h < cnt; h += gridDim.x) {
-        const int32_t v = A.huge[h];
+        const int64_t item = A.huge[h];
+        const int32_t v = (int32_t)(uint32_t)item;
+        const int64_t j = item >> 32;
         const int64_t b = A.rp[v], e = A.rp[v + 1];
+        const uint32_t deg = (uint32_t)(e - b);
+        const int64_t pb = b + j * JP_PIECE, pe_ = min(e, pb + JP_PIECE);
         const uint64_t kv = vkey(A.k, (uint32_t)v);
-        if (threadIdx.x == 0) s_sum = 0;
-        __syncthreads();
         uint32_t lc = 0;
-        for (int64_t x = b + threadIdx.x; x < e; x += JP_HUGE_THREADS) {
-            uint32_t w = (uint32_t)__ldg(A.ci + x);
+        uint32_t lw[4] = {0u, 0u, 0u, 0u};
+        for (int64_t x = pb + threadIdx.x; x < pe_; x += JP_HUGE_THREADS) {
+            const uint32_t w = (uint32_t)__ldg(A.ci + x);
             if (in_set(A.inS, w)) lc += vkey(A.k, w) > kv ? 1u : 0u;
-            else set_forbidden(A.bits, b + v, e - b + 1, A.color[w]);
+            else note_colour(lw, A.bits, b, v, deg, A.color[w]);
         }
-        for (int d = 16; d; d >>= 1) lc += __shfl_xor_sync(FULL, lc, d);
-        if (lane_id() == 0) atomicAdd(&s_sum, lc);
-        __syncthreads();
+        lc = __reduce_add_sync(FULL, lc);
+#pragma unroll
+        for (int q = 0; q < 4; q++) lw[q] = __reduce_or_sync(FULL, lw[q]);
+        if (lane_id() == 0) {
+            if (lc) atomicAdd(&A.rec[v].cnt, lc);
+#pragma unroll
+            for (int q = 0; q < 4; q++)
+                if (lw[q]) atomicOr(&A.rec[v].win[q], lw[q]);
+        }
+    }
+}
+
+// huge rows whose count is 0 are ready for level 0
+__global__ void k_jp_huge_ready(JpArgs A) {
+    const uint32_t cnt = *A.huge_cnt;
+    for (uint32_t h = blockIdx.x * blockDim.x + threadIdx.x; h < cnt; h += gridDim.x * blockDim.x) {
+        const int64_t item = A.huge[h];
+        if ((item >> 32) != 0) continue;
+        const int32_t v = (int32_t)(uint32_t)item;
+        if (A.rec[v].cnt != 0) continue;
+        const int64_t b = A.rp[v], e = A.rp[v + 1];
         const uint32_t nt = n_tasks(e - b);
-        if (threadIdx.x == 0) {
-            A.cnt[v] = s_sum;
-            s_slot = (s_sum == 0) ? (int64_t)atomicAdd(A.out_cnt, nt) : -1;
+        const int64_t slot = atomicAdd(A.out_cnt, nt);
+        put_tasks(A.tout, slot, v, b, e, nt);
+    }
+}
+
+// ---------------------------------------------------------------- one level
+// Ready vertices found during a level are staged in shared memory and appended to the
+// next task list once per CTA (one global reservation per CTA and level, tasks of a
+// hub written by the whole CTA); a full stage falls back to a per-lane append.
+constexpr int JP_STAGE = 1024;
+
+struct JpStage {
+    uint32_t n;                  // entries appended this level (may exceed JP_STAGE)
+    uint32_t base;               // global slot of the CTA's first task
+    uint32_t total;              // tasks of the staged entries
+    uint32_t wsum[32];           // scan scratch (one per warp)
+    int32_t v[JP_STAGE];
+    uint32_t deg[JP_STAGE];
+    int64_t b[JP_STAGE];
+    uint32_t off[JP_STAGE + 1];  // exclusive prefix of the task counts
+};
+
+__device__ __forceinline__ void stage_ready(const JpArgs &A, JpStage &st, int32_t w, int64_t b, uint32_t deg) {
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(A.ci + b));  // the row is read next level
+    const uint32_t slot = atomicAdd(&st.n, 1u);
+    if (slot < JP_STAGE) {
+        st.v[slot] = w;
+        st.deg[slot] = deg;
+        st.b[slot] = b;
+    } else {
+        const uint32_t nt = n_tasks(deg);
+        put_tasks(A.tout, atomicAdd(A.out_cnt, nt), w, b, b + deg, nt);
+    }
+}
+
+// CTA-wide: reserve the staged entries' tasks with one global atomic and write them
+__device__ __forceinline__ void stage_flush(const JpArgs &A, JpStage &st) {
+    __syncthreads();
+    const uint32_t n = min(st.n, (uint32_t)JP_STAGE);
+    const uint32_t per = (JP_STAGE + blockDim.x - 1) / blockDim.x;
+    const uint32_t i0 = threadIdx.x * per;
+    uint32_t loc = 0;
+    for (uint32_t i = i0; i < min(n, i0 + per); i++) loc += n_tasks(st.deg[i]);
+    // block exclusive scan of loc
+    uint32_t incl = loc;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, d);
+        if (lane_id() >= d) incl += y;
+    }
+    const int wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    if (lane_id() == 31) st.wsum[wid] = incl;
+    __syncthreads();
+    if (wid == 0) {
+        uint32_t x = lane_id() < nw ? st.wsum[lane_id()] : 0u, xi = x;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(FULL, xi, d);
+            if (lane_id() >= d) xi += y;
         }
-        __syncthreads();
-        if (s_slot >= 0)
-            for (uint32_t q = threadIdx.x; q < nt; q += JP_HUGE_THREADS) {
-                JpTask t;
-                t.b = b;
-                t.e = e;
-                t.v = v;
-                t.j = q;
-                t.pad = 0;
-                A.tout[s_slot + q] = t;
+        if (lane_id() < nw) st.wsum[lane_id()] = xi - x;
+        if (lane_id() == 31) {
+            st.total = xi;
+            st.base = xi ? atomicAdd(A.out_cnt, xi) : 0u;
+        }
+    }
+    __syncthreads();
+    uint32_t o = st.wsum[wid] + incl - loc;
+    for (uint32_t i = i0; i < min(n, i0 + per); i++) {
+        st.off[i] = o;
+        o += n_tasks(st.deg[i]);
+    }
+    if (threadIdx.x == 0) st.off[n] = st.total;
+    __syncthreads();
+    const uint32_t total = st.total, base = st.base;
+    for (uint32_t q = threadIdx.x; q < total; q += blockDim.x) {
+        uint32_t lo = 0, hi = n - 1;  // last entry with off <= q
+        while (lo < hi) {
+            const uint32_t mid = (lo + hi + 1) >> 1;
+            if (st.off[mid] <= q) lo = mid;
+            else hi = mid - 1;
+        }
+        JpTask t;
+        t.b = st.b[lo];
+        t.e = st.b[lo] + st.deg[lo];
+        t.v = st.v[lo];
+        t.j = q - st.off[lo];
+        t.pad = 0;
+        A.tout[base + q] = t;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) st.n = 0;
+}
+
+// Decrement the counts of the lower S-neighbours w[0..U) (flags low[]); returns the
+// previous counts (1 = the push that makes w ready)
+template <int U>
+__device__ __forceinline__ void jp_decrement(const JpArgs &A, const uint32_t (&w)[U], const bool (&low)[U],
+                                             uint32_t (&old)[U]) {
+#pragma unroll
+    for (int u = 0; u < U; u++) old[u] = low[u] ? atomicSub(&A.rec[w[u]].cnt, 1u) : 0u;
+}
+
+// forbidden bit of colour c for the lower S-neighbours (fire-and-forget), then the
+// records of the vertices that became ready go to the stage
+template <int U>
+__device__ __forceinline__ void jp_mark(const JpArgs &A, JpStage &st, const uint32_t (&w)[U], const bool (&low)[U],
+                                        const uint32_t (&old)[U], uint32_t c) {
+    if (c <= JP_WIN) {
+        const uint32_t q = (c - 1) >> 5, bit = 1u << ((c - 1) & 31);
+#pragma unroll
+        for (int u = 0; u < U; u++)
+            if (low[u]) atomicOr(&A.rec[w[u]].win[q], bit);
+    } else {  // dense core: the overflow bitmap needs the row of w
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            if (low[u]) {
+                const uint4 h = __ldcg(reinterpret_cast<const uint4 *>(A.rec + w[u]));
+                set_overflow(A.bits, (int64_t)(((uint64_t)h.w << 32) | h.z), (int32_t)w[u], h.y, c);
             }
-        __syncthreads();
-    }
-}
-
-// ---------------------------------------------------------------- push rounds
-// Push the colour c of a vertex to the lower S-neighbours w[0..U) (flags in low[]):
-// the row bounds of w and the decrement are issued together, then the bitmap bit.
-template <int U>
-__device__ __forceinline__ uint32_t jp_push_arcs(const JpArgs &A, const uint32_t (&w)[U], bool (&low)[U], uint32_t c,
-                                                 int64_t (&wb)[U], int64_t (&we)[U]) {
-    uint32_t old[U];
-#pragma unroll
-    for (int u = 0; u < U; u++) {
-        if (low[u]) {
-            wb[u] = A.rp[w[u]];
-            we[u] = A.rp[w[u] + 1];
-            old[u] = atomicSub(A.cnt + w[u], 1u);
         }
     }
-    uint32_t ready = 0;
 #pragma unroll
     for (int u = 0; u < U; u++) {
-        if (low[u]) {
-            set_forbidden(A.bits, wb[u] + w[u], we[u] - wb[u] + 1, c);
-            if (old[u] == 1u) ready |= 1u << u;
-        }
-    }
-    return ready;
-}
-
-template <int U>
-__device__ __forceinline__ void jp_enqueue(const JpArgs &A, const uint32_t (&w)[U], uint32_t ready,
-                                           const int64_t (&wb)[U], const int64_t (&we)[U]) {
-    uint32_t nt = 0;
-#pragma unroll
-    for (int u = 0; u < U; u++)
-        if ((ready >> u) & 1u) nt += n_tasks(we[u] - wb[u]);
-    int64_t slot = warp_reserve(nt, A.out_cnt);
-#pragma unroll
-    for (int u = 0; u < U; u++) {
-        if ((ready >> u) & 1u) {
-            uint32_t k = n_tasks(we[u] - wb[u]);
-            put_tasks(A.tout, slot, (int32_t)w[u], wb[u], we[u], k);
-            slot += k;
+        if (low[u] && old[u] == 1u) {
+            const uint4 h = __ldcg(reinterpret_cast<const uint4 *>(A.rec + w[u]));
+            stage_ready(A, st, (int32_t)w[u], (int64_t)(((uint64_t)h.w << 32) | h.z), h.y);
         }
     }
 }
 
-__global__ void __launch_bounds__(JP_THREADS) k_jp_push(JpArgs A) {
-    const uint32_t cnt = *A.in_cnt;
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        *A.clear_cnt = 0;
-        if (A.hist && A.round < 2048) A.hist[A.round] = cnt;
-    }
+// One level of push JP: every task of tin[0, cnt) colours its vertex (the first chunk
+// writes the colour) and pushes it to the lower S-neighbours of its chunk; vertices
+// whose count reaches 0 are appended to A.tout (counter A.out_cnt).  CTA-wide.
+__device__ __forceinline__ void jp_level(const JpArgs &A, JpStage &st, uint32_t cnt, const JpTask *tin,
+                                         int64_t warp_g, int64_t nwarps) {
     const int lane = lane_id();
-    const int64_t warp_g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     // task index t = it*32*nwarps + lane*nwarps + warp: consecutive tasks (the chunks
     // of one hub) land on different warps
     for (int64_t base = warp_g; base - warp_g < cnt; base += nwarps * 32) {
@@ -306,8 +451,8 @@ __global__ void __launch_bounds__(JP_THREADS) k_jp_push(JpArgs A) {
         uint32_t j = 0;
         int64_t b = 0, e = 0;
         if (t < cnt) {
-            const longlong2 *p = reinterpret_cast<const longlong2 *>(A.tin + t);
-            longlong2 q0 = __ldcg(p), q1 = __ldcg(p + 1);
+            const longlong2 *p = reinterpret_cast<const longlong2 *>(tin + t);
+            const longlong2 q0 = __ldcg(p), q1 = __ldcg(p + 1);
             b = q0.x;
             e = q0.y;
             v = (int32_t)(uint32_t)q1.x;
@@ -316,24 +461,24 @@ __global__ void __launch_bounds__(JP_THREADS) k_jp_push(JpArgs A) {
         const uint64_t kv = v >= 0 ? vkey(A.k, (uint32_t)v) : 0;
         // ---- short rows: one lane does the whole task
         const bool small = v >= 0 && e - b <= JP_LANE;
-        {
+        if (__any_sync(FULL, small)) {
             uint32_t w[JP_LANE];
             bool low[JP_LANE];
 #pragma unroll
             for (int u = 0; u < JP_LANE; u++) {
                 low[u] = small && b + u < e;
-                w[u] = low[u] ? (uint32_t)__ldg(A.ci + b + u) : 0u;
-            }
-            uint32_t c = 0;
-            if (small) {
-                c = lane_mex(A.bits, b + v, e - b + 1);
-                A.color[v] = c;
+                w[u] = low[u] ? (uint32_t)JP_LDCI(A.ci + b + u) : 0u;
             }
 #pragma unroll
             for (int u = 0; u < JP_LANE; u++) low[u] = low[u] && in_set(A.inS, w[u]) && vkey(A.k, w[u]) < kv;
-            int64_t wb[JP_LANE], we[JP_LANE];
-            uint32_t ready = jp_push_arcs<JP_LANE>(A, w, low, c, wb, we);
-            jp_enqueue<JP_LANE>(A, w, ready, wb, we);
+            uint32_t old[JP_LANE];
+            jp_decrement<JP_LANE>(A, w, low, old);
+            uint32_t c = 1;
+            if (small) {
+                c = lane_mex(A.rec + v, (uint32_t)(e - b));
+                A.color[v] = c;
+            }
+            jp_mark<JP_LANE>(A, st, w, low, old, c);
         }
         // ---- longer rows: the warp takes these tasks one by one (<= JP_CHUNK arcs)
         unsigned bigm = __ballot_sync(FULL, v >= 0 && !small);
@@ -350,19 +495,105 @@ __global__ void __launch_bounds__(JP_THREADS) k_jp_push(JpArgs A) {
             bool low[U];
 #pragma unroll
             for (int u = 0; u < U; u++) {
-                int64_t x = cb + u * 32 + lane;
+                const int64_t x = cb + u * 32 + lane;
                 low[u] = x < te;
-                w[u] = low[u] ? (uint32_t)__ldg(A.ci + x) : 0u;
+                w[u] = low[u] ? (uint32_t)JP_LDCI(A.ci + x) : 0u;
             }
-            const uint32_t c = warp_mex(A.bits, tb + tv, te - tb + 1);
-            if (tj == 0 && lane == 0) A.color[tv] = c;
 #pragma unroll
             for (int u = 0; u < U; u++) low[u] = low[u] && in_set(A.inS, w[u]) && vkey(A.k, w[u]) < tk;
-            int64_t wb[U], we[U];
-            uint32_t ready = jp_push_arcs<U>(A, w, low, c, wb, we);
-            jp_enqueue<U>(A, w, ready, wb, we);
+            uint32_t old[U];
+            jp_decrement<U>(A, w, low, old);  // the decrements do not wait for the mex
+            const uint32_t c = warp_mex(A.rec + tv, A.bits, tb + tv, (uint32_t)(te - tb));
+            if (tj == 0 && lane == 0) A.color[tv] = c;
+            jp_mark<U>(A, st, w, low, old, c);
         }
     }
+    stage_flush(A, st);
+}
+
+// host-driven level (fallback when cooperative launch is unavailable)
+__global__ void __launch_bounds__(JP_THREADS) k_jp_push(JpArgs A) {
+    __shared__ JpStage st;
+    if (threadIdx.x == 0) st.n = 0;
+    __syncthreads();
+    const uint32_t cnt = *A.in_cnt;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        *A.clear_cnt = 0;
+        if (A.hist && A.round < 1024) A.hist[A.round] = cnt;
+    }
+    const int64_t warp_g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    jp_level(A, st, cnt, A.tin, warp_g, nwarps);
+}
+
+// ---------------------------------------------------------------- persistent levels
+// All levels in ONE cooperative launch: a level is jp_level over the task list of the
+// previous level, then a software grid barrier (one arrival atomic per CTA on a
+// monotone counter that the CTAs poll).  The barrier orders the pushes of level r
+// before the mex reads of level r+1, so no per-push fence is needed.  Counters:
+// ring[r%3] = tasks of level r, ring[(r+1)%3] = tasks appended for level r+1,
+// ring[(r+2)%3] (read before the previous barrier) is cleared for level r+2.
+constexpr int JL_THREADS = 512;
+#ifndef SYM_JL_MINB
+#define SYM_JL_MINB 1
+#endif
+constexpr uint64_t JL_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
+
+struct JlCtl {
+    uint32_t *ring;    // [3]
+    uint32_t *bar;     // arrivals (monotone)
+    uint32_t *err;     // 1 = timeout / max levels
+    uint32_t *levels;  // out: number of levels run
+    JpTask *tq0, *tq1;
+    uint32_t max_levels;
+};
+
+__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *p) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// epoch = arrivals expected after this barrier (wrap-safe comparison)
+__device__ __forceinline__ void grid_barrier(const JlCtl &C, uint32_t &epoch) {
+    __syncthreads();
+    epoch += gridDim.x;
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(C.bar, 1u);
+        while ((int32_t)(ld_acquire_u32(C.bar) - epoch) < 0) {
+        }
+    }
+    __syncthreads();
+}
+
+__global__ void __launch_bounds__(JL_THREADS, SYM_JL_MINB) k_jp_levels(JpArgs A, JlCtl C) {
+    __shared__ JpStage st;
+    if (threadIdx.x == 0) st.n = 0;
+    __syncthreads();
+    // warp-in-CTA major: consecutive tasks (the chunks of one row) go to different SMs
+    const int64_t warp_g = (int64_t)(threadIdx.x >> 5) * gridDim.x + blockIdx.x;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    uint32_t epoch = 0;
+    const uint64_t t0 = globaltimer_ns();
+    uint32_t r = 0;
+    for (;; r++) {
+        const uint32_t cnt = __ldcg(C.ring + r % 3);
+        if (cnt == 0 || __ldcg(C.err) != 0) break;
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            C.ring[(r + 2) % 3] = 0;
+            if (A.hist && r < 1024) {  // stats: tasks and start time (32 ns units) of the first levels
+                A.hist[r] = cnt;
+                A.hist[1024 + r] = (uint32_t)((globaltimer_ns() - t0) >> 5);
+            }
+            if (r + 1 >= C.max_levels || globaltimer_ns() - t0 > JL_TIMEOUT_NS) atomicExch(C.err, 1u);
+        }
+        A.out_cnt = C.ring + (r + 1) % 3;
+        A.tout = (r & 1) ? C.tq0 : C.tq1;
+        jp_level(A, st, cnt, (r & 1) ? C.tq1 : C.tq0, warp_g, nwarps);
+        grid_barrier(C, epoch);
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) *C.levels = r;
 }
 
 // ---------------------------------------------------------------- fix-up kernels
@@ -415,339 +646,133 @@ __global__ void k_color_max(const uint32_t *color, int64_t n, uint32_t *mx) {
 
 // ---------------------------------------------------------------- host side
 void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
-    w.cnt = a.take<uint32_t>((size_t)n + 1);
+    w.rec = a.take<uint8_t>(((size_t)n + 1) * sizeof(JpRec));
     w.bits = a.take<uint32_t>((size_t)((nnz + n) / 32 + 2));
     w.bits_words = (nnz + n) / 32 + 2;
-    w.queue_cap = n + nnz / JP_CHUNK + 2;  // tasks in one round <= all tasks
+    w.queue_cap = n + nnz / JP_CHUNK + 2;  // tasks in one level <= all tasks
     w.task = a.take<int64_t>(2 * (size_t)w.queue_cap * (sizeof(JpTask) / sizeof(int64_t)));
     w.vlist = a.take<int32_t>((size_t)n + 1);
     w.mark = a.take<uint8_t>((size_t)n + 1);
-    w.queue = a.take<int32_t>((size_t)(nnz / JP_BUDGET + 2));  // deferred init rows
+    w.queue = a.take<int64_t>((size_t)(nnz / JP_BUDGET + 2));  // huge-row pieces (<= nnz/JP_BUDGET)
+    w.sync = a.take<uint32_t>(64);  // levels kernel: barrier words, apart from the task counters
 }
 
 // JP over (rp, ci) for the vertex set S (list/implicit) with membership inS; the
-// bitmap layout follows this CSR (offset rp[v] + v, deg+1 bits).
-// ---------------------------------------------------------------- asynchronous JP
-// No global rounds: a persistent grid of warps colours vertices as soon as they are
-// ready.  A lane that makes a short-row vertex (deg <= JP_LANE) ready colours it
-// itself next (per-lane continuation stack, no queue hop); longer rows are split into
-// JP_CHUNK-arc tasks appended to one global queue that idle warps claim.  Pushes set
-// the forbidden bit, fence, then decrement; the decrement that reaches 0 is followed
-// by a fence before the bitmap is read, so every higher neighbour's colour is seen.
-// Termination: an exact count of coloured vertices (flushed before a warp waits).
-// A warp waiting on an empty queue slot also watches the count, an error flag and a
-// %globaltimer deadline, so a bug cannot hang the device.
-constexpr int JA_STACK = 16;
-constexpr uint64_t JA_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
-
-struct JaArgs {
-    const int64_t *rp;
-    const int32_t *ci;
-    const uint8_t *inS;
-    uint32_t *color;
-    uint32_t *cnt;
-    uint32_t *bits;
-    JpTask *q;
-    int64_t qcap;
-    uint32_t *head, *tail, *done, *err;
-    const uint32_t *target;  // vertices to colour by tasks
-    Key k;
-};
-
-__device__ __forceinline__ uint64_t globaltimer_ns() {
-    uint64_t t;
-    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
-    return t;
-}
-
-__device__ __forceinline__ int32_t ld_volatile_i32(const int32_t *p) {
-    int32_t v;
-    asm volatile("ld.volatile.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-
-__device__ __forceinline__ void st_volatile_i32(int32_t *p, int32_t v) {
-    asm volatile("st.volatile.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
-// lane-level enqueue of all chunk tasks of vertex w (flag field v written last)
-__device__ __forceinline__ void ja_enqueue(const JaArgs &A, int32_t w, int64_t wb, int64_t we) {
-    const uint32_t nt = n_tasks(we - wb);
-    const uint32_t slot = atomicAdd(A.tail, nt);
-    for (uint32_t q = 0; q < nt; q++) {
-        JpTask *t = A.q + slot + q;
-        t->b = wb;
-        t->e = we;
-        t->j = q;
-    }
-    __threadfence();
-    for (uint32_t q = 0; q < nt; q++) st_volatile_i32(&A.q[slot + q].v, w);
-}
-
-struct JaStack {
-    int32_t v[JA_STACK];
-    int64_t b[JA_STACK], e[JA_STACK];
-    int sp;
-};
-
-__device__ __forceinline__ void ja_ready(const JaArgs &A, JaStack &st, int32_t w, int64_t wb, int64_t we) {
-    if (we - wb <= JP_LANE && st.sp < JA_STACK) {
-        st.v[st.sp] = w;
-        st.b[st.sp] = wb;
-        st.e[st.sp] = we;
-        st.sp++;
-    } else {
-        ja_enqueue(A, w, wb, we);
-    }
-}
-
-// colour a short-row vertex and push to its lower S-neighbours (one lane)
-__device__ __forceinline__ void ja_lane_vertex(const JaArgs &A, JaStack &st, int32_t v, int64_t b, int64_t e,
-                                               uint32_t &ncol) {
-    const uint64_t kv = vkey(A.k, (uint32_t)v);
-    __threadfence();  // acquire: the decrement that made v ready precedes these reads
-    const uint32_t c = lane_mex(A.bits, b + v, e - b + 1);
-    A.color[v] = c;
-    ncol++;
-    uint32_t w[JP_LANE];
-    bool low[JP_LANE];
-    int64_t wb[JP_LANE], we[JP_LANE];
-#pragma unroll
-    for (int u = 0; u < JP_LANE; u++) {
-        low[u] = b + u < e;
-        w[u] = low[u] ? (uint32_t)__ldg(A.ci + b + u) : 0u;
-    }
-#pragma unroll
-    for (int u = 0; u < JP_LANE; u++) {
-        low[u] = low[u] && in_set(A.inS, w[u]) && vkey(A.k, w[u]) < kv;
-        if (low[u]) {
-            wb[u] = A.rp[w[u]];
-            we[u] = A.rp[w[u] + 1];
-        }
-    }
-#pragma unroll
-    for (int u = 0; u < JP_LANE; u++)
-        if (low[u]) set_forbidden(A.bits, wb[u] + w[u], we[u] - wb[u] + 1, c);
-    __threadfence();  // release: the forbidden bits precede the decrements
-#pragma unroll
-    for (int u = 0; u < JP_LANE; u++)
-        if (low[u] && atomicSub(A.cnt + w[u], 1u) == 1u) ja_ready(A, st, (int32_t)w[u], wb[u], we[u]);
-}
-
-__global__ void __launch_bounds__(JP_THREADS) k_jp_async(JaArgs A) {
-    const int lane = lane_id();
-    JaStack st;
-    st.sp = 0;
-    uint32_t ncol = 0;
-    const uint64_t t0 = globaltimer_ns();
-    const uint32_t target = *A.target;
-    for (;;) {
-        // 1. drain the lanes' continuation stacks
-        while (__any_sync(FULL, st.sp > 0)) {
-            if (st.sp > 0) {
-                st.sp--;
-                ja_lane_vertex(A, st, st.v[st.sp], st.b[st.sp], st.e[st.sp], ncol);
-            }
-        }
-        // 2. flush the coloured count, then claim one queued task for the warp
-        uint32_t sum = ncol;
-        for (int d = 16; d; d >>= 1) sum += __shfl_xor_sync(FULL, sum, d);
-        ncol = 0;
-        int32_t tv = -1;
-        uint32_t idx = 0;
-        bool quit = false;
-        if (lane == 0) {
-            if (sum) atomicAdd(A.done, sum);
-            idx = atomicAdd(A.head, 1u);
-            uint32_t spins = 0;
-            for (;;) {
-                tv = idx < A.qcap ? ld_volatile_i32(&A.q[idx].v) : -1;
-                if (tv >= 0) break;
-                if ((++spins & 63u) == 0) {
-                    if (ld_volatile_u32(A.done) >= target || ld_volatile_u32(A.err)) {
-                        quit = true;
-                        break;
-                    }
-                    if (globaltimer_ns() - t0 > JA_TIMEOUT_NS) {
-                        atomicExch(A.err, 1u);
-                        quit = true;
-                        break;
-                    }
-                }
-                __nanosleep(64);
-            }
-        }
-        quit = __shfl_sync(FULL, quit, 0);
-        if (quit) return;
-        tv = __shfl_sync(FULL, tv, 0);
-        idx = __shfl_sync(FULL, idx, 0);
-        __threadfence();
-        const int64_t tb = __ldcg(&A.q[idx].b), te = __ldcg(&A.q[idx].e);
-        const uint32_t tj = __ldcg(&A.q[idx].j);
-        // 3. process the chunk with the whole warp
-        const uint64_t tk = vkey(A.k, (uint32_t)tv);
-        const int64_t cb = tb + (int64_t)tj * JP_CHUNK;
-        constexpr int U = JP_CHUNK / 32;
-        uint32_t w[U];
-        bool low[U];
-#pragma unroll
-        for (int u = 0; u < U; u++) {
-            int64_t x = cb + u * 32 + lane;
-            low[u] = x < te;
-            w[u] = low[u] ? (uint32_t)__ldg(A.ci + x) : 0u;
-        }
-        const uint32_t c = warp_mex(A.bits, tb + tv, te - tb + 1);
-        if (tj == 0 && lane == 0) {
-            A.color[tv] = c;
-            ncol++;
-        }
-        int64_t wb[U], we[U];
-#pragma unroll
-        for (int u = 0; u < U; u++) {
-            low[u] = low[u] && in_set(A.inS, w[u]) && vkey(A.k, w[u]) < tk;
-            if (low[u]) {
-                wb[u] = A.rp[w[u]];
-                we[u] = A.rp[w[u] + 1];
-            }
-        }
-#pragma unroll
-        for (int u = 0; u < U; u++)
-            if (low[u]) set_forbidden(A.bits, wb[u] + w[u], we[u] - wb[u] + 1, c);
-        __threadfence();
-#pragma unroll
-        for (int u = 0; u < U; u++)
-            if (low[u] && atomicSub(A.cnt + w[u], 1u) == 1u) ja_ready(A, st, (int32_t)w[u], wb[u], we[u]);
-    }
-}
-
-// target = #S vertices with phase arcs (the others were coloured by the init pass)
-__global__ void k_jp_count_targets(const int64_t *__restrict__ rp, const int32_t *list, const uint32_t *list_cnt,
-                                   int64_t implicit_n, uint32_t *target) {
-    const uint32_t cnt = list ? *list_cnt : (uint32_t)implicit_n;
-    uint32_t local = 0;
-    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
-        int64_t v = list ? list[i] : (int64_t)i;
-        local += rp[v + 1] > rp[v] ? 1u : 0u;
-    }
-    for (int d = 16; d; d >>= 1) local += __shfl_xor_sync(FULL, local, d);
-    if (lane_id() == 0 && local) atomicAdd(target, local);
-}
-
-static int jp_run_async(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
-                        const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n,
-                        int phase) {
+// overflow bitmap layout follows this CSR (offset rp[v] + v, deg+1 bits).
+// Init pass: records, level-0 tasks into tq0 (count in ring[0]).
+static int jp_init(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, const int64_t *rp, const int32_t *ci,
+                   const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n, JpTask *tq0) {
     Ctl *ctl = f.ctl;
     cudaStream_t s = f.stream;
-    const Key k = stream_key(f.p.seed, TAG_VERTEX, 0);
-    JpTask *q = reinterpret_cast<JpTask *>(w.task);
-    const int64_t qcap = 2 * w.queue_cap;
-    // counters: ring[0] = tail (init writes the first ready tasks there), ring[1] =
-    // head, ring[2] = done, flag = error, q_head = target
     SYM_CUDA(cudaMemsetAsync(ctl->ring, 0, sizeof(ctl->ring) + sizeof(ctl->huge), s));
-    SYM_CUDA(cudaMemsetAsync(&ctl->flag, 0, sizeof(uint32_t), s));
-    SYM_CUDA(cudaMemsetAsync(&ctl->q_head, 0, sizeof(uint32_t), s));
     SYM_CUDA(cudaMemsetAsync(w.bits, 0, sizeof(uint32_t) * (size_t)w.bits_words, s));
-    SYM_CUDA(cudaMemsetAsync(q, 0xff, sizeof(JpTask) * (size_t)qcap, s));
-    prof_begin("jp_init", s);
-    JpArgs A;
     A.rp = rp;
     A.ci = ci;
     A.inS = inS;
     A.color = color;
-    A.cnt = w.cnt;
+    A.rec = reinterpret_cast<JpRec *>(w.rec);
     A.bits = w.bits;
-    A.k = k;
+    A.k = stream_key(f.p.seed, TAG_VERTEX, 0);
     A.huge = w.queue;
     A.hist = nullptr;
     A.in_list = list0;
     A.in_cnt = cnt0;
     A.implicit_n = implicit_n;
     A.tin = nullptr;
-    A.tout = q;
+    A.tout = tq0;
     A.out_cnt = &ctl->ring[0];
     A.clear_cnt = &ctl->ring[3];
     A.huge_cnt = &ctl->huge[1];
-    A.huge_clear = &ctl->huge[0];
-    A.round = 0;
-    k_jp_init<<<num_sms() * (2048 / JP_THREADS), JP_THREADS, 0, s>>>(A);
-    SYM_LAUNCH_CHECK();
-    k_jp_init_huge<<<num_sms() * 2, JP_HUGE_THREADS, 0, s>>>(A);
-    SYM_LAUNCH_CHECK();
-    k_jp_count_targets<<<num_sms() * 4, 256, 0, s>>>(rp, list0, cnt0, implicit_n, &ctl->q_head);
-    prof_end(s, -1);
-    SYM_LAUNCH_CHECK();
-    JaArgs J;
-    J.rp = rp;
-    J.ci = ci;
-    J.inS = inS;
-    J.color = color;
-    J.cnt = w.cnt;
-    J.bits = w.bits;
-    J.q = q;
-    J.qcap = qcap;
-    J.tail = &ctl->ring[0];
-    J.head = &ctl->ring[1];
-    J.done = &ctl->ring[2];
-    J.err = &ctl->flag;
-    J.target = &ctl->q_head;
-    J.k = k;
-    int per_sm = 0;
-    SYM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_jp_async, JP_THREADS, 0));
-    if (per_sm < 1) per_sm = 1;
-    // algorithmic bytes of the asynchronous pass: every arc of the phase
-    // CSR read once (4 B) + per vertex the row bounds of the task (8 B) and the
-    // colour write (4 B); counter/bitmap atomics are L2 traffic
-    const int64_t phase_nnz = rp == f.g.rp ? f.g.nnz : (rp == f.split.rp_in ? f.split.nnz_in : -1);
-    const double jp_bytes = phase_nnz >= 0 ? 4.0 * (double)phase_nnz + 12.0 * (double)f.g.n : -1.0;
-    prof_begin("jp_async", s);
-    k_jp_async<<<num_sms() * per_sm, JP_THREADS, 0, s>>>(J);
-    prof_end(s, jp_bytes);
-    SYM_LAUNCH_CHECK();
-    uint32_t err = 0;
-    SYM_TRY(read_u32(&ctl->flag, &err, s));
-    if (err) {
-        set_error("asynchronous JP stalled (device timeout)");
-        return SYM_ECUDA;
-    }
-    if (f.stats) f.stats->rounds[phase] = 0;
-    return SYM_OK;
-}
-
-static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
-                  const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n, int phase) {
-    if (!getenv("SYM_JP_ROUNDS")) return jp_run_async(f, w, color, rp, ci, inS, list0, cnt0, implicit_n, phase);
-    Ctl *ctl = f.ctl;
-    cudaStream_t s = f.stream;
-    const Key k = stream_key(f.p.seed, TAG_VERTEX, 0);
-    JpTask *tq[2] = {reinterpret_cast<JpTask *>(w.task), reinterpret_cast<JpTask *>(w.task) + w.queue_cap};
-    SYM_CUDA(cudaMemsetAsync(ctl->ring, 0, sizeof(ctl->ring) + sizeof(ctl->huge), s));
-    SYM_CUDA(cudaMemsetAsync(w.bits, 0, sizeof(uint32_t) * (size_t)w.bits_words, s));
-    JpArgs A;
-    A.rp = rp;
-    A.ci = ci;
-    A.inS = inS;
-    A.color = color;
-    A.cnt = w.cnt;
-    A.bits = w.bits;
-    A.k = k;
-    A.huge = w.queue;
-    A.hist = ctl->hist + phase * 2048;
-    A.in_list = list0;
-    A.in_cnt = cnt0;
-    A.implicit_n = implicit_n;
-    A.tin = nullptr;
-    A.tout = tq[0];
-    A.out_cnt = &ctl->ring[0];
-    A.clear_cnt = &ctl->ring[2];
-    A.huge_cnt = &ctl->huge[1];
-    A.huge_clear = &ctl->huge[0];
     A.round = 0;
     prof_begin("jp_init", s);
     k_jp_init<<<num_sms() * (2048 / JP_THREADS), JP_THREADS, 0, s>>>(A);
     SYM_LAUNCH_CHECK();
-    k_jp_init_huge<<<num_sms() * 2, JP_HUGE_THREADS, 0, s>>>(A);
+    k_jp_init_huge<<<num_sms() * 4, JP_HUGE_THREADS, 0, s>>>(A);
+    SYM_LAUNCH_CHECK();
+    k_jp_huge_ready<<<num_sms(), 256, 0, s>>>(A);
     prof_end(s, -1);
     SYM_LAUNCH_CHECK();
+    return SYM_OK;
+}
+
+// algorithmic bytes of the level pass: every arc of the phase CSR read
+// once (4 B) + per vertex its task (row bounds, 16 B) and colour write (4 B); the
+// pushes are L2 atomics on the 32-B records (not HBM bytes)
+static double jp_alg_bytes(const FlowArgs &f, const int64_t *rp) {
+    const int64_t phase_nnz = rp == f.g.rp ? f.g.nnz : (rp == f.split.rp_in ? f.split.nnz_in : -1);
+    return phase_nnz >= 0 ? 4.0 * (double)phase_nnz + 20.0 * (double)f.g.n : -1.0;
+}
+
+static int coop_supported() {
+    static int ok = -1;
+    if (ok < 0) {
+        int dev = 0, v = 0;
+        ok = (cudaGetDevice(&dev) == cudaSuccess &&
+              cudaDeviceGetAttribute(&v, cudaDevAttrCooperativeLaunch, dev) == cudaSuccess && v)
+                 ? 1
+                 : 0;
+    }
+    return ok;
+}
+
+// default driver: every level in one persistent cooperative launch
+static int jp_run_levels(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
+                         const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n,
+                         int phase) {
+    Ctl *ctl = f.ctl;
+    cudaStream_t s = f.stream;
+    JpTask *tq[2] = {reinterpret_cast<JpTask *>(w.task), reinterpret_cast<JpTask *>(w.task) + w.queue_cap};
+    SYM_CUDA(cudaMemsetAsync(w.sync, 0, 64 * sizeof(uint32_t), s));
+    JpArgs A;
+    SYM_TRY(jp_init(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n, tq[0]));
+    A.hist = f.stats ? ctl->hist + phase * 2048 : nullptr;
+    JlCtl C;
+    C.ring = ctl->ring;
+    C.bar = &w.sync[0];
+    C.err = &w.sync[32];
+    C.levels = &w.sync[33];
+    C.tq0 = tq[0];
+    C.tq1 = tq[1];
+    C.max_levels = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
+    static int grid = 0;
+    if (grid == 0) {
+        int per_sm = 0;
+        SYM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_jp_levels, JL_THREADS, 0));
+        if (per_sm < 1) {
+            set_error("k_jp_levels does not fit on an SM");
+            return SYM_ECUDA;
+        }
+        grid = num_sms() * per_sm;
+    }
+    void *args[] = {&A, &C};
+    prof_begin("jp_levels", s);
+    SYM_CUDA(cudaLaunchCooperativeKernel((const void *)k_jp_levels, dim3(grid), dim3(JL_THREADS), args, 0, s));
+    prof_end(s, jp_alg_bytes(f, rp));
+    uint32_t err = 0, levels = 0;
+    SYM_TRY(read_u32(C.err, &err, s));
+    if (err) {
+        SYM_TRY(read_u32(C.levels, &levels, s));
+        const bool rounds = f.p.max_rounds && levels + 1 >= f.p.max_rounds;
+        set_error(rounds ? "JP did not converge within max_rounds" : "JP levels kernel timed out");
+        return rounds ? SYM_EROUNDS : SYM_ECUDA;
+    }
+    if (f.stats) {
+        SYM_TRY(read_u32(C.levels, &levels, s));
+        f.stats->rounds[phase] = levels;
+    }
+    return SYM_OK;
+}
+
+// fallback: one k_jp_push launch per level, host polls in growing batches
+static int jp_run_rounds(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
+                         const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n,
+                         int phase) {
+    Ctl *ctl = f.ctl;
+    cudaStream_t s = f.stream;
+    JpTask *tq[2] = {reinterpret_cast<JpTask *>(w.task), reinterpret_cast<JpTask *>(w.task) + w.queue_cap};
+    JpArgs A;
+    SYM_TRY(jp_init(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n, tq[0]));
+    A.hist = f.stats ? ctl->hist + phase * 2048 : nullptr;
     const uint32_t maxr = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
     const int grid = num_sms() * 2;  // frontiers are small: a short grid launches and drains fast
     int r = 0, batch = 8;
@@ -758,7 +783,7 @@ static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t 
             A.tout = tq[(r + 1) & 1];
             A.out_cnt = &ctl->ring[(r + 1) % 3];
             A.clear_cnt = &ctl->ring[(r + 2) % 3];
-            A.round = r < 2048 ? r : 2047;
+            A.round = r;
             prof_begin("jp_push", s);
             k_jp_push<<<grid, JP_THREADS, 0, s>>>(A);
             prof_end(s, -1);
@@ -775,6 +800,14 @@ static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t 
     }
     if (f.stats) f.stats->rounds[phase] = (uint32_t)r;
     return SYM_OK;
+}
+
+static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
+                  const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n, int phase) {
+    const char *mode = getenv("SYM_JP_MODE");
+    if ((mode && mode[0] == 'r') || !coop_supported())
+        return jp_run_rounds(f, w, color, rp, ci, inS, list0, cnt0, implicit_n, phase);
+    return jp_run_levels(f, w, color, rp, ci, inS, list0, cnt0, implicit_n, phase);
 }
 
 int run_color(const FlowArgs &f, ColorWs &w, uint32_t *color) {
