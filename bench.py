@@ -32,10 +32,10 @@ METRIC = "MIS/MM/COLOR edges/s at 1/2/4/8 B200; % of HBM roofline; vs CPU oracle
 # class from one `ncu --set full` capture of this step (profiles/r1_ncu_summary.md);
 # None where no capture was taken for the current code.
 TRAFFIC = {
-    "split": 4.51e9,       # k_split<DEGK> at R-MAT s24 (profiles/r1_ncu.md): 2.22 GB read + 2.29 GB written
-    "mm_round0": 0.717e9,  # k_round0<MM> on the RAND-4 intra CSR
-    "jp_init": 1.90e9,
-    "jp_async": 25.04e9,   # 20.0 GB read + 5.04 GB written: random record/bitmap traffic
+    "split": 4.51e9,       # k_split<DEGK> / <RAND> at R-MAT s24 (profiles/r1b_ncu.md): 2.22 GB read + 2.29 GB written
+    "mm_round0": 0.719e9,  # k_round0<MM> on the RAND-4 intra CSR
+    "jp_init": 2.36e9,     # k_jp_init: 1.75 GB read + 0.61 GB written (records)
+    "jp_levels": 10.21e9,  # k_jp_levels: 7.43 GB read + 2.78 GB written (records, tasks, colours, columns)
 }
 
 
@@ -53,6 +53,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--profile-only", action="store_true", help="short run for ncu (no JSON contract)")
+    ap.add_argument("--sequential", action="store_true", help="one stream, the five calls in order")
     return ap.parse_args()
 
 
@@ -181,13 +182,21 @@ def main():
     m = nnz // 2
     seed = args.seed + rank
 
-    def step():
+    def step_sequential(rp=rp, ci=ci):
         dD = sb.sym_decompose(rp, ci, "degk", 2, seed)
         I = sb.sym_mis(rp, ci, "degk", 2, seed, decomp=dD)
         C = sb.sym_color(rp, ci, "degk", 2, seed, decomp=dD)
         dR = sb.sym_decompose(rp, ci, "rand", 4, seed)
         M = sb.sym_mm(rp, ci, "rand", 4, seed, decomp=dR)
         return I, C, M
+
+    from paper_conf_ipps_nayyaroddeengk17_b200.schedule import ConcurrentStep
+    _cs = ConcurrentStep(dev, seed)
+
+    def step_concurrent(rp=rp, ci=ci):
+        return _cs(rp, ci)
+
+    step = step_sequential if args.sequential else step_concurrent
 
     if args.profile_only:
         for _ in range(max(1, args.warmup)):
@@ -223,9 +232,7 @@ def main():
     ms_step = ms / args.steps
     value = world * m / (ms_step * 1e-3)
 
-    # ---- per-problem breakdown + per-kernel-class device times (profiling hook, separate pass)
-    sb.sym_profile_enable(True)
-    sb.sym_profile_collect()
+    # ---- per-problem breakdown (events between the calls, no profiling hook) ...
     steps_p = max(1, min(args.steps, 3))
     evs = [torch.cuda.Event(enable_timing=True) for _ in range(6)]
     brk = {"decompose_deg2": 0.0, "mis_deg2": 0.0, "color_deg2": 0.0, "decompose_rand4": 0.0, "mm_rand4": 0.0}
@@ -244,6 +251,14 @@ def main():
         torch.cuda.synchronize()
         for i, k in enumerate(brk):
             brk[k] += evs[i].elapsed_time(evs[i + 1]) / steps_p
+    # ... and per-kernel-class device times through the library's event hook (separate pass)
+    sb.sym_profile_enable(True)
+    step_sequential()  # first profiled call allocates the hook's counters
+    torch.cuda.synchronize()
+    sb.sym_profile_collect()
+    for _ in range(steps_p):
+        step_sequential()
+    torch.cuda.synchronize()
     prof = sb.sym_profile_collect()
     sb.sym_profile_enable(False)
     _, st_mis = sb.sym_mis(rp, ci, "degk", 2, seed, stats=True, flags=2)
@@ -276,6 +291,14 @@ def main():
     # the dominant kernel = the class with the most device time in the step
     dominant_overall = max(prof, key=lambda k: prof[k]["ms"]) if prof else None
     roof = roof_of(dominant_overall) if dominant_overall else None
+    if roof is not None and dominant_overall == "jp_levels":
+        # JP is bound by its dependency depth, not by bytes: one level = a burst of
+        # scattered record atomics + one grid barrier
+        levels = st_col["rounds"][0]
+        roof["latency_model"] = {
+            "levels": levels, "us_per_level": roof["ms_per_launch"] * 1e3 / max(1, levels),
+            "grid_barrier_us": 1.4, "note": "depth-bound: levels x (push burst + grid barrier); "
+            "HBM frac is reported for the algorithmic bytes only"}
     rooflines = {k: roof_of(k) for k in prof if roof_of(k)}
 
     # ---- e2e through the public API with pinned host buffers
@@ -290,11 +313,7 @@ def main():
         for _ in range(args.e2e_steps):
             rpd = rp_h.to(dev, non_blocking=True)
             cid = ci_h.to(dev, non_blocking=True)
-            dD = sb.sym_decompose(rpd, cid, "degk", 2, seed)
-            I = sb.sym_mis(rpd, cid, "degk", 2, seed, decomp=dD)
-            C = sb.sym_color(rpd, cid, "degk", 2, seed, decomp=dD)
-            dR = sb.sym_decompose(rpd, cid, "rand", 4, seed)
-            M = sb.sym_mm(rpd, cid, "rand", 4, seed, decomp=dR)
+            I, C, M = step(rpd, cid)
             res = [x.cpu() for x in (I, C, M)]
             outs_bytes = sum(x.numel() * x.element_size() for x in res)
             del rpd, cid
@@ -357,6 +376,8 @@ def main():
             "config": {"workload": f"rmat{args.scale}-ef{args.ef}: DEG2{{MIS,COLOR}} + RAND4{{MM}}",
                        "n": n, "m": m, "arcs": nnz, "seed": seed, "graph_seed": 1,
                        "parallelism": "replicas" if world > 1 else "single",
+                       "schedule": "sequential (one stream)" if args.sequential else
+                       "2 streams: [DEG2 decomposition -> COLOR-Deg2] || [RAND4 decomposition -> MM-Rand4 -> MIS-Deg2]",
                        "l2": "inputs exceed L2 (col_idx %.2f GB > 126 MB)" % (nnz * 4 / 1e9),
                        "generate_s": round(gen_s, 2)},
             "breakdown_ms": brk,

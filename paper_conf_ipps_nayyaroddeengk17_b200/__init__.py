@@ -48,7 +48,10 @@ _WS: dict = {}
 
 
 def _workspace(nbytes: int, device) -> torch.Tensor:
-    key = torch.device(device).index
+    """Per (device, stream) scratch: calls on different streams (e.g. independent problems
+    run concurrently from several host threads) never share a workspace."""
+    device = torch.device(device)
+    key = (device.index, torch.cuda.current_stream(device).cuda_stream)
     buf = _WS.get(key)
     if buf is None or buf.numel() < nbytes:
         _WS.pop(key, None)

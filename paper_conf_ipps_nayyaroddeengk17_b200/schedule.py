@@ -1,0 +1,66 @@
+"""Concurrent schedule of one step of the hot path (MIS-Deg2 + COLOR-Deg2 + MM-Rand4).
+
+The three problems are independent once the DEG2 decomposition exists (P:288, P:234
+use it; MM-Rand has its own RAND decomposition), so they run on two CUDA
+streams from two host threads (ctypes releases the GIL; the library keeps no
+per-call global state and every stream gets its own workspace):
+
+    stream A (high priority): DEG2 decomposition -> COLOR-Deg2.  Its JP kernel is
+                              persistent and depth-bound (1 CTA/SM, mostly waiting
+                              on its grid barrier), so it leaves SM slots idle.
+    stream B:                 RAND4 decomposition -> MM-Rand4 -> MIS-Deg2 (after
+                              stream A's decomposition) -- fills those slots.
+
+Every call is the public API (sym_decompose / sym_mis / sym_mm / sym_color); results
+are bit-identical to running the five calls in order (tests/test_gpu_concurrent.py).
+"""
+from __future__ import annotations
+
+import concurrent.futures as cf
+
+import torch
+
+from . import sym_color, sym_decompose, sym_mis, sym_mm
+
+
+class ConcurrentStep:
+    def __init__(self, device, seed: int, k: int = 2, p: int = 4):
+        self.dev = torch.device(device)
+        self.seed, self.k, self.p = seed, k, p
+        self.sA = torch.cuda.Stream(self.dev, priority=-1)
+        self.sB = torch.cuda.Stream(self.dev)
+        self.pool = cf.ThreadPoolExecutor(1)
+
+    def __call__(self, rp: torch.Tensor, ci: torch.Tensor):
+        """-> (in_set, color, mate) of MIS-Deg{k}, COLOR-Deg{k}, MM-Rand{p} on (rp, ci)."""
+        seed, k, p = self.seed, self.k, self.p
+        main = torch.cuda.current_stream(self.dev)
+        self.sA.wait_stream(main)
+        self.sB.wait_stream(main)
+        with torch.cuda.stream(self.sA):
+            dD = sym_decompose(rp, ci, "degk", k, seed)
+            evD = torch.cuda.Event()
+            evD.record(self.sA)
+
+        def side():
+            with torch.cuda.device(self.dev), torch.cuda.stream(self.sB):
+                dR = sym_decompose(rp, ci, "rand", p, seed)
+                M = sym_mm(rp, ci, "rand", p, seed, decomp=dR)
+                self.sB.wait_event(evD)
+                I = sym_mis(rp, ci, "degk", k, seed, decomp=dD)
+            return I, M
+
+        fut = self.pool.submit(side)
+        with torch.cuda.stream(self.sA):
+            C = sym_color(rp, ci, "degk", k, seed, decomp=dD)
+        I, M = fut.result()
+        # tensors used on both streams: keep the caching allocator from reusing them early
+        for t in (dD.row_ptr_in, dD.col_in, dD.row_ptr_x, dD.col_x, rp, ci):
+            t.record_stream(self.sA)
+            t.record_stream(self.sB)
+        for t in (I, M):
+            t.record_stream(self.sB)
+        C.record_stream(self.sA)
+        main.wait_stream(self.sA)
+        main.wait_stream(self.sB)
+        return I, C, M

@@ -9,7 +9,7 @@ d = sb.sym_decompose(rp, ci, "degk", 2, 42)
 for _ in range(2):
     col, st = sb.sym_color(rp, ci, "degk", 2, 42, decomp=d, stats=True)
 torch.cuda.synchronize()
-ws = sb._WS[0]
+ws = sb._WS[(0, torch.cuda.current_stream(dev).cuda_stream)]
 off = ((ws.data_ptr() + 255) & ~255) - ws.data_ptr()
 h = ws[off + 136: off + 136 + 8192].cpu().numpy().view(np.uint32)
 cnt, ts = h[:1024].astype(np.int64), h[1024:2048].astype(np.int64) * 32 / 1000.0
