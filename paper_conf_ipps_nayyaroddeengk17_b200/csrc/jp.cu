@@ -23,6 +23,7 @@
 // ~5e4 scattered pushes, so the cost per level is the latency of that burst plus one
 // grid barrier: all levels run inside ONE persistent cooperative kernel (k_jp_levels)
 // with a software grid barrier between levels.
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 
@@ -73,14 +74,11 @@ struct JpArgs {
     const int32_t *in_list;    // init: vertex list (nullable = implicit)
     const uint32_t *in_cnt;
     int64_t implicit_n;
-    const JpTask *tin;
-    JpTask *tout;
-    uint32_t *out_cnt;
-    uint32_t *clear_cnt;
+    JpTask *tout;         // the task queue (monotone; level r owns [lo_r, hi_r))
+    uint32_t *out_cnt;    // init: task counter (the low half of the levels kernel's W)
     int64_t *huge;        // init: (piece << 32 | v) items of the huge rows
     uint32_t *huge_cnt;
     uint32_t *hist;
-    int round;
     Key k;
 };
 
@@ -312,9 +310,15 @@ __global__ void k_jp_huge_ready(JpArgs A) {
 }
 
 // ---------------------------------------------------------------- one level
-// Ready vertices found during a level are staged in shared memory and appended to the
-// next task list once per CTA (one global reservation per CTA and level, tasks of a
-// hub written by the whole CTA); a full stage falls back to a per-lane append.
+// Tasks live in ONE monotone queue (every vertex is enqueued exactly once): level r
+// owns slots [lo_r, hi_r).  A 64-bit word W = (arrivals << 32 | tasks reserved) is
+// both the grid barrier and the task allocator: at the end of a level each CTA adds
+// (1 << 32 | its staged tasks) once -- reservation and arrival in one atomic -- then
+// writes its tasks; the last arriver publishes (r+1 << 32 | hi_{r+1}) in the word G
+// that the other CTAs poll.  Tasks may land after the barrier, so the queue is
+// pre-filled with -1 and a reader waits until its task's three 8-byte words are
+// written.  Ready vertices are staged in shared memory (one reservation per CTA and
+// level, a hub's tasks written by the whole CTA); a full stage reserves per warp.
 constexpr int JP_STAGE = 1024;
 
 struct JpStage {
@@ -328,28 +332,71 @@ struct JpStage {
     uint32_t off[JP_STAGE + 1];  // exclusive prefix of the task counts
 };
 
-__device__ __forceinline__ void stage_ready(const JpArgs &A, JpStage &st, int32_t w, int64_t b, uint32_t deg) {
+struct JlCtl {
+    unsigned long long *W;  // (arrivals << 32) | tasks reserved (low half = init's counter)
+    unsigned long long *G;  // (level + 1) << 32 | end of that level's tasks, by the last arriver
+    uint32_t *err;          // 1 = timeout / max levels
+    uint32_t *levels;       // out: number of levels run
+    uint32_t max_levels;
+};
+
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void st_release_u64(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ void write_task(JpTask *q, int64_t b, int64_t e, int32_t v, uint32_t j) {
+    longlong2 *p = reinterpret_cast<longlong2 *>(q);
+    p[0] = make_longlong2(b, e);
+    p[1] = make_longlong2((long long)(((uint64_t)j << 32) | (uint32_t)v), 0);
+}
+
+// a task of the current level; waits (bounded by the writer CTA's progress: all CTAs
+// are co-resident) until its writer's stores are visible
+__device__ __forceinline__ void read_task(const JpTask *q, int64_t &b, int64_t &e, int32_t &v, uint32_t &j) {
+    const volatile long long *p = reinterpret_cast<const volatile long long *>(q);
+    long long x0, x1, x2;
+    do {
+        x0 = p[0];
+        x1 = p[1];
+        x2 = p[2];
+    } while (x0 == -1 || x1 == -1 || x2 == -1);
+    b = x0;
+    e = x1;
+    v = (int32_t)(uint32_t)(unsigned long long)x2;
+    j = (uint32_t)((unsigned long long)x2 >> 32);
+}
+
+__device__ __forceinline__ void stage_ready(const JpArgs &A, const JlCtl &C, JpStage &st, int32_t w, int64_t b,
+                                            uint32_t deg) {
     asm volatile("prefetch.global.L2 [%0];" ::"l"(A.ci + b));  // the row is read next level
     const uint32_t slot = atomicAdd(&st.n, 1u);
     if (slot < JP_STAGE) {
         st.v[slot] = w;
         st.deg[slot] = deg;
         st.b[slot] = b;
-    } else {
+    } else {  // stage full: reserve directly (no arrival)
         const uint32_t nt = n_tasks(deg);
-        put_tasks(A.tout, atomicAdd(A.out_cnt, nt), w, b, b + deg, nt);
+        const uint32_t base = (uint32_t)atomicAdd(C.W, (unsigned long long)nt);
+        for (uint32_t q = 0; q < nt; q++) write_task(A.tout + base + q, b, b + deg, w, q);
     }
 }
 
-// CTA-wide: reserve the staged entries' tasks with one global atomic and write them
-__device__ __forceinline__ void stage_flush(const JpArgs &A, JpStage &st) {
+// CTA-wide end of a level: one atomic = arrival + reservation of the staged entries'
+// tasks, then the tasks, then wait for the level's last arrival; returns hi_{r+1}
+__device__ __forceinline__ uint32_t stage_flush_barrier(const JpArgs &A, const JlCtl &C, JpStage &st, uint32_t r,
+                                                        uint32_t arrivals_expected) {
     __syncthreads();
     const uint32_t n = min(st.n, (uint32_t)JP_STAGE);
     const uint32_t per = (JP_STAGE + blockDim.x - 1) / blockDim.x;
     const uint32_t i0 = threadIdx.x * per;
     uint32_t loc = 0;
     for (uint32_t i = i0; i < min(n, i0 + per); i++) loc += n_tasks(st.deg[i]);
-    // block exclusive scan of loc
     uint32_t incl = loc;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
@@ -360,7 +407,8 @@ __device__ __forceinline__ void stage_flush(const JpArgs &A, JpStage &st) {
     if (lane_id() == 31) st.wsum[wid] = incl;
     __syncthreads();
     if (wid == 0) {
-        uint32_t x = lane_id() < nw ? st.wsum[lane_id()] : 0u, xi = x;
+        const uint32_t x = lane_id() < nw ? st.wsum[lane_id()] : 0u;
+        uint32_t xi = x;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
             const uint32_t y = __shfl_up_sync(FULL, xi, d);
@@ -368,8 +416,12 @@ __device__ __forceinline__ void stage_flush(const JpArgs &A, JpStage &st) {
         }
         if (lane_id() < nw) st.wsum[lane_id()] = xi - x;
         if (lane_id() == 31) {
+            __threadfence();  // this CTA's pushes (counts, bits, colours) before its arrival
+            const unsigned long long old = atomicAdd(C.W, (1ull << 32) | xi);
             st.total = xi;
-            st.base = xi ? atomicAdd(A.out_cnt, xi) : 0u;
+            st.base = (uint32_t)old;
+            if ((uint32_t)(old >> 32) + 1u == arrivals_expected)  // last arriver: publish the level's end
+                st_release_u64(C.G, ((unsigned long long)(r + 1) << 32) | (uint32_t)(old + xi));
         }
     }
     __syncthreads();
@@ -378,7 +430,6 @@ __device__ __forceinline__ void stage_flush(const JpArgs &A, JpStage &st) {
         st.off[i] = o;
         o += n_tasks(st.deg[i]);
     }
-    if (threadIdx.x == 0) st.off[n] = st.total;
     __syncthreads();
     const uint32_t total = st.total, base = st.base;
     for (uint32_t q = threadIdx.x; q < total; q += blockDim.x) {
@@ -388,16 +439,17 @@ __device__ __forceinline__ void stage_flush(const JpArgs &A, JpStage &st) {
             if (st.off[mid] <= q) lo = mid;
             else hi = mid - 1;
         }
-        JpTask t;
-        t.b = st.b[lo];
-        t.e = st.b[lo] + st.deg[lo];
-        t.v = st.v[lo];
-        t.j = q - st.off[lo];
-        t.pad = 0;
-        A.tout[base + q] = t;
+        write_task(A.tout + base + q, st.b[lo], st.b[lo] + st.deg[lo], st.v[lo], q - st.off[lo]);
+    }
+    if (threadIdx.x == 0) {
+        st.n = 0;
+        unsigned long long g;
+        while (((g = ld_acquire_u64(C.G)) >> 32) < r + 1) {
+        }
+        st.base = (uint32_t)g;
     }
     __syncthreads();
-    if (threadIdx.x == 0) st.n = 0;
+    return st.base;
 }
 
 // Decrement the counts of the lower S-neighbours w[0..U) (flags low[]); returns the
@@ -412,8 +464,8 @@ __device__ __forceinline__ void jp_decrement(const JpArgs &A, const uint32_t (&w
 // forbidden bit of colour c for the lower S-neighbours (fire-and-forget), then the
 // records of the vertices that became ready go to the stage
 template <int U>
-__device__ __forceinline__ void jp_mark(const JpArgs &A, JpStage &st, const uint32_t (&w)[U], const bool (&low)[U],
-                                        const uint32_t (&old)[U], uint32_t c) {
+__device__ __forceinline__ void jp_mark(const JpArgs &A, const JlCtl &C, JpStage &st, const uint32_t (&w)[U],
+                                        const bool (&low)[U], const uint32_t (&old)[U], uint32_t c) {
     if (c <= JP_WIN) {
         const uint32_t q = (c - 1) >> 5, bit = 1u << ((c - 1) & 31);
 #pragma unroll
@@ -432,17 +484,18 @@ __device__ __forceinline__ void jp_mark(const JpArgs &A, JpStage &st, const uint
     for (int u = 0; u < U; u++) {
         if (low[u] && old[u] == 1u) {
             const uint4 h = __ldcg(reinterpret_cast<const uint4 *>(A.rec + w[u]));
-            stage_ready(A, st, (int32_t)w[u], (int64_t)(((uint64_t)h.w << 32) | h.z), h.y);
+            stage_ready(A, C, st, (int32_t)w[u], (int64_t)(((uint64_t)h.w << 32) | h.z), h.y);
         }
     }
 }
 
-// One level of push JP: every task of tin[0, cnt) colours its vertex (the first chunk
-// writes the colour) and pushes it to the lower S-neighbours of its chunk; vertices
-// whose count reaches 0 are appended to A.tout (counter A.out_cnt).  CTA-wide.
-__device__ __forceinline__ void jp_level(const JpArgs &A, JpStage &st, uint32_t cnt, const JpTask *tin,
+// One level of push JP over the tasks [lo, hi) of the queue: every task colours its
+// vertex (the first chunk writes the colour) and pushes it to the lower S-neighbours
+// of its chunk; vertices whose count reaches 0 are staged for the next level.
+__device__ __forceinline__ void jp_level(const JpArgs &A, const JlCtl &C, JpStage &st, uint32_t lo, uint32_t hi,
                                          int64_t warp_g, int64_t nwarps) {
     const int lane = lane_id();
+    const uint32_t cnt = hi - lo;
     // task index t = it*32*nwarps + lane*nwarps + warp: consecutive tasks (the chunks
     // of one hub) land on different warps
     for (int64_t base = warp_g; base - warp_g < cnt; base += nwarps * 32) {
@@ -450,14 +503,7 @@ __device__ __forceinline__ void jp_level(const JpArgs &A, JpStage &st, uint32_t 
         int32_t v = -1;
         uint32_t j = 0;
         int64_t b = 0, e = 0;
-        if (t < cnt) {
-            const longlong2 *p = reinterpret_cast<const longlong2 *>(tin + t);
-            const longlong2 q0 = __ldcg(p), q1 = __ldcg(p + 1);
-            b = q0.x;
-            e = q0.y;
-            v = (int32_t)(uint32_t)q1.x;
-            j = (uint32_t)((uint64_t)q1.x >> 32);
-        }
+        if (t < cnt) read_task(A.tout + lo + t, b, e, v, j);
         const uint64_t kv = v >= 0 ? vkey(A.k, (uint32_t)v) : 0;
         // ---- short rows: one lane does the whole task
         const bool small = v >= 0 && e - b <= JP_LANE;
@@ -478,7 +524,7 @@ __device__ __forceinline__ void jp_level(const JpArgs &A, JpStage &st, uint32_t 
                 c = lane_mex(A.rec + v, (uint32_t)(e - b));
                 A.color[v] = c;
             }
-            jp_mark<JP_LANE>(A, st, w, low, old, c);
+            jp_mark<JP_LANE>(A, C, st, w, low, old, c);
         }
         // ---- longer rows: the warp takes these tasks one by one (<= JP_CHUNK arcs)
         unsigned bigm = __ballot_sync(FULL, v >= 0 && !small);
@@ -505,67 +551,21 @@ __device__ __forceinline__ void jp_level(const JpArgs &A, JpStage &st, uint32_t 
             jp_decrement<U>(A, w, low, old);  // the decrements do not wait for the mex
             const uint32_t c = warp_mex(A.rec + tv, A.bits, tb + tv, (uint32_t)(te - tb));
             if (tj == 0 && lane == 0) A.color[tv] = c;
-            jp_mark<U>(A, st, w, low, old, c);
+            jp_mark<U>(A, C, st, w, low, old, c);
         }
     }
-    stage_flush(A, st);
-}
-
-// host-driven level (fallback when cooperative launch is unavailable)
-__global__ void __launch_bounds__(JP_THREADS) k_jp_push(JpArgs A) {
-    __shared__ JpStage st;
-    if (threadIdx.x == 0) st.n = 0;
-    __syncthreads();
-    const uint32_t cnt = *A.in_cnt;
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        *A.clear_cnt = 0;
-        if (A.hist && A.round < 1024) A.hist[A.round] = cnt;
-    }
-    const int64_t warp_g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    jp_level(A, st, cnt, A.tin, warp_g, nwarps);
 }
 
 // ---------------------------------------------------------------- persistent levels
-// All levels in ONE cooperative launch: a level is jp_level over the task list of the
-// previous level, then a software grid barrier (one arrival atomic per CTA on a
-// monotone counter that the CTAs poll).  The barrier orders the pushes of level r
-// before the mex reads of level r+1, so no per-push fence is needed.  Counters:
-// ring[r%3] = tasks of level r, ring[(r+1)%3] = tasks appended for level r+1,
-// ring[(r+2)%3] (read before the previous barrier) is cleared for level r+2.
+// All levels in ONE cooperative launch (grid = one or more CTAs per SM, all
+// co-resident): level r = jp_level over [lo_r, hi_r), then stage_flush_barrier.  The
+// barrier orders the pushes of level r before the mex reads of level r+1, so no
+// per-push fence is needed.
 constexpr int JL_THREADS = 512;
 #ifndef SYM_JL_MINB
 #define SYM_JL_MINB 1
 #endif
 constexpr uint64_t JL_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
-
-struct JlCtl {
-    uint32_t *ring;    // [3]
-    uint32_t *bar;     // arrivals (monotone)
-    uint32_t *err;     // 1 = timeout / max levels
-    uint32_t *levels;  // out: number of levels run
-    JpTask *tq0, *tq1;
-    uint32_t max_levels;
-};
-
-__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *p) {
-    uint32_t v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-
-// epoch = arrivals expected after this barrier (wrap-safe comparison)
-__device__ __forceinline__ void grid_barrier(const JlCtl &C, uint32_t &epoch) {
-    __syncthreads();
-    epoch += gridDim.x;
-    if (threadIdx.x == 0) {
-        __threadfence();
-        atomicAdd(C.bar, 1u);
-        while ((int32_t)(ld_acquire_u32(C.bar) - epoch) < 0) {
-        }
-    }
-    __syncthreads();
-}
 
 __global__ void __launch_bounds__(JL_THREADS, SYM_JL_MINB) k_jp_levels(JpArgs A, JlCtl C) {
     __shared__ JpStage st;
@@ -574,24 +574,22 @@ __global__ void __launch_bounds__(JL_THREADS, SYM_JL_MINB) k_jp_levels(JpArgs A,
     // warp-in-CTA major: consecutive tasks (the chunks of one row) go to different SMs
     const int64_t warp_g = (int64_t)(threadIdx.x >> 5) * gridDim.x + blockIdx.x;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    uint32_t epoch = 0;
     const uint64_t t0 = globaltimer_ns();
+    uint32_t lo = 0, hi = (uint32_t)__ldcg(C.W);  // level 0 = the init pass's tasks
     uint32_t r = 0;
     for (;; r++) {
-        const uint32_t cnt = __ldcg(C.ring + r % 3);
-        if (cnt == 0 || __ldcg(C.err) != 0) break;
+        if (hi == lo || __ldcg(C.err) != 0) break;
         if (blockIdx.x == 0 && threadIdx.x == 0) {
-            C.ring[(r + 2) % 3] = 0;
             if (A.hist && r < 1024) {  // stats: tasks and start time (32 ns units) of the first levels
-                A.hist[r] = cnt;
+                A.hist[r] = hi - lo;
                 A.hist[1024 + r] = (uint32_t)((globaltimer_ns() - t0) >> 5);
             }
             if (r + 1 >= C.max_levels || globaltimer_ns() - t0 > JL_TIMEOUT_NS) atomicExch(C.err, 1u);
         }
-        A.out_cnt = C.ring + (r + 1) % 3;
-        A.tout = (r & 1) ? C.tq0 : C.tq1;
-        jp_level(A, st, cnt, (r & 1) ? C.tq1 : C.tq0, warp_g, nwarps);
-        grid_barrier(C, epoch);
+        jp_level(A, C, st, lo, hi, warp_g, nwarps);
+        const uint32_t next = stage_flush_barrier(A, C, st, r, (r + 1) * gridDim.x);
+        lo = hi;
+        hi = next;
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *C.levels = r;
 }
@@ -659,12 +657,13 @@ void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
 
 // JP over (rp, ci) for the vertex set S (list/implicit) with membership inS; the
 // overflow bitmap layout follows this CSR (offset rp[v] + v, deg+1 bits).
-// Init pass: records, level-0 tasks into tq0 (count in ring[0]).
+// Init pass: records and the level-0 tasks at the head of the queue (counter *qcnt).
 static int jp_init(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, const int64_t *rp, const int32_t *ci,
-                   const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n, JpTask *tq0) {
+                   const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n, JpTask *q,
+                   uint32_t *qcnt) {
     Ctl *ctl = f.ctl;
     cudaStream_t s = f.stream;
-    SYM_CUDA(cudaMemsetAsync(ctl->ring, 0, sizeof(ctl->ring) + sizeof(ctl->huge), s));
+    SYM_CUDA(cudaMemsetAsync(ctl->huge, 0, sizeof(ctl->huge), s));
     SYM_CUDA(cudaMemsetAsync(w.bits, 0, sizeof(uint32_t) * (size_t)w.bits_words, s));
     A.rp = rp;
     A.ci = ci;
@@ -678,12 +677,9 @@ static int jp_init(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, co
     A.in_list = list0;
     A.in_cnt = cnt0;
     A.implicit_n = implicit_n;
-    A.tin = nullptr;
-    A.tout = tq0;
-    A.out_cnt = &ctl->ring[0];
-    A.clear_cnt = &ctl->ring[3];
+    A.tout = q;
+    A.out_cnt = qcnt;
     A.huge_cnt = &ctl->huge[1];
-    A.round = 0;
     prof_begin("jp_init", s);
     k_jp_init<<<num_sms() * (2048 / JP_THREADS), JP_THREADS, 0, s>>>(A);
     SYM_LAUNCH_CHECK();
@@ -696,47 +692,27 @@ static int jp_init(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, co
 }
 
 // algorithmic bytes of the level pass: every arc of the phase CSR read
-// once (4 B) + per vertex its task (row bounds, 16 B) and colour write (4 B); the
+// once (4 B) + per vertex its task (32 B written + read) and colour write (4 B); the
 // pushes are L2 atomics on the 32-B records (not HBM bytes)
 static double jp_alg_bytes(const FlowArgs &f, const int64_t *rp) {
     const int64_t phase_nnz = rp == f.g.rp ? f.g.nnz : (rp == f.split.rp_in ? f.split.nnz_in : -1);
-    return phase_nnz >= 0 ? 4.0 * (double)phase_nnz + 20.0 * (double)f.g.n : -1.0;
+    return phase_nnz >= 0 ? 4.0 * (double)phase_nnz + 68.0 * (double)f.g.n : -1.0;
 }
 
-static int coop_supported() {
-    static int ok = -1;
-    if (ok < 0) {
-        int dev = 0, v = 0;
-        ok = (cudaGetDevice(&dev) == cudaSuccess &&
-              cudaDeviceGetAttribute(&v, cudaDevAttrCooperativeLaunch, dev) == cudaSuccess && v)
-                 ? 1
-                 : 0;
-    }
-    return ok;
-}
-
-// default driver: every level in one persistent cooperative launch
-static int jp_run_levels(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
-                         const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n,
-                         int phase) {
+// every level in one persistent cooperative launch
+static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
+                  const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n, int phase) {
     Ctl *ctl = f.ctl;
     cudaStream_t s = f.stream;
-    JpTask *tq[2] = {reinterpret_cast<JpTask *>(w.task), reinterpret_cast<JpTask *>(w.task) + w.queue_cap};
-    SYM_CUDA(cudaMemsetAsync(w.sync, 0, 64 * sizeof(uint32_t), s));
-    JpArgs A;
-    SYM_TRY(jp_init(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n, tq[0]));
-    A.hist = f.stats ? ctl->hist + phase * 2048 : nullptr;
-    JlCtl C;
-    C.ring = ctl->ring;
-    C.bar = &w.sync[0];
-    C.err = &w.sync[32];
-    C.levels = &w.sync[33];
-    C.tq0 = tq[0];
-    C.tq1 = tq[1];
-    C.max_levels = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
     static int grid = 0;
     if (grid == 0) {
-        int per_sm = 0;
+        int dev = 0, coop = 0, per_sm = 0;
+        SYM_CUDA(cudaGetDevice(&dev));
+        SYM_CUDA(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev));
+        if (!coop) {
+            set_error("JP needs cooperative launch (persistent levels kernel), unsupported on this device");
+            return SYM_ECUDA;
+        }
         SYM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_jp_levels, JL_THREADS, 0));
         if (per_sm < 1) {
             set_error("k_jp_levels does not fit on an SM");
@@ -744,6 +720,26 @@ static int jp_run_levels(const FlowArgs &f, ColorWs &w, uint32_t *color, const i
         }
         grid = num_sms() * per_sm;
     }
+    JpTask *q = reinterpret_cast<JpTask *>(w.task);
+    const int64_t qcap = 2 * w.queue_cap;  // >= n + nnz/JP_CHUNK: every vertex is enqueued once
+    if (qcap >= (int64_t)0xffffffff) {
+        set_error("JP task queue exceeds 2^32 entries");
+        return SYM_EINVAL;
+    }
+    // W (u64) = sync[0..1], G (u64) = sync[2..3], err = sync[32], levels = sync[33]
+    SYM_CUDA(cudaMemsetAsync(w.sync, 0, 64 * sizeof(uint32_t), s));
+    SYM_CUDA(cudaMemsetAsync(q, 0xff, sizeof(JpTask) * (size_t)qcap, s));
+    JlCtl C;
+    C.W = reinterpret_cast<unsigned long long *>(w.sync);
+    C.G = reinterpret_cast<unsigned long long *>(w.sync + 2);
+    C.err = &w.sync[32];
+    C.levels = &w.sync[33];
+    C.max_levels = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
+    // arrivals (levels x grid) must not overflow the high half of W
+    C.max_levels = std::min<uint64_t>(C.max_levels, 0xffffffffull / (uint64_t)grid - 1);
+    JpArgs A;
+    SYM_TRY(jp_init(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n, q, w.sync /* low half of W */));
+    A.hist = f.stats ? ctl->hist + phase * 2048 : nullptr;
     void *args[] = {&A, &C};
     prof_begin("jp_levels", s);
     SYM_CUDA(cudaLaunchCooperativeKernel((const void *)k_jp_levels, dim3(grid), dim3(JL_THREADS), args, 0, s));
@@ -761,53 +757,6 @@ static int jp_run_levels(const FlowArgs &f, ColorWs &w, uint32_t *color, const i
         f.stats->rounds[phase] = levels;
     }
     return SYM_OK;
-}
-
-// fallback: one k_jp_push launch per level, host polls in growing batches
-static int jp_run_rounds(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
-                         const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n,
-                         int phase) {
-    Ctl *ctl = f.ctl;
-    cudaStream_t s = f.stream;
-    JpTask *tq[2] = {reinterpret_cast<JpTask *>(w.task), reinterpret_cast<JpTask *>(w.task) + w.queue_cap};
-    JpArgs A;
-    SYM_TRY(jp_init(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n, tq[0]));
-    A.hist = f.stats ? ctl->hist + phase * 2048 : nullptr;
-    const uint32_t maxr = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
-    const int grid = num_sms() * 2;  // frontiers are small: a short grid launches and drains fast
-    int r = 0, batch = 8;
-    for (;;) {
-        for (int bb = 0; bb < batch; bb++, r++) {
-            A.tin = tq[r & 1];
-            A.in_cnt = &ctl->ring[r % 3];
-            A.tout = tq[(r + 1) & 1];
-            A.out_cnt = &ctl->ring[(r + 1) % 3];
-            A.clear_cnt = &ctl->ring[(r + 2) % 3];
-            A.round = r;
-            prof_begin("jp_push", s);
-            k_jp_push<<<grid, JP_THREADS, 0, s>>>(A);
-            prof_end(s, -1);
-            SYM_LAUNCH_CHECK();
-        }
-        uint32_t left = 0;
-        SYM_TRY(read_u32(&ctl->ring[r % 3], &left, s));
-        if (left == 0) break;
-        if ((uint32_t)r >= maxr) {
-            set_error("JP did not converge within max_rounds");
-            return SYM_EROUNDS;
-        }
-        if (batch < 256) batch *= 2;
-    }
-    if (f.stats) f.stats->rounds[phase] = (uint32_t)r;
-    return SYM_OK;
-}
-
-static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
-                  const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n, int phase) {
-    const char *mode = getenv("SYM_JP_MODE");
-    if ((mode && mode[0] == 'r') || !coop_supported())
-        return jp_run_rounds(f, w, color, rp, ci, inS, list0, cnt0, implicit_n, phase);
-    return jp_run_levels(f, w, color, rp, ci, inS, list0, cnt0, implicit_n, phase);
 }
 
 int run_color(const FlowArgs &f, ColorWs &w, uint32_t *color) {
