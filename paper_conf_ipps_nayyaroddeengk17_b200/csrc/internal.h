@@ -161,13 +161,21 @@ struct MmWs {
 };
 
 struct ColorWs {
-    uint8_t *rec = nullptr;        // 32-B per-vertex records (count, degree, row, colours 1..128)
-    uint32_t *bits = nullptr;      // overflow forbidden-colour bitmaps, (deg+1) bits per vertex
-    int64_t bits_words = 0;
-    int64_t *queue = nullptr;      // init pass: (piece << 32 | v) items of the huge rows
+    int32_t *cid = nullptr;        // original -> compact id (S vertices with phase arcs)
+    int32_t *ov = nullptr;         // compact id -> original
+    uint32_t *ldeg = nullptr;      // lower degrees (build) / fill cursors
+    uint32_t *rfull = nullptr;     // bitmap words per compact vertex
+    uint32_t *ccol = nullptr;      // colours by compact id
+    unsigned long long *rec = nullptr;  // 8-B records: count | R << 24 | bitmap offset << 32
+    uint32_t *seg = nullptr;       // per compact vertex: forbidden-colour bitmap + lower list
+    int64_t seg_words = 0;
+    uint32_t *tcnt = nullptr;      // build scan scratch (per tile)
+    unsigned long long *tsum = nullptr;
+    int64_t ntiles = 0;
+    int64_t *queue = nullptr;      // build: (piece << 32 | h) items of the huge rows
     int32_t *vlist = nullptr;
     uint8_t *mark = nullptr;       // COLOR-RAND V'
-    int64_t *task = nullptr;       // two task lists (ping-pong), queue_cap each
+    int64_t *task = nullptr;       // the task queue, queue_cap tasks
     int64_t queue_cap = 0;
     uint32_t *sync = nullptr;      // levels kernel: barrier / error / level-count words
 };
