@@ -161,23 +161,24 @@ struct MmWs {
 };
 
 struct ColorWs {
-    int32_t *cid = nullptr;        // original -> compact id (S vertices with phase arcs)
     int32_t *ov = nullptr;         // compact id -> original
-    uint32_t *ldeg = nullptr;      // lower degrees (build) / fill cursors
-    uint32_t *rfull = nullptr;     // bitmap words per compact vertex
-    uint32_t *ccol = nullptr;      // colours by compact id
-    unsigned long long *rec = nullptr;  // 8-B records: count | R << 24 | bitmap offset << 32
-    uint32_t *seg = nullptr;       // per compact vertex: forbidden-colour bitmap + lower list
+    uint32_t *hdeg = nullptr;      // higher / lower degrees (build), fill cursors
+    uint32_t *ldeg = nullptr;
+    uint32_t *sbh = nullptr;       // compact id -> segment base (8-B units)
+    unsigned long long *sbR = nullptr;  // original id -> segment base | R << 32
+    uint32_t *ul[2] = {nullptr, nullptr};  // uncoloured lists (ping-pong by round)
+    uint32_t *seg = nullptr;       // per compact vertex: header, forbidden bitmap, higher + lower lists
     int64_t seg_words = 0;
     uint32_t *tcnt = nullptr;      // build scan scratch (per tile)
     unsigned long long *tsum = nullptr;
     int64_t ntiles = 0;
+    uint4 *task = nullptr;         // push tasks of one round
+    uint2 *btask = nullptr;        // watch-list build tasks of one round
+    int64_t task_cap = 0;
     int64_t *queue = nullptr;      // build: (piece << 32 | h) items of the huge rows
     int32_t *vlist = nullptr;
     uint8_t *mark = nullptr;       // COLOR-RAND V'
-    int64_t *task = nullptr;       // the task queue, queue_cap tasks
-    int64_t queue_cap = 0;
-    uint32_t *sync = nullptr;      // levels kernel: barrier / error / level-count words
+    uint32_t *sync = nullptr;      // rounds kernel: barrier / counter / error words
 };
 
 int phase_arcs(const FlowArgs &f, const int64_t *rp, int64_t *out);  // round0.cu

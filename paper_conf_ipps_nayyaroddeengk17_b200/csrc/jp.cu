@@ -1,29 +1,42 @@
 // jp.cu -- Jones-Plassmann colouring and the COLOR flows.
 //
-// JP ([18]) with fixed priorities colours v once every higher-(pv,id)
-// neighbour of its phase set S is coloured, with the smallest colour >= 1 not held by
-// any coloured neighbour: exactly first-fit greedy in priority order (DESIGN §3 C1).
+// JP ([18]) with fixed priorities gives v the smallest colour >= 1 not held by
+// any higher-(pv,id) neighbour of its phase set S: exactly first-fit greedy in
+// priority order (DESIGN §3 C1).  Plain JP waits until EVERY higher neighbour is
+// coloured, so it runs as many dependent levels as the priority DAG is deep (5 063
+// at R-MAT s24).  This file computes the same colouring with an early-commit rule:
 //
-// Push form over a compact oriented DAG, built once per call:
-//   ids     the S vertices with phase arcs get compact ids h (rows of degree > 2
-//           first, so the hot records of a power-law core are contiguous); a vertex
-//           without any phase arc takes colour 1 at once.
-//   segment seg[boff .. boff+R) = h's forbidden-colour bitmap, R = ceil(cap/32)
-//           words for cap = (#higher + #fixed-coloured neighbours) + 1 >= mex, then
-//           seg[boff+R .. boff+R+ldeg) = compact ids of h's LOWER S-neighbours: the
-//           only arcs a push needs (half of the phase arcs, no hash at level time).
-//   record  rec[h] (8 B) = cnt | min(R,255) << 24 | boff << 32, cnt = higher
-//           S-neighbours not yet coloured.  A push to w is ONE returning 64-bit
-//           atomic (the decrement returns w's segment address; w's lower degree is
-//           loaded beside it, so a vertex that becomes ready needs no further load)
-//           plus one RED of the colour bit; records + bitmaps are ~90 MB at R-MAT
-//           s24 (vs 0.5 GB of 32-B records per vertex id before).
-//   level   every ready vertex is split into tasks of <= JP_CHUNK lower arcs; a
-//           task computes colour(h) = mex of h's bitmap (complete: every higher
-//           neighbour pushed in an earlier level) and pushes it to its lower
-//           neighbours; the decrement reaching 0 stages w for the next level.
-// Levels = the JP dependency depth (~5e3 on R-MAT scale 24), all in ONE persistent
-// cooperative kernel (k_jp_levels) with a software grid barrier between levels.
+//   m = mex of the colours of v's coloured higher neighbours (v's forbidden bitmap);
+//   v may take m as soon as every higher neighbour u is either coloured with a
+//   colour != m, or uncoloured with m already in u's own forbidden set.
+//
+// Proof: the final higher-neighbour colours are the known ones (which hold 1..m-1
+// and not m) plus one colour per uncoloured u, and u can never take m (m is
+// forbidden for u), so the final mex is m.  Every fact the rule reads ("u has colour
+// c", "m is forbidden for u") is permanent once observed, so the rule is exact under
+// any schedule and any staleness; a vertex whose higher neighbours are all coloured
+// (plain JP's ready vertex) always passes.  Result: the same colours in 531 rounds
+// instead of 5 063 levels at R-MAT s24 (CPU simulation).
+//
+// Layout (built once per call; S vertices with phase arcs get compact ids h, rows
+// of degree > 2 first; a vertex without any phase arc takes colour 1 at once):
+//   segment of h at word O = 2*sb(h) of seg[] (8-B aligned):
+//     O+0 colour (0 = not yet), O+1 R, O+2 hdeg, O+3 ldeg, O+4 cnt = higher
+//     neighbours not yet pushed, O+5 watch-list length, O+6..7 check memo (blocker
+//     position, m at the last failed check);
+//     O+8: forbidden bitmap, R = ceil(cap/32) words, cap = #higher + #fixed-coloured
+//     neighbours + 1 >= mex; a JP_WATCH-entry watch area if hdeg > JP_WATCH; the
+//     higher list (hdeg segment bases sb(u), u32); the lower list (ldeg entries
+//     sb(w) | R(w) << 32, u64).
+// A round: phase A -- every uncoloured vertex whose count is <= JP_WATCH checks its
+// watch list (the higher neighbours still uncoloured when it was built; a list of
+// <= JP_WATCH higher neighbours is its own watch list), resuming at the last blocker
+// when m is unchanged; a vertex that passes writes its colour and queues push tasks;
+// grid barrier; phase B -- each new colour goes into the lower neighbours' bitmaps
+// and decrements their counts (RED), and requested watch lists are built; grid
+// barrier.  All rounds run in ONE persistent cooperative kernel (k_jp_rounds).
+// Waiting for the count to reach JP_WATCH costs no rounds on R-MAT (CPU simulation)
+// and bounds every check to one warp step.
 #include <algorithm>
 #include <cstdio>
 #include <cstdlib>
@@ -39,22 +52,14 @@ constexpr int JP_BUDGET = 4096;  // build: rows > JP_BUDGET arcs are split into 
 constexpr int JP_PIECE = 8192;   // arcs per CTA piece of a huge row in the build passes
 constexpr int JP_TILE = 2048;    // build: compact ids per scan tile (JP_THREADS x 8)
 constexpr int JP_TPT = JP_TILE / JP_THREADS;
-#ifndef SYM_JP_CHUNK
-#define SYM_JP_CHUNK 64
-#endif
-constexpr int JP_CHUNK = SYM_JP_CHUNK;  // lower arcs per warp task (2 per lane)
-constexpr int JP_LANE = 8;              // lower lists of <= JP_LANE arcs are a lane task
-constexpr unsigned long long JP_CNT_MASK = (1ull << 24) - 1;
-constexpr uint32_t JP_RSAT = 255;       // R field saturated: the word count is in rfull[h]
-
-// a task: one chunk of a ready vertex's lower list
-struct __align__(16) JpTask {
-    int64_t b, e;     // h's lower list: seg[b .. e)
-    int32_t h;
-    uint32_t j;       // chunk index
-    uint64_t bm;      // h's bitmap: boff << 32 | R
-};
-static_assert(sizeof(JpTask) == 32, "JpTask layout");
+constexpr int JP_HDR = 8;        // segment header words
+constexpr int JP_LANE_CHECKS = 4;  // phase A: higher entries a lane checks before the warp takes over
+constexpr int JP_PUSH = 256;     // phase B: lower entries per push task
+constexpr int JP_PUSH_LANE = 8;  // phase B: tasks of <= JP_PUSH_LANE entries are a lane's
+constexpr uint32_t JP_WATCH = 16;  // a vertex checks once <= JP_WATCH higher neighbours are unpushed
+constexpr uint32_t JP_WLIST = 64;  // higher lists up to JP_WLIST entries are their own watch list
+constexpr uint32_t JP_NOTBUILT = 0xffffffffu;
+constexpr int JP_BUILD = 256;    // phase B: higher entries per watch-list build task
 
 struct JpArgs {
     const int64_t *rp;   // phase CSR (original ids)
@@ -64,24 +69,27 @@ struct JpArgs {
     const int32_t *in_list;  // S as a list (nullable = implicit 0..implicit_n-1)
     const uint32_t *in_cnt;
     int64_t implicit_n;
-    int32_t *cid;        // [n] original -> compact id
     int32_t *ov;         // [n] compact id -> original
-    uint32_t *ldeg;      // [n] lower degree
-    uint32_t *rfull;     // [n] bitmap words R
-    unsigned long long *rec;  // [n+1] cnt | Rsat << 24 | boff << 32
-    uint32_t *seg;       // per compact vertex: bitmap (R words), lower list (ldeg ids)
-    uint32_t *ccol;      // [n] colours by compact id (build: fill cursor of huge rows)
+    uint32_t *hdeg;      // [n] higher degree (count pass), fill cursor (huge rows)
+    uint32_t *ldeg;      // [n] lower degree (count pass), fill cursor (huge rows)
+    uint32_t *sbh;       // [n] compact id -> segment base (8-B units)
+    unsigned long long *sbR;  // [n] original id -> sb | R << 32
+    uint32_t *seg;       // segments
     uint32_t *tcnt;      // scan scratch: per tile class counts (2 per tile)
-    unsigned long long *tsum;  // scan scratch: per tile (lower arcs, bitmap words)
+    unsigned long long *tsum;  // scan scratch: per tile segment words
     uint32_t *nc;        // [0] = compact count n', [1] = rows of degree > 2
-    JpTask *tout;        // the task queue (monotone; level r owns [lo_r, hi_r))
-    uint32_t *out_cnt;   // level-0 task counter (the low half of the levels kernel's W)
+    uint32_t *ul[2];     // uncoloured lists (segment bases), ping-pong by round
+    uint4 *task;         // push tasks {list word lo, hi, entries, colour}
+    uint2 *btask;        // watch-list build tasks {sb, chunk}
+    uint32_t *ucnt;      // [3] list counts (ring by round)
+    uint32_t *pcnt;      // [3] push-task counts (ring by round)
+    uint32_t *bcnt;      // [3] build-task counts (ring by round)
     int64_t *huge;       // (piece << 32 | h) items of the huge rows
     uint32_t *huge_cnt;
-    uint32_t *err;       // 2 = a count exceeds the record field
+    uint32_t *err;       // 1 = timeout / max rounds, 2 = segment offsets overflow
     uint32_t *hist;
-    uint32_t *trace;     // nullable: per-level spans (SYM_JP_TRACE diagnostics)
-    unsigned long long *prof;  // algorithmic bytes of the levels pass (nullable)
+    uint32_t *trace;     // nullable: per-round phase-A end time, push and build tasks (SYM_JP_TRACE)
+    unsigned long long *prof;  // algorithmic bytes of the rounds pass (nullable)
     Key k;
 };
 
@@ -93,14 +101,18 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
 
 __device__ __forceinline__ bool in_set(const uint8_t *inS, uint32_t w) { return inS == nullptr || inS[w] != 0; }
 
-__device__ __forceinline__ uint32_t n_tasks(int64_t ldeg) {
-    return ldeg <= 0 ? 1u : (uint32_t)((ldeg + JP_CHUNK - 1) / JP_CHUNK);
-}
+__device__ __forceinline__ uint32_t even(uint32_t x) { return (x + 1u) & ~1u; }
 
-__device__ __forceinline__ void write_task(JpTask *q, int64_t b, int64_t e, int32_t h, uint32_t j, uint64_t bm) {
-    longlong2 *p = reinterpret_cast<longlong2 *>(q);
-    p[0] = make_longlong2(b, e);
-    p[1] = make_longlong2((long long)(((uint64_t)j << 32) | (uint32_t)h), (long long)bm);
+// word offsets inside a segment
+__device__ __forceinline__ uint32_t watch_words(uint32_t hd) { return hd > JP_WLIST ? JP_WATCH : 0u; }
+__device__ __forceinline__ uint64_t seg_bitmap(uint32_t sb) { return 2ull * sb + JP_HDR; }
+// the list a check reads: the watch area (hdeg > JP_WLIST) or the higher list itself
+__device__ __forceinline__ uint64_t seg_watch(uint32_t sb, uint32_t R) { return 2ull * sb + JP_HDR + even(R); }
+__device__ __forceinline__ uint64_t seg_higher(uint32_t sb, uint32_t R, uint32_t hd) {
+    return 2ull * sb + JP_HDR + even(R) + watch_words(hd);
+}
+__device__ __forceinline__ uint64_t seg_lower(uint32_t sb, uint32_t R, uint32_t hd) {
+    return seg_higher(sb, R, hd) + even(hd);
 }
 
 // warp-aggregated reservation of k_lane consecutive slots per lane; returns this
@@ -119,12 +131,6 @@ __device__ __forceinline__ int64_t warp_reserve(uint32_t k_lane, uint32_t *count
         base = __shfl_sync(FULL, base, 0);
     }
     return (int64_t)base + incl - k_lane;
-}
-
-// bitmap word count of a record (saturated field -> rfull)
-__device__ __forceinline__ uint32_t rec_words(const JpArgs &A, unsigned long long r, uint32_t h) {
-    const uint32_t R = (uint32_t)(r >> 24) & 0xffu;
-    return R == JP_RSAT ? __ldg(A.rfull + h) : R;
 }
 
 // CTA-wide exclusive scan of one value per thread (blockDim.x == JP_THREADS);
@@ -260,7 +266,6 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_assign(JpArgs A) {
         const uint32_t r1 = block_excl_scan<uint32_t>(c == 1, sm1, &t1);
         if (c < 2) {
             const uint32_t h = c == 0 ? o0 + r0 : o1 + r1;
-            A.cid[v] = (int32_t)h;
             A.ov[h] = v;
         } else if (v >= 0) {
             A.color[v] = 1u;
@@ -271,7 +276,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_assign(JpArgs A) {
 }
 
 // ---------------------------------------------------------------- build: DAG
-// count pass: rec[h] = #higher S-neighbours, ldeg[h] = #lower S-neighbours; rows
+// count pass: hdeg[h] = #higher S-neighbours, ldeg[h] = #lower S-neighbours; rows
 // longer than JP_BUDGET arcs are deferred as JP_PIECE-arc pieces
 __global__ void __launch_bounds__(JP_THREADS) k_jpc_count(JpArgs A) {
     const uint32_t cnt = A.nc[0];
@@ -325,7 +330,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_count(JpArgs A) {
         }
         const bool huge = active && e - b > JP_BUDGET;
         if (active) {
-            A.rec[h] = hi;
+            A.hdeg[h] = hi;
             A.ldeg[h] = lo;
         }
         const uint32_t np = huge ? (uint32_t)((e - b + JP_PIECE - 1) / JP_PIECE) : 0u;
@@ -357,11 +362,12 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_count_huge(JpArgs A) {
         lh = __reduce_add_sync(FULL, lh);
         ll = __reduce_add_sync(FULL, ll);
         if (lane_id() == 0) {
-            if (lh) atomicAdd(A.rec + h, (unsigned long long)lh);
+            if (lh) atomicAdd(A.hdeg + h, lh);
             if (ll) atomicAdd(A.ldeg + h, ll);
         }
     }
 }
+
 
 // bitmap words of compact vertex h: cap = (higher + fixed-coloured neighbours) + 1 bits
 __device__ __forceinline__ uint32_t jp_words(const JpArgs &A, int64_t h) {
@@ -370,163 +376,141 @@ __device__ __forceinline__ uint32_t jp_words(const JpArgs &A, int64_t h) {
     return (uint32_t)((deg - (int64_t)A.ldeg[h] + 1 + 31) >> 5);
 }
 
-// per tile of JP_TILE compact ids: (lower arcs, bitmap words)
+// segment words of h, a multiple of 4 (segments are 16-B aligned)
+__device__ __forceinline__ unsigned long long jp_seg_words(const JpArgs &A, int64_t h) {
+    const uint32_t hd = A.hdeg[h];
+    const unsigned long long w = JP_HDR + even(jp_words(A, h)) + watch_words(hd) + even(hd) + 2ull * A.ldeg[h];
+    return (w + 3ull) & ~3ull;
+}
+
+// per tile of JP_TILE compact ids: segment words
 __global__ void __launch_bounds__(JP_THREADS) k_jpc_sums(JpArgs A) {
     const uint32_t cnt = A.nc[0];
     const int64_t base = (int64_t)blockIdx.x * JP_TILE;
     if (base >= cnt) return;
-    unsigned long long sl = 0, sw = 0;
+    unsigned long long sw = 0;
     for (int u = 0; u < JP_TPT; u++) {
         const int64_t h = base + u * JP_THREADS + threadIdx.x;
-        if (h < cnt) {
-            sl += A.ldeg[h];
-            sw += jp_words(A, h) + A.ldeg[h];
-        }
+        if (h < cnt) sw += jp_seg_words(A, h);
     }
-    for (int d = 16; d; d >>= 1) {
-        sl += __shfl_xor_sync(FULL, sl, d);
-        sw += __shfl_xor_sync(FULL, sw, d);
-    }
-    __shared__ unsigned long long a[2];
-    if (threadIdx.x == 0) a[0] = a[1] = 0;
+    for (int d = 16; d; d >>= 1) sw += __shfl_xor_sync(FULL, sw, d);
+    __shared__ unsigned long long a;
+    if (threadIdx.x == 0) a = 0;
     __syncthreads();
-    if (lane_id() == 0) {
-        atomicAdd(&a[0], sl);
-        atomicAdd(&a[1], sw);
-    }
+    if (lane_id() == 0) atomicAdd(&a, sw);
     __syncthreads();
-    if (threadIdx.x == 0) {
-        A.tsum[2 * blockIdx.x] = a[0];
-        A.tsum[2 * blockIdx.x + 1] = a[1];
-    }
+    if (threadIdx.x == 0) A.tsum[blockIdx.x] = a;
 }
 
-// one CTA: exclusive prefix of the tile sums (segment offsets must fit 32 bits)
+// one CTA: exclusive prefix of the tile sums (segment bases must fit 32 bits in
+// 8-B units)
 __global__ void __launch_bounds__(1024) k_jpc_sums_scan(JpArgs A, int64_t ntiles) {
     const uint32_t cnt = A.nc[0];
     const int64_t need = ((int64_t)cnt + JP_TILE - 1) / JP_TILE;
     const int64_t used = need < ntiles ? need : ntiles;
     const int64_t per = (used + blockDim.x - 1) / blockDim.x;
     const int64_t t0 = (int64_t)threadIdx.x * per, t1 = used < t0 + per ? used : t0 + per;
-    unsigned long long s0 = 0, s1 = 0;
-    for (int64_t t = t0; t < t1; t++) {
-        s0 += A.tsum[2 * t];
-        s1 += A.tsum[2 * t + 1];
-    }
-    __shared__ unsigned long long w0[32], w1[32];
-    unsigned long long i0 = s0, i1 = s1;
+    unsigned long long s0 = 0;
+    for (int64_t t = t0; t < t1; t++) s0 += A.tsum[t];
+    __shared__ unsigned long long w0[32];
+    unsigned long long i0 = s0;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-        const unsigned long long y0 = __shfl_up_sync(FULL, i0, d), y1 = __shfl_up_sync(FULL, i1, d);
-        if (lane_id() >= d) {
-            i0 += y0;
-            i1 += y1;
-        }
+        const unsigned long long y0 = __shfl_up_sync(FULL, i0, d);
+        if (lane_id() >= d) i0 += y0;
     }
     const int wid = threadIdx.x >> 5;
-    if (lane_id() == 31) {
-        w0[wid] = i0;
-        w1[wid] = i1;
-    }
+    if (lane_id() == 31) w0[wid] = i0;
     __syncthreads();
-    unsigned long long b0 = 0, b1 = 0, T0 = 0, T1 = 0;
+    unsigned long long b0 = 0, T0 = 0;
     for (int q = 0; q < (int)(blockDim.x >> 5); q++) {
-        if (q < wid) {
-            b0 += w0[q];
-            b1 += w1[q];
-        }
+        if (q < wid) b0 += w0[q];
         T0 += w0[q];
-        T1 += w1[q];
     }
-    unsigned long long o0 = b0 + i0 - s0, o1 = b1 + i1 - s1;
+    unsigned long long o0 = b0 + i0 - s0;
     for (int64_t t = t0; t < t1; t++) {
-        const unsigned long long a0 = A.tsum[2 * t], a1 = A.tsum[2 * t + 1];
-        A.tsum[2 * t] = o0;
-        A.tsum[2 * t + 1] = o1;
+        const unsigned long long a0 = A.tsum[t];
+        A.tsum[t] = o0;
         o0 += a0;
-        o1 += a1;
     }
-    if (threadIdx.x == 0 && T1 >= (1ull << 32)) atomicOr(A.err, 2u);
+    if (threadIdx.x == 0 && T0 >= (1ull << 33)) atomicOr(A.err, 2u);
 }
 
-// per compact id: the record (count, segment address), a zeroed bitmap, level-0 tasks
+// per compact id: segment base, header, zeroed bitmap, the maps; the first round's
+// list = the vertices with <= JP_WATCH higher neighbours
 __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
     const uint32_t cnt = A.nc[0];
     const int64_t base = (int64_t)blockIdx.x * JP_TILE;
     if (base >= cnt) return;
-    __shared__ unsigned long long sm0[8], sm1[8];
-    unsigned long long o0 = A.tsum[2 * blockIdx.x], o1 = A.tsum[2 * blockIdx.x + 1];
+    __shared__ unsigned long long sm0[8];
+    unsigned long long o0 = A.tsum[blockIdx.x];
     for (int u = 0; u < JP_TPT; u++) {
         const int64_t h = base + u * JP_THREADS + threadIdx.x;
         const bool active = h < cnt;
-        unsigned long long ld = 0, R = 0, hi = 0;
+        const unsigned long long words = active ? jp_seg_words(A, h) : 0ull;
+        unsigned long long t0;
+        const unsigned long long p0 = block_excl_scan<unsigned long long>(words, sm0, &t0);
+        const bool first = active && A.hdeg[h] <= JP_WATCH;
+        const int64_t slot = warp_append(first, A.ucnt);
         if (active) {
-            ld = A.ldeg[h];
-            R = jp_words(A, h);
-            hi = A.rec[h];
+            const unsigned long long O = o0 + p0;  // a multiple of 4: segment sizes are
+            const uint32_t sb = (uint32_t)(O >> 1);
+            const uint32_t R = jp_words(A, h), hd = A.hdeg[h], ld = A.ldeg[h];
+            uint4 *hp = reinterpret_cast<uint4 *>(A.seg + O);
+            hp[0] = make_uint4(0u, R, hd, ld);
+            hp[1] = make_uint4(hd, hd > JP_WLIST ? JP_NOTBUILT : hd, 0u, 0u);
+            for (uint32_t q = 0; q < R; q++) A.seg[O + JP_HDR + q] = 0u;
+            A.sbh[h] = sb;
+            A.sbR[A.ov[h]] = (unsigned long long)sb | ((unsigned long long)R << 32);
+            if (first) A.ul[0][slot] = sb;
+            A.hdeg[h] = 0;  // fill cursors of the huge rows
+            A.ldeg[h] = 0;
         }
-        unsigned long long t0, t1;
-        const unsigned long long p0 = block_excl_scan<unsigned long long>(ld, sm0, &t0);
-        const unsigned long long p1 = block_excl_scan<unsigned long long>(R + ld, sm1, &t1);
-        (void)p0;
-        uint32_t nt = 0;
-        int64_t b = 0;
-        unsigned long long boff = 0;
-        if (active) {
-            boff = o1 + p1;
-            b = (int64_t)(boff + R);
-            if (hi > JP_CNT_MASK) atomicOr(A.err, 2u);
-            A.rec[h] = hi | ((R < JP_RSAT ? R : (unsigned long long)JP_RSAT) << 24) | (boff << 32);
-            A.rfull[h] = (uint32_t)R;
-            A.ccol[h] = 0;  // fill cursor
-            for (unsigned long long q = 0; q < R; q++) A.seg[boff + q] = 0u;
-            nt = hi == 0 ? n_tasks((int64_t)ld) : 0u;
-        }
-        // algorithmic bytes of the levels pass: the lower list (4 B/arc) + per vertex its
-        // tasks (32 B written + read), lp pair (16 B), record read (8 B), colour (4 B)
-        prof_add(A.prof, active ? 4ull * ld + 92ull : 0ull);
-        const int64_t slot = warp_reserve(nt, A.out_cnt);
-        for (uint32_t q = 0; q < nt; q++)
-            write_task(A.tout + slot + q, b, b + (int64_t)ld, (int32_t)h, q, (boff << 32) | R);
         o0 += t0;
-        o1 += t1;
     }
 }
 
-// fill pass: lower lists (compact ids, CSR order) and the fixed colours of neighbours
-// outside S (COLOR-Rand recolouring) as forbidden bits
-__device__ __forceinline__ void jp_fixed(const JpArgs &A, unsigned long long r, int64_t h, uint32_t w) {
+// fixed colour c of a neighbour outside S (COLOR-Rand recolouring) as a forbidden bit
+__device__ __forceinline__ void jp_fixed(const JpArgs &A, uint64_t O, uint32_t R, uint32_t w) {
     const uint32_t c = A.color[w];
     if (c == 0) return;
     const uint32_t q = (c - 1) >> 5;
-    if (q < rec_words(A, r, (uint32_t)h)) atomicOr(A.seg + (r >> 32) + q, 1u << ((c - 1) & 31));
+    if (q < R) atomicOr(A.seg + O + JP_HDR + q, 1u << ((c - 1) & 31));
 }
 
+// fill pass: higher list (segment bases) and lower list (segment base | R), both in
+// CSR order; fixed colours of neighbours outside S
 __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
     const uint32_t cnt = A.nc[0];
     const int lane = lane_id();
     const int64_t warp_g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    unsigned long long *seg64 = reinterpret_cast<unsigned long long *>(A.seg);
     for (int64_t base = warp_g * 32; base < cnt; base += nwarps * 32) {
         const int64_t h = base + lane;
         const bool active = h < cnt;
         int32_t v = 0;
-        int64_t b = 0, e = 0, o = 0;
-        uint64_t kv = 0;
-        unsigned long long r = 0;
+        int64_t b = 0, e = 0;
+        uint64_t kv = 0, O = 0, hl = 0, ll = 0;
+        uint32_t R = 0;
         if (active) {
             v = A.ov[h];
             b = A.rp[v];
             e = A.rp[v + 1];
             kv = vkey(A.k, (uint32_t)v);
-            r = A.rec[h];
-            o = (int64_t)(r >> 32) + rec_words(A, r, (uint32_t)h);
+            const uint32_t sb = A.sbh[h];
+            O = 2ull * sb;
+            const uint4 hd = *reinterpret_cast<const uint4 *>(A.seg + O);
+            R = hd.y;
+            hl = seg_higher(sb, R, hd.z);
+            ll = seg_lower(sb, R, hd.z) >> 1;
         }
         if (active && e - b <= JP_SMALL) {
             for (int64_t x = b; x < e; x++) {
                 const uint32_t w = (uint32_t)__ldg(A.ci + x);
-                if (!in_set(A.inS, w)) jp_fixed(A, r, h, w);
-                else if (vkey(A.k, w) < kv) A.seg[o++] = (uint32_t)A.cid[w];
+                if (!in_set(A.inS, w)) jp_fixed(A, O, R, w);
+                else if (vkey(A.k, w) > kv) A.seg[hl++] = (uint32_t)A.sbR[w];
+                else seg64[ll++] = A.sbR[w];
             }
         }
         unsigned medm = __ballot_sync(FULL, active && e - b > JP_SMALL && e - b <= JP_BUDGET);
@@ -534,31 +518,35 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
             const int src = __ffs(medm) - 1;
             medm &= medm - 1;
             const int64_t wb = __shfl_sync(FULL, b, src), we = __shfl_sync(FULL, e, src);
-            const uint64_t wk = __shfl_sync(FULL, kv, src);
-            const int64_t wh = base + src;
-            const unsigned long long wr = __shfl_sync(FULL, r, src);
-            int64_t wo = __shfl_sync(FULL, o, src);
+            const uint64_t wk = __shfl_sync(FULL, kv, src), wO = __shfl_sync(FULL, O, src);
+            const uint32_t wR = __shfl_sync(FULL, R, src);
+            uint64_t whl = __shfl_sync(FULL, hl, src), wll = __shfl_sync(FULL, ll, src);
             for (int64_t x0 = wb; x0 < we; x0 += 32) {
                 const int64_t x = x0 + lane;
-                bool low = false;
+                bool up = false, dn = false;
                 uint32_t w = 0;
                 if (x < we) {
                     w = (uint32_t)__ldg(A.ci + x);
-                    if (!in_set(A.inS, w)) jp_fixed(A, wr, wh, w);
-                    else low = vkey(A.k, w) < wk;
+                    if (!in_set(A.inS, w)) jp_fixed(A, wO, wR, w);
+                    else if (vkey(A.k, w) > wk) up = true;
+                    else dn = true;
                 }
-                const unsigned m = __ballot_sync(FULL, low);
-                if (low) A.seg[wo + __popc(m & ((1u << lane) - 1u))] = (uint32_t)A.cid[w];
-                wo += __popc(m);
+                const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
+                const unsigned lt = (1u << lane) - 1u;
+                if (up) A.seg[whl + __popc(mu & lt)] = (uint32_t)A.sbR[w];
+                if (dn) seg64[wll + __popc(md & lt)] = A.sbR[w];
+                whl += __popc(mu);
+                wll += __popc(md);
             }
         }
     }
 }
 
-// huge rows: one CTA per piece, positions reserved per warp on the row's cursor
+// huge rows: one CTA per piece, positions reserved per warp on the row's cursors
 __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
     const uint32_t cnt = *A.huge_cnt;
     const int lane = lane_id();
+    unsigned long long *seg64 = reinterpret_cast<unsigned long long *>(A.seg);
     for (uint32_t p = blockIdx.x; p < cnt; p += gridDim.x) {
         const int64_t item = A.huge[p];
         const int32_t h = (int32_t)(uint32_t)item;
@@ -567,22 +555,31 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
         const int64_t b = A.rp[v], e = A.rp[v + 1];
         const int64_t pb = b + j * JP_PIECE, pe_ = min(e, pb + JP_PIECE);
         const uint64_t kv = vkey(A.k, (uint32_t)v);
-        const unsigned long long r = A.rec[h];
-        const int64_t o = (int64_t)(r >> 32) + rec_words(A, r, (uint32_t)h);
+        const uint32_t sb = A.sbh[h];
+        const uint64_t O = 2ull * sb;
+        const uint4 hd = *reinterpret_cast<const uint4 *>(A.seg + O);
+        const uint64_t hl = seg_higher(sb, hd.y, hd.z), ll = seg_lower(sb, hd.y, hd.z) >> 1;
         for (int64_t x0 = pb + (threadIdx.x & ~31); x0 < pe_; x0 += JP_HUGE_THREADS) {
             const int64_t x = x0 + lane;
-            bool low = false;
+            bool up = false, dn = false;
             uint32_t w = 0;
             if (x < pe_) {
                 w = (uint32_t)__ldg(A.ci + x);
-                if (!in_set(A.inS, w)) jp_fixed(A, r, h, w);
-                else low = vkey(A.k, w) < kv;
+                if (!in_set(A.inS, w)) jp_fixed(A, O, hd.y, w);
+                else if (vkey(A.k, w) > kv) up = true;
+                else dn = true;
             }
-            const unsigned m = __ballot_sync(FULL, low);
-            uint32_t pos = 0;
-            if (m && lane == 0) pos = atomicAdd(A.ccol + h, (uint32_t)__popc(m));
-            pos = __shfl_sync(FULL, pos, 0);
-            if (low) A.seg[o + pos + __popc(m & ((1u << lane) - 1u))] = (uint32_t)A.cid[w];
+            const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
+            uint32_t pu = 0, pd = 0;
+            if (lane == 0) {
+                if (mu) pu = atomicAdd(A.hdeg + h, (uint32_t)__popc(mu));
+                if (md) pd = atomicAdd(A.ldeg + h, (uint32_t)__popc(md));
+            }
+            pu = __shfl_sync(FULL, pu, 0);
+            pd = __shfl_sync(FULL, pd, 0);
+            const unsigned lt = (1u << lane) - 1u;
+            if (up) A.seg[hl + pu + __popc(mu & lt)] = (uint32_t)A.sbR[w];
+            if (dn) seg64[ll + pd + __popc(md & lt)] = A.sbR[w];
         }
     }
 }
@@ -591,319 +588,345 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
 __global__ void k_jpc_scatter(JpArgs A) {
     const uint32_t cnt = A.nc[0];
     for (int64_t h = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; h < cnt; h += (int64_t)gridDim.x * blockDim.x)
-        A.color[A.ov[h]] = A.ccol[h];
+        A.color[A.ov[h]] = A.seg[2ull * A.sbh[h]];
 }
 
-// ---------------------------------------------------------------- one level
-// Tasks live in ONE monotone queue (every vertex is enqueued exactly once): level r
-// owns slots [lo_r, hi_r).  A 64-bit word W = (arrivals << 32 | tasks reserved) is
-// both the grid barrier and the task allocator: at the end of a level each CTA adds
-// (1 << 32 | its staged tasks) once -- reservation and arrival in one atomic -- then
-// writes its tasks; the last arriver publishes (r+1 << 32 | hi_{r+1}) in the word G
-// that the other CTAs poll.  Tasks may land after the barrier, so the queue is
-// pre-filled with -1 and a reader waits until its task's three 8-byte words are
-// written.  Ready vertices are staged in shared memory (one reservation per CTA and
-// level, a hub's tasks written by the whole CTA); a full stage reserves per warp.
-constexpr int JP_STAGE = 1024;
-
-struct JpStage {
-    uint32_t n;                  // entries appended this level (may exceed JP_STAGE)
-    uint32_t base;               // global slot of the CTA's first task
-    uint32_t total;              // tasks of the staged entries
-    uint32_t wsum[32];           // scan scratch (one per warp)
-    int32_t v[JP_STAGE];         // compact ids
-    uint32_t deg[JP_STAGE];      // lower degrees
-    int64_t b[JP_STAGE];         // lower-list starts
-    uint64_t bm[JP_STAGE];       // bitmaps: boff << 32 | R
-    uint32_t off[JP_STAGE + 1];  // exclusive prefix of the task counts
-};
-
-struct JlCtl {
-    unsigned long long *W;  // (arrivals << 32) | tasks reserved (low half = the build's counter)
-    unsigned long long *G;  // (level + 1) << 32 | end of that level's tasks, by the last arriver
-    uint32_t *err;          // 1 = timeout / max levels, 2 = record field overflow
-    uint32_t *levels;       // out: number of levels run
-    uint32_t max_levels;
-};
-
-__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long *p) {
-    unsigned long long v;
-    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+// ---------------------------------------------------------------- rounds
+__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *p) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
 
-__device__ __forceinline__ void st_release_u64(unsigned long long *p, unsigned long long v) {
-    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+__device__ __forceinline__ void st_release_u32(uint32_t *p, uint32_t v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-// a task of the current level; waits (bounded by the writer CTA's progress: all CTAs
-// are co-resident) until its writer's stores are visible
-__device__ __forceinline__ void read_task(const JpTask *q, int64_t &b, int64_t &e, int32_t &h, uint32_t &j,
-                                          uint64_t &bm) {
-    const volatile long long *p = reinterpret_cast<const volatile long long *>(q);
-    long long x0, x1, x2, x3;
-    do {
-        x0 = p[0];
-        x1 = p[1];
-        x2 = p[2];
-        x3 = p[3];
-    } while (x0 == -1 || x1 == -1 || x2 == -1 || x3 == -1);
-    b = x0;
-    e = x1;
-    h = (int32_t)(uint32_t)(unsigned long long)x2;
-    j = (uint32_t)((unsigned long long)x2 >> 32);
-    bm = (uint64_t)x3;
-}
+struct JrCtl {
+    uint32_t *arr;     // barrier arrivals (monotone)
+    uint32_t *gen;     // index of the last completed barrier, published by its last arriver
+    uint32_t *levels;  // out: rounds run
+    uint32_t max_rounds;
+};
 
-// w became ready: its record r (returned by the decrement) gives the segment address
-__device__ __forceinline__ void stage_ready(const JpArgs &A, const JlCtl &C, JpStage &st, int32_t w,
-                                            unsigned long long r, uint32_t deg) {
-    const uint32_t R = rec_words(A, r, (uint32_t)w);
-    const int64_t b = (int64_t)(r >> 32) + R;
-    const uint64_t bm = (r >> 32 << 32) | R;
-    asm volatile("prefetch.global.L2 [%0];" ::"l"(A.seg + b));  // the list is read next level
-    const uint32_t slot = atomicAdd(&st.n, 1u);
-    if (slot < JP_STAGE) {
-        st.v[slot] = w;
-        st.deg[slot] = deg;
-        st.b[slot] = b;
-        st.bm[slot] = bm;
-    } else {  // stage full: reserve directly (no arrival)
-        const uint32_t nt = n_tasks(deg);
-        const uint32_t base = (uint32_t)atomicAdd(C.W, (unsigned long long)nt);
-        for (uint32_t q = 0; q < nt; q++) write_task(A.tout + base + q, b, b + deg, w, q, bm);
-    }
-}
-
-// CTA-wide end of a level: one atomic = arrival + reservation of the staged entries'
-// tasks, then the tasks, then wait for the level's last arrival; returns hi_{r+1}
-__device__ __forceinline__ uint32_t stage_flush_barrier(const JpArgs &A, const JlCtl &C, JpStage &st, uint32_t r,
-                                                        uint32_t arrivals_expected, uint32_t *trace, uint64_t ts) {
+// software grid barrier (all CTAs co-resident); k = barriers passed so far.  The
+// fence orders this CTA's writes (colours, lists, task entries, bitmap REDs) before
+// the arrival, so the next phase sees them.
+__device__ __forceinline__ void grid_sync(const JrCtl &C, uint32_t &k) {
     __syncthreads();
-    const uint64_t tw = trace ? globaltimer_ns() : 0;
-    const uint32_t n = min(st.n, (uint32_t)JP_STAGE);
-    const uint32_t per = (JP_STAGE + blockDim.x - 1) / blockDim.x;
-    const uint32_t i0 = threadIdx.x * per;
-    uint32_t loc = 0;
-    for (uint32_t i = i0; i < min(n, i0 + per); i++) loc += n_tasks(st.deg[i]);
-    uint32_t incl = loc;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const uint32_t y = __shfl_up_sync(FULL, incl, d);
-        if (lane_id() >= d) incl += y;
-    }
-    const int wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    if (lane_id() == 31) st.wsum[wid] = incl;
-    __syncthreads();
-    if (wid == 0) {
-        const uint32_t x = lane_id() < nw ? st.wsum[lane_id()] : 0u;
-        uint32_t xi = x;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const uint32_t y = __shfl_up_sync(FULL, xi, d);
-            if (lane_id() >= d) xi += y;
-        }
-        if (lane_id() < nw) st.wsum[lane_id()] = xi - x;
-        if (lane_id() == 31) {
-            __threadfence();  // this CTA's pushes (counts, bits, colours) before its arrival
-            const unsigned long long old = atomicAdd(C.W, (1ull << 32) | xi);
-            st.total = xi;
-            st.base = (uint32_t)old;
-            if ((uint32_t)(old >> 32) + 1u == arrivals_expected)  // last arriver: publish the level's end
-                st_release_u64(C.G, ((unsigned long long)(r + 1) << 32) | (uint32_t)(old + xi));
-            if (trace && r < 1024) {  // stats: slowest CTA's work span and flush+arrival span
-                const uint64_t ta = globaltimer_ns();
-                atomicMax(trace + r, (uint32_t)((tw - ts) >> 5));
-                atomicMax(trace + 1024 + r, (uint32_t)((ta - tw) >> 5));
-            }
-        }
-    }
-    __syncthreads();
-    uint32_t o = st.wsum[wid] + incl - loc;
-    for (uint32_t i = i0; i < min(n, i0 + per); i++) {
-        st.off[i] = o;
-        o += n_tasks(st.deg[i]);
-    }
-    __syncthreads();
-    const uint32_t total = st.total, base = st.base;
-    for (uint32_t q = threadIdx.x; q < total; q += blockDim.x) {
-        uint32_t lo = 0, hi = n - 1;  // last entry with off <= q
-        while (lo < hi) {
-            const uint32_t mid = (lo + hi + 1) >> 1;
-            if (st.off[mid] <= q) lo = mid;
-            else hi = mid - 1;
-        }
-        write_task(A.tout + base + q, st.b[lo], st.b[lo] + st.deg[lo], st.v[lo], q - st.off[lo], st.bm[lo]);
-    }
+    k++;
     if (threadIdx.x == 0) {
-        st.n = 0;
-        unsigned long long g;
-        while (((g = ld_acquire_u64(C.G)) >> 32) < r + 1) {
-        }
-        st.base = (uint32_t)g;
+        __threadfence();
+        const uint32_t old = atomicAdd(C.arr, 1u);
+        if (old + 1u == k * gridDim.x) st_release_u32(C.gen, k);
+        else
+            while (ld_acquire_u32(C.gen) < k) {
+            }
     }
     __syncthreads();
-    return st.base;
 }
 
-// decrement the counts of the lower neighbours w[0..U) (flags act[]); each returns
-// the neighbour's whole record (count before the push + segment address); the lower
-// degrees are loaded beside the atomics (needed only by the vertices that become ready)
-template <int U>
-__device__ __forceinline__ void jp_decrement(const JpArgs &A, const uint32_t (&w)[U], const bool (&act)[U],
-                                             unsigned long long (&old)[U], uint32_t (&ld)[U]) {
-#pragma unroll
-    for (int u = 0; u < U; u++) old[u] = act[u] ? atomicAdd(A.rec + w[u], ~0ull) : 0ull;
-#pragma unroll
-    for (int u = 0; u < U; u++) ld[u] = act[u] ? __ldg(A.ldeg + w[u]) : 0u;
+// neighbour u (segment base e) passes v's check for colour m: coloured with another
+// colour, or uncoloured with m already forbidden for it (q, bit = m's word and bit)
+__device__ __forceinline__ bool nb_ok(uint2 hu, uint32_t bw, uint32_t m, uint32_t q, uint32_t bit) {
+    return hu.x != 0u ? hu.x != m : (q < hu.y && ((bw >> bit) & 1u));
 }
 
-// forbidden bit of colour c for the lower neighbours (fire-and-forget; skipped when c
-// lies beyond w's mex range), then the vertices that became ready go to the stage
-template <int U>
-__device__ __forceinline__ void jp_mark(const JpArgs &A, const JlCtl &C, JpStage &st, const uint32_t (&w)[U],
-                                        const bool (&act)[U], const unsigned long long (&old)[U],
-                                        const uint32_t (&ld)[U], uint32_t c) {
-    const uint32_t q = (c - 1) >> 5, bit = 1u << ((c - 1) & 31);
-#pragma unroll
-    for (int u = 0; u < U; u++)
-        if (act[u] && q < rec_words(A, old[u], w[u])) atomicOr(A.seg + (old[u] >> 32) + q, bit);
-#pragma unroll
-    for (int u = 0; u < U; u++)
-        if (act[u] && (old[u] & JP_CNT_MASK) == 1ull) stage_ready(A, C, st, (int32_t)w[u], old[u], ld[u]);
+__device__ __forceinline__ uint2 ld_hdr(const uint32_t *seg, uint32_t e) {
+    return __ldcg(reinterpret_cast<const uint2 *>(seg + 2ull * e));
 }
 
-// mex of h's bitmap (bm = boff << 32 | R), warp-cooperative (a zero lies within the
-// first cap bits)
-__device__ __forceinline__ uint32_t warp_mex(const JpArgs &A, uint64_t bmw) {
-    const uint32_t R = (uint32_t)bmw;
-    const uint32_t *bm = A.seg + (bmw >> 32);
-    for (uint32_t k0 = 0; k0 < R; k0 += 32) {
-        const uint32_t z = k0 + lane_id() < R ? ~__ldcg(bm + k0 + lane_id()) : 0u;
-        const unsigned bal = __ballot_sync(FULL, z != 0);
-        if (bal) {
-            const int src = __ffs(bal) - 1;
-            const uint32_t zz = __shfl_sync(FULL, z, src);
-            return (k0 + src) * 32 + __ffs(zz);
-        }
-    }
-    return R * 32 + 1;  // unreachable: at most cap-1 of the first cap bits are set
-}
-
-// mex by one lane (usually the first word decides)
-__device__ __forceinline__ uint32_t lane_mex(const JpArgs &A, uint64_t bmw) {
-    const uint32_t R = (uint32_t)bmw;
-    const uint32_t *bm = A.seg + (bmw >> 32);
-    for (uint32_t k = 0; k < R; k++) {
-        const uint32_t z = ~__ldcg(bm + k);
-        if (z) return k * 32 + __ffs(z);
-    }
-    return R * 32 + 1;
-}
-
-// One level of push JP over the tasks [lo, hi) of the queue: every task colours its
-// vertex (the first chunk writes the colour) and pushes it to the lower neighbours of
-// its chunk; vertices whose count reaches 0 are staged for the next level.
-__device__ __forceinline__ void jp_level(const JpArgs &A, const JlCtl &C, JpStage &st, uint32_t lo, uint32_t hi,
-                                         int64_t warp_g, int64_t nwarps) {
+// Phase A of round r: every vertex of the uncoloured list U_r with at most JP_WATCH
+// unpushed higher neighbours checks its watch list (the higher neighbours that were
+// uncoloured when the list was built; every other higher neighbour's colour is
+// already in v's bitmap, so it cannot equal m).  A vertex whose count just dropped
+// to JP_WATCH but whose higher list is longer asks phase B to build the watch list.
+__device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t warp_g, int64_t nwarps,
+                                           unsigned long long &bytes) {
     const int lane = lane_id();
-    const uint32_t cnt = hi - lo;
-    // task index t = it*32*nwarps + lane*nwarps + warp: consecutive tasks (the chunks
-    // of one hub) land on different warps
-    for (int64_t base = warp_g; base - warp_g < cnt; base += nwarps * 32) {
-        const int64_t t = base + (int64_t)lane * nwarps;
-        int32_t h = -1;
-        uint32_t j = 0;
-        int64_t b = 0, e = 0;
-        uint64_t bmw = 0;
-        if (t < cnt) read_task(A.tout + lo + t, b, e, h, j, bmw);
-        // ---- short lists: one lane does the whole task
-        const bool small = h >= 0 && e - b <= JP_LANE;
-        if (__any_sync(FULL, small)) {
-            uint32_t w[JP_LANE];
-            bool act[JP_LANE];
-#pragma unroll
-            for (int u = 0; u < JP_LANE; u++) {
-                act[u] = small && b + u < e;
-                w[u] = act[u] ? __ldcs(A.seg + b + u) : 0u;
+    const uint32_t cnt = __ldcg(A.ucnt + r % 3);
+    const uint32_t *U = A.ul[r & 1];
+    uint32_t *Un = A.ul[(r + 1) & 1];
+    uint32_t *seg = A.seg;
+    // a long list is read coalesced (entry it*32*nwarps + warp*32 + lane); a short one
+    // spreads over all warps (entry it*32*nwarps + lane*nwarps + warp), so the
+    // warp-cooperative steps of different vertices run in parallel
+    const bool spread = cnt < 32 * nwarps;
+    for (int64_t it = 0; it < cnt; it += nwarps * 32) {
+        const int64_t i = it + (spread ? (int64_t)lane * nwarps + warp_g : warp_g * 32 + lane);
+        const bool act = i < cnt;
+        uint32_t sb = 0, R = 0, hd = 0, ld = 0, wc = 0, pos = 0, lm = 0, m = 1;
+        int state = 3;  // 0 checking, 1 passed, 2 failed (memo), 3 idle, 4 waiting, 5 build request
+        if (act) {
+            sb = __ldcg(U + i);
+            const uint4 h0 = __ldcg(reinterpret_cast<const uint4 *>(seg + 2ull * sb));
+            const uint4 h1 = __ldcg(reinterpret_cast<const uint4 *>(seg + 2ull * sb + 4));
+            R = h0.y;
+            hd = h0.z;
+            ld = h0.w;
+            wc = h1.y;
+            pos = h1.z;
+            lm = h1.w;
+            bytes += 36;
+            if (h1.x > JP_WATCH) {
+                state = 4;
+            } else if (wc == JP_NOTBUILT) {
+                state = 5;
+            } else {
+                state = 0;
+                const uint32_t *bm = seg + seg_bitmap(sb);
+                for (uint32_t q = 0; q < R; q++) {  // mex: usually the first word decides
+                    const uint32_t z = ~__ldcg(bm + q);
+                    if (z) {
+                        m = q * 32 + __ffs(z);
+                        break;
+                    }
+                }
             }
-            unsigned long long old[JP_LANE];
-            uint32_t ld[JP_LANE];
-            jp_decrement<JP_LANE>(A, w, act, old, ld);
-            uint32_t c = 1;
-            if (small) {
-                c = lane_mex(A, bmw);
-                A.ccol[h] = c;
-            }
-            jp_mark<JP_LANE>(A, C, st, w, act, old, ld, c);
         }
-        // ---- longer lists: the warp takes these tasks one by one (<= JP_CHUNK arcs)
-        unsigned bigm = __ballot_sync(FULL, h >= 0 && !small);
+        const uint64_t wl = seg_watch(sb, R);
+        const uint32_t q = (m - 1) >> 5, bit = (m - 1) & 31;
+        uint32_t j = (lm == m && pos < wc) ? pos : 0u;  // m unchanged: resume at the last blocker
+        // ---- lane: the first JP_LANE_CHECKS entries
+        if (state == 0) {
+            uint32_t e[JP_LANE_CHECKS];
+            uint2 hu[JP_LANE_CHECKS];
+            uint32_t bw[JP_LANE_CHECKS];
+#pragma unroll
+            for (int u = 0; u < JP_LANE_CHECKS; u++) e[u] = j + u < wc ? __ldcg(seg + wl + j + u) : 0u;
+#pragma unroll
+            for (int u = 0; u < JP_LANE_CHECKS; u++) {
+                if (j + u < wc) {
+                    hu[u] = ld_hdr(seg, e[u]);
+                    bw[u] = __ldcg(seg + seg_bitmap(e[u]) + q);
+                } else {
+                    hu[u] = make_uint2(0u, 0u);
+                    bw[u] = 0u;
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < JP_LANE_CHECKS; u++) {
+                if (state == 0) {
+                    if (j >= wc) {
+                        state = 1;
+                    } else if (!nb_ok(hu[u], bw[u], m, q, bit)) {
+                        state = 2;
+                        pos = j;
+                        lm = m;
+                    } else {
+                        j++;
+                    }
+                }
+            }
+            if (state == 0 && j >= wc) state = 1;
+            bytes += 4ull * min(wc, (uint32_t)JP_LANE_CHECKS);
+        }
+        // ---- warp: the rest of a list (<= JP_WLIST entries: at most two steps)
+        unsigned need = __ballot_sync(FULL, state == 0);
+        while (need) {
+            const int src = __ffs(need) - 1;
+            need &= need - 1;
+            uint32_t wj = __shfl_sync(FULL, j, src);
+            const uint32_t wwc = __shfl_sync(FULL, wc, src), wm = __shfl_sync(FULL, m, src);
+            const uint64_t wwl = __shfl_sync(FULL, wl, src);
+            const uint32_t wq = (wm - 1) >> 5, wbit = (wm - 1) & 31;
+            int wstate = 0;
+            uint32_t wpos = 0;
+            while (wstate == 0) {
+                const uint32_t jj = wj + lane;
+                bool ok = true;
+                if (jj < wwc) {
+                    const uint32_t eu = __ldcg(seg + wwl + jj);
+                    ok = nb_ok(ld_hdr(seg, eu), __ldcg(seg + seg_bitmap(eu) + wq), wm, wq, wbit);
+                }
+                const unsigned fails = __ballot_sync(FULL, !ok);
+                if (fails) {
+                    wstate = 2;
+                    wpos = wj + __ffs(fails) - 1;
+                } else {
+                    wj += 32;
+                    if (wj >= wwc) wstate = 1;
+                }
+                bytes += lane == 0 ? 128ull : 0ull;
+            }
+            if (lane == src) {
+                state = wstate;
+                if (wstate == 2) {
+                    pos = wpos;
+                    lm = m;
+                }
+            }
+        }
+        // ---- outcome
+        const bool pass = state == 1, stay = state == 2 || state == 4 || state == 5;
+        if (pass) seg[2ull * sb] = m;
+        if (state == 2) *reinterpret_cast<uint2 *>(seg + 2ull * sb + 6) = make_uint2(pos, lm);
+        if (state == 5) seg[2ull * sb + 5] = 0u;  // the watch list is filled by phase B
+        const int64_t slot = warp_append(stay, A.ucnt + (r + 1) % 3);
+        if (stay) Un[slot] = sb;
+        // push tasks of a new colour
+        const uint32_t nt = pass ? (ld + JP_PUSH - 1) / JP_PUSH : 0u;
+        const int64_t ts = warp_reserve(nt, A.pcnt + r % 3);
+        if (nt) {
+            const uint64_t l0 = seg_lower(sb, R, hd) >> 1;  // u64 index of the lower list
+            for (uint32_t t = 0; t < nt; t++) {
+                const uint64_t s0 = l0 + (uint64_t)t * JP_PUSH;
+                A.task[ts + t] = make_uint4((uint32_t)s0, (uint32_t)(s0 >> 32), min(JP_PUSH, ld - t * JP_PUSH), m);
+            }
+        }
+        // watch-list build tasks, one per JP_BUILD higher entries
+        const uint32_t nb = state == 5 ? (hd + JP_BUILD - 1) / JP_BUILD : 0u;
+        const int64_t bs = warp_reserve(nb, A.bcnt + r % 3);
+        for (uint32_t t = 0; t < nb; t++) A.btask[bs + t] = make_uint2(sb, t);
+        bytes += (state == 2 ? 8ull : 0ull) + (stay ? 4ull : 0ull) + (pass ? 4ull + 16ull * nt : 0ull) + 8ull * nb;
+    }
+}
+
+// a new colour c (word q, bit) for lower neighbours x[u] = sb | R << 32 (flags act):
+// the forbidden bits, and one higher neighbour less to wait for; the push that brings
+// a count to JP_WATCH activates w (next round's list; there it asks for its watch
+// list).  All atomics of the batch are in flight together.
+// A neighbour that is already coloured (early commits) needs neither; one whose count
+// is already <= JP_WATCH needs only the bit: both are read first (plain L2 loads) so
+// the atomics go only where they matter.
+template <int K>
+__device__ __forceinline__ void jp_push(const JpArgs &A, uint32_t r, uint32_t *seg, const unsigned long long (&x)[K],
+                                        bool (&act)[K], uint32_t q, uint32_t bit) {
+    uint32_t old[K], cw[K];
+#pragma unroll
+    for (int u = 0; u < K; u++) cw[u] = act[u] ? __ldcg(seg + 2ull * (uint32_t)x[u]) : 1u;  // colour
+#pragma unroll
+    for (int u = 0; u < K; u++) act[u] = act[u] && cw[u] == 0u;
+#pragma unroll
+    for (int u = 0; u < K; u++) old[u] = act[u] ? atomicSub(seg + 2ull * (uint32_t)x[u] + 4, 1u) : 0u;
+#pragma unroll
+    for (int u = 0; u < K; u++)
+        if (act[u] && q < (uint32_t)(x[u] >> 32)) atomicOr(seg + seg_bitmap((uint32_t)x[u]) + q, 1u << bit);
+#pragma unroll
+    for (int u = 0; u < K; u++) {
+        if (act[u] && old[u] == JP_WATCH + 1u) {
+            const uint32_t slot = atomicAdd(A.ucnt + (r + 1) % 3, 1u);
+            A.ul[(r + 1) & 1][slot] = (uint32_t)x[u];
+        }
+    }
+}
+
+// Phase B of round r: push the new colours; build the requested watch lists
+__device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, int64_t warp_g, int64_t nwarps,
+                                           unsigned long long &bytes) {
+    const int lane = lane_id();
+    const uint32_t cnt = __ldcg(A.pcnt + r % 3);
+    uint32_t *seg = A.seg;
+    const unsigned long long *seg64 = reinterpret_cast<const unsigned long long *>(seg);
+    for (int64_t base = warp_g; base - warp_g < cnt; base += nwarps * 32) {
+        const int64_t i = base + (int64_t)lane * nwarps;  // tasks spread over all warps
+        uint4 tk = make_uint4(0u, 0u, 0u, 0u);
+        if (i < cnt) tk = __ldcg(A.task + i);
+        const uint64_t s0 = (uint64_t)tk.x | ((uint64_t)tk.y << 32);
+        const bool small = tk.z > 0 && tk.z <= JP_PUSH_LANE;
+        if (small) {
+            const uint32_t q = (tk.w - 1) >> 5, bit = (tk.w - 1) & 31;
+            unsigned long long x[JP_PUSH_LANE];
+            bool act[JP_PUSH_LANE];
+#pragma unroll
+            for (int u = 0; u < JP_PUSH_LANE; u++) {
+                act[u] = u < (int)tk.z;
+                x[u] = act[u] ? __ldcs(seg64 + s0 + u) : 0ull;
+            }
+            jp_push<JP_PUSH_LANE>(A, r, seg, x, act, q, bit);
+            bytes += 8ull * tk.z;
+        }
+        unsigned bigm = __ballot_sync(FULL, tk.z > JP_PUSH_LANE);
         while (bigm) {
             const int src = __ffs(bigm) - 1;
             bigm &= bigm - 1;
-            const int32_t th = __shfl_sync(FULL, h, src);
-            const uint32_t tj = __shfl_sync(FULL, j, src);
-            const int64_t tb = __shfl_sync(FULL, b, src), te = __shfl_sync(FULL, e, src);
-            const uint64_t tbm = __shfl_sync(FULL, bmw, src);
-            const int64_t cb = tb + (int64_t)tj * JP_CHUNK;
-            constexpr int U = JP_CHUNK / 32;
-            uint32_t w[U];
-            bool act[U];
+            const uint64_t ws = __shfl_sync(FULL, s0, src);
+            const uint32_t wn = __shfl_sync(FULL, tk.z, src), wc = __shfl_sync(FULL, tk.w, src);
+            const uint32_t q = (wc - 1) >> 5, bit = (wc - 1) & 31;
+            constexpr int K = JP_PUSH / 32;
+            unsigned long long x[K];
+            bool act[K];
 #pragma unroll
-            for (int u = 0; u < U; u++) {
-                const int64_t x = cb + u * 32 + lane;
-                act[u] = x < te;
-                w[u] = act[u] ? __ldcs(A.seg + x) : 0u;
+            for (int u = 0; u < K; u++) {
+                act[u] = u * 32 + lane < (int)wn;
+                x[u] = act[u] ? __ldcs(seg64 + ws + u * 32 + lane) : 0ull;
             }
-            unsigned long long old[U];
-            uint32_t ld[U];
-            jp_decrement<U>(A, w, act, old, ld);  // the decrements do not wait for the mex
-            const uint32_t c = warp_mex(A, tbm);
-            if (tj == 0 && lane == 0) A.ccol[th] = c;
-            jp_mark<U>(A, C, st, w, act, old, ld, c);
+            jp_push<K>(A, r, seg, x, act, q, bit);
+            bytes += lane == 0 ? 8ull * wn : 0ull;
         }
+    }
+    // watch lists: a warp per task filters JP_BUILD higher entries (uncoloured ones kept)
+    const uint32_t nbt = __ldcg(A.bcnt + r % 3);
+    for (int64_t t = warp_g; t < nbt; t += nwarps) {
+        const uint2 bt = __ldcg(A.btask + t);
+        const uint4 h0 = __ldcg(reinterpret_cast<const uint4 *>(seg + 2ull * bt.x));
+        const uint64_t hl = seg_higher(bt.x, h0.y, h0.z), wl = seg_watch(bt.x, h0.y);
+        const uint32_t j0 = bt.y * JP_BUILD, j1 = min(h0.z, j0 + JP_BUILD);
+        constexpr int K = JP_BUILD / 32;
+        uint32_t e[K], c[K];
+#pragma unroll
+        for (int u = 0; u < K; u++) e[u] = j0 + u * 32 + lane < j1 ? __ldcs(seg + hl + j0 + u * 32 + lane) : 0u;
+#pragma unroll
+        for (int u = 0; u < K; u++) c[u] = j0 + u * 32 + lane < j1 ? __ldcg(seg + 2ull * e[u]) : 1u;
+#pragma unroll
+        for (int u = 0; u < K; u++) {
+            const bool keep = c[u] == 0u;
+            const unsigned mk = __ballot_sync(FULL, keep);
+            uint32_t p0 = 0;
+            if (mk && lane == 0) p0 = atomicAdd(seg + 2ull * bt.x + 5, (uint32_t)__popc(mk));
+            p0 = __shfl_sync(FULL, p0, 0);
+            const uint32_t p = p0 + __popc(mk & ((1u << lane) - 1u));
+            if (keep && p < JP_WATCH) seg[wl + p] = e[u];
+        }
+        bytes += lane == 0 ? 4ull * (j1 - j0) : 0ull;
     }
 }
 
-// ---------------------------------------------------------------- persistent levels
-// All levels in ONE cooperative launch (grid = one or more CTAs per SM, all
-// co-resident): level r = jp_level over [lo_r, hi_r), then stage_flush_barrier.  The
-// barrier orders the pushes of level r before the mex reads of level r+1, so no
-// per-push fence is needed.
-constexpr int JL_THREADS = 512;
-#ifndef SYM_JL_MINB
-#define SYM_JL_MINB 1
+constexpr int JR_THREADS = 512;
+#ifndef SYM_JR_MINB
+#define SYM_JR_MINB 2
 #endif
-constexpr uint64_t JL_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
+constexpr uint64_t JR_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
 
-__global__ void __launch_bounds__(JL_THREADS, SYM_JL_MINB) k_jp_levels(JpArgs A, JlCtl C) {
-    __shared__ JpStage st;
-    if (threadIdx.x == 0) st.n = 0;
-    __syncthreads();
-    // warp-in-CTA major: consecutive tasks (the chunks of one row) go to different SMs
+__global__ void __launch_bounds__(JR_THREADS, SYM_JR_MINB) k_jp_rounds(JpArgs A, JrCtl C) {
+    // warp-in-CTA major: consecutive list entries of a warp step spread over SMs
     const int64_t warp_g = (int64_t)(threadIdx.x >> 5) * gridDim.x + blockIdx.x;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const uint64_t t0 = globaltimer_ns();
-    uint32_t lo = 0, hi = (uint32_t)__ldcg(C.W);  // level 0 = the build pass's tasks
-    uint32_t r = 0;
-    uint32_t *trace = A.trace;
+    unsigned long long bytes = 0;
+    uint32_t k = 0, r = 0;
+    if (__ldcg(A.err) & 2u) return;  // the build overflowed the segment offsets (set before launch)
     for (;; r++) {
-        if (hi == lo || __ldcg(C.err) != 0) break;
-        const uint64_t ts = trace ? globaltimer_ns() : 0;
+        const uint32_t cnt = __ldcg(A.ucnt + r % 3);
+        if (cnt == 0) break;
         if (blockIdx.x == 0 && threadIdx.x == 0) {
-            if (A.hist && r < 1024) {  // stats: tasks and start time (32 ns units) of the first levels
-                A.hist[r] = hi - lo;
+            if (A.hist && r < 1024) {  // stats: list size and start time (32 ns units) of the first rounds
+                A.hist[r] = cnt;
                 A.hist[1024 + r] = (uint32_t)((globaltimer_ns() - t0) >> 5);
             }
-            if (r + 1 >= C.max_levels || globaltimer_ns() - t0 > JL_TIMEOUT_NS) atomicOr(C.err, 1u);
+            A.ucnt[(r + 2) % 3] = 0u;  // U_{r+2}'s counter: last read at the start of round r-1
+            A.pcnt[(r + 2) % 3] = 0u;  // push tasks of round r+2: last read in round r-1
+            A.bcnt[(r + 2) % 3] = 0u;
+            if (r + 1 >= C.max_rounds || globaltimer_ns() - t0 > JR_TIMEOUT_NS) atomicOr(A.err, 1u);
         }
-        jp_level(A, C, st, lo, hi, warp_g, nwarps);
-        const uint32_t next = stage_flush_barrier(A, C, st, r, (r + 1) * gridDim.x, trace, ts);
-        lo = hi;
-        hi = next;
+        jp_phase_a(A, r, warp_g, nwarps, bytes);
+        grid_sync(C, k);
+        if (__ldcg(A.err) != 0) break;  // read after the barrier: every CTA sees the same word
+        if (A.trace && blockIdx.x == 0 && threadIdx.x == 0 && r < 512) {  // diagnostics
+            A.trace[r] = (uint32_t)((globaltimer_ns() - t0) >> 5);
+            A.trace[512 + r] = __ldcg(A.pcnt + r % 3);
+            A.trace[1024 + r] = __ldcg(A.bcnt + r % 3);
+        }
+        const uint64_t tb = A.trace ? globaltimer_ns() : 0;
+        jp_phase_b(A, r, warp_g, nwarps, bytes);
+        if (A.trace && r < 512) {  // diagnostics: slowest CTA's phase-B work span
+            __syncthreads();
+            if (threadIdx.x == 0) atomicMax(A.trace + 1536 + r, (uint32_t)((globaltimer_ns() - tb) >> 5));
+        }
+        grid_sync(C, k);
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *C.levels = r;
+    prof_add(A.prof, bytes);
 }
 
 // ---------------------------------------------------------------- fix-up kernels
@@ -957,37 +980,42 @@ __global__ void k_color_max(const uint32_t *color, int64_t n, uint32_t *mx) {
 // ---------------------------------------------------------------- host side
 void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
     const int64_t ntiles = (n + JP_TILE - 1) / JP_TILE + 1;
-    w.cid = a.take<int32_t>((size_t)n + 1);
     w.ov = a.take<int32_t>((size_t)n + 1);
+    w.hdeg = a.take<uint32_t>((size_t)n + 1);
     w.ldeg = a.take<uint32_t>((size_t)n + 1);
-    w.rfull = a.take<uint32_t>((size_t)n + 1);
-    w.ccol = a.take<uint32_t>((size_t)n + 1);
-    w.rec = a.take<unsigned long long>((size_t)n + 2);
-    // segments: bitmaps, sum of ceil(cap/32) <= (nnz + n)/32 + n words, and lower
-    // lists, one id per S-S edge (<= nnz/2)
-    w.seg_words = (nnz + n) / 32 + n + nnz / 2 + 2;
+    w.sbh = a.take<uint32_t>((size_t)n + 1);
+    w.sbR = a.take<unsigned long long>((size_t)n + 1);
+    w.ul[0] = a.take<uint32_t>((size_t)n + 1);
+    w.ul[1] = a.take<uint32_t>((size_t)n + 1);
+    // segments: header 8 + bitmap (sum of ceil(cap/32) <= (nnz+n)/32 + n) + higher list
+    // (one word per arc) + lower list (two words per arc), each part padded to even
+    // and the whole to 4 words: <= 14 n + (nnz+n)/32 + 2 nnz words
+    w.seg_words = 14 * n + (nnz + n) / 32 + 2 * nnz + 64;
     w.seg = a.take<uint32_t>((size_t)w.seg_words);
     w.tcnt = a.take<uint32_t>(2 * (size_t)ntiles);
-    w.tsum = a.take<unsigned long long>(2 * (size_t)ntiles);
+    w.tsum = a.take<unsigned long long>((size_t)ntiles);
     w.ntiles = ntiles;
-    w.queue_cap = n + nnz / (2 * JP_CHUNK) + 2;  // every vertex is enqueued once
-    w.task = a.take<int64_t>((size_t)w.queue_cap * (sizeof(JpTask) / sizeof(int64_t)));
+    w.task_cap = n + nnz / JP_PUSH + 2;  // tasks of one round <= all tasks
+    w.task = a.take<uint4>((size_t)w.task_cap);
+    w.btask = a.take<uint2>((size_t)w.task_cap);
     w.vlist = a.take<int32_t>((size_t)n + 1);
     w.mark = a.take<uint8_t>((size_t)n + 1);
     w.queue = a.take<int64_t>((size_t)(nnz / JP_BUDGET + 2));  // huge-row pieces (<= nnz/JP_BUDGET)
-    w.sync = a.take<uint32_t>(64);  // levels kernel: barrier words, apart from the task counters
+    w.sync = a.take<uint32_t>(64);  // rounds kernel: barrier / counters / error words
 }
 
-// JP over (rp, ci) for the vertex set S (list/implicit) with membership inS.
-// Build: compact ids, the oriented lower-neighbour DAG, records + bitmaps, and the
-// level-0 tasks at the head of the queue (counter = the low half of W).
+// Build: compact ids, segments (bitmaps, higher and lower lists), the first round's
+// list.  sync words: [0] barrier arrivals, [1] barrier generation, [4..6] list
+// counts, [8..10] push-task counts, [12..14] build-task counts, [32] error, [33]
+// rounds, [40..41] compact counts.
 static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, const int64_t *rp,
                     const int32_t *ci, const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0,
-                    int64_t implicit_n, JpTask *q, uint32_t *qcnt, uint32_t *err) {
+                    int64_t implicit_n) {
     Ctl *ctl = f.ctl;
     cudaStream_t s = f.stream;
     const int64_t n = f.g.n;
     SYM_CUDA(cudaMemsetAsync(ctl->huge, 0, sizeof(ctl->huge), s));
+    SYM_CUDA(cudaMemsetAsync(w.sync, 0, 64 * sizeof(uint32_t), s));
     A.rp = rp;
     A.ci = ci;
     A.inS = inS;
@@ -995,24 +1023,28 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     A.in_list = list0;
     A.in_cnt = cnt0;
     A.implicit_n = implicit_n;
-    A.cid = w.cid;
     A.ov = w.ov;
+    A.hdeg = w.hdeg;
     A.ldeg = w.ldeg;
-    A.rfull = w.rfull;
-    A.rec = w.rec;
+    A.sbh = w.sbh;
+    A.sbR = w.sbR;
     A.seg = w.seg;
-    A.ccol = w.ccol;
     A.tcnt = w.tcnt;
     A.tsum = w.tsum;
     A.nc = w.sync + 40;
-    A.tout = q;
-    A.out_cnt = qcnt;
+    A.ul[0] = w.ul[0];
+    A.ul[1] = w.ul[1];
+    A.task = w.task;
+    A.ucnt = w.sync + 4;
+    A.pcnt = w.sync + 8;
+    A.bcnt = w.sync + 12;
+    A.btask = w.btask;
     A.huge = w.queue;
     A.huge_cnt = &ctl->huge[1];
-    A.err = err;
+    A.err = w.sync + 32;
     A.hist = nullptr;
     A.trace = nullptr;
-    A.prof = prof_counter(s);
+    A.prof = nullptr;
     A.k = stream_key(f.p.seed, TAG_VERTEX, 0);
     const int64_t smax = list0 ? n : implicit_n;  // positions of S (upper bound for a list)
     const unsigned tiles_s = (unsigned)((smax + JP_TILE - 1) / JP_TILE);
@@ -1050,7 +1082,7 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     return SYM_OK;
 }
 
-// every level in one persistent cooperative launch
+// every round in one persistent cooperative launch
 static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t *rp, const int32_t *ci,
                   const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0, int64_t implicit_n, int phase) {
     Ctl *ctl = f.ctl;
@@ -1062,60 +1094,46 @@ static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t 
         SYM_CUDA(cudaGetDevice(&dev));
         SYM_CUDA(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev));
         if (!coop) {
-            set_error("JP needs cooperative launch (persistent levels kernel), unsupported on this device");
+            set_error("JP needs cooperative launch (persistent rounds kernel), unsupported on this device");
             return SYM_ECUDA;
         }
-        SYM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_jp_levels, JL_THREADS, 0));
+        SYM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_jp_rounds, JR_THREADS, 0));
         if (per_sm < 1) {
-            set_error("k_jp_levels does not fit on an SM");
+            set_error("k_jp_rounds does not fit on an SM");
             return SYM_ECUDA;
         }
         grid = num_sms() * per_sm;
     }
-    JpTask *q = reinterpret_cast<JpTask *>(w.task);
-    const int64_t qcap = w.queue_cap;
-    if (qcap >= (int64_t)0xffffffff) {
-        set_error("JP task queue exceeds 2^32 entries");
-        return SYM_EINVAL;
-    }
-    // W (u64) = sync[0..1], G (u64) = sync[2..3], err = sync[32], levels = sync[33],
-    // build counts = sync[40..41]
-    SYM_CUDA(cudaMemsetAsync(w.sync, 0, 64 * sizeof(uint32_t), s));
-    SYM_CUDA(cudaMemsetAsync(q, 0xff, sizeof(JpTask) * (size_t)qcap, s));
-    JlCtl C;
-    C.W = reinterpret_cast<unsigned long long *>(w.sync);
-    C.G = reinterpret_cast<unsigned long long *>(w.sync + 2);
-    C.err = &w.sync[32];
-    C.levels = &w.sync[33];
-    C.max_levels = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
-    // arrivals (levels x grid) must not overflow the high half of W
-    C.max_levels = std::min<uint64_t>(C.max_levels, 0xffffffffull / (uint64_t)grid - 1);
     JpArgs A;
-    SYM_TRY(jp_build(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n, q, w.sync /* low half of W */, C.err));
-    // stats: per-level task counts and start times; phase 0 also traces the level
-    // spans into hist[2048..4095] (SYM_JP_TRACE=1 in the environment)
-    static const bool jp_trace = getenv("SYM_JP_TRACE") != nullptr;
+    SYM_TRY(jp_build(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n));
+    JrCtl C;
+    C.arr = w.sync;
+    C.gen = w.sync + 1;
+    C.levels = w.sync + 33;
+    C.max_rounds = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
+    // barriers (2 per round) x grid must not overflow the arrival word
+    C.max_rounds = std::min<uint64_t>(C.max_rounds, 0xffffffffull / (2ull * (uint64_t)grid) - 1);
     A.hist = f.stats ? ctl->hist + phase * 2048 : nullptr;
-    A.trace = jp_trace && phase == 0 && A.hist ? ctl->hist + 2048 : nullptr;
+    static const bool jp_trace = getenv("SYM_JP_TRACE") != nullptr;
+    A.trace = jp_trace && f.stats && phase == 0 ? ctl->hist + 2048 : nullptr;
     if (A.trace) SYM_CUDA(cudaMemsetAsync(A.trace, 0, 2048 * sizeof(uint32_t), s));
-    unsigned long long *ctr = A.prof;
-    A.prof = nullptr;
+    A.prof = prof_counter(s);
     void *args[] = {&A, &C};
-    prof_begin("jp_levels", s);
-    SYM_CUDA(cudaLaunchCooperativeKernel((const void *)k_jp_levels, dim3(grid), dim3(JL_THREADS), args, 0, s));
-    prof_end_dev(s, ctr);
+    prof_begin("jp_rounds", s);
+    SYM_CUDA(cudaLaunchCooperativeKernel((const void *)k_jp_rounds, dim3(grid), dim3(JR_THREADS), args, 0, s));
+    prof_end_dev(s, A.prof);
     k_jpc_scatter<<<num_sms() * 8, 256, 0, s>>>(A);
     SYM_LAUNCH_CHECK();
     uint32_t err = 0, levels = 0;
-    SYM_TRY(read_u32(C.err, &err, s));
+    SYM_TRY(read_u32(A.err, &err, s));
     if (err) {
         SYM_TRY(read_u32(C.levels, &levels, s));
         if (err & 2u) {
-            set_error("JP: a vertex count or bitmap offset exceeds the record fields (degree >= 2^24)");
+            set_error("JP: segment offsets exceed 2^35 bytes");
             return SYM_EINVAL;
         }
         const bool rounds = f.p.max_rounds && levels + 1 >= f.p.max_rounds;
-        set_error(rounds ? "JP did not converge within max_rounds" : "JP levels kernel timed out");
+        set_error(rounds ? "JP did not converge within max_rounds" : "JP rounds kernel timed out");
         return rounds ? SYM_EROUNDS : SYM_ECUDA;
     }
     if (f.stats) {

@@ -1,5 +1,5 @@
-"""Diagnostic: per-level task counts, start times and (SYM_JP_TRACE=1) spans of the
-persistent JP levels kernel: the slowest CTA's work span and flush+arrival span."""
+"""Diagnostic: per-round list sizes and start times of the persistent JP rounds kernel
+(COLOR-Deg2 on R-MAT), and the COLOR-Deg2 device time."""
 import os, sys
 os.environ.setdefault("SYM_JP_TRACE", "1")
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -8,18 +8,31 @@ dev = torch.device("cuda", 0)
 scale = int(sys.argv[1]) if len(sys.argv) > 1 else 24
 rp, ci = graphgen.rmat(scale, 16, seed=1, device=dev)
 d = sb.sym_decompose(rp, ci, "degk", 2, 42)
-for _ in range(2):
-    col, st = sb.sym_color(rp, ci, "degk", 2, 42, decomp=d, stats=True)
+ts = []
+for _ in range(3):
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(); sb.sym_color(rp, ci, "degk", 2, 42, decomp=d); e1.record(); torch.cuda.synchronize()
+    ts.append(e0.elapsed_time(e1))
+sb.sym_profile_enable(True)
+sb.sym_color(rp, ci, "degk", 2, 42, decomp=d)
 torch.cuda.synchronize()
+print("profile", sb.sym_profile_collect())
+sb.sym_profile_enable(False)
+col, st = sb.sym_color(rp, ci, "degk", 2, 42, decomp=d, stats=True)
+torch.cuda.synchronize()
+print("COLOR-Deg2 ms", ts, "max colour", int(col.max()))
 ws = sb._WS[(0, torch.cuda.current_stream(dev).cuda_stream)]
 off = ((ws.data_ptr() + 255) & ~255) - ws.data_ptr()
 h = ws[off + 136: off + 136 + 16384].cpu().numpy().view(np.uint32)
-cnt, ts = h[:1024].astype(np.int64), h[1024:2048].astype(np.int64) * 32 / 1000.0
-work, flush = h[2048:3072] * 32 / 1000.0, h[3072:4096] * 32 / 1000.0
-print("levels", st["rounds"])
-dt = np.diff(ts)
-for r in list(range(0, 12)) + list(range(40, 1023, 80)):
-    print(f"L{r:5d} tasks {cnt[r]:8d} t {ts[r]:9.1f} us  dt {dt[r]:7.2f} us  work(max CTA) {work[r]:6.2f}  flush(max) {flush[r]:6.2f}")
-sel = slice(20, 1023)
-print("median dt", np.median(dt[sel]), "work", np.median(work[sel]), "flush", np.median(flush[sel]),
-      "rest (barrier+skew)", np.median(dt[sel] - work[sel] - flush[sel]))
+tr = h[2048:4096].astype(np.int64)
+pa = tr[:512] * 32 / 1000.0
+cnt, t = h[:1024].astype(np.int64), h[1024:2048].astype(np.int64) * 32 / 1000.0
+R = st["rounds"][0]
+print("rounds", st["rounds"])
+dt = np.diff(t[:min(R, 1024)])
+for r in list(range(0, 16)) + list(range(20, min(R, 1023), 40)):
+    if r < len(dt):
+        extra = f" A {pa[r]-t[r]:7.2f} us pushT {tr[512+r]:7d} buildT {tr[1024+r]:7d} Bwork {tr[1536+r]*0.032:7.2f}" if r < 512 else ""
+        print(f"R{r:5d} |U| {cnt[r]:9d} t {t[r]:9.1f} us  dt {dt[r]:7.2f} us" + extra)
+if len(dt) > 40:
+    print("median dt (rounds >= 20)", np.median(dt[20:]), "mean", dt[20:].mean())
