@@ -164,11 +164,16 @@ struct ColorWs {
     int32_t *ov = nullptr;         // compact id -> original
     uint32_t *hdeg = nullptr;      // higher / lower degrees (build), fill cursors
     uint32_t *ldeg = nullptr;
-    uint32_t *sbh = nullptr;       // compact id -> segment base (8-B units)
-    unsigned long long *sbR = nullptr;  // original id -> segment base | R << 32
-    uint32_t *ul[2] = {nullptr, nullptr};  // uncoloured lists (ping-pong by round)
-    uint32_t *seg = nullptr;       // per compact vertex: header, forbidden bitmap, higher + lower lists
-    int64_t seg_words = 0;
+    uint32_t *cidR = nullptr;      // original id -> list id (compact id | min(R,31) << 27)
+    uint32_t *col = nullptr;       // hot per-vertex state: colour, count, bitmap word 0,
+    uint32_t *cnt = nullptr;       //   offset of the extra bitmap words
+    uint32_t *bm0 = nullptr;
+    uint32_t *xo = nullptr;
+    uint4 *meta = nullptr;         // per-vertex own data (2 x 16 B)
+    uint32_t *ul[2] = {nullptr, nullptr};  // active lists (ping-pong by round)
+    uint32_t *lst = nullptr;       // watch / higher / lower lists
+    int64_t lst_words = 0;
+    uint32_t *xb = nullptr;        // bitmap words for colours > 32
     uint32_t *tcnt = nullptr;      // build scan scratch (per tile)
     unsigned long long *tsum = nullptr;
     int64_t ntiles = 0;

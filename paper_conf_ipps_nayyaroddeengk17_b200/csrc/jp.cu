@@ -8,35 +8,38 @@
 //
 //   m = mex of the colours of v's coloured higher neighbours (v's forbidden bitmap);
 //   v may take m as soon as every higher neighbour u is either coloured with a
-//   colour != m, or uncoloured with m already in u's own forbidden set.
+//   colour != m, or uncoloured and unable to take m: m is already forbidden for u,
+//   or m > cap(u) (u's colour is at most cap(u) = #higher + #fixed-coloured + 1).
 //
 // Proof: the final higher-neighbour colours are the known ones (which hold 1..m-1
-// and not m) plus one colour per uncoloured u, and u can never take m (m is
-// forbidden for u), so the final mex is m.  Every fact the rule reads ("u has colour
-// c", "m is forbidden for u") is permanent once observed, so the rule is exact under
-// any schedule and any staleness; a vertex whose higher neighbours are all coloured
-// (plain JP's ready vertex) always passes.  Result: the same colours in 531 rounds
-// instead of 5 063 levels at R-MAT s24 (CPU simulation).
+// and not m) plus one colour per uncoloured u, and u can never take m, so the final
+// mex is m.  Every fact the rule reads ("u has colour c", "m is forbidden for u") is
+// permanent once observed, so the rule is exact under any schedule and staleness; a
+// vertex whose higher neighbours are all coloured (plain JP's ready vertex) always
+// passes.  Result: the same colours in ~530 rounds instead of 5 063 levels at R-MAT
+// s24 (CPU simulation and GPU).
 //
-// Layout (built once per call; S vertices with phase arcs get compact ids h, rows
-// of degree > 2 first; a vertex without any phase arc takes colour 1 at once):
-//   segment of h at word O = 2*sb(h) of seg[] (8-B aligned):
-//     O+0 colour (0 = not yet), O+1 R, O+2 hdeg, O+3 ldeg, O+4 cnt = higher
-//     neighbours not yet pushed, O+5 watch-list length, O+6..7 check memo (blocker
-//     position, m at the last failed check);
-//     O+8: forbidden bitmap, R = ceil(cap/32) words, cap = #higher + #fixed-coloured
-//     neighbours + 1 >= mex; a JP_WATCH-entry watch area if hdeg > JP_WATCH; the
-//     higher list (hdeg segment bases sb(u), u32); the lower list (ldeg entries
-//     sb(w) | R(w) << 32, u64).
-// A round: phase A -- every uncoloured vertex whose count is <= JP_WATCH checks its
-// watch list (the higher neighbours still uncoloured when it was built; a list of
-// <= JP_WATCH higher neighbours is its own watch list), resuming at the last blocker
-// when m is unchanged; a vertex that passes writes its colour and queues push tasks;
-// grid barrier; phase B -- each new colour goes into the lower neighbours' bitmaps
-// and decrements their counts (RED), and requested watch lists are built; grid
-// barrier.  All rounds run in ONE persistent cooperative kernel (k_jp_rounds).
-// Waiting for the count to reach JP_WATCH costs no rounds on R-MAT (CPU simulation)
-// and bounds every check to one warp step.
+// Layout (built once per call; S vertices with phase arcs get compact ids h, rows of
+// degree > 2 first; a vertex without any phase arc takes colour 1 at once).  The
+// per-vertex state other vertices touch is split into compact arrays so the hot set
+// stays in L2 (4 x 4 B per vertex, 90 MB at R-MAT s24):
+//   col[h]  colour (0 = not yet)          cnt[h]  higher neighbours not yet pushed
+//   bm0[h]  forbidden colours 1..32       xo[h]   offset of h's words for colours
+//                                                 33..32R in xb[] (R-1 words)
+// with R = ceil(cap/32).  meta[h] (32 B, read by h itself) = {R, hdeg, ldeg, watch
+// length, blocker position, m at the last failed check, list offset}; lst[off..]
+// = [watch area of JP_WATCH ids if hdeg > JP_WLIST] [higher ids] [lower ids], each
+// id = h | min(R,31) << 27.
+// A round: phase A -- every vertex whose count is <= JP_WATCH checks its watch list
+// (the higher neighbours still uncoloured when it was built; a list of <= JP_WLIST
+// higher neighbours is its own watch list), resuming at the last blocker when m is
+// unchanged; a vertex that passes writes its colour and queues push tasks; grid
+// barrier; phase B -- each new colour goes into the uncoloured lower neighbours'
+// bitmaps and decrements their counts (the push that brings a count to JP_WATCH
+// activates the vertex), and requested watch lists are built; grid barrier.  All
+// rounds run in ONE persistent cooperative kernel (k_jp_rounds).  Waiting for the
+// count to reach JP_WATCH costs no rounds on R-MAT (CPU simulation) and bounds every
+// check to two warp steps.
 #include <algorithm>
 #include <cstdio>
 #include <cstdlib>
@@ -52,14 +55,16 @@ constexpr int JP_BUDGET = 4096;  // build: rows > JP_BUDGET arcs are split into 
 constexpr int JP_PIECE = 8192;   // arcs per CTA piece of a huge row in the build passes
 constexpr int JP_TILE = 2048;    // build: compact ids per scan tile (JP_THREADS x 8)
 constexpr int JP_TPT = JP_TILE / JP_THREADS;
-constexpr int JP_HDR = 8;        // segment header words
-constexpr int JP_LANE_CHECKS = 4;  // phase A: higher entries a lane checks before the warp takes over
+constexpr int JP_LANE_CHECKS = 4;  // phase A: entries a lane checks before the warp takes over
 constexpr int JP_PUSH = 256;     // phase B: lower entries per push task
 constexpr int JP_PUSH_LANE = 8;  // phase B: tasks of <= JP_PUSH_LANE entries are a lane's
 constexpr uint32_t JP_WATCH = 16;  // a vertex checks once <= JP_WATCH higher neighbours are unpushed
 constexpr uint32_t JP_WLIST = 64;  // higher lists up to JP_WLIST entries are their own watch list
 constexpr uint32_t JP_NOTBUILT = 0xffffffffu;
 constexpr int JP_BUILD = 256;    // phase B: higher entries per watch-list build task
+constexpr uint32_t JP_HBITS = 27;  // list id = h | min(R, 31) << 27
+constexpr uint32_t JP_HMASK = (1u << JP_HBITS) - 1u;
+constexpr uint32_t JP_R5 = 31u;
 
 struct JpArgs {
     const int64_t *rp;   // phase CSR (original ids)
@@ -72,23 +77,25 @@ struct JpArgs {
     int32_t *ov;         // [n] compact id -> original
     uint32_t *hdeg;      // [n] higher degree (count pass), fill cursor (huge rows)
     uint32_t *ldeg;      // [n] lower degree (count pass), fill cursor (huge rows)
-    uint32_t *sbh;       // [n] compact id -> segment base (8-B units)
-    unsigned long long *sbR;  // [n] original id -> sb | R << 32
-    uint32_t *seg;       // segments
+    uint32_t *cidR;      // [n] original id -> list id (h | min(R,31) << 27)
+    uint32_t *col, *cnt, *bm0, *xo;  // [n] hot per-vertex state (see the header)
+    uint4 *meta;         // [2n] per-vertex own data
+    uint32_t *lst;       // watch / higher / lower lists
+    uint32_t *xb;        // bitmap words for colours > 32
     uint32_t *tcnt;      // scan scratch: per tile class counts (2 per tile)
-    unsigned long long *tsum;  // scan scratch: per tile segment words
+    unsigned long long *tsum;  // scan scratch: per tile (list words, extra bitmap words)
     uint32_t *nc;        // [0] = compact count n', [1] = rows of degree > 2
-    uint32_t *ul[2];     // uncoloured lists (segment bases), ping-pong by round
-    uint4 *task;         // push tasks {list word lo, hi, entries, colour}
-    uint2 *btask;        // watch-list build tasks {sb, chunk}
+    uint32_t *ul[2];     // active lists (compact ids), ping-pong by round
+    uint4 *task;         // push tasks {list index lo, hi, entries, colour}
+    uint2 *btask;        // watch-list build tasks {h, chunk}
     uint32_t *ucnt;      // [3] list counts (ring by round)
     uint32_t *pcnt;      // [3] push-task counts (ring by round)
     uint32_t *bcnt;      // [3] build-task counts (ring by round)
     int64_t *huge;       // (piece << 32 | h) items of the huge rows
     uint32_t *huge_cnt;
-    uint32_t *err;       // 1 = timeout / max rounds, 2 = segment offsets overflow
+    uint32_t *err;       // 1 = timeout / max rounds, 2 = offsets overflow
     uint32_t *hist;
-    uint32_t *trace;     // nullable: per-round phase-A end time, push and build tasks (SYM_JP_TRACE)
+    uint32_t *trace;     // nullable: per-round diagnostics (SYM_JP_TRACE)
     unsigned long long *prof;  // algorithmic bytes of the rounds pass (nullable)
     Key k;
 };
@@ -101,19 +108,9 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
 
 __device__ __forceinline__ bool in_set(const uint8_t *inS, uint32_t w) { return inS == nullptr || inS[w] != 0; }
 
-__device__ __forceinline__ uint32_t even(uint32_t x) { return (x + 1u) & ~1u; }
-
-// word offsets inside a segment
 __device__ __forceinline__ uint32_t watch_words(uint32_t hd) { return hd > JP_WLIST ? JP_WATCH : 0u; }
-__device__ __forceinline__ uint64_t seg_bitmap(uint32_t sb) { return 2ull * sb + JP_HDR; }
-// the list a check reads: the watch area (hdeg > JP_WLIST) or the higher list itself
-__device__ __forceinline__ uint64_t seg_watch(uint32_t sb, uint32_t R) { return 2ull * sb + JP_HDR + even(R); }
-__device__ __forceinline__ uint64_t seg_higher(uint32_t sb, uint32_t R, uint32_t hd) {
-    return 2ull * sb + JP_HDR + even(R) + watch_words(hd);
-}
-__device__ __forceinline__ uint64_t seg_lower(uint32_t sb, uint32_t R, uint32_t hd) {
-    return seg_higher(sb, R, hd) + even(hd);
-}
+
+__device__ __forceinline__ uint64_t meta_off(const uint4 &m1) { return (uint64_t)m1.z | ((uint64_t)m1.w << 32); }
 
 // warp-aggregated reservation of k_lane consecutive slots per lane; returns this
 // lane's first slot.  All lanes must call it.
@@ -376,141 +373,169 @@ __device__ __forceinline__ uint32_t jp_words(const JpArgs &A, int64_t h) {
     return (uint32_t)((deg - (int64_t)A.ldeg[h] + 1 + 31) >> 5);
 }
 
-// segment words of h, a multiple of 4 (segments are 16-B aligned)
-__device__ __forceinline__ unsigned long long jp_seg_words(const JpArgs &A, int64_t h) {
-    const uint32_t hd = A.hdeg[h];
-    const unsigned long long w = JP_HDR + even(jp_words(A, h)) + watch_words(hd) + even(hd) + 2ull * A.ldeg[h];
-    return (w + 3ull) & ~3ull;
-}
-
-// per tile of JP_TILE compact ids: segment words
+// per tile of JP_TILE compact ids: list words and extra bitmap words
 __global__ void __launch_bounds__(JP_THREADS) k_jpc_sums(JpArgs A) {
     const uint32_t cnt = A.nc[0];
     const int64_t base = (int64_t)blockIdx.x * JP_TILE;
     if (base >= cnt) return;
-    unsigned long long sw = 0;
+    unsigned long long sl = 0, sx = 0;
     for (int u = 0; u < JP_TPT; u++) {
         const int64_t h = base + u * JP_THREADS + threadIdx.x;
-        if (h < cnt) sw += jp_seg_words(A, h);
+        if (h < cnt) {
+            const uint32_t hd = A.hdeg[h];
+            sl += watch_words(hd) + hd + A.ldeg[h];
+            sx += jp_words(A, h) - 1u;
+        }
     }
-    for (int d = 16; d; d >>= 1) sw += __shfl_xor_sync(FULL, sw, d);
-    __shared__ unsigned long long a;
-    if (threadIdx.x == 0) a = 0;
+    for (int d = 16; d; d >>= 1) {
+        sl += __shfl_xor_sync(FULL, sl, d);
+        sx += __shfl_xor_sync(FULL, sx, d);
+    }
+    __shared__ unsigned long long a[2];
+    if (threadIdx.x == 0) a[0] = a[1] = 0;
     __syncthreads();
-    if (lane_id() == 0) atomicAdd(&a, sw);
+    if (lane_id() == 0) {
+        atomicAdd(&a[0], sl);
+        atomicAdd(&a[1], sx);
+    }
     __syncthreads();
-    if (threadIdx.x == 0) A.tsum[blockIdx.x] = a;
+    if (threadIdx.x == 0) {
+        A.tsum[2 * blockIdx.x] = a[0];
+        A.tsum[2 * blockIdx.x + 1] = a[1];
+    }
 }
 
-// one CTA: exclusive prefix of the tile sums (segment bases must fit 32 bits in
-// 8-B units)
+// one CTA: exclusive prefix of the tile sums (extra bitmap offsets must fit 32 bits,
+// compact ids 27 bits)
 __global__ void __launch_bounds__(1024) k_jpc_sums_scan(JpArgs A, int64_t ntiles) {
     const uint32_t cnt = A.nc[0];
     const int64_t need = ((int64_t)cnt + JP_TILE - 1) / JP_TILE;
     const int64_t used = need < ntiles ? need : ntiles;
     const int64_t per = (used + blockDim.x - 1) / blockDim.x;
     const int64_t t0 = (int64_t)threadIdx.x * per, t1 = used < t0 + per ? used : t0 + per;
-    unsigned long long s0 = 0;
-    for (int64_t t = t0; t < t1; t++) s0 += A.tsum[t];
-    __shared__ unsigned long long w0[32];
-    unsigned long long i0 = s0;
+    unsigned long long s0 = 0, s1 = 0;
+    for (int64_t t = t0; t < t1; t++) {
+        s0 += A.tsum[2 * t];
+        s1 += A.tsum[2 * t + 1];
+    }
+    __shared__ unsigned long long w0[32], w1[32];
+    unsigned long long i0 = s0, i1 = s1;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-        const unsigned long long y0 = __shfl_up_sync(FULL, i0, d);
-        if (lane_id() >= d) i0 += y0;
+        const unsigned long long y0 = __shfl_up_sync(FULL, i0, d), y1 = __shfl_up_sync(FULL, i1, d);
+        if (lane_id() >= d) {
+            i0 += y0;
+            i1 += y1;
+        }
     }
     const int wid = threadIdx.x >> 5;
-    if (lane_id() == 31) w0[wid] = i0;
+    if (lane_id() == 31) {
+        w0[wid] = i0;
+        w1[wid] = i1;
+    }
     __syncthreads();
-    unsigned long long b0 = 0, T0 = 0;
+    unsigned long long b0 = 0, b1 = 0, T1 = 0;
     for (int q = 0; q < (int)(blockDim.x >> 5); q++) {
-        if (q < wid) b0 += w0[q];
-        T0 += w0[q];
+        if (q < wid) {
+            b0 += w0[q];
+            b1 += w1[q];
+        }
+        T1 += w1[q];
     }
-    unsigned long long o0 = b0 + i0 - s0;
+    unsigned long long o0 = b0 + i0 - s0, o1 = b1 + i1 - s1;
     for (int64_t t = t0; t < t1; t++) {
-        const unsigned long long a0 = A.tsum[t];
-        A.tsum[t] = o0;
+        const unsigned long long a0 = A.tsum[2 * t], a1 = A.tsum[2 * t + 1];
+        A.tsum[2 * t] = o0;
+        A.tsum[2 * t + 1] = o1;
         o0 += a0;
+        o1 += a1;
     }
-    if (threadIdx.x == 0 && T0 >= (1ull << 33)) atomicOr(A.err, 2u);
+    if (threadIdx.x == 0 && (T1 >= (1ull << 32) || cnt > JP_HMASK)) atomicOr(A.err, 2u);
 }
 
-// per compact id: segment base, header, zeroed bitmap, the maps; the first round's
-// list = the vertices with <= JP_WATCH higher neighbours
+// per compact id: list offset, meta, hot state, zeroed extra bitmap words, the list
+// id map; the first round's list = the vertices with <= JP_WATCH higher neighbours
 __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
     const uint32_t cnt = A.nc[0];
     const int64_t base = (int64_t)blockIdx.x * JP_TILE;
     if (base >= cnt) return;
-    __shared__ unsigned long long sm0[8];
-    unsigned long long o0 = A.tsum[blockIdx.x];
+    __shared__ unsigned long long sm0[8], sm1[8];
+    unsigned long long o0 = A.tsum[2 * blockIdx.x], o1 = A.tsum[2 * blockIdx.x + 1];
     for (int u = 0; u < JP_TPT; u++) {
         const int64_t h = base + u * JP_THREADS + threadIdx.x;
         const bool active = h < cnt;
-        const unsigned long long words = active ? jp_seg_words(A, h) : 0ull;
-        unsigned long long t0;
-        const unsigned long long p0 = block_excl_scan<unsigned long long>(words, sm0, &t0);
-        const bool first = active && A.hdeg[h] <= JP_WATCH;
+        uint32_t hd = 0, ld = 0, R = 1;
+        if (active) {
+            hd = A.hdeg[h];
+            ld = A.ldeg[h];
+            R = jp_words(A, h);
+        }
+        unsigned long long t0, t1;
+        const unsigned long long p0 =
+            block_excl_scan<unsigned long long>(active ? watch_words(hd) + hd + ld : 0ull, sm0, &t0);
+        const unsigned long long p1 = block_excl_scan<unsigned long long>(active ? R - 1u : 0ull, sm1, &t1);
+        const bool first = active && hd <= JP_WATCH;
         const int64_t slot = warp_append(first, A.ucnt);
         if (active) {
-            const unsigned long long O = o0 + p0;  // a multiple of 4: segment sizes are
-            const uint32_t sb = (uint32_t)(O >> 1);
-            const uint32_t R = jp_words(A, h), hd = A.hdeg[h], ld = A.ldeg[h];
-            uint4 *hp = reinterpret_cast<uint4 *>(A.seg + O);
-            hp[0] = make_uint4(0u, R, hd, ld);
-            hp[1] = make_uint4(hd, hd > JP_WLIST ? JP_NOTBUILT : hd, 0u, 0u);
-            for (uint32_t q = 0; q < R; q++) A.seg[O + JP_HDR + q] = 0u;
-            A.sbh[h] = sb;
-            A.sbR[A.ov[h]] = (unsigned long long)sb | ((unsigned long long)R << 32);
-            if (first) A.ul[0][slot] = sb;
+            const unsigned long long off = o0 + p0;
+            const uint32_t x0 = (uint32_t)(o1 + p1);
+            A.meta[2 * h] = make_uint4(R, hd, ld, hd > JP_WLIST ? JP_NOTBUILT : hd);
+            A.meta[2 * h + 1] = make_uint4(0u, 0u, (uint32_t)off, (uint32_t)(off >> 32));
+            A.col[h] = 0u;
+            A.cnt[h] = hd;
+            A.bm0[h] = 0u;
+            A.xo[h] = x0;
+            for (uint32_t q = 1; q < R; q++) A.xb[x0 + q - 1] = 0u;
+            A.cidR[A.ov[h]] = (uint32_t)h | (min(R, JP_R5) << JP_HBITS);
+            if (first) A.ul[0][slot] = (uint32_t)h;
             A.hdeg[h] = 0;  // fill cursors of the huge rows
             A.ldeg[h] = 0;
         }
         o0 += t0;
+        o1 += t1;
     }
 }
 
 // fixed colour c of a neighbour outside S (COLOR-Rand recolouring) as a forbidden bit
-__device__ __forceinline__ void jp_fixed(const JpArgs &A, uint64_t O, uint32_t R, uint32_t w) {
+__device__ __forceinline__ void jp_fixed(const JpArgs &A, int64_t h, uint32_t R, uint32_t x0, uint32_t w) {
     const uint32_t c = A.color[w];
     if (c == 0) return;
-    const uint32_t q = (c - 1) >> 5;
-    if (q < R) atomicOr(A.seg + O + JP_HDR + q, 1u << ((c - 1) & 31));
+    const uint32_t q = (c - 1) >> 5, bit = 1u << ((c - 1) & 31);
+    if (q == 0) atomicOr(A.bm0 + h, bit);
+    else if (q < R) atomicOr(A.xb + x0 + q - 1, bit);
 }
 
-// fill pass: higher list (segment bases) and lower list (segment base | R), both in
-// CSR order; fixed colours of neighbours outside S
+// fill pass: higher and lower lists (list ids, CSR order); fixed colours of
+// neighbours outside S
 __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
     const uint32_t cnt = A.nc[0];
     const int lane = lane_id();
     const int64_t warp_g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    unsigned long long *seg64 = reinterpret_cast<unsigned long long *>(A.seg);
     for (int64_t base = warp_g * 32; base < cnt; base += nwarps * 32) {
         const int64_t h = base + lane;
         const bool active = h < cnt;
         int32_t v = 0;
         int64_t b = 0, e = 0;
-        uint64_t kv = 0, O = 0, hl = 0, ll = 0;
-        uint32_t R = 0;
+        uint64_t kv = 0, hl = 0, ll = 0;
+        uint32_t R = 0, x0 = 0;
         if (active) {
             v = A.ov[h];
             b = A.rp[v];
             e = A.rp[v + 1];
             kv = vkey(A.k, (uint32_t)v);
-            const uint32_t sb = A.sbh[h];
-            O = 2ull * sb;
-            const uint4 hd = *reinterpret_cast<const uint4 *>(A.seg + O);
-            R = hd.y;
-            hl = seg_higher(sb, R, hd.z);
-            ll = seg_lower(sb, R, hd.z) >> 1;
+            const uint4 m0 = A.meta[2 * h], m1 = A.meta[2 * h + 1];
+            R = m0.x;
+            x0 = A.xo[h];
+            hl = meta_off(m1) + watch_words(m0.y);
+            ll = hl + m0.y;
         }
         if (active && e - b <= JP_SMALL) {
             for (int64_t x = b; x < e; x++) {
                 const uint32_t w = (uint32_t)__ldg(A.ci + x);
-                if (!in_set(A.inS, w)) jp_fixed(A, O, R, w);
-                else if (vkey(A.k, w) > kv) A.seg[hl++] = (uint32_t)A.sbR[w];
-                else seg64[ll++] = A.sbR[w];
+                if (!in_set(A.inS, w)) jp_fixed(A, h, R, x0, w);
+                else if (vkey(A.k, w) > kv) A.lst[hl++] = A.cidR[w];
+                else A.lst[ll++] = A.cidR[w];
             }
         }
         unsigned medm = __ballot_sync(FULL, active && e - b > JP_SMALL && e - b <= JP_BUDGET);
@@ -518,23 +543,24 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
             const int src = __ffs(medm) - 1;
             medm &= medm - 1;
             const int64_t wb = __shfl_sync(FULL, b, src), we = __shfl_sync(FULL, e, src);
-            const uint64_t wk = __shfl_sync(FULL, kv, src), wO = __shfl_sync(FULL, O, src);
-            const uint32_t wR = __shfl_sync(FULL, R, src);
+            const uint64_t wk = __shfl_sync(FULL, kv, src);
+            const int64_t wh = base + src;
+            const uint32_t wR = __shfl_sync(FULL, R, src), wx0 = __shfl_sync(FULL, x0, src);
             uint64_t whl = __shfl_sync(FULL, hl, src), wll = __shfl_sync(FULL, ll, src);
-            for (int64_t x0 = wb; x0 < we; x0 += 32) {
-                const int64_t x = x0 + lane;
+            for (int64_t xb0 = wb; xb0 < we; xb0 += 32) {
+                const int64_t x = xb0 + lane;
                 bool up = false, dn = false;
                 uint32_t w = 0;
                 if (x < we) {
                     w = (uint32_t)__ldg(A.ci + x);
-                    if (!in_set(A.inS, w)) jp_fixed(A, wO, wR, w);
+                    if (!in_set(A.inS, w)) jp_fixed(A, wh, wR, wx0, w);
                     else if (vkey(A.k, w) > wk) up = true;
                     else dn = true;
                 }
                 const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
                 const unsigned lt = (1u << lane) - 1u;
-                if (up) A.seg[whl + __popc(mu & lt)] = (uint32_t)A.sbR[w];
-                if (dn) seg64[wll + __popc(md & lt)] = A.sbR[w];
+                if (up) A.lst[whl + __popc(mu & lt)] = A.cidR[w];
+                if (dn) A.lst[wll + __popc(md & lt)] = A.cidR[w];
                 whl += __popc(mu);
                 wll += __popc(md);
             }
@@ -546,7 +572,6 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
 __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
     const uint32_t cnt = *A.huge_cnt;
     const int lane = lane_id();
-    unsigned long long *seg64 = reinterpret_cast<unsigned long long *>(A.seg);
     for (uint32_t p = blockIdx.x; p < cnt; p += gridDim.x) {
         const int64_t item = A.huge[p];
         const int32_t h = (int32_t)(uint32_t)item;
@@ -555,17 +580,16 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
         const int64_t b = A.rp[v], e = A.rp[v + 1];
         const int64_t pb = b + j * JP_PIECE, pe_ = min(e, pb + JP_PIECE);
         const uint64_t kv = vkey(A.k, (uint32_t)v);
-        const uint32_t sb = A.sbh[h];
-        const uint64_t O = 2ull * sb;
-        const uint4 hd = *reinterpret_cast<const uint4 *>(A.seg + O);
-        const uint64_t hl = seg_higher(sb, hd.y, hd.z), ll = seg_lower(sb, hd.y, hd.z) >> 1;
-        for (int64_t x0 = pb + (threadIdx.x & ~31); x0 < pe_; x0 += JP_HUGE_THREADS) {
-            const int64_t x = x0 + lane;
+        const uint4 m0 = A.meta[2 * h], m1 = A.meta[2 * h + 1];
+        const uint32_t x0 = A.xo[h];
+        const uint64_t hl = meta_off(m1) + watch_words(m0.y), ll = hl + m0.y;
+        for (int64_t xb0 = pb + (threadIdx.x & ~31); xb0 < pe_; xb0 += JP_HUGE_THREADS) {
+            const int64_t x = xb0 + lane;
             bool up = false, dn = false;
             uint32_t w = 0;
             if (x < pe_) {
                 w = (uint32_t)__ldg(A.ci + x);
-                if (!in_set(A.inS, w)) jp_fixed(A, O, hd.y, w);
+                if (!in_set(A.inS, w)) jp_fixed(A, h, m0.x, x0, w);
                 else if (vkey(A.k, w) > kv) up = true;
                 else dn = true;
             }
@@ -578,8 +602,8 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
             pu = __shfl_sync(FULL, pu, 0);
             pd = __shfl_sync(FULL, pd, 0);
             const unsigned lt = (1u << lane) - 1u;
-            if (up) A.seg[hl + pu + __popc(mu & lt)] = (uint32_t)A.sbR[w];
-            if (dn) seg64[ll + pd + __popc(md & lt)] = A.sbR[w];
+            if (up) A.lst[hl + pu + __popc(mu & lt)] = A.cidR[w];
+            if (dn) A.lst[ll + pd + __popc(md & lt)] = A.cidR[w];
         }
     }
 }
@@ -588,7 +612,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
 __global__ void k_jpc_scatter(JpArgs A) {
     const uint32_t cnt = A.nc[0];
     for (int64_t h = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; h < cnt; h += (int64_t)gridDim.x * blockDim.x)
-        A.color[A.ov[h]] = A.seg[2ull * A.sbh[h]];
+        A.color[A.ov[h]] = A.col[h];
 }
 
 // ---------------------------------------------------------------- rounds
@@ -626,28 +650,37 @@ __device__ __forceinline__ void grid_sync(const JrCtl &C, uint32_t &k) {
     __syncthreads();
 }
 
-// neighbour u (segment base e) passes v's check for colour m: coloured with another
-// colour, or uncoloured with m already forbidden for it (q, bit = m's word and bit)
-__device__ __forceinline__ bool nb_ok(uint2 hu, uint32_t bw, uint32_t m, uint32_t q, uint32_t bit) {
-    return hu.x != 0u ? hu.x != m : (q < hu.y && ((bw >> bit) & 1u));
+// Can higher neighbour e (list id) not take colour m (word q, bit)?  Coloured: its
+// colour differs; uncoloured: m is forbidden for it, or m > cap (q >= R).  c = its
+// colour, w = its bitmap word q when q < R (loaded by the caller).
+__device__ __forceinline__ bool nb_ok(const JpArgs &A, uint32_t e, uint32_t c, uint32_t w, uint32_t m, uint32_t q,
+                                      uint32_t bit) {
+    if (c != 0u) return c != m;
+    const uint32_t R5 = e >> JP_HBITS;
+    if (q == 0u || q < R5) return (w >> bit) & 1u;
+    if (R5 < JP_R5) return true;  // m > 32 R >= cap: the neighbour's colour is below m
+    const uint32_t hu = e & JP_HMASK;  // saturated R field: the full count
+    const uint32_t R = __ldg(&A.meta[2 * hu].x);
+    return q >= R || ((__ldcg(A.xb + __ldcg(A.xo + hu) + q - 1) >> bit) & 1u);
 }
 
-__device__ __forceinline__ uint2 ld_hdr(const uint32_t *seg, uint32_t e) {
-    return __ldcg(reinterpret_cast<const uint2 *>(seg + 2ull * e));
+// the neighbour's bitmap word q (q == 0: bm0; q < R: in xb; else unused)
+__device__ __forceinline__ uint32_t nb_word_addr_free(const JpArgs &A, uint32_t e, uint32_t q) {
+    const uint32_t hu = e & JP_HMASK;
+    return q == 0u ? __ldcg(A.bm0 + hu) : (q < (e >> JP_HBITS) ? __ldcg(A.xo + hu) : 0u);
 }
 
-// Phase A of round r: every vertex of the uncoloured list U_r with at most JP_WATCH
-// unpushed higher neighbours checks its watch list (the higher neighbours that were
-// uncoloured when the list was built; every other higher neighbour's colour is
-// already in v's bitmap, so it cannot equal m).  A vertex whose count just dropped
-// to JP_WATCH but whose higher list is longer asks phase B to build the watch list.
+// Phase A of round r: every active vertex (count <= JP_WATCH) checks its watch list
+// (the higher neighbours that were uncoloured when the list was built; every other
+// higher neighbour's colour is already in v's bitmap, so it cannot equal m).  A
+// vertex whose higher list is longer than JP_WLIST asks phase B for its watch list
+// first.
 __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t warp_g, int64_t nwarps,
                                            unsigned long long &bytes) {
     const int lane = lane_id();
     const uint32_t cnt = __ldcg(A.ucnt + r % 3);
     const uint32_t *U = A.ul[r & 1];
     uint32_t *Un = A.ul[(r + 1) & 1];
-    uint32_t *seg = A.seg;
     // a long list is read coalesced (entry it*32*nwarps + warp*32 + lane); a short one
     // spreads over all warps (entry it*32*nwarps + lane*nwarps + warp), so the
     // warp-cooperative steps of different vertices run in parallel
@@ -655,61 +688,63 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
     for (int64_t it = 0; it < cnt; it += nwarps * 32) {
         const int64_t i = it + (spread ? (int64_t)lane * nwarps + warp_g : warp_g * 32 + lane);
         const bool act = i < cnt;
-        uint32_t sb = 0, R = 0, hd = 0, ld = 0, wc = 0, pos = 0, lm = 0, m = 1;
-        int state = 3;  // 0 checking, 1 passed, 2 failed (memo), 3 idle, 4 waiting, 5 build request
+        uint32_t h = 0, R = 1, hd = 0, ld = 0, wc = 0, pos = 0, lm = 0, m = 1;
+        uint64_t off = 0;
+        int state = 3;  // 0 checking, 1 passed, 2 failed (memo), 3 idle, 5 build request
         if (act) {
-            sb = __ldcg(U + i);
-            const uint4 h0 = __ldcg(reinterpret_cast<const uint4 *>(seg + 2ull * sb));
-            const uint4 h1 = __ldcg(reinterpret_cast<const uint4 *>(seg + 2ull * sb + 4));
-            R = h0.y;
-            hd = h0.z;
-            ld = h0.w;
-            wc = h1.y;
-            pos = h1.z;
-            lm = h1.w;
-            bytes += 36;
-            if (h1.x > JP_WATCH) {
-                state = 4;
-            } else if (wc == JP_NOTBUILT) {
+            h = __ldcg(U + i);
+            const uint4 m0 = __ldcg(A.meta + 2 * h), m1 = __ldcg(A.meta + 2 * h + 1);
+            R = m0.x;
+            hd = m0.y;
+            ld = m0.z;
+            wc = m0.w;
+            pos = m1.x;
+            lm = m1.y;
+            off = meta_off(m1);
+            bytes += 40;
+            if (wc == JP_NOTBUILT) {
                 state = 5;
             } else {
                 state = 0;
-                const uint32_t *bm = seg + seg_bitmap(sb);
-                for (uint32_t q = 0; q < R; q++) {  // mex: usually the first word decides
-                    const uint32_t z = ~__ldcg(bm + q);
-                    if (z) {
-                        m = q * 32 + __ffs(z);
-                        break;
+                const uint32_t z0 = ~__ldcg(A.bm0 + h);
+                if (z0) {
+                    m = __ffs(z0);
+                } else {  // colours > 32
+                    const uint32_t *xw = A.xb + __ldcg(A.xo + h);
+                    for (uint32_t k = 1; k < R; k++) {
+                        const uint32_t z = ~__ldcg(xw + k - 1);
+                        if (z) {
+                            m = k * 32 + __ffs(z);
+                            break;
+                        }
                     }
+                    if (m == 1) m = R * 32 + 1;  // unreachable: a zero lies within cap bits
                 }
             }
         }
-        const uint64_t wl = seg_watch(sb, R);
         const uint32_t q = (m - 1) >> 5, bit = (m - 1) & 31;
         uint32_t j = (lm == m && pos < wc) ? pos : 0u;  // m unchanged: resume at the last blocker
-        // ---- lane: the first JP_LANE_CHECKS entries
+        // ---- lane: the first JP_LANE_CHECKS entries (all loads of a stage in flight)
         if (state == 0) {
-            uint32_t e[JP_LANE_CHECKS];
-            uint2 hu[JP_LANE_CHECKS];
-            uint32_t bw[JP_LANE_CHECKS];
+            uint32_t e[JP_LANE_CHECKS], c[JP_LANE_CHECKS], w[JP_LANE_CHECKS];
 #pragma unroll
-            for (int u = 0; u < JP_LANE_CHECKS; u++) e[u] = j + u < wc ? __ldcg(seg + wl + j + u) : 0u;
+            for (int u = 0; u < JP_LANE_CHECKS; u++) e[u] = j + u < wc ? __ldcg(A.lst + off + j + u) : 0u;
 #pragma unroll
             for (int u = 0; u < JP_LANE_CHECKS; u++) {
-                if (j + u < wc) {
-                    hu[u] = ld_hdr(seg, e[u]);
-                    bw[u] = __ldcg(seg + seg_bitmap(e[u]) + q);
-                } else {
-                    hu[u] = make_uint2(0u, 0u);
-                    bw[u] = 0u;
-                }
+                c[u] = j + u < wc ? __ldcg(A.col + (e[u] & JP_HMASK)) : 1u;
+                w[u] = j + u < wc ? nb_word_addr_free(A, e[u], q) : 0u;
+            }
+            if (q > 0) {
+#pragma unroll
+                for (int u = 0; u < JP_LANE_CHECKS; u++)
+                    if (j + u < wc && c[u] == 0u && q < (e[u] >> JP_HBITS)) w[u] = __ldcg(A.xb + w[u] + q - 1);
             }
 #pragma unroll
             for (int u = 0; u < JP_LANE_CHECKS; u++) {
                 if (state == 0) {
                     if (j >= wc) {
                         state = 1;
-                    } else if (!nb_ok(hu[u], bw[u], m, q, bit)) {
+                    } else if (!nb_ok(A, e[u], c[u], w[u], m, q, bit)) {
                         state = 2;
                         pos = j;
                         lm = m;
@@ -719,7 +754,7 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
                 }
             }
             if (state == 0 && j >= wc) state = 1;
-            bytes += 4ull * min(wc, (uint32_t)JP_LANE_CHECKS);
+            bytes += 12ull * min(wc, (uint32_t)JP_LANE_CHECKS);
         }
         // ---- warp: the rest of a list (<= JP_WLIST entries: at most two steps)
         unsigned need = __ballot_sync(FULL, state == 0);
@@ -728,7 +763,7 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
             need &= need - 1;
             uint32_t wj = __shfl_sync(FULL, j, src);
             const uint32_t wwc = __shfl_sync(FULL, wc, src), wm = __shfl_sync(FULL, m, src);
-            const uint64_t wwl = __shfl_sync(FULL, wl, src);
+            const uint64_t woff = __shfl_sync(FULL, off, src);
             const uint32_t wq = (wm - 1) >> 5, wbit = (wm - 1) & 31;
             int wstate = 0;
             uint32_t wpos = 0;
@@ -736,8 +771,11 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
                 const uint32_t jj = wj + lane;
                 bool ok = true;
                 if (jj < wwc) {
-                    const uint32_t eu = __ldcg(seg + wwl + jj);
-                    ok = nb_ok(ld_hdr(seg, eu), __ldcg(seg + seg_bitmap(eu) + wq), wm, wq, wbit);
+                    const uint32_t eu = __ldcg(A.lst + woff + jj);
+                    const uint32_t cu = __ldcg(A.col + (eu & JP_HMASK));
+                    uint32_t wu = nb_word_addr_free(A, eu, wq);
+                    if (wq > 0 && cu == 0u && wq < (eu >> JP_HBITS)) wu = __ldcg(A.xb + wu + wq - 1);
+                    ok = nb_ok(A, eu, cu, wu, wm, wq, wbit);
                 }
                 const unsigned fails = __ballot_sync(FULL, !ok);
                 if (fails) {
@@ -747,7 +785,7 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
                     wj += 32;
                     if (wj >= wwc) wstate = 1;
                 }
-                bytes += lane == 0 ? 128ull : 0ull;
+                bytes += lane == 0 ? 384ull : 0ull;
             }
             if (lane == src) {
                 state = wstate;
@@ -758,17 +796,17 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
             }
         }
         // ---- outcome
-        const bool pass = state == 1, stay = state == 2 || state == 4 || state == 5;
-        if (pass) seg[2ull * sb] = m;
-        if (state == 2) *reinterpret_cast<uint2 *>(seg + 2ull * sb + 6) = make_uint2(pos, lm);
-        if (state == 5) seg[2ull * sb + 5] = 0u;  // the watch list is filled by phase B
+        const bool pass = state == 1, stay = state == 2 || state == 5;
+        if (pass) A.col[h] = m;
+        if (state == 2) *reinterpret_cast<uint2 *>(A.meta + 2 * h + 1) = make_uint2(pos, lm);
+        if (state == 5) reinterpret_cast<uint32_t *>(A.meta + 2 * h)[3] = 0u;  // filled by phase B
         const int64_t slot = warp_append(stay, A.ucnt + (r + 1) % 3);
-        if (stay) Un[slot] = sb;
+        if (stay) Un[slot] = h;
         // push tasks of a new colour
         const uint32_t nt = pass ? (ld + JP_PUSH - 1) / JP_PUSH : 0u;
         const int64_t ts = warp_reserve(nt, A.pcnt + r % 3);
         if (nt) {
-            const uint64_t l0 = seg_lower(sb, R, hd) >> 1;  // u64 index of the lower list
+            const uint64_t l0 = off + watch_words(hd) + hd;  // the lower list
             for (uint32_t t = 0; t < nt; t++) {
                 const uint64_t s0 = l0 + (uint64_t)t * JP_PUSH;
                 A.task[ts + t] = make_uint4((uint32_t)s0, (uint32_t)(s0 >> 32), min(JP_PUSH, ld - t * JP_PUSH), m);
@@ -777,36 +815,45 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
         // watch-list build tasks, one per JP_BUILD higher entries
         const uint32_t nb = state == 5 ? (hd + JP_BUILD - 1) / JP_BUILD : 0u;
         const int64_t bs = warp_reserve(nb, A.bcnt + r % 3);
-        for (uint32_t t = 0; t < nb; t++) A.btask[bs + t] = make_uint2(sb, t);
+        for (uint32_t t = 0; t < nb; t++) A.btask[bs + t] = make_uint2(h, t);
         bytes += (state == 2 ? 8ull : 0ull) + (stay ? 4ull : 0ull) + (pass ? 4ull + 16ull * nt : 0ull) + 8ull * nb;
     }
 }
 
-// a new colour c (word q, bit) for lower neighbours x[u] = sb | R << 32 (flags act):
-// the forbidden bits, and one higher neighbour less to wait for; the push that brings
-// a count to JP_WATCH activates w (next round's list; there it asks for its watch
-// list).  All atomics of the batch are in flight together.
-// A neighbour that is already coloured (early commits) needs neither; one whose count
-// is already <= JP_WATCH needs only the bit: both are read first (plain L2 loads) so
-// the atomics go only where they matter.
+// A new colour c (word q, bit) for lower neighbours e[u] (list ids, flags act): a
+// neighbour already coloured (early commit) needs nothing; otherwise its forbidden
+// bit and one higher neighbour less to wait for.  The push that brings a count to
+// JP_WATCH activates the neighbour (next round's list).  Each stage's loads/atomics
+// are in flight together.
 template <int K>
-__device__ __forceinline__ void jp_push(const JpArgs &A, uint32_t r, uint32_t *seg, const unsigned long long (&x)[K],
-                                        bool (&act)[K], uint32_t q, uint32_t bit) {
-    uint32_t old[K], cw[K];
+__device__ __forceinline__ void jp_push(const JpArgs &A, uint32_t r, const uint32_t (&e)[K], bool (&act)[K],
+                                        uint32_t q, uint32_t bit) {
+    uint32_t old[K], x[K];
 #pragma unroll
-    for (int u = 0; u < K; u++) cw[u] = act[u] ? __ldcg(seg + 2ull * (uint32_t)x[u]) : 1u;  // colour
+    for (int u = 0; u < K; u++) act[u] = act[u] && __ldcg(A.col + (e[u] & JP_HMASK)) == 0u;
 #pragma unroll
-    for (int u = 0; u < K; u++) act[u] = act[u] && cw[u] == 0u;
+    for (int u = 0; u < K; u++) old[u] = act[u] ? atomicSub(A.cnt + (e[u] & JP_HMASK), 1u) : 0u;
+    if (q == 0) {
 #pragma unroll
-    for (int u = 0; u < K; u++) old[u] = act[u] ? atomicSub(seg + 2ull * (uint32_t)x[u] + 4, 1u) : 0u;
+        for (int u = 0; u < K; u++)
+            if (act[u]) atomicOr(A.bm0 + (e[u] & JP_HMASK), 1u << bit);
+    } else {
 #pragma unroll
-    for (int u = 0; u < K; u++)
-        if (act[u] && q < (uint32_t)(x[u] >> 32)) atomicOr(seg + seg_bitmap((uint32_t)x[u]) + q, 1u << bit);
+        for (int u = 0; u < K; u++) {
+            const uint32_t hw = e[u] & JP_HMASK, R5 = e[u] >> JP_HBITS;
+            bool go = act[u] && q < R5;
+            if (act[u] && !go && R5 == JP_R5) go = q < __ldg(&A.meta[2 * hw].x);
+            x[u] = go ? __ldcg(A.xo + hw) : 0xffffffffu;
+        }
+#pragma unroll
+        for (int u = 0; u < K; u++)
+            if (x[u] != 0xffffffffu) atomicOr(A.xb + x[u] + q - 1, 1u << bit);
+    }
 #pragma unroll
     for (int u = 0; u < K; u++) {
         if (act[u] && old[u] == JP_WATCH + 1u) {
             const uint32_t slot = atomicAdd(A.ucnt + (r + 1) % 3, 1u);
-            A.ul[(r + 1) & 1][slot] = (uint32_t)x[u];
+            A.ul[(r + 1) & 1][slot] = e[u] & JP_HMASK;
         }
     }
 }
@@ -816,8 +863,6 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, int64_t 
                                            unsigned long long &bytes) {
     const int lane = lane_id();
     const uint32_t cnt = __ldcg(A.pcnt + r % 3);
-    uint32_t *seg = A.seg;
-    const unsigned long long *seg64 = reinterpret_cast<const unsigned long long *>(seg);
     for (int64_t base = warp_g; base - warp_g < cnt; base += nwarps * 32) {
         const int64_t i = base + (int64_t)lane * nwarps;  // tasks spread over all warps
         uint4 tk = make_uint4(0u, 0u, 0u, 0u);
@@ -826,15 +871,15 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, int64_t 
         const bool small = tk.z > 0 && tk.z <= JP_PUSH_LANE;
         if (small) {
             const uint32_t q = (tk.w - 1) >> 5, bit = (tk.w - 1) & 31;
-            unsigned long long x[JP_PUSH_LANE];
+            uint32_t e[JP_PUSH_LANE];
             bool act[JP_PUSH_LANE];
 #pragma unroll
             for (int u = 0; u < JP_PUSH_LANE; u++) {
                 act[u] = u < (int)tk.z;
-                x[u] = act[u] ? __ldcs(seg64 + s0 + u) : 0ull;
+                e[u] = act[u] ? __ldcs(A.lst + s0 + u) : 0u;
             }
-            jp_push<JP_PUSH_LANE>(A, r, seg, x, act, q, bit);
-            bytes += 8ull * tk.z;
+            jp_push<JP_PUSH_LANE>(A, r, e, act, q, bit);
+            bytes += 4ull * tk.z;
         }
         unsigned bigm = __ballot_sync(FULL, tk.z > JP_PUSH_LANE);
         while (bigm) {
@@ -844,41 +889,42 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, int64_t 
             const uint32_t wn = __shfl_sync(FULL, tk.z, src), wc = __shfl_sync(FULL, tk.w, src);
             const uint32_t q = (wc - 1) >> 5, bit = (wc - 1) & 31;
             constexpr int K = JP_PUSH / 32;
-            unsigned long long x[K];
+            uint32_t e[K];
             bool act[K];
 #pragma unroll
             for (int u = 0; u < K; u++) {
                 act[u] = u * 32 + lane < (int)wn;
-                x[u] = act[u] ? __ldcs(seg64 + ws + u * 32 + lane) : 0ull;
+                e[u] = act[u] ? __ldcs(A.lst + ws + u * 32 + lane) : 0u;
             }
-            jp_push<K>(A, r, seg, x, act, q, bit);
-            bytes += lane == 0 ? 8ull * wn : 0ull;
+            jp_push<K>(A, r, e, act, q, bit);
+            bytes += lane == 0 ? 4ull * wn : 0ull;
         }
     }
     // watch lists: a warp per task filters JP_BUILD higher entries (uncoloured ones kept)
     const uint32_t nbt = __ldcg(A.bcnt + r % 3);
     for (int64_t t = warp_g; t < nbt; t += nwarps) {
         const uint2 bt = __ldcg(A.btask + t);
-        const uint4 h0 = __ldcg(reinterpret_cast<const uint4 *>(seg + 2ull * bt.x));
-        const uint64_t hl = seg_higher(bt.x, h0.y, h0.z), wl = seg_watch(bt.x, h0.y);
-        const uint32_t j0 = bt.y * JP_BUILD, j1 = min(h0.z, j0 + JP_BUILD);
+        const uint4 m0 = __ldcg(A.meta + 2 * bt.x), m1 = __ldcg(A.meta + 2 * bt.x + 1);
+        const uint64_t wl = meta_off(m1), hl = wl + watch_words(m0.y);
+        uint32_t *wcp = reinterpret_cast<uint32_t *>(A.meta + 2 * bt.x) + 3;
+        const uint32_t j0 = bt.y * JP_BUILD, j1 = min(m0.y, j0 + JP_BUILD);
         constexpr int K = JP_BUILD / 32;
         uint32_t e[K], c[K];
 #pragma unroll
-        for (int u = 0; u < K; u++) e[u] = j0 + u * 32 + lane < j1 ? __ldcs(seg + hl + j0 + u * 32 + lane) : 0u;
+        for (int u = 0; u < K; u++) e[u] = j0 + u * 32 + lane < j1 ? __ldcs(A.lst + hl + j0 + u * 32 + lane) : 0u;
 #pragma unroll
-        for (int u = 0; u < K; u++) c[u] = j0 + u * 32 + lane < j1 ? __ldcg(seg + 2ull * e[u]) : 1u;
+        for (int u = 0; u < K; u++) c[u] = j0 + u * 32 + lane < j1 ? __ldcg(A.col + (e[u] & JP_HMASK)) : 1u;
 #pragma unroll
         for (int u = 0; u < K; u++) {
             const bool keep = c[u] == 0u;
             const unsigned mk = __ballot_sync(FULL, keep);
             uint32_t p0 = 0;
-            if (mk && lane == 0) p0 = atomicAdd(seg + 2ull * bt.x + 5, (uint32_t)__popc(mk));
+            if (mk && lane == 0) p0 = atomicAdd(wcp, (uint32_t)__popc(mk));
             p0 = __shfl_sync(FULL, p0, 0);
             const uint32_t p = p0 + __popc(mk & ((1u << lane) - 1u));
-            if (keep && p < JP_WATCH) seg[wl + p] = e[u];
+            if (keep && p < JP_WATCH) A.lst[wl + p] = e[u];
         }
-        bytes += lane == 0 ? 4ull * (j1 - j0) : 0ull;
+        bytes += lane == 0 ? 8ull * (j1 - j0) : 0ull;
     }
 }
 
@@ -983,17 +1029,21 @@ void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
     w.ov = a.take<int32_t>((size_t)n + 1);
     w.hdeg = a.take<uint32_t>((size_t)n + 1);
     w.ldeg = a.take<uint32_t>((size_t)n + 1);
-    w.sbh = a.take<uint32_t>((size_t)n + 1);
-    w.sbR = a.take<unsigned long long>((size_t)n + 1);
+    w.cidR = a.take<uint32_t>((size_t)n + 1);
+    w.col = a.take<uint32_t>((size_t)n + 1);
+    w.cnt = a.take<uint32_t>((size_t)n + 1);
+    w.bm0 = a.take<uint32_t>((size_t)n + 1);
+    w.xo = a.take<uint32_t>((size_t)n + 1);
+    w.meta = a.take<uint4>(2 * (size_t)n + 2);
     w.ul[0] = a.take<uint32_t>((size_t)n + 1);
     w.ul[1] = a.take<uint32_t>((size_t)n + 1);
-    // segments: header 8 + bitmap (sum of ceil(cap/32) <= (nnz+n)/32 + n) + higher list
-    // (one word per arc) + lower list (two words per arc), each part padded to even
-    // and the whole to 4 words: <= 14 n + (nnz+n)/32 + 2 nnz words
-    w.seg_words = 14 * n + (nnz + n) / 32 + 2 * nnz + 64;
-    w.seg = a.take<uint32_t>((size_t)w.seg_words);
+    // lists: watch areas (<= JP_WATCH per vertex) + one id per arc (higher or lower)
+    w.lst_words = (int64_t)JP_WATCH * n + nnz + 2;
+    w.lst = a.take<uint32_t>((size_t)w.lst_words);
+    // extra bitmap words: sum of ceil(cap/32) - 1 <= (nnz + n)/32
+    w.xb = a.take<uint32_t>((size_t)((nnz + n) / 32 + 2));
     w.tcnt = a.take<uint32_t>(2 * (size_t)ntiles);
-    w.tsum = a.take<unsigned long long>((size_t)ntiles);
+    w.tsum = a.take<unsigned long long>(2 * (size_t)ntiles);
     w.ntiles = ntiles;
     w.task_cap = n + nnz / JP_PUSH + 2;  // tasks of one round <= all tasks
     w.task = a.take<uint4>((size_t)w.task_cap);
@@ -1004,7 +1054,7 @@ void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
     w.sync = a.take<uint32_t>(64);  // rounds kernel: barrier / counters / error words
 }
 
-// Build: compact ids, segments (bitmaps, higher and lower lists), the first round's
+// Build: compact ids, hot state, meta, higher and lower lists, the first round's
 // list.  sync words: [0] barrier arrivals, [1] barrier generation, [4..6] list
 // counts, [8..10] push-task counts, [12..14] build-task counts, [32] error, [33]
 // rounds, [40..41] compact counts.
@@ -1026,9 +1076,14 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     A.ov = w.ov;
     A.hdeg = w.hdeg;
     A.ldeg = w.ldeg;
-    A.sbh = w.sbh;
-    A.sbR = w.sbR;
-    A.seg = w.seg;
+    A.cidR = w.cidR;
+    A.col = w.col;
+    A.cnt = w.cnt;
+    A.bm0 = w.bm0;
+    A.xo = w.xo;
+    A.meta = w.meta;
+    A.lst = w.lst;
+    A.xb = w.xb;
     A.tcnt = w.tcnt;
     A.tsum = w.tsum;
     A.nc = w.sync + 40;
@@ -1129,7 +1184,7 @@ static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t 
     if (err) {
         SYM_TRY(read_u32(C.levels, &levels, s));
         if (err & 2u) {
-            set_error("JP: segment offsets exceed 2^35 bytes");
+            set_error("JP: more than 2^27 vertices or 2^32 extra bitmap words");
             return SYM_EINVAL;
         }
         const bool rounds = f.p.max_rounds && levels + 1 >= f.p.max_rounds;
