@@ -56,10 +56,19 @@ constexpr int JP_PIECE = 8192;   // arcs per CTA piece of a huge row in the buil
 constexpr int JP_TILE = 2048;    // build: compact ids per scan tile (JP_THREADS x 8)
 constexpr int JP_TPT = JP_TILE / JP_THREADS;
 constexpr int JP_LANE_CHECKS = 4;  // phase A: entries a lane checks before the warp takes over
-constexpr int JP_PUSH = 256;     // phase B: lower entries per push task
+#ifndef SYM_JP_PUSH
+#define SYM_JP_PUSH 256
+#endif
+#ifndef SYM_JP_WATCH
+#define SYM_JP_WATCH 64
+#endif
+#ifndef SYM_JP_WLIST
+#define SYM_JP_WLIST 64
+#endif
+constexpr int JP_PUSH = SYM_JP_PUSH;  // phase B: lower entries per push task
 constexpr int JP_PUSH_LANE = 8;  // phase B: tasks of <= JP_PUSH_LANE entries are a lane's
-constexpr uint32_t JP_WATCH = 16;  // a vertex checks once <= JP_WATCH higher neighbours are unpushed
-constexpr uint32_t JP_WLIST = 64;  // higher lists up to JP_WLIST entries are their own watch list
+constexpr uint32_t JP_WATCH = SYM_JP_WATCH;  // a vertex checks once <= JP_WATCH higher neighbours are unpushed
+constexpr uint32_t JP_WLIST = SYM_JP_WLIST;  // higher lists up to JP_WLIST entries are their own watch list
 constexpr uint32_t JP_NOTBUILT = 0xffffffffu;
 constexpr int JP_BUILD = 256;    // phase B: higher entries per watch-list build task
 constexpr uint32_t JP_HBITS = 27;  // list id = h | min(R, 31) << 27
@@ -506,7 +515,8 @@ __device__ __forceinline__ void jp_fixed(const JpArgs &A, int64_t h, uint32_t R,
 }
 
 // fill pass: higher and lower lists (list ids, CSR order); fixed colours of
-// neighbours outside S
+// neighbours outside S.  Columns and lists stream (evict-first) so the id map stays
+// in L2 for the gathers.
 __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
     const uint32_t cnt = A.nc[0];
     const int lane = lane_id();
@@ -532,10 +542,10 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
         }
         if (active && e - b <= JP_SMALL) {
             for (int64_t x = b; x < e; x++) {
-                const uint32_t w = (uint32_t)__ldg(A.ci + x);
+                const uint32_t w = (uint32_t)__ldcs(A.ci + x);
                 if (!in_set(A.inS, w)) jp_fixed(A, h, R, x0, w);
-                else if (vkey(A.k, w) > kv) A.lst[hl++] = A.cidR[w];
-                else A.lst[ll++] = A.cidR[w];
+                else if (vkey(A.k, w) > kv) __stcs(A.lst + hl++, A.cidR[w]);
+                else __stcs(A.lst + ll++, A.cidR[w]);
             }
         }
         unsigned medm = __ballot_sync(FULL, active && e - b > JP_SMALL && e - b <= JP_BUDGET);
@@ -552,15 +562,15 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
                 bool up = false, dn = false;
                 uint32_t w = 0;
                 if (x < we) {
-                    w = (uint32_t)__ldg(A.ci + x);
+                    w = (uint32_t)__ldcs(A.ci + x);
                     if (!in_set(A.inS, w)) jp_fixed(A, wh, wR, wx0, w);
                     else if (vkey(A.k, w) > wk) up = true;
                     else dn = true;
                 }
                 const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
                 const unsigned lt = (1u << lane) - 1u;
-                if (up) A.lst[whl + __popc(mu & lt)] = A.cidR[w];
-                if (dn) A.lst[wll + __popc(md & lt)] = A.cidR[w];
+                if (up) __stcs(A.lst + whl + __popc(mu & lt), A.cidR[w]);
+                if (dn) __stcs(A.lst + wll + __popc(md & lt), A.cidR[w]);
                 whl += __popc(mu);
                 wll += __popc(md);
             }
@@ -588,7 +598,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
             bool up = false, dn = false;
             uint32_t w = 0;
             if (x < pe_) {
-                w = (uint32_t)__ldg(A.ci + x);
+                w = (uint32_t)__ldcs(A.ci + x);
                 if (!in_set(A.inS, w)) jp_fixed(A, h, m0.x, x0, w);
                 else if (vkey(A.k, w) > kv) up = true;
                 else dn = true;
@@ -602,8 +612,8 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
             pu = __shfl_sync(FULL, pu, 0);
             pd = __shfl_sync(FULL, pd, 0);
             const unsigned lt = (1u << lane) - 1u;
-            if (up) A.lst[hl + pu + __popc(mu & lt)] = A.cidR[w];
-            if (dn) A.lst[ll + pd + __popc(md & lt)] = A.cidR[w];
+            if (up) __stcs(A.lst + hl + pu + __popc(mu & lt), A.cidR[w]);
+            if (dn) __stcs(A.lst + ll + pd + __popc(md & lt), A.cidR[w]);
         }
     }
 }
