@@ -50,7 +50,10 @@ namespace sym {
 
 constexpr int JP_THREADS = 256;
 constexpr int JP_HUGE_THREADS = 512;
-constexpr int JP_SMALL = 32;     // build: rows <= JP_SMALL arcs are handled by one lane
+#ifndef SYM_JP_SMALL
+#define SYM_JP_SMALL 32
+#endif
+constexpr int JP_SMALL = SYM_JP_SMALL;  // build: rows <= JP_SMALL arcs are handled by one lane
 constexpr int JP_BUDGET = 4096;  // build: rows > JP_BUDGET arcs are split into pieces
 constexpr int JP_PIECE = 8192;   // arcs per CTA piece of a huge row in the build passes
 constexpr int JP_TILE = 2048;    // build: compact ids per scan tile (JP_THREADS x 8)
@@ -578,42 +581,60 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
     }
 }
 
-// huge rows: one CTA per piece, positions reserved per warp on the row's cursors
+// huge rows: one CTA per piece; each warp counts its 512-arc slice (ballots), reserves
+// its positions on the row's two cursors with one atomic each, then writes (the
+// slice is re-read from L2)
 __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
+    constexpr int SLICE = JP_PIECE / (JP_HUGE_THREADS / 32);
     const uint32_t cnt = *A.huge_cnt;
     const int lane = lane_id();
+    const unsigned lt = (1u << lane) - 1u;
     for (uint32_t p = blockIdx.x; p < cnt; p += gridDim.x) {
         const int64_t item = A.huge[p];
         const int32_t h = (int32_t)(uint32_t)item;
         const int64_t j = item >> 32;
         const int32_t v = A.ov[h];
         const int64_t b = A.rp[v], e = A.rp[v + 1];
-        const int64_t pb = b + j * JP_PIECE, pe_ = min(e, pb + JP_PIECE);
+        const int64_t sb0 = b + j * JP_PIECE + (int64_t)(threadIdx.x >> 5) * SLICE;
+        const int64_t se = min(e, sb0 + SLICE);
         const uint64_t kv = vkey(A.k, (uint32_t)v);
         const uint4 m0 = A.meta[2 * h], m1 = A.meta[2 * h + 1];
         const uint32_t x0 = A.xo[h];
         const uint64_t hl = meta_off(m1) + watch_words(m0.y), ll = hl + m0.y;
-        for (int64_t xb0 = pb + (threadIdx.x & ~31); xb0 < pe_; xb0 += JP_HUGE_THREADS) {
-            const int64_t x = xb0 + lane;
+        uint32_t nu = 0, nd = 0;
+        for (int64_t x = sb0 + lane; x - lane < se; x += 32) {
+            bool up = false, dn = false;
+            if (x < se) {
+                const uint32_t w = (uint32_t)__ldg(A.ci + x);
+                if (in_set(A.inS, w)) {
+                    up = vkey(A.k, w) > kv;
+                    dn = !up;
+                }
+            }
+            nu += __popc(__ballot_sync(FULL, up));
+            nd += __popc(__ballot_sync(FULL, dn));
+        }
+        uint32_t pu = 0, pd = 0;
+        if (lane == 0) {
+            if (nu) pu = atomicAdd(A.hdeg + h, nu);
+            if (nd) pd = atomicAdd(A.ldeg + h, nd);
+        }
+        pu = __shfl_sync(FULL, pu, 0);
+        pd = __shfl_sync(FULL, pd, 0);
+        for (int64_t x = sb0 + lane; x - lane < se; x += 32) {
             bool up = false, dn = false;
             uint32_t w = 0;
-            if (x < pe_) {
-                w = (uint32_t)__ldcs(A.ci + x);
+            if (x < se) {
+                w = (uint32_t)__ldg(A.ci + x);
                 if (!in_set(A.inS, w)) jp_fixed(A, h, m0.x, x0, w);
                 else if (vkey(A.k, w) > kv) up = true;
                 else dn = true;
             }
             const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
-            uint32_t pu = 0, pd = 0;
-            if (lane == 0) {
-                if (mu) pu = atomicAdd(A.hdeg + h, (uint32_t)__popc(mu));
-                if (md) pd = atomicAdd(A.ldeg + h, (uint32_t)__popc(md));
-            }
-            pu = __shfl_sync(FULL, pu, 0);
-            pd = __shfl_sync(FULL, pd, 0);
-            const unsigned lt = (1u << lane) - 1u;
             if (up) __stcs(A.lst + hl + pu + __popc(mu & lt), A.cidR[w]);
             if (dn) __stcs(A.lst + ll + pd + __popc(md & lt), A.cidR[w]);
+            pu += __popc(mu);
+            pd += __popc(md);
         }
     }
 }

@@ -8,12 +8,11 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 OUT = os.path.join(ROOT, "build", "variants")
 VARIANTS = {
-    "w32": ["-DSYM_JP_WATCH=32"],
-    "w48": ["-DSYM_JP_WATCH=48"],
-    "w64": ["-DSYM_JP_WATCH=64"],
-    "w64l128": ["-DSYM_JP_WATCH=64", "-DSYM_JP_WLIST=128"],
-    "w128l128": ["-DSYM_JP_WATCH=128", "-DSYM_JP_WLIST=128"],
-    "w32l32": ["-DSYM_JP_WATCH=32", "-DSYM_JP_WLIST=32"],
+    "base": [],
+    "nopf": ["-DSYM_JP_NOPF"],
+    "small8": ["-DSYM_JP_SMALL=8"],
+    "small16": ["-DSYM_JP_SMALL=16"],
+    "minb1": ["-DSYM_JR_MINB=1"],
 }
 
 if sys.argv[1] == "build":
