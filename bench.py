@@ -34,8 +34,10 @@ METRIC = "MIS/MM/COLOR edges/s at 1/2/4/8 B200; % of HBM roofline; vs CPU oracle
 TRAFFIC = {
     "split": 4.51e9,       # k_split<DEGK> / <RAND> at R-MAT s24 (profiles/r1b_ncu.md): 2.22 GB read + 2.29 GB written
     "mm_round0": 0.719e9,  # k_round0<MM> on the RAND-4 intra CSR
-    "jp_init": 2.36e9,     # k_jp_init: 1.75 GB read + 0.61 GB written (records)
-    "jp_levels": 10.21e9,  # k_jp_levels: 7.43 GB read + 2.78 GB written (records, tasks, colours, columns)
+    # COLOR-Deg2 at R-MAT s24 (profiles/r1e_color_launches.csv): the build kernels
+    # (k_jpc_*: compact ids, counts, lists) and the early-commit rounds kernel
+    "jp_build": 13.07e9,
+    "jp_rounds": 14.31e9,  # k_jp_rounds: 12.05 GB read + 2.26 GB written (lists, hot records, meta)
 }
 
 
@@ -53,7 +55,10 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=4)
     ap.add_argument("--profile-only", action="store_true", help="short run for ncu (no JSON contract)")
-    ap.add_argument("--sequential", action="store_true", help="one stream, the five calls in order")
+    ap.add_argument("--sequential", action="store_true", help="one stream, the five calls in order (default)")
+    ap.add_argument("--concurrent", action="store_true",
+                    help="two streams (schedule.ConcurrentStep); slower since the early-commit JP kernel "
+                         "holds every SM's register file")
     return ap.parse_args()
 
 
@@ -196,6 +201,7 @@ def main():
     def step_concurrent(rp=rp, ci=ci):
         return _cs(rp, ci)
 
+    args.sequential = not args.concurrent
     step = step_sequential if args.sequential else step_concurrent
 
     if args.profile_only:
@@ -291,14 +297,14 @@ def main():
     # the dominant kernel = the class with the most device time in the step
     dominant_overall = max(prof, key=lambda k: prof[k]["ms"]) if prof else None
     roof = roof_of(dominant_overall) if dominant_overall else None
-    if roof is not None and dominant_overall == "jp_levels":
-        # JP is bound by its dependency depth, not by bytes: one level = a burst of
-        # scattered record atomics + one grid barrier
-        levels = st_col["rounds"][0]
+    if roof is not None and dominant_overall == "jp_rounds":
+        # the colouring is bound by its number of dependent rounds, not by bytes: a
+        # round = checks, grid barrier, pushes, grid barrier
+        rounds = st_col["rounds"][0]
         roof["latency_model"] = {
-            "levels": levels, "us_per_level": roof["ms_per_launch"] * 1e3 / max(1, levels),
-            "grid_barrier_us": 1.4, "note": "depth-bound: levels x (push burst + grid barrier); "
-            "HBM frac is reported for the algorithmic bytes only"}
+            "rounds": rounds, "plain_jp_levels": 5063, "us_per_round": roof["ms_per_launch"] * 1e3 / max(1, rounds),
+            "grid_barriers_per_round": 2, "note": "round-bound: rounds x (dependent L2/DRAM round trips + 2 grid "
+            "barriers); HBM frac is reported for the algorithmic bytes only"}
     rooflines = {k: roof_of(k) for k in prof if roof_of(k)}
 
     # ---- e2e through the public API with pinned host buffers: every step copies its

@@ -164,11 +164,10 @@ struct ColorWs {
     int32_t *ov = nullptr;         // compact id -> original
     uint32_t *hdeg = nullptr;      // higher / lower degrees (build), fill cursors
     uint32_t *ldeg = nullptr;
-    uint32_t *cidR = nullptr;      // original id -> list id (compact id | min(R,31) << 27)
-    uint32_t *col = nullptr;       // hot per-vertex state: colour, count, bitmap word 0,
-    uint32_t *cnt = nullptr;       //   offset of the extra bitmap words
-    uint32_t *bm0 = nullptr;
-    uint32_t *xo = nullptr;
+    uint32_t *abits = nullptr;     // S vertices with phase arcs (bitmap) and the
+    uint32_t *apre = nullptr;      //   exclusive popcount prefix per word: compact id = rank
+    uint4 *hot = nullptr;          // hot per-vertex state {colour, count, bitmap word 0,
+                                   //   offset of the extra bitmap words}
     uint4 *meta = nullptr;         // per-vertex own data (2 x 16 B)
     uint32_t *ul[2] = {nullptr, nullptr};  // active lists (ping-pong by round)
     uint32_t *lst = nullptr;       // watch / higher / lower lists

@@ -19,17 +19,16 @@
 // passes.  Result: the same colours in ~530 rounds instead of 5 063 levels at R-MAT
 // s24 (CPU simulation and GPU).
 //
-// Layout (built once per call; S vertices with phase arcs get compact ids h, rows of
-// degree > 2 first; a vertex without any phase arc takes colour 1 at once).  The
-// per-vertex state other vertices touch is split into compact arrays so the hot set
-// stays in L2 (4 x 4 B per vertex, 90 MB at R-MAT s24):
-//   col[h]  colour (0 = not yet)          cnt[h]  higher neighbours not yet pushed
-//   bm0[h]  forbidden colours 1..32       xo[h]   offset of h's words for colours
-//                                                 33..32R in xb[] (R-1 words)
-// with R = ceil(cap/32).  meta[h] (32 B, read by h itself) = {R, hdeg, ldeg, watch
+// Layout (built once per call; the S vertices with phase arcs get compact ids h =
+// their rank in id order; a vertex without any phase arc takes colour 1 at once).  The
+// per-vertex state other vertices touch is one 16-B record in a compact array, so a
+// check or a push touches ONE sector and the hot set (90 MB at R-MAT s24) is mostly
+// L2-resident: hot[h] = {colour (0 = not yet), count = higher neighbours not yet
+// pushed, forbidden colours 1..32, offset of h's words for colours 33..32R in xb[]
+// (R-1 words) | min(R,31) << 27}, R = ceil(cap/32).  meta[h] (32 B, read by h itself) = {R, hdeg, ldeg, watch
 // length, blocker position, m at the last failed check, list offset}; lst[off..]
-// = [watch area of JP_WATCH ids if hdeg > JP_WLIST] [higher ids] [lower ids], each
-// id = h | min(R,31) << 27.
+// = [watch area of JP_WATCH ids if hdeg > JP_WLIST] [higher ids] [lower ids] (compact
+// ids).
 // A round: phase A -- every vertex whose count is <= JP_WATCH checks its watch list
 // (the higher neighbours still uncoloured when it was built; a list of <= JP_WLIST
 // higher neighbours is its own watch list), resuming at the last blocker when m is
@@ -74,7 +73,7 @@ constexpr uint32_t JP_WATCH = SYM_JP_WATCH;  // a vertex checks once <= JP_WATCH
 constexpr uint32_t JP_WLIST = SYM_JP_WLIST;  // higher lists up to JP_WLIST entries are their own watch list
 constexpr uint32_t JP_NOTBUILT = 0xffffffffu;
 constexpr int JP_BUILD = 256;    // phase B: higher entries per watch-list build task
-constexpr uint32_t JP_HBITS = 27;  // list id = h | min(R, 31) << 27
+constexpr uint32_t JP_HBITS = 27;  // hot.w = offset of the extra bitmap words | min(R, 31) << 27
 constexpr uint32_t JP_HMASK = (1u << JP_HBITS) - 1u;
 constexpr uint32_t JP_R5 = 31u;
 
@@ -89,8 +88,9 @@ struct JpArgs {
     int32_t *ov;         // [n] compact id -> original
     uint32_t *hdeg;      // [n] higher degree (count pass), fill cursor (huge rows)
     uint32_t *ldeg;      // [n] lower degree (count pass), fill cursor (huge rows)
-    uint32_t *cidR;      // [n] original id -> list id (h | min(R,31) << 27)
-    uint32_t *col, *cnt, *bm0, *xo;  // [n] hot per-vertex state (see the header)
+    uint32_t *abits;     // [n/32] S vertices with phase arcs (rank = compact id)
+    uint32_t *apre;      // [n/32] exclusive prefix of the bitmap words' popcounts
+    uint4 *hot;          // [n] hot per-vertex state {col, cnt, bm0, xo} (see the header)
     uint4 *meta;         // [2n] per-vertex own data
     uint32_t *lst;       // watch / higher / lower lists
     uint32_t *xb;        // bitmap words for colours > 32
@@ -168,119 +168,106 @@ __device__ __forceinline__ T block_excl_scan(T x, T *sm, T *total) {
 }
 
 // ---------------------------------------------------------------- build: compact ids
-// class of position i of S: 0 = degree > 2, 1 = 1..2 arcs, 2 = no phase arc
-__device__ __forceinline__ int jp_class(const JpArgs &A, int64_t i, uint32_t cnt, int32_t &v) {
-    v = -1;
-    if (i >= cnt) return 2;
-    v = A.in_list ? A.in_list[i] : (int32_t)i;
-    const int64_t d = A.rp[v + 1] - A.rp[v];
-    return d > 2 ? 0 : (d > 0 ? 1 : 2);
+// The S vertices with phase arcs are numbered by rank in id order:
+//   h(v) = apre[v >> 5] + popc(abits[v >> 5] & lanes below v)
+// so a list id is computed from 4 MB of bitmap + prefix (L2/L1-resident at R-MAT
+// s24) instead of gathered from an n-entry map.  A vertex of S without phase arcs
+// takes colour 1 at once.
+__device__ __forceinline__ uint32_t jp_rank(const JpArgs &A, uint32_t v) {
+    return __ldg(A.apre + (v >> 5)) + __popc(__ldg(A.abits + (v >> 5)) & ((1u << (v & 31)) - 1u));
 }
 
-__device__ __forceinline__ uint32_t s_count(const JpArgs &A) {
-    return A.in_list ? *A.in_cnt : (uint32_t)A.implicit_n;
+// implicit S = 0..n-1: one bitmap word per warp step (ballot of "has phase arcs")
+__global__ void k_jpc_bits(JpArgs A, int64_t n) {
+    const int64_t nw = (n + 31) >> 5;
+    for (int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nw;
+         w += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        const int64_t v = (w << 5) + lane_id();
+        const bool in = v < n;
+        const bool arcs = in && A.rp[v + 1] > A.rp[v];
+        const unsigned b = __ballot_sync(FULL, arcs);
+        if (lane_id() == 0) A.abits[w] = b;
+        if (in && !arcs) A.color[v] = 1u;
+    }
 }
 
-// per tile of JP_TILE positions of S: the number of class-0 and class-1 vertices
-__global__ void __launch_bounds__(JP_THREADS) k_jpc_tiles(JpArgs A) {
-    const uint32_t cnt = s_count(A);
+// S given as a list (COLOR-Rand recolouring): bits of the listed vertices
+__global__ void k_jpc_mark(JpArgs A) {
+    const uint32_t cnt = *A.in_cnt;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
+        const uint32_t v = (uint32_t)A.in_list[i];
+        if (A.rp[v + 1] > A.rp[v]) atomicOr(A.abits + (v >> 5), 1u << (v & 31));
+        else A.color[v] = 1u;
+    }
+}
+
+// per tile of JP_TILE bitmap words: set bits
+__global__ void __launch_bounds__(JP_THREADS) k_jpc_tiles(JpArgs A, int64_t nwords) {
     const int64_t base = (int64_t)blockIdx.x * JP_TILE;
-    if (base >= cnt) return;
-    int c0 = 0, c1 = 0;
+    uint32_t c = 0;
     for (int u = 0; u < JP_TPT; u++) {
-        int32_t v;
-        const int c = jp_class(A, base + u * JP_THREADS + threadIdx.x, cnt, v);
-        c0 += c == 0;
-        c1 += c == 1;
+        const int64_t w = base + u * JP_THREADS + threadIdx.x;
+        if (w < nwords) c += __popc(A.abits[w]);
     }
-    __shared__ int s0, s1;
-    if (threadIdx.x == 0) s0 = s1 = 0;
+    c = __reduce_add_sync(FULL, c);
+    __shared__ uint32_t s0;
+    if (threadIdx.x == 0) s0 = 0;
     __syncthreads();
-    c0 = __reduce_add_sync(FULL, c0);
-    c1 = __reduce_add_sync(FULL, c1);
-    if (lane_id() == 0) {
-        if (c0) atomicAdd(&s0, c0);
-        if (c1) atomicAdd(&s1, c1);
-    }
+    if (lane_id() == 0 && c) atomicAdd(&s0, c);
     __syncthreads();
-    if (threadIdx.x == 0) {
-        A.tcnt[2 * blockIdx.x] = (uint32_t)s0;
-        A.tcnt[2 * blockIdx.x + 1] = (uint32_t)s1;
-    }
+    if (threadIdx.x == 0) A.tcnt[blockIdx.x] = s0;
 }
 
-// one CTA: exclusive prefix of the tile counts per class (class 1 after all class 0)
+// one CTA: exclusive prefix of the tile counts; n' = the total
 __global__ void __launch_bounds__(1024) k_jpc_tiles_scan(JpArgs A, int64_t ntiles) {
-    const uint32_t cnt = s_count(A);
-    const int64_t need = ((int64_t)cnt + JP_TILE - 1) / JP_TILE;
-    const int64_t used = need < ntiles ? need : ntiles;
-    const int64_t per = (used + blockDim.x - 1) / blockDim.x;
-    const int64_t t0 = (int64_t)threadIdx.x * per, t1 = used < t0 + per ? used : t0 + per;
-    uint32_t s0 = 0, s1 = 0;
-    for (int64_t t = t0; t < t1; t++) {
-        s0 += A.tcnt[2 * t];
-        s1 += A.tcnt[2 * t + 1];
-    }
-    __shared__ uint32_t w0[32], w1[32];
-    uint32_t i0 = s0, i1 = s1;
+    const int64_t per = (ntiles + blockDim.x - 1) / blockDim.x;
+    const int64_t t0 = (int64_t)threadIdx.x * per, t1 = ntiles < t0 + per ? ntiles : t0 + per;
+    uint32_t s0 = 0;
+    for (int64_t t = t0; t < t1; t++) s0 += A.tcnt[t];
+    __shared__ uint32_t w0[32];
+    uint32_t i0 = s0;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-        const uint32_t y0 = __shfl_up_sync(FULL, i0, d), y1 = __shfl_up_sync(FULL, i1, d);
-        if (lane_id() >= d) {
-            i0 += y0;
-            i1 += y1;
-        }
+        const uint32_t y0 = __shfl_up_sync(FULL, i0, d);
+        if (lane_id() >= d) i0 += y0;
     }
     const int wid = threadIdx.x >> 5;
-    if (lane_id() == 31) {
-        w0[wid] = i0;
-        w1[wid] = i1;
-    }
+    if (lane_id() == 31) w0[wid] = i0;
     __syncthreads();
-    uint32_t b0 = 0, b1 = 0, T0 = 0, T1 = 0;
+    uint32_t b0 = 0, T0 = 0;
     for (int q = 0; q < (int)(blockDim.x >> 5); q++) {
-        if (q < wid) {
-            b0 += w0[q];
-            b1 += w1[q];
-        }
+        if (q < wid) b0 += w0[q];
         T0 += w0[q];
-        T1 += w1[q];
     }
-    uint32_t o0 = b0 + i0 - s0, o1 = T0 + b1 + i1 - s1;
+    uint32_t o0 = b0 + i0 - s0;
     for (int64_t t = t0; t < t1; t++) {
-        const uint32_t a0 = A.tcnt[2 * t], a1 = A.tcnt[2 * t + 1];
-        A.tcnt[2 * t] = o0;
-        A.tcnt[2 * t + 1] = o1;
+        const uint32_t a0 = A.tcnt[t];
+        A.tcnt[t] = o0;
         o0 += a0;
-        o1 += a1;
     }
-    if (threadIdx.x == 0) {
-        A.nc[0] = T0 + T1;
-        A.nc[1] = T0;
-    }
+    if (threadIdx.x == 0) A.nc[0] = T0;
 }
 
-// compact ids in (class, position) order; vertices without phase arcs: colour 1
-__global__ void __launch_bounds__(JP_THREADS) k_jpc_assign(JpArgs A) {
-    const uint32_t cnt = s_count(A);
+// word prefixes and the compact id -> original map
+__global__ void __launch_bounds__(JP_THREADS) k_jpc_assign(JpArgs A, int64_t nwords) {
     const int64_t base = (int64_t)blockIdx.x * JP_TILE;
-    if (base >= cnt) return;
-    __shared__ uint32_t sm0[8], sm1[8];
-    uint32_t o0 = A.tcnt[2 * blockIdx.x], o1 = A.tcnt[2 * blockIdx.x + 1];
+    __shared__ uint32_t sm0[8];
+    uint32_t o0 = A.tcnt[blockIdx.x];
     for (int u = 0; u < JP_TPT; u++) {
-        int32_t v;
-        const int c = jp_class(A, base + u * JP_THREADS + threadIdx.x, cnt, v);
-        uint32_t t0, t1;
-        const uint32_t r0 = block_excl_scan<uint32_t>(c == 0, sm0, &t0);
-        const uint32_t r1 = block_excl_scan<uint32_t>(c == 1, sm1, &t1);
-        if (c < 2) {
-            const uint32_t h = c == 0 ? o0 + r0 : o1 + r1;
-            A.ov[h] = v;
-        } else if (v >= 0) {
-            A.color[v] = 1u;
+        const int64_t w = base + u * JP_THREADS + threadIdx.x;
+        const uint32_t bits = w < nwords ? A.abits[w] : 0u;
+        uint32_t t0;
+        const uint32_t p0 = block_excl_scan<uint32_t>(__popc(bits), sm0, &t0);
+        if (w < nwords) {
+            A.apre[w] = o0 + p0;
+            uint32_t b = bits, h = o0 + p0;
+            while (b) {
+                const int k = __ffs(b) - 1;
+                b &= b - 1;
+                A.ov[h++] = (int32_t)((w << 5) + k);
+            }
         }
         o0 += t0;
-        o1 += t1;
     }
 }
 
@@ -462,7 +449,7 @@ __global__ void __launch_bounds__(1024) k_jpc_sums_scan(JpArgs A, int64_t ntiles
         o0 += a0;
         o1 += a1;
     }
-    if (threadIdx.x == 0 && (T1 >= (1ull << 32) || cnt > JP_HMASK)) atomicOr(A.err, 2u);
+    if (threadIdx.x == 0 && T1 > JP_HMASK) atomicOr(A.err, 2u);
 }
 
 // per compact id: list offset, meta, hot state, zeroed extra bitmap words, the list
@@ -493,12 +480,8 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
             const uint32_t x0 = (uint32_t)(o1 + p1);
             A.meta[2 * h] = make_uint4(R, hd, ld, hd > JP_WLIST ? JP_NOTBUILT : hd);
             A.meta[2 * h + 1] = make_uint4(0u, 0u, (uint32_t)off, (uint32_t)(off >> 32));
-            A.col[h] = 0u;
-            A.cnt[h] = hd;
-            A.bm0[h] = 0u;
-            A.xo[h] = x0;
+            A.hot[h] = make_uint4(0u, hd, 0u, (x0 & JP_HMASK) | (min(R, JP_R5) << JP_HBITS));
             for (uint32_t q = 1; q < R; q++) A.xb[x0 + q - 1] = 0u;
-            A.cidR[A.ov[h]] = (uint32_t)h | (min(R, JP_R5) << JP_HBITS);
             if (first) A.ul[0][slot] = (uint32_t)h;
             A.hdeg[h] = 0;  // fill cursors of the huge rows
             A.ldeg[h] = 0;
@@ -513,7 +496,7 @@ __device__ __forceinline__ void jp_fixed(const JpArgs &A, int64_t h, uint32_t R,
     const uint32_t c = A.color[w];
     if (c == 0) return;
     const uint32_t q = (c - 1) >> 5, bit = 1u << ((c - 1) & 31);
-    if (q == 0) atomicOr(A.bm0 + h, bit);
+    if (q == 0) atomicOr(&A.hot[h].z, bit);
     else if (q < R) atomicOr(A.xb + x0 + q - 1, bit);
 }
 
@@ -539,7 +522,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
             kv = vkey(A.k, (uint32_t)v);
             const uint4 m0 = A.meta[2 * h], m1 = A.meta[2 * h + 1];
             R = m0.x;
-            x0 = A.xo[h];
+            x0 = A.hot[h].w & JP_HMASK;
             hl = meta_off(m1) + watch_words(m0.y);
             ll = hl + m0.y;
         }
@@ -547,8 +530,8 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
             for (int64_t x = b; x < e; x++) {
                 const uint32_t w = (uint32_t)__ldcs(A.ci + x);
                 if (!in_set(A.inS, w)) jp_fixed(A, h, R, x0, w);
-                else if (vkey(A.k, w) > kv) __stcs(A.lst + hl++, A.cidR[w]);
-                else __stcs(A.lst + ll++, A.cidR[w]);
+                else if (vkey(A.k, w) > kv) __stcs(A.lst + hl++, jp_rank(A, w));
+                else __stcs(A.lst + ll++, jp_rank(A, w));
             }
         }
         unsigned medm = __ballot_sync(FULL, active && e - b > JP_SMALL && e - b <= JP_BUDGET);
@@ -572,8 +555,8 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
                 }
                 const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
                 const unsigned lt = (1u << lane) - 1u;
-                if (up) __stcs(A.lst + whl + __popc(mu & lt), A.cidR[w]);
-                if (dn) __stcs(A.lst + wll + __popc(md & lt), A.cidR[w]);
+                if (up) __stcs(A.lst + whl + __popc(mu & lt), jp_rank(A, w));
+                if (dn) __stcs(A.lst + wll + __popc(md & lt), jp_rank(A, w));
                 whl += __popc(mu);
                 wll += __popc(md);
             }
@@ -599,7 +582,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
         const int64_t se = min(e, sb0 + SLICE);
         const uint64_t kv = vkey(A.k, (uint32_t)v);
         const uint4 m0 = A.meta[2 * h], m1 = A.meta[2 * h + 1];
-        const uint32_t x0 = A.xo[h];
+        const uint32_t x0 = A.hot[h].w & JP_HMASK;
         const uint64_t hl = meta_off(m1) + watch_words(m0.y), ll = hl + m0.y;
         uint32_t nu = 0, nd = 0;
         for (int64_t x = sb0 + lane; x - lane < se; x += 32) {
@@ -631,8 +614,8 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
                 else dn = true;
             }
             const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
-            if (up) __stcs(A.lst + hl + pu + __popc(mu & lt), A.cidR[w]);
-            if (dn) __stcs(A.lst + ll + pd + __popc(md & lt), A.cidR[w]);
+            if (up) __stcs(A.lst + hl + pu + __popc(mu & lt), jp_rank(A, w));
+            if (dn) __stcs(A.lst + ll + pd + __popc(md & lt), jp_rank(A, w));
             pu += __popc(mu);
             pd += __popc(md);
         }
@@ -643,7 +626,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
 __global__ void k_jpc_scatter(JpArgs A) {
     const uint32_t cnt = A.nc[0];
     for (int64_t h = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; h < cnt; h += (int64_t)gridDim.x * blockDim.x)
-        A.color[A.ov[h]] = A.col[h];
+        A.color[A.ov[h]] = A.hot[h].x;
 }
 
 // ---------------------------------------------------------------- rounds
@@ -684,21 +667,24 @@ __device__ __forceinline__ void grid_sync(const JrCtl &C, uint32_t &k) {
 // Can higher neighbour e (list id) not take colour m (word q, bit)?  Coloured: its
 // colour differs; uncoloured: m is forbidden for it, or m > cap (q >= R).  c = its
 // colour, w = its bitmap word q when q < R (loaded by the caller).
-__device__ __forceinline__ bool nb_ok(const JpArgs &A, uint32_t e, uint32_t c, uint32_t w, uint32_t m, uint32_t q,
-                                      uint32_t bit) {
+__device__ __forceinline__ bool nb_ok(const JpArgs &A, uint32_t e, uint32_t c, uint32_t w, uint32_t R5, uint32_t m,
+                                      uint32_t q, uint32_t bit) {
     if (c != 0u) return c != m;
-    const uint32_t R5 = e >> JP_HBITS;
     if (q == 0u || q < R5) return (w >> bit) & 1u;
     if (R5 < JP_R5) return true;  // m > 32 R >= cap: the neighbour's colour is below m
-    const uint32_t hu = e & JP_HMASK;  // saturated R field: the full count
-    const uint32_t R = __ldg(&A.meta[2 * hu].x);
-    return q >= R || ((__ldcg(A.xb + __ldcg(A.xo + hu) + q - 1) >> bit) & 1u);
+    const uint32_t R = __ldg(&A.meta[2 * e].x);  // saturated R field: the full count
+    return q >= R || ((__ldcg(A.xb + (__ldcg(&A.hot[e].w) & JP_HMASK) + q - 1) >> bit) & 1u);
 }
 
-// the neighbour's bitmap word q (q == 0: bm0; q < R: in xb; else unused)
-__device__ __forceinline__ uint32_t nb_word_addr_free(const JpArgs &A, uint32_t e, uint32_t q) {
-    const uint32_t hu = e & JP_HMASK;
-    return q == 0u ? __ldcg(A.bm0 + hu) : (q < (e >> JP_HBITS) ? __ldcg(A.xo + hu) : 0u);
+// a neighbour's colour c, R field and bitmap word q (q == 0: bm0; q < R: offset of
+// its words in xb, resolved by the caller; else unused) from ONE 16-B load of its
+// hot record
+__device__ __forceinline__ void nb_load(const JpArgs &A, uint32_t e, uint32_t q, uint32_t &c, uint32_t &w,
+                                        uint32_t &R5) {
+    const uint4 s = __ldcg(A.hot + e);
+    c = s.x;
+    R5 = s.w >> JP_HBITS;
+    w = q == 0u ? s.z : (q < R5 ? (s.w & JP_HMASK) : 0u);
 }
 
 // Phase A of round r: every active vertex (count <= JP_WATCH) checks its watch list
@@ -737,11 +723,12 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
                 state = 5;
             } else {
                 state = 0;
-                const uint32_t z0 = ~__ldcg(A.bm0 + h);
+                const uint4 hs = __ldcg(A.hot + h);
+                const uint32_t z0 = ~hs.z;
                 if (z0) {
                     m = __ffs(z0);
                 } else {  // colours > 32
-                    const uint32_t *xw = A.xb + __ldcg(A.xo + h);
+                    const uint32_t *xw = A.xb + (hs.w & JP_HMASK);
                     for (uint32_t k = 1; k < R; k++) {
                         const uint32_t z = ~__ldcg(xw + k - 1);
                         if (z) {
@@ -757,25 +744,27 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
         uint32_t j = (lm == m && pos < wc) ? pos : 0u;  // m unchanged: resume at the last blocker
         // ---- lane: the first JP_LANE_CHECKS entries (all loads of a stage in flight)
         if (state == 0) {
-            uint32_t e[JP_LANE_CHECKS], c[JP_LANE_CHECKS], w[JP_LANE_CHECKS];
+            uint32_t e[JP_LANE_CHECKS], c[JP_LANE_CHECKS], w[JP_LANE_CHECKS], r5[JP_LANE_CHECKS];
 #pragma unroll
             for (int u = 0; u < JP_LANE_CHECKS; u++) e[u] = j + u < wc ? __ldcg(A.lst + off + j + u) : 0u;
 #pragma unroll
             for (int u = 0; u < JP_LANE_CHECKS; u++) {
-                c[u] = j + u < wc ? __ldcg(A.col + (e[u] & JP_HMASK)) : 1u;
-                w[u] = j + u < wc ? nb_word_addr_free(A, e[u], q) : 0u;
+                c[u] = 1u;
+                w[u] = 0u;
+                r5[u] = 0u;
+                if (j + u < wc) nb_load(A, e[u], q, c[u], w[u], r5[u]);
             }
             if (q > 0) {
 #pragma unroll
                 for (int u = 0; u < JP_LANE_CHECKS; u++)
-                    if (j + u < wc && c[u] == 0u && q < (e[u] >> JP_HBITS)) w[u] = __ldcg(A.xb + w[u] + q - 1);
+                    if (j + u < wc && c[u] == 0u && q < r5[u]) w[u] = __ldcg(A.xb + w[u] + q - 1);
             }
 #pragma unroll
             for (int u = 0; u < JP_LANE_CHECKS; u++) {
                 if (state == 0) {
                     if (j >= wc) {
                         state = 1;
-                    } else if (!nb_ok(A, e[u], c[u], w[u], m, q, bit)) {
+                    } else if (!nb_ok(A, e[u], c[u], w[u], r5[u], m, q, bit)) {
                         state = 2;
                         pos = j;
                         lm = m;
@@ -803,10 +792,10 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
                 bool ok = true;
                 if (jj < wwc) {
                     const uint32_t eu = __ldcg(A.lst + woff + jj);
-                    const uint32_t cu = __ldcg(A.col + (eu & JP_HMASK));
-                    uint32_t wu = nb_word_addr_free(A, eu, wq);
-                    if (wq > 0 && cu == 0u && wq < (eu >> JP_HBITS)) wu = __ldcg(A.xb + wu + wq - 1);
-                    ok = nb_ok(A, eu, cu, wu, wm, wq, wbit);
+                    uint32_t cu, wu, ru;
+                    nb_load(A, eu, wq, cu, wu, ru);
+                    if (wq > 0 && cu == 0u && wq < ru) wu = __ldcg(A.xb + wu + wq - 1);
+                    ok = nb_ok(A, eu, cu, wu, ru, wm, wq, wbit);
                 }
                 const unsigned fails = __ballot_sync(FULL, !ok);
                 if (fails) {
@@ -828,7 +817,7 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t 
         }
         // ---- outcome
         const bool pass = state == 1, stay = state == 2 || state == 5;
-        if (pass) A.col[h] = m;
+        if (pass) A.hot[h].x = m;
         if (state == 2) *reinterpret_cast<uint2 *>(A.meta + 2 * h + 1) = make_uint2(pos, lm);
         if (state == 5) reinterpret_cast<uint32_t *>(A.meta + 2 * h)[3] = 0u;  // filled by phase B
         const int64_t slot = warp_append(stay, A.ucnt + (r + 1) % 3);
@@ -861,20 +850,27 @@ __device__ __forceinline__ void jp_push(const JpArgs &A, uint32_t r, const uint3
                                         uint32_t q, uint32_t bit) {
     uint32_t old[K], x[K];
 #pragma unroll
-    for (int u = 0; u < K; u++) act[u] = act[u] && __ldcg(A.col + (e[u] & JP_HMASK)) == 0u;
+    for (int u = 0; u < K; u++) {  // colour, R field and extra-word offset in one 16-B load
+        x[u] = 0xffffffffu;
+        if (act[u]) {
+            const uint4 s = __ldcg(A.hot + e[u]);
+            act[u] = s.x == 0u;
+            x[u] = s.w;
+        }
+    }
 #pragma unroll
-    for (int u = 0; u < K; u++) old[u] = act[u] ? atomicSub(A.cnt + (e[u] & JP_HMASK), 1u) : 0u;
+    for (int u = 0; u < K; u++) old[u] = act[u] ? atomicSub(&A.hot[e[u]].y, 1u) : 0u;
     if (q == 0) {
 #pragma unroll
         for (int u = 0; u < K; u++)
-            if (act[u]) atomicOr(A.bm0 + (e[u] & JP_HMASK), 1u << bit);
+            if (act[u]) atomicOr(&A.hot[e[u]].z, 1u << bit);
     } else {
 #pragma unroll
         for (int u = 0; u < K; u++) {
-            const uint32_t hw = e[u] & JP_HMASK, R5 = e[u] >> JP_HBITS;
+            const uint32_t R5 = x[u] >> JP_HBITS;
             bool go = act[u] && q < R5;
-            if (act[u] && !go && R5 == JP_R5) go = q < __ldg(&A.meta[2 * hw].x);
-            x[u] = go ? __ldcg(A.xo + hw) : 0xffffffffu;
+            if (act[u] && !go && R5 == JP_R5) go = q < __ldg(&A.meta[2 * e[u]].x);
+            x[u] = go ? (x[u] & JP_HMASK) : 0xffffffffu;
         }
 #pragma unroll
         for (int u = 0; u < K; u++)
@@ -884,7 +880,7 @@ __device__ __forceinline__ void jp_push(const JpArgs &A, uint32_t r, const uint3
     for (int u = 0; u < K; u++) {
         if (act[u] && old[u] == JP_WATCH + 1u) {
             const uint32_t slot = atomicAdd(A.ucnt + (r + 1) % 3, 1u);
-            A.ul[(r + 1) & 1][slot] = e[u] & JP_HMASK;
+            A.ul[(r + 1) & 1][slot] = e[u];
         }
     }
 }
@@ -944,7 +940,7 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, int64_t 
 #pragma unroll
         for (int u = 0; u < K; u++) e[u] = j0 + u * 32 + lane < j1 ? __ldcs(A.lst + hl + j0 + u * 32 + lane) : 0u;
 #pragma unroll
-        for (int u = 0; u < K; u++) c[u] = j0 + u * 32 + lane < j1 ? __ldcg(A.col + (e[u] & JP_HMASK)) : 1u;
+        for (int u = 0; u < K; u++) c[u] = j0 + u * 32 + lane < j1 ? __ldcg(&A.hot[e[u]].x) : 1u;
 #pragma unroll
         for (int u = 0; u < K; u++) {
             const bool keep = c[u] == 0u;
@@ -1060,11 +1056,9 @@ void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
     w.ov = a.take<int32_t>((size_t)n + 1);
     w.hdeg = a.take<uint32_t>((size_t)n + 1);
     w.ldeg = a.take<uint32_t>((size_t)n + 1);
-    w.cidR = a.take<uint32_t>((size_t)n + 1);
-    w.col = a.take<uint32_t>((size_t)n + 1);
-    w.cnt = a.take<uint32_t>((size_t)n + 1);
-    w.bm0 = a.take<uint32_t>((size_t)n + 1);
-    w.xo = a.take<uint32_t>((size_t)n + 1);
+    w.abits = a.take<uint32_t>((size_t)(n + 31) / 32 + 1);
+    w.apre = a.take<uint32_t>((size_t)(n + 31) / 32 + 1);
+    w.hot = a.take<uint4>((size_t)n + 1);
     w.meta = a.take<uint4>(2 * (size_t)n + 2);
     w.ul[0] = a.take<uint32_t>((size_t)n + 1);
     w.ul[1] = a.take<uint32_t>((size_t)n + 1);
@@ -1107,11 +1101,9 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     A.ov = w.ov;
     A.hdeg = w.hdeg;
     A.ldeg = w.ldeg;
-    A.cidR = w.cidR;
-    A.col = w.col;
-    A.cnt = w.cnt;
-    A.bm0 = w.bm0;
-    A.xo = w.xo;
+    A.abits = w.abits;
+    A.apre = w.apre;
+    A.hot = w.hot;
     A.meta = w.meta;
     A.lst = w.lst;
     A.xb = w.xb;
@@ -1132,20 +1124,23 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     A.trace = nullptr;
     A.prof = nullptr;
     A.k = stream_key(f.p.seed, TAG_VERTEX, 0);
-    const int64_t smax = list0 ? n : implicit_n;  // positions of S (upper bound for a list)
-    const unsigned tiles_s = (unsigned)((smax + JP_TILE - 1) / JP_TILE);
+    const int64_t nwords = (n + 31) / 32;
+    const unsigned tiles_w = (unsigned)((nwords + JP_TILE - 1) / JP_TILE);
     const unsigned tiles_c = (unsigned)((n + JP_TILE - 1) / JP_TILE);  // compact ids <= n
     prof_begin("jp_build", s);
-    if (tiles_s) {
-        k_jpc_tiles<<<tiles_s, JP_THREADS, 0, s>>>(A);
-        SYM_LAUNCH_CHECK();
+    if (list0) {
+        SYM_CUDA(cudaMemsetAsync(w.abits, 0, sizeof(uint32_t) * (size_t)nwords, s));
+        k_jpc_mark<<<num_sms() * 8, 256, 0, s>>>(A);
+    } else {
+        k_jpc_bits<<<num_sms() * 8, 256, 0, s>>>(A, implicit_n);
     }
-    k_jpc_tiles_scan<<<1, 1024, 0, s>>>(A, tiles_s);
     SYM_LAUNCH_CHECK();
-    if (tiles_s) {
-        k_jpc_assign<<<tiles_s, JP_THREADS, 0, s>>>(A);
-        SYM_LAUNCH_CHECK();
-    }
+    k_jpc_tiles<<<tiles_w, JP_THREADS, 0, s>>>(A, nwords);
+    SYM_LAUNCH_CHECK();
+    k_jpc_tiles_scan<<<1, 1024, 0, s>>>(A, tiles_w);
+    SYM_LAUNCH_CHECK();
+    k_jpc_assign<<<tiles_w, JP_THREADS, 0, s>>>(A, nwords);
+    SYM_LAUNCH_CHECK();
     k_jpc_count<<<num_sms() * (2048 / JP_THREADS), JP_THREADS, 0, s>>>(A);
     SYM_LAUNCH_CHECK();
     k_jpc_count_huge<<<num_sms() * 4, JP_HUGE_THREADS, 0, s>>>(A);

@@ -5,11 +5,15 @@ use it; MM-Rand has its own RAND decomposition), so they run on two CUDA
 streams from two host threads (ctypes releases the GIL; the library keeps no
 per-call global state and every stream gets its own workspace):
 
-    stream A (high priority): DEG2 decomposition -> COLOR-Deg2.  Its JP kernel is
-                              persistent and depth-bound (1 CTA/SM, mostly waiting
-                              on its grid barrier), so it leaves SM slots idle.
+    stream A (high priority): DEG2 decomposition -> COLOR-Deg2.
     stream B:                 RAND4 decomposition -> MM-Rand4 -> MIS-Deg2 (after
-                              stream A's decomposition) -- fills those slots.
+                              stream A's decomposition).
+
+This paid off while COLOR's persistent kernel held one 512-thread CTA per SM (levels
+JP, 60.4 vs 65.9 ms per step); the early-commit rounds kernel holds two CTAs of 64
+registers per thread -- every SM's register file -- so stream B can only interleave
+and the step is slower than the five calls in order (51.2 vs 48.8 ms).  bench.py
+therefore runs the calls in order by default (--concurrent selects this schedule).
 
 Every call is the public API (sym_decompose / sym_mis / sym_mm / sym_color); results
 are bit-identical to running the five calls in order (tests/test_gpu_concurrent.py).

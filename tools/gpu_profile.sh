@@ -12,7 +12,7 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
     python bench.py --profile-only --steps 1 --warmup 0 > /dev/null 2>&1
 NCU="ncu --set full --import-source on --clock-control none"
 PB="python bench.py --profile-only --steps 1 --warmup 0"
-timeout 600 $NCU -k regex:'^k_jp_(init|levels)$' -c 2 -o $O/jp $PB > /dev/null 2>&1
+timeout 600 $NCU -k regex:'^k_jp(_rounds|c_fill)$' -c 2 -o $O/jp $PB > /dev/null 2>&1
 timeout 600 $NCU -k regex:'^k_split' -c 2 -o $O/split $PB > /dev/null 2>&1
 timeout 600 $NCU -k regex:'^k_(round0|mm_round)' -c 3 -o $O/mm $PB > /dev/null 2>&1
 timeout 600 $NCU -k regex:'^k_mis_round' -c 4 -o $O/mis $PB > /dev/null 2>&1

@@ -9,9 +9,6 @@ sys.path.insert(0, ROOT)
 OUT = os.path.join(ROOT, "build", "variants")
 VARIANTS = {
     "base": [],
-    "nopf": ["-DSYM_JP_NOPF"],
-    "small8": ["-DSYM_JP_SMALL=8"],
-    "small16": ["-DSYM_JP_SMALL=16"],
     "minb1": ["-DSYM_JR_MINB=1"],
 }
 
