@@ -292,13 +292,18 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_count(JpArgs A) {
             kv = vkey(A.k, (uint32_t)v);
         }
         uint32_t hi = 0, lo = 0;
-        if (active && e - b <= JP_SMALL) {
-            for (int64_t x = b; x < e; x++) {
-                const uint32_t w = (uint32_t)__ldg(A.ci + x);
-                if (in_set(A.inS, w)) {
-                    const bool up = vkey(A.k, w) > kv;
-                    hi += up;
-                    lo += !up;
+        if (active && e - b <= JP_SMALL) {  // batches of 4 arcs: their loads in flight together
+            for (int64_t xq = b; xq < e; xq += 4) {
+                uint32_t w[4];
+#pragma unroll
+                for (int u = 0; u < 4; u++) w[u] = xq + u < e ? (uint32_t)__ldcs(A.ci + xq + u) : 0u;
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    if (xq + u < e && in_set(A.inS, w[u])) {
+                        const bool up = vkey(A.k, w[u]) > kv;
+                        hi += up;
+                        lo += !up;
+                    }
                 }
             }
         }
@@ -526,12 +531,27 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
             hl = meta_off(m1) + watch_words(m0.y);
             ll = hl + m0.y;
         }
-        if (active && e - b <= JP_SMALL) {
-            for (int64_t x = b; x < e; x++) {
-                const uint32_t w = (uint32_t)__ldcs(A.ci + x);
-                if (!in_set(A.inS, w)) jp_fixed(A, h, R, x0, w);
-                else if (vkey(A.k, w) > kv) __stcs(A.lst + hl++, jp_rank(A, w));
-                else __stcs(A.lst + ll++, jp_rank(A, w));
+        if (active && e - b <= JP_SMALL) {  // batches of 4 arcs: their loads in flight together
+            for (int64_t xq = b; xq < e; xq += 4) {
+                uint32_t w[4], rk[4];
+                bool ok[4], sv[4];
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    ok[u] = xq + u < e;
+                    w[u] = ok[u] ? (uint32_t)__ldcs(A.ci + xq + u) : 0u;
+                }
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    sv[u] = ok[u] && in_set(A.inS, w[u]);
+                    rk[u] = sv[u] ? jp_rank(A, w[u]) : 0u;
+                }
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    if (!ok[u]) continue;
+                    if (!sv[u]) jp_fixed(A, h, R, x0, w[u]);
+                    else if (vkey(A.k, w[u]) > kv) __stcs(A.lst + hl++, rk[u]);
+                    else __stcs(A.lst + ll++, rk[u]);
+                }
             }
         }
         unsigned medm = __ballot_sync(FULL, active && e - b > JP_SMALL && e - b <= JP_BUDGET);
@@ -543,22 +563,32 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
             const int64_t wh = base + src;
             const uint32_t wR = __shfl_sync(FULL, R, src), wx0 = __shfl_sync(FULL, x0, src);
             uint64_t whl = __shfl_sync(FULL, hl, src), wll = __shfl_sync(FULL, ll, src);
-            for (int64_t xb0 = wb; xb0 < we; xb0 += 32) {
-                const int64_t x = xb0 + lane;
-                bool up = false, dn = false;
-                uint32_t w = 0;
-                if (x < we) {
-                    w = (uint32_t)__ldcs(A.ci + x);
-                    if (!in_set(A.inS, w)) jp_fixed(A, wh, wR, wx0, w);
-                    else if (vkey(A.k, w) > wk) up = true;
-                    else dn = true;
+            const unsigned lt = (1u << lane) - 1u;
+            for (int64_t xb0 = wb; xb0 < we; xb0 += 128) {  // 4 steps of 32 arcs in flight
+                uint32_t w[4], rk[4];
+                bool up[4], dn[4];
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    const int64_t x = xb0 + u * 32 + lane;
+                    w[u] = x < we ? (uint32_t)__ldcs(A.ci + x) : 0u;
                 }
-                const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
-                const unsigned lt = (1u << lane) - 1u;
-                if (up) __stcs(A.lst + whl + __popc(mu & lt), jp_rank(A, w));
-                if (dn) __stcs(A.lst + wll + __popc(md & lt), jp_rank(A, w));
-                whl += __popc(mu);
-                wll += __popc(md);
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    const bool ok = xb0 + u * 32 + lane < we;
+                    const bool sv = ok && in_set(A.inS, w[u]);
+                    up[u] = sv && vkey(A.k, w[u]) > wk;
+                    dn[u] = sv && !up[u];
+                    rk[u] = sv ? jp_rank(A, w[u]) : 0u;
+                    if (ok && !sv) jp_fixed(A, wh, wR, wx0, w[u]);
+                }
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    const unsigned mu = __ballot_sync(FULL, up[u]), md = __ballot_sync(FULL, dn[u]);
+                    if (up[u]) __stcs(A.lst + whl + __popc(mu & lt), rk[u]);
+                    if (dn[u]) __stcs(A.lst + wll + __popc(md & lt), rk[u]);
+                    whl += __popc(mu);
+                    wll += __popc(md);
+                }
             }
         }
     }
