@@ -57,7 +57,10 @@ constexpr int JP_BUDGET = 4096;  // build: rows > JP_BUDGET arcs are split into 
 constexpr int JP_PIECE = 8192;   // arcs per CTA piece of a huge row in the build passes
 constexpr int JP_TILE = 2048;    // build: compact ids per scan tile (JP_THREADS x 8)
 constexpr int JP_TPT = JP_TILE / JP_THREADS;
-constexpr int JP_LANE_CHECKS = 4;  // phase A: entries a lane checks before the warp takes over
+#ifndef SYM_JP_LANE_CHECKS
+#define SYM_JP_LANE_CHECKS 4
+#endif
+constexpr int JP_LANE_CHECKS = SYM_JP_LANE_CHECKS;  // phase A: entries a lane checks before the warp takes over
 #ifndef SYM_JP_PUSH
 #define SYM_JP_PUSH 256
 #endif
@@ -985,7 +988,10 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, int64_t 
     }
 }
 
-constexpr int JR_THREADS = 512;
+#ifndef SYM_JR_THREADS
+#define SYM_JR_THREADS 512
+#endif
+constexpr int JR_THREADS = SYM_JR_THREADS;
 #ifndef SYM_JR_MINB
 #define SYM_JR_MINB 2
 #endif

@@ -9,7 +9,10 @@ sys.path.insert(0, ROOT)
 OUT = os.path.join(ROOT, "build", "variants")
 VARIANTS = {
     "base": [],
-    "minb1": ["-DSYM_JR_MINB=1"],
+    "t1024": ["-DSYM_JR_THREADS=1024", "-DSYM_JR_MINB=1"],
+    "t256": ["-DSYM_JR_THREADS=256", "-DSYM_JR_MINB=4"],
+    "lc8": ["-DSYM_JP_LANE_CHECKS=8"],
+    "push128": ["-DSYM_JP_PUSH=128"],
 }
 
 if sys.argv[1] == "build":
