@@ -169,7 +169,11 @@ int sym_mm(const sym_graph *g, const sym_params *p, const sym_decomp *decomp, vo
            int32_t *mate, sym_stats *stats, sym_stream_t stream);
 
 /* Vertex colouring.  color uint32[n] (device): colours >= 1, proper on G.
-   NONE: Jones-Plassmann = first-fit in priority order.
+   NONE: Jones-Plassmann = first-fit in priority order.  Computed by
+         early-commit rounds (a vertex takes its greedy colour as soon as it is
+         determined): same colours, ~10x fewer rounds than JP levels
+         on R-MAT; stats->rounds[phase] = those rounds.  Limits: compact ids and
+         extra bitmap words < 2^27 (else SYM_EINVAL).
    DEGK: COLOR-Degk (Alg 9): C_H on G_H; G_L coloured with max(C_H)+1 ..
          max(C_H)+k+1 (reading: JP replaces the speculative 3-slot loop).
    RAND: COLOR-Rand (Alg 8): JP on the parts with one palette; the
@@ -267,8 +271,8 @@ int sym_shard_mm_round(const sym_graph_shard *g, const sym_params *p, int round,
 /* ---- kernel profiling hook (measurement only; off by default) ----
    sym_profile_enable(1) makes every later call record a CUDA event pair on its
    stream around each hot-kernel launch, grouped by kernel class ("split",
-   "mis_round", "mis_huge", "mm_round0", "mm_round", "mm_huge", "jp_init",
-   "jp_round", "jp_huge", ...).  sym_profile_collect() synchronises those events and
+   "mis_round", "mis_huge", "mm_round0", "mm_round", "mm_huge", "jp_build",
+   "jp_rounds", ...).  sym_profile_collect() synchronises those events and
    returns, per class: launches, summed device milliseconds, and the algorithmic
    bytes those launches had to move when the library knows them exactly from host
    sizes (split = 8 B/arc + 24 B/vertex; first MM round = 4 B/arc + 24

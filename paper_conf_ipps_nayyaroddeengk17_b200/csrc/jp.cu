@@ -481,8 +481,13 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
         const unsigned long long p0 =
             block_excl_scan<unsigned long long>(active ? watch_words(hd) + hd + ld : 0ull, sm0, &t0);
         const unsigned long long p1 = block_excl_scan<unsigned long long>(active ? R - 1u : 0ull, sm1, &t1);
-        const bool first = active && hd <= JP_WATCH;
-        const int64_t slot = warp_append(first, A.ucnt);
+        // Round 0 can only colour vertices without higher neighbours (nothing is coloured
+        // and, without fixed colours -- S given implicitly -- nothing is forbidden), so
+        // the other active vertices start in round 1's list.
+        const bool ready = active && hd == 0, later = active && hd > 0 && hd <= JP_WATCH;
+        const bool r0 = ready || (later && A.in_list != nullptr);
+        const bool first = r0 || later;
+        const int64_t s0 = warp_append(r0, A.ucnt), s1 = warp_append(first && !r0, A.ucnt + 1);
         if (active) {
             const unsigned long long off = o0 + p0;
             const uint32_t x0 = (uint32_t)(o1 + p1);
@@ -490,7 +495,8 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
             A.meta[2 * h + 1] = make_uint4(0u, 0u, (uint32_t)off, (uint32_t)(off >> 32));
             A.hot[h] = make_uint4(0u, hd, 0u, (x0 & JP_HMASK) | (min(R, JP_R5) << JP_HBITS));
             for (uint32_t q = 1; q < R; q++) A.xb[x0 + q - 1] = 0u;
-            if (first) A.ul[0][slot] = (uint32_t)h;
+            if (r0) A.ul[0][s0] = (uint32_t)h;
+            else if (first) A.ul[1][s1] = (uint32_t)h;
             A.hdeg[h] = 0;  // fill cursors of the huge rows
             A.ldeg[h] = 0;
         }
