@@ -7,11 +7,10 @@ import json, os, subprocess, sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 OUT = os.path.join(ROOT, "build", "variants")
-VARIANTS = {
+VARIANTS = {  # the last comparison run (DESIGN §7 records the others)
     "base": [],
-    "t1024": ["-DSYM_JR_THREADS=1024", "-DSYM_JR_MINB=1"],
-    "t256": ["-DSYM_JR_THREADS=256", "-DSYM_JR_MINB=4"],
-    "lc8": ["-DSYM_JP_LANE_CHECKS=8"],
+    "minb1": ["-DSYM_JR_MINB=1"],
+    "w32": ["-DSYM_JP_WATCH=32"],
     "push128": ["-DSYM_JP_PUSH=128"],
 }
 
