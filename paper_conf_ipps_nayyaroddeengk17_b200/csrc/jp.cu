@@ -1104,8 +1104,11 @@ void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
     w.meta = a.take<uint4>(2 * (size_t)n + 2);
     w.ul[0] = a.take<uint32_t>((size_t)n + 1);
     w.ul[1] = a.take<uint32_t>((size_t)n + 1);
-    // lists: watch areas (<= JP_WATCH per vertex) + one id per arc (higher or lower)
-    w.lst_words = (int64_t)JP_WATCH * n + nnz + 2;
+    // lists: one id per arc (higher or lower) + watch areas of JP_WATCH ids for the
+    // rows with > JP_WLIST higher neighbours (fewer than nnz / JP_WLIST rows, so the
+    // areas take < nnz words)
+    static_assert(JP_WATCH <= JP_WLIST, "watch areas must fit the nnz bound");
+    w.lst_words = std::min<int64_t>((int64_t)JP_WATCH * n, nnz) + nnz + 2;
     w.lst = a.take<uint32_t>((size_t)w.lst_words);
     // extra bitmap words: sum of ceil(cap/32) - 1 <= (nnz + n)/32
     w.xb = a.take<uint32_t>((size_t)((nnz + n) / 32 + 2));
