@@ -53,7 +53,7 @@ def parse():
     ap.add_argument("--cpu-scale", type=int, default=20, help="R-MAT scale of the bounded oracle sample")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=4)
+    ap.add_argument("--e2e-steps", type=int, default=8)
     ap.add_argument("--profile-only", action="store_true", help="short run for ncu (no JSON contract)")
     ap.add_argument("--sequential", action="store_true", help="one stream, the five calls in order (default)")
     ap.add_argument("--concurrent", action="store_true",
