@@ -164,8 +164,8 @@ struct ColorWs {
     int32_t *ov = nullptr;         // compact id -> original
     uint32_t *hdeg = nullptr;      // higher / lower degrees (build), fill cursors
     uint32_t *ldeg = nullptr;
-    uint32_t *abits = nullptr;     // S vertices with phase arcs (bitmap) and the
-    uint32_t *apre = nullptr;      //   exclusive popcount prefix per word: compact id = rank
+    uint32_t *arank = nullptr;     // per 32 ids {bitmap of S vertices with phase arcs,
+                                   //   exclusive popcount prefix}: compact id = rank
     uint4 *hot = nullptr;          // hot per-vertex state {colour, count, bitmap word 0,
                                    //   offset of the extra bitmap words}
     uint4 *meta = nullptr;         // per-vertex own data (2 x 16 B)

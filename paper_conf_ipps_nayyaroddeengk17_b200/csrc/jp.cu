@@ -91,8 +91,8 @@ struct JpArgs {
     int32_t *ov;         // [n] compact id -> original
     uint32_t *hdeg;      // [n] higher degree (count pass), fill cursor (huge rows)
     uint32_t *ldeg;      // [n] lower degree (count pass), fill cursor (huge rows)
-    uint32_t *abits;     // [n/32] S vertices with phase arcs (rank = compact id)
-    uint32_t *apre;      // [n/32] exclusive prefix of the bitmap words' popcounts
+    uint32_t *arank;     // [2 n/32] per 32 ids: {bitmap of the S vertices with phase arcs,
+                         //   exclusive prefix of the popcounts} (rank = compact id)
     uint4 *hot;          // [n] hot per-vertex state {col, cnt, bm0, xo} (see the header)
     uint4 *meta;         // [2n] per-vertex own data
     uint32_t *lst;       // watch / higher / lower lists
@@ -172,12 +172,13 @@ __device__ __forceinline__ T block_excl_scan(T x, T *sm, T *total) {
 
 // ---------------------------------------------------------------- build: compact ids
 // The S vertices with phase arcs are numbered by rank in id order:
-//   h(v) = apre[v >> 5] + popc(abits[v >> 5] & lanes below v)
+//   h(v) = prefix[v >> 5] + popc(bits[v >> 5] & lanes below v)  (one 8-B load)
 // so a list id is computed from 4 MB of bitmap + prefix (L2/L1-resident at R-MAT
 // s24) instead of gathered from an n-entry map.  A vertex of S without phase arcs
 // takes colour 1 at once.
 __device__ __forceinline__ uint32_t jp_rank(const JpArgs &A, uint32_t v) {
-    return __ldg(A.apre + (v >> 5)) + __popc(__ldg(A.abits + (v >> 5)) & ((1u << (v & 31)) - 1u));
+    const uint2 x = __ldg(reinterpret_cast<const uint2 *>(A.arank) + (v >> 5));
+    return x.y + __popc(x.x & ((1u << (v & 31)) - 1u));
 }
 
 // implicit S = 0..n-1: one bitmap word per warp step (ballot of "has phase arcs")
@@ -189,7 +190,7 @@ __global__ void k_jpc_bits(JpArgs A, int64_t n) {
         const bool in = v < n;
         const bool arcs = in && A.rp[v + 1] > A.rp[v];
         const unsigned b = __ballot_sync(FULL, arcs);
-        if (lane_id() == 0) A.abits[w] = b;
+        if (lane_id() == 0) A.arank[2 * w] = b;
         if (in && !arcs) A.color[v] = 1u;
     }
 }
@@ -199,7 +200,7 @@ __global__ void k_jpc_mark(JpArgs A) {
     const uint32_t cnt = *A.in_cnt;
     for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
         const uint32_t v = (uint32_t)A.in_list[i];
-        if (A.rp[v + 1] > A.rp[v]) atomicOr(A.abits + (v >> 5), 1u << (v & 31));
+        if (A.rp[v + 1] > A.rp[v]) atomicOr(A.arank + 2 * (v >> 5), 1u << (v & 31));
         else A.color[v] = 1u;
     }
 }
@@ -210,7 +211,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_tiles(JpArgs A, int64_t nwor
     uint32_t c = 0;
     for (int u = 0; u < JP_TPT; u++) {
         const int64_t w = base + u * JP_THREADS + threadIdx.x;
-        if (w < nwords) c += __popc(A.abits[w]);
+        if (w < nwords) c += __popc(A.arank[2 * w]);
     }
     c = __reduce_add_sync(FULL, c);
     __shared__ uint32_t s0;
@@ -258,11 +259,11 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_assign(JpArgs A, int64_t nwo
     uint32_t o0 = A.tcnt[blockIdx.x];
     for (int u = 0; u < JP_TPT; u++) {
         const int64_t w = base + u * JP_THREADS + threadIdx.x;
-        const uint32_t bits = w < nwords ? A.abits[w] : 0u;
+        const uint32_t bits = w < nwords ? A.arank[2 * w] : 0u;
         uint32_t t0;
         const uint32_t p0 = block_excl_scan<uint32_t>(__popc(bits), sm0, &t0);
         if (w < nwords) {
-            A.apre[w] = o0 + p0;
+            A.arank[2 * w + 1] = o0 + p0;
             uint32_t b = bits, h = o0 + p0;
             while (b) {
                 const int k = __ffs(b) - 1;
@@ -317,12 +318,17 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_count(JpArgs A) {
             const int64_t wb = __shfl_sync(FULL, b, src), we = __shfl_sync(FULL, e, src);
             const uint64_t wk = __shfl_sync(FULL, kv, src);
             uint32_t lh = 0, ll = 0;
-            for (int64_t x = wb + lane; x < we; x += 32) {
-                const uint32_t w = (uint32_t)__ldg(A.ci + x);
-                if (in_set(A.inS, w)) {
-                    const bool up = vkey(A.k, w) > wk;
-                    lh += up;
-                    ll += !up;
+            for (int64_t xb0 = wb + lane; xb0 < we; xb0 += 128) {  // 4 steps of 32 arcs in flight
+                uint32_t w[4];
+#pragma unroll
+                for (int u = 0; u < 4; u++) w[u] = xb0 + u * 32 < we ? (uint32_t)__ldcs(A.ci + xb0 + u * 32) : 0u;
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    if (xb0 + u * 32 < we && in_set(A.inS, w[u])) {
+                        const bool up = vkey(A.k, w[u]) > wk;
+                        lh += up;
+                        ll += !up;
+                    }
                 }
             }
             lh = __reduce_add_sync(FULL, lh);
@@ -1098,8 +1104,7 @@ void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
     w.ov = a.take<int32_t>((size_t)n + 1);
     w.hdeg = a.take<uint32_t>((size_t)n + 1);
     w.ldeg = a.take<uint32_t>((size_t)n + 1);
-    w.abits = a.take<uint32_t>((size_t)(n + 31) / 32 + 1);
-    w.apre = a.take<uint32_t>((size_t)(n + 31) / 32 + 1);
+    w.arank = a.take<uint32_t>(2 * ((size_t)(n + 31) / 32 + 1));
     w.hot = a.take<uint4>((size_t)n + 1);
     w.meta = a.take<uint4>(2 * (size_t)n + 2);
     w.ul[0] = a.take<uint32_t>((size_t)n + 1);
@@ -1146,8 +1151,7 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     A.ov = w.ov;
     A.hdeg = w.hdeg;
     A.ldeg = w.ldeg;
-    A.abits = w.abits;
-    A.apre = w.apre;
+    A.arank = w.arank;
     A.hot = w.hot;
     A.meta = w.meta;
     A.lst = w.lst;
@@ -1174,7 +1178,7 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     const unsigned tiles_c = (unsigned)((n + JP_TILE - 1) / JP_TILE);  // compact ids <= n
     prof_begin("jp_build", s);
     if (list0) {
-        SYM_CUDA(cudaMemsetAsync(w.abits, 0, sizeof(uint32_t) * (size_t)nwords, s));
+        SYM_CUDA(cudaMemsetAsync(w.arank, 0, 2 * sizeof(uint32_t) * (size_t)nwords, s));
         k_jpc_mark<<<num_sms() * 8, 256, 0, s>>>(A);
     } else {
         k_jpc_bits<<<num_sms() * 8, 256, 0, s>>>(A, implicit_n);
