@@ -649,20 +649,28 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
         }
         pu = __shfl_sync(FULL, pu, 0);
         pd = __shfl_sync(FULL, pd, 0);
-        for (int64_t x = sb0 + lane; x - lane < se; x += 32) {
-            bool up = false, dn = false;
-            uint32_t w = 0;
-            if (x < se) {
-                w = (uint32_t)__ldg(A.ci + x);
-                if (!in_set(A.inS, w)) jp_fixed(A, h, m0.x, x0, w);
-                else if (vkey(A.k, w) > kv) up = true;
-                else dn = true;
+        for (int64_t xq = sb0 + lane; xq - lane < se; xq += 128) {  // 4 steps of 32 arcs in flight
+            uint32_t w[4], rk[4];
+            bool up[4], dn[4];
+#pragma unroll
+            for (int u = 0; u < 4; u++) w[u] = xq + u * 32 < se ? (uint32_t)__ldg(A.ci + xq + u * 32) : 0u;
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const bool ok = xq + u * 32 < se;
+                const bool sv = ok && in_set(A.inS, w[u]);
+                up[u] = sv && vkey(A.k, w[u]) > kv;
+                dn[u] = sv && !up[u];
+                rk[u] = sv ? jp_rank(A, w[u]) : 0u;
+                if (ok && !sv) jp_fixed(A, h, m0.x, x0, w[u]);
             }
-            const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
-            if (up) __stcs(A.lst + hl + pu + __popc(mu & lt), jp_rank(A, w));
-            if (dn) __stcs(A.lst + ll + pd + __popc(md & lt), jp_rank(A, w));
-            pu += __popc(mu);
-            pd += __popc(md);
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const unsigned mu = __ballot_sync(FULL, up[u]), md = __ballot_sync(FULL, dn[u]);
+                if (up[u]) __stcs(A.lst + hl + pu + __popc(mu & lt), rk[u]);
+                if (dn[u]) __stcs(A.lst + ll + pd + __popc(md & lt), rk[u]);
+                pu += __popc(mu);
+                pd += __popc(md);
+            }
         }
     }
 }
