@@ -343,6 +343,9 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_count(JpArgs A) {
             A.hdeg[h] = hi;
             A.ldeg[h] = lo;
         }
+        // algorithmic bytes: the row's columns (huge rows: k_jpc_count_huge), row pair,
+        // id map entry, the two counts
+        prof_add(A.prof, active ? (huge ? 0ull : 4ull * (uint64_t)(e - b)) + 28ull : 0ull);
         const uint32_t np = huge ? (uint32_t)((e - b + JP_PIECE - 1) / JP_PIECE) : 0u;
         const int64_t ps = warp_reserve(np, A.huge_cnt);
         for (uint32_t q = 0; q < np; q++) A.huge[ps + q] = ((int64_t)q << 32) | (uint32_t)h;
@@ -375,6 +378,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_count_huge(JpArgs A) {
             if (lh) atomicAdd(A.hdeg + h, lh);
             if (ll) atomicAdd(A.ldeg + h, ll);
         }
+        prof_add(A.prof, threadIdx.x == 0 ? 4ull * (uint64_t)(pe_ - pb) : 0ull);
     }
 }
 
@@ -506,6 +510,8 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
             A.hdeg[h] = 0;  // fill cursors of the huge rows
             A.ldeg[h] = 0;
         }
+        // algorithmic bytes: counts read, meta + hot record + zeroed extra words written
+        prof_add(A.prof, active ? 8ull + 48ull + 4ull * (R - 1u) : 0ull);
         o0 += t0;
         o1 += t1;
     }
@@ -606,6 +612,9 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
                 }
             }
         }
+        // algorithmic bytes: the row's columns read + list ids written (huge rows:
+        // k_jpc_fill_huge), row pair, id map, meta + hot record read
+        prof_add(A.prof, active ? (e - b > JP_BUDGET ? 0ull : 8ull * (uint64_t)(e - b)) + 68ull : 0ull);
     }
 }
 
@@ -672,6 +681,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
                 pd += __popc(md);
             }
         }
+        prof_add(A.prof, lane == 0 && se > sb0 ? 8ull * (uint64_t)(se - sb0) : 0ull);
     }
 }
 
@@ -1184,6 +1194,8 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     const int64_t nwords = (n + 31) / 32;
     const unsigned tiles_w = (unsigned)((nwords + JP_TILE - 1) / JP_TILE);
     const unsigned tiles_c = (unsigned)((n + JP_TILE - 1) / JP_TILE);  // compact ids <= n
+    unsigned long long *ctr = prof_counter(s);  // algorithmic bytes of the build (profiling)
+    A.prof = ctr;
     prof_begin("jp_build", s);
     if (list0) {
         SYM_CUDA(cudaMemsetAsync(w.arank, 0, 2 * sizeof(uint32_t) * (size_t)nwords, s));
@@ -1216,7 +1228,8 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     SYM_LAUNCH_CHECK();
     k_jpc_fill_huge<<<num_sms() * 4, JP_HUGE_THREADS, 0, s>>>(A);
     SYM_LAUNCH_CHECK();
-    prof_end(s, -1);
+    prof_end_dev(s, ctr);
+    A.prof = nullptr;
     return SYM_OK;
 }
 

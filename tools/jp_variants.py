@@ -9,9 +9,9 @@ sys.path.insert(0, ROOT)
 OUT = os.path.join(ROOT, "build", "variants")
 VARIANTS = {  # the last comparison run (DESIGN §7 records the others)
     "base": [],
-    "minb1": ["-DSYM_JR_MINB=1"],
-    "w32": ["-DSYM_JP_WATCH=32"],
-    "push128": ["-DSYM_JP_PUSH=128"],
+    "lc2": ["-DSYM_JP_LANE_CHECKS=2"],
+    "lc1": ["-DSYM_JP_LANE_CHECKS=1"],
+    "push512": ["-DSYM_JP_PUSH=512"],
 }
 
 if sys.argv[1] == "build":
