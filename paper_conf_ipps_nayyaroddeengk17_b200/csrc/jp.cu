@@ -75,6 +75,9 @@ constexpr int JP_PUSH_LANE = 8;  // phase B: tasks of <= JP_PUSH_LANE entries ar
 constexpr uint32_t JP_WATCH = SYM_JP_WATCH;  // a vertex checks once <= JP_WATCH higher neighbours are unpushed
 constexpr uint32_t JP_WLIST = SYM_JP_WLIST;  // higher lists up to JP_WLIST entries are their own watch list
 constexpr uint32_t JP_NOTBUILT = 0xffffffffu;
+#ifndef SYM_JR_BARRIER_RED
+#define SYM_JR_BARRIER_RED 1  // grid barrier: 1 = release-RED arrival + polling the counter (29.5 vs 30.9 ms)
+#endif
 constexpr int JP_BUILD = 256;    // phase B: higher entries per watch-list build task
 constexpr uint32_t JP_HBITS = 27;  // hot.w = offset of the extra bitmap words | min(R, 31) << 27
 constexpr uint32_t JP_HMASK = (1u << JP_HBITS) - 1u;
@@ -717,12 +720,20 @@ __device__ __forceinline__ void grid_sync(const JrCtl &C, uint32_t &k) {
     __syncthreads();
     k++;
     if (threadIdx.x == 0) {
+#if SYM_JR_BARRIER_RED
+        // arrival = one release reduction (no return); every CTA polls the counter
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(C.arr) : "memory");
+        const uint32_t target = k * gridDim.x;
+        while (ld_acquire_u32(C.arr) < target) {
+        }
+#else
         __threadfence();
         const uint32_t old = atomicAdd(C.arr, 1u);
         if (old + 1u == k * gridDim.x) st_release_u32(C.gen, k);
         else
             while (ld_acquire_u32(C.gen) < k) {
             }
+#endif
     }
     __syncthreads();
 }
