@@ -75,6 +75,9 @@ constexpr int JP_PUSH_LANE = 8;  // phase B: tasks of <= JP_PUSH_LANE entries ar
 constexpr uint32_t JP_WATCH = SYM_JP_WATCH;  // a vertex checks once <= JP_WATCH higher neighbours are unpushed
 constexpr uint32_t JP_WLIST = SYM_JP_WLIST;  // higher lists up to JP_WLIST entries are their own watch list
 constexpr uint32_t JP_NOTBUILT = 0xffffffffu;
+#ifndef SYM_JR_POLL
+#define SYM_JR_POLL 0
+#endif
 #ifndef SYM_JR_BARRIER_RED
 #define SYM_JR_BARRIER_RED 1  // grid barrier: 1 = release-RED arrival + polling the counter (29.5 vs 30.9 ms)
 #endif
@@ -716,7 +719,11 @@ struct JrCtl {
 // software grid barrier (all CTAs co-resident); k = barriers passed so far.  The
 // fence orders this CTA's writes (colours, lists, task entries, bitmap REDs) before
 // the arrival, so the next phase sees them.
-__device__ __forceinline__ void grid_sync(const JrCtl &C, uint32_t &k) {
+// After the barrier, thread 0 loads up to three counters into sm[0..2] (one L2 read
+// per CTA instead of one per warp) -- visible to the CTA after the final bar.sync.
+__device__ __forceinline__ void grid_sync(const JrCtl &C, uint32_t &k, const uint32_t *p0 = nullptr,
+                                          const uint32_t *p1 = nullptr, const uint32_t *p2 = nullptr,
+                                          uint32_t *sm = nullptr) {
     __syncthreads();
     k++;
     if (threadIdx.x == 0) {
@@ -724,8 +731,16 @@ __device__ __forceinline__ void grid_sync(const JrCtl &C, uint32_t &k) {
         // arrival = one release reduction (no return); every CTA polls the counter
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(C.arr) : "memory");
         const uint32_t target = k * gridDim.x;
+#if SYM_JR_POLL == 1  // relaxed polling, one acquire fence at the end
+        while (ld_volatile_u32(C.arr) < target) {
+        }
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+#elif SYM_JR_POLL == 2  // acquire polling with a short back-off
+        while (ld_acquire_u32(C.arr) < target) __nanosleep(40);
+#else
         while (ld_acquire_u32(C.arr) < target) {
         }
+#endif
 #else
         __threadfence();
         const uint32_t old = atomicAdd(C.arr, 1u);
@@ -734,6 +749,9 @@ __device__ __forceinline__ void grid_sync(const JrCtl &C, uint32_t &k) {
             while (ld_acquire_u32(C.gen) < k) {
             }
 #endif
+        if (p0) sm[0] = __ldcg(p0);
+        if (p1) sm[1] = __ldcg(p1);
+        if (p2) sm[2] = __ldcg(p2);
     }
     __syncthreads();
 }
@@ -766,10 +784,9 @@ __device__ __forceinline__ void nb_load(const JpArgs &A, uint32_t e, uint32_t q,
 // higher neighbour's colour is already in v's bitmap, so it cannot equal m).  A
 // vertex whose higher list is longer than JP_WLIST asks phase B for its watch list
 // first.
-__device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, int64_t warp_g, int64_t nwarps,
-                                           unsigned long long &bytes) {
+__device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t cnt, int64_t warp_g,
+                                           int64_t nwarps, unsigned long long &bytes) {
     const int lane = lane_id();
-    const uint32_t cnt = __ldcg(A.ucnt + r % 3);
     const uint32_t *U = A.ul[r & 1];
     uint32_t *Un = A.ul[(r + 1) & 1];
     // a long list is read coalesced (entry it*32*nwarps + warp*32 + lane); a short one
@@ -960,10 +977,9 @@ __device__ __forceinline__ void jp_push(const JpArgs &A, uint32_t r, const uint3
 }
 
 // Phase B of round r: push the new colours; build the requested watch lists
-__device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, int64_t warp_g, int64_t nwarps,
-                                           unsigned long long &bytes) {
+__device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, uint32_t cnt, uint32_t nbt,
+                                           int64_t warp_g, int64_t nwarps, unsigned long long &bytes) {
     const int lane = lane_id();
-    const uint32_t cnt = __ldcg(A.pcnt + r % 3);
     for (int64_t base = warp_g; base - warp_g < cnt; base += nwarps * 32) {
         const int64_t i = base + (int64_t)lane * nwarps;  // tasks spread over all warps
         uint4 tk = make_uint4(0u, 0u, 0u, 0u);
@@ -1002,7 +1018,6 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, int64_t 
         }
     }
     // watch lists: a warp per task filters JP_BUILD higher entries (uncoloured ones kept)
-    const uint32_t nbt = __ldcg(A.bcnt + r % 3);
     for (int64_t t = warp_g; t < nbt; t += nwarps) {
         const uint2 bt = __ldcg(A.btask + t);
         const uint4 m0 = __ldcg(A.meta + 2 * bt.x), m1 = __ldcg(A.meta + 2 * bt.x + 1);
@@ -1046,8 +1061,11 @@ __global__ void __launch_bounds__(JR_THREADS, SYM_JR_MINB) k_jp_rounds(JpArgs A,
     unsigned long long bytes = 0;
     uint32_t k = 0, r = 0;
     if (__ldcg(A.err) & 2u) return;  // the build overflowed the segment offsets (set before launch)
+    __shared__ uint32_t s_val[3];    // counters loaded once per CTA by the barriers
+    if (threadIdx.x == 0) s_val[0] = __ldcg(A.ucnt);
+    __syncthreads();
     for (;; r++) {
-        const uint32_t cnt = __ldcg(A.ucnt + r % 3);
+        const uint32_t cnt = s_val[0];
         if (cnt == 0) break;
         if (blockIdx.x == 0 && threadIdx.x == 0) {
             if (A.hist && r < 1024) {  // stats: list size and start time (32 ns units) of the first rounds
@@ -1059,21 +1077,22 @@ __global__ void __launch_bounds__(JR_THREADS, SYM_JR_MINB) k_jp_rounds(JpArgs A,
             A.bcnt[(r + 2) % 3] = 0u;
             if (r + 1 >= C.max_rounds || globaltimer_ns() - t0 > JR_TIMEOUT_NS) atomicOr(A.err, 1u);
         }
-        jp_phase_a(A, r, warp_g, nwarps, bytes);
-        grid_sync(C, k);
-        if (__ldcg(A.err) != 0) break;  // read after the barrier: every CTA sees the same word
+        jp_phase_a(A, r, cnt, warp_g, nwarps, bytes);
+        grid_sync(C, k, A.pcnt + r % 3, A.bcnt + r % 3, A.err, s_val);
+        if (s_val[2] != 0) break;  // read after the barrier: every CTA sees the same word
+        const uint32_t pc = s_val[0], bc = s_val[1];
         if (A.trace && blockIdx.x == 0 && threadIdx.x == 0 && r < 512) {  // diagnostics
             A.trace[r] = (uint32_t)((globaltimer_ns() - t0) >> 5);
             A.trace[512 + r] = __ldcg(A.pcnt + r % 3);
             A.trace[1024 + r] = __ldcg(A.bcnt + r % 3);
         }
         const uint64_t tb = A.trace ? globaltimer_ns() : 0;
-        jp_phase_b(A, r, warp_g, nwarps, bytes);
+        jp_phase_b(A, r, pc, bc, warp_g, nwarps, bytes);
         if (A.trace && r < 512) {  // diagnostics: slowest CTA's phase-B work span
             __syncthreads();
             if (threadIdx.x == 0) atomicMax(A.trace + 1536 + r, (uint32_t)((globaltimer_ns() - tb) >> 5));
         }
-        grid_sync(C, k);
+        grid_sync(C, k, A.ucnt + (r + 1) % 3, nullptr, nullptr, s_val);
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *C.levels = r;
     prof_add(A.prof, bytes);

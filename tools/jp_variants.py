@@ -10,8 +10,6 @@ OUT = os.path.join(ROOT, "build", "variants")
 VARIANTS = {  # the last comparison run (DESIGN §7 records the others)
     "base": [],
     "lc2": ["-DSYM_JP_LANE_CHECKS=2"],
-    "bar_atom": ["-DSYM_JR_BARRIER_RED=0"],
-    "minb1": ["-DSYM_JR_MINB=1"],
 }
 
 if sys.argv[1] == "build":
