@@ -911,11 +911,33 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
         if (pass) A.hot[h].x = m;
         if (state == 2) *reinterpret_cast<uint2 *>(A.meta + 2 * h + 1) = make_uint2(pos, lm);
         if (state == 5) reinterpret_cast<uint32_t *>(A.meta + 2 * h)[3] = 0u;  // filled by phase B
-        const int64_t slot = warp_append(stay, A.ucnt + (r + 1) % 3);
+        // the three reservations (next list, push tasks, build tasks): warp scans, then
+        // lane 0 issues the three atomics back to back (one round trip, not three)
+        const uint32_t nt = pass ? (ld + JP_PUSH - 1) / JP_PUSH : 0u;
+        const uint32_t nb = state == 5 ? (hd + JP_BUILD - 1) / JP_BUILD : 0u;
+        uint32_t xs = stay ? 1u : 0u, xt = nt, xb_ = nb;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t ys = __shfl_up_sync(FULL, xs, d), yt = __shfl_up_sync(FULL, xt, d),
+                           yb = __shfl_up_sync(FULL, xb_, d);
+            if (lane >= d) {
+                xs += ys;
+                xt += yt;
+                xb_ += yb;
+            }
+        }
+        const uint32_t Ts = __shfl_sync(FULL, xs, 31), Tt = __shfl_sync(FULL, xt, 31), Tb = __shfl_sync(FULL, xb_, 31);
+        uint32_t bsv = 0, btv = 0, bbv = 0;
+        if (lane == 0) {
+            if (Ts) bsv = atomicAdd(A.ucnt + (r + 1) % 3, Ts);
+            if (Tt) btv = atomicAdd(A.pcnt + r % 3, Tt);
+            if (Tb) bbv = atomicAdd(A.bcnt + r % 3, Tb);
+        }
+        const int64_t slot = (int64_t)__shfl_sync(FULL, bsv, 0) + xs - (stay ? 1u : 0u);
+        const int64_t ts = (int64_t)__shfl_sync(FULL, btv, 0) + xt - nt;
+        const int64_t bs = (int64_t)__shfl_sync(FULL, bbv, 0) + xb_ - nb;
         if (stay) Un[slot] = h;
         // push tasks of a new colour
-        const uint32_t nt = pass ? (ld + JP_PUSH - 1) / JP_PUSH : 0u;
-        const int64_t ts = warp_reserve(nt, A.pcnt + r % 3);
         if (nt) {
             const uint64_t l0 = off + watch_words(hd) + hd;  // the lower list
             for (uint32_t t = 0; t < nt; t++) {
@@ -924,8 +946,6 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
             }
         }
         // watch-list build tasks, one per JP_BUILD higher entries
-        const uint32_t nb = state == 5 ? (hd + JP_BUILD - 1) / JP_BUILD : 0u;
-        const int64_t bs = warp_reserve(nb, A.bcnt + r % 3);
         for (uint32_t t = 0; t < nb; t++) A.btask[bs + t] = make_uint2(h, t);
         bytes += (state == 2 ? 8ull : 0ull) + (stay ? 4ull : 0ull) + (pass ? 4ull + 16ull * nt : 0ull) + 8ull * nb;
     }
@@ -1030,15 +1050,21 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, uint32_t
         for (int u = 0; u < K; u++) e[u] = j0 + u * 32 + lane < j1 ? __ldcs(A.lst + hl + j0 + u * 32 + lane) : 0u;
 #pragma unroll
         for (int u = 0; u < K; u++) c[u] = j0 + u * 32 + lane < j1 ? __ldcg(&A.hot[e[u]].x) : 1u;
+        unsigned mk[K];
+        uint32_t tot = 0;
 #pragma unroll
         for (int u = 0; u < K; u++) {
-            const bool keep = c[u] == 0u;
-            const unsigned mk = __ballot_sync(FULL, keep);
-            uint32_t p0 = 0;
-            if (mk && lane == 0) p0 = atomicAdd(wcp, (uint32_t)__popc(mk));
-            p0 = __shfl_sync(FULL, p0, 0);
-            const uint32_t p = p0 + __popc(mk & ((1u << lane) - 1u));
-            if (keep && p < JP_WATCH) A.lst[wl + p] = e[u];
+            mk[u] = __ballot_sync(FULL, c[u] == 0u);
+            tot += __popc(mk[u]);
+        }
+        uint32_t p0 = 0;
+        if (tot && lane == 0) p0 = atomicAdd(wcp, tot);  // one reservation per task
+        p0 = __shfl_sync(FULL, p0, 0);
+#pragma unroll
+        for (int u = 0; u < K; u++) {
+            const uint32_t p = p0 + __popc(mk[u] & ((1u << lane) - 1u));
+            if (c[u] == 0u && p < JP_WATCH) A.lst[wl + p] = e[u];
+            p0 += __popc(mk[u]);
         }
         bytes += lane == 0 ? 8ull * (j1 - j0) : 0ull;
     }
