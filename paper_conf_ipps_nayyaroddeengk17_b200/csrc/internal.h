@@ -177,7 +177,7 @@ struct ColorWs {
     unsigned long long *tsum = nullptr;
     int64_t ntiles = 0;
     uint4 *task = nullptr;         // push tasks of one round
-    uint2 *btask = nullptr;        // watch-list build tasks of one round
+    uint4 *btask = nullptr;        // watch-list build tasks of one round
     int64_t task_cap = 0;
     int64_t *queue = nullptr;      // build: (piece << 32 | h) items of the huge rows
     int32_t *vlist = nullptr;

@@ -75,6 +75,9 @@ constexpr int JP_PUSH_LANE = 8;  // phase B: tasks of <= JP_PUSH_LANE entries ar
 constexpr uint32_t JP_WATCH = SYM_JP_WATCH;  // a vertex checks once <= JP_WATCH higher neighbours are unpushed
 constexpr uint32_t JP_WLIST = SYM_JP_WLIST;  // higher lists up to JP_WLIST entries are their own watch list
 constexpr uint32_t JP_NOTBUILT = 0xffffffffu;
+#ifndef SYM_JP_PUSH_FILTER0
+#define SYM_JP_PUSH_FILTER0 0  // 1: also filter colours 1..32 (a load on the chain; 26.3 vs 26.05 ms)
+#endif
 #ifndef SYM_JR_POLL
 #define SYM_JR_POLL 0
 #endif
@@ -108,7 +111,8 @@ struct JpArgs {
     uint32_t *nc;        // [0] = compact count n', [1] = rows of degree > 2
     uint32_t *ul[2];     // active lists (compact ids), ping-pong by round
     uint4 *task;         // push tasks {list index lo, hi, entries, colour}
-    uint2 *btask;        // watch-list build tasks {h, chunk}
+    uint4 *btask;        // watch-list build tasks {h, chunk | offset bits 32.. << 24, hdeg, offset
+                         //   bits 0..31} -- everything the task needs, no meta load
     uint32_t *ucnt;      // [3] list counts (ring by round)
     uint32_t *pcnt;      // [3] push-task counts (ring by round)
     uint32_t *bcnt;      // [3] build-task counts (ring by round)
@@ -946,7 +950,8 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
             }
         }
         // watch-list build tasks, one per JP_BUILD higher entries
-        for (uint32_t t = 0; t < nb; t++) A.btask[bs + t] = make_uint2(h, t);
+        for (uint32_t t = 0; t < nb; t++)
+            A.btask[bs + t] = make_uint4(h, t | ((uint32_t)(off >> 32) << 24), hd, (uint32_t)off);
         bytes += (state == 2 ? 8ull : 0ull) + (stay ? 4ull : 0ull) + (pass ? 4ull + 16ull * nt : 0ull) + 8ull * nb;
     }
 }
@@ -963,7 +968,11 @@ __device__ __forceinline__ void jp_push(const JpArgs &A, uint32_t r, const uint3
 #pragma unroll
     for (int u = 0; u < K; u++) {  // colour, R field and extra-word offset in one 16-B load
         x[u] = 0xffffffffu;
+#if SYM_JP_PUSH_FILTER0
         if (act[u]) {
+#else
+        if (act[u] && q > 0) {  // colours 1..32: no filter load, the atomics go straight out
+#endif
             const uint4 s = __ldcg(A.hot + e[u]);
             act[u] = s.x == 0u;
             x[u] = s.w;
@@ -1039,11 +1048,10 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, uint32_t
     }
     // watch lists: a warp per task filters JP_BUILD higher entries (uncoloured ones kept)
     for (int64_t t = warp_g; t < nbt; t += nwarps) {
-        const uint2 bt = __ldcg(A.btask + t);
-        const uint4 m0 = __ldcg(A.meta + 2 * bt.x), m1 = __ldcg(A.meta + 2 * bt.x + 1);
-        const uint64_t wl = meta_off(m1), hl = wl + watch_words(m0.y);
+        const uint4 bt = __ldcg(A.btask + t);
+        const uint64_t wl = ((uint64_t)(bt.y >> 24) << 32) | bt.w, hl = wl + watch_words(bt.z);
         uint32_t *wcp = reinterpret_cast<uint32_t *>(A.meta + 2 * bt.x) + 3;
-        const uint32_t j0 = bt.y * JP_BUILD, j1 = min(m0.y, j0 + JP_BUILD);
+        const uint32_t j0 = (bt.y & 0xffffffu) * JP_BUILD, j1 = min(bt.z, j0 + JP_BUILD);
         constexpr int K = JP_BUILD / 32;
         uint32_t e[K], c[K];
 #pragma unroll
@@ -1196,7 +1204,7 @@ void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
     w.ntiles = ntiles;
     w.task_cap = n + nnz / JP_PUSH + 2;  // tasks of one round <= all tasks
     w.task = a.take<uint4>((size_t)w.task_cap);
-    w.btask = a.take<uint2>((size_t)w.task_cap);
+    w.btask = a.take<uint4>((size_t)w.task_cap);
     w.vlist = a.take<int32_t>((size_t)n + 1);
     w.mark = a.take<uint8_t>((size_t)n + 1);
     w.queue = a.take<int64_t>((size_t)(nnz / JP_BUDGET + 2));  // huge-row pieces (<= nnz/JP_BUDGET)

@@ -9,7 +9,7 @@ sys.path.insert(0, ROOT)
 OUT = os.path.join(ROOT, "build", "variants")
 VARIANTS = {  # the last comparison run (DESIGN §7 records the others)
     "base": [],
-    "lc2": ["-DSYM_JP_LANE_CHECKS=2"],
+    "filter0": ["-DSYM_JP_PUSH_FILTER0=1"],
 }
 
 if sys.argv[1] == "build":
