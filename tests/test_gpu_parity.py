@@ -171,3 +171,18 @@ def test_generator_cpu_gpu_identical():
     c = G.grid(300, 200, 0.6, 2)
     d = G.grid(300, 200, 0.6, 2, device=DEV)
     assert torch.equal(c[1], d[1].cpu())
+
+
+@pytest.mark.parametrize("fn", ["sym_color", "sym_mis", "sym_mm"])
+def test_max_rounds_is_reported(fn):
+    """params.max_rounds caps the round loop: SYM_EROUNDS, not a wrong result.  The
+    early-commit colouring needs tens of rounds on R-MAT s12 (plain JP: more)."""
+    rp, ci = G.rmat(12, 16, 1)
+    rpd, cid = rp.cuda(), ci.cuda()
+    with pytest.raises(sb.SymError) as ei:
+        getattr(sb, fn)(rpd, cid, "none", 0, 42, max_rounds=2)
+    assert ei.value.code == 6  # SYM_EROUNDS
+    # and with room to finish, the result equals the oracle
+    got = getattr(sb, fn)(rpd, cid, "none", 0, 42, max_rounds=100000).cpu().numpy()
+    ref = getattr(O, fn[4:])(rp, ci, "none", 0, 42)
+    assert (got.astype(np.int64) == ref.astype(np.int64)).all()
