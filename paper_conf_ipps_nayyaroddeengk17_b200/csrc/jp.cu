@@ -1162,8 +1162,7 @@ __global__ void k_color_conflicts(const int64_t *__restrict__ rp_x, const int32_
             for (int64_t x = rp_x[v]; x < rp_x[v + 1] && !conf; x++) conf = color[ci_x[x]] == cv;
             mark[v] = conf ? 1 : 0;
         }
-        int64_t s = warp_append(conf, cnt);
-        if (s >= 0) list[s] = (int32_t)v;
+        cta_append2(conf, false, (int32_t)v, n, list, cnt, cnt);  // one atomic per CTA
     }
 }
 

@@ -223,10 +223,7 @@ __global__ void k_mis_classify_cross(const int64_t *__restrict__ rp_x, int64_t n
         bool valid = v < n;
         bool bnd = valid && (rp_x[v + 1] > rp_x[v]);
         if (valid) st[v] = bnd ? ST_INACTIVE : ST_UNDEC;
-        int64_t sI = warp_append(valid && !bnd, cnt_front);
-        int64_t sB = warp_append(bnd, cnt_back);
-        if (sI >= 0) vlist[sI] = (int32_t)v;
-        if (sB >= 0) vlist[n - 1 - sB] = (int32_t)v;
+        cta_append2(valid && !bnd, bnd, (int32_t)v, n, vlist, cnt_front, cnt_back);
     }
 }
 

@@ -30,33 +30,7 @@ __global__ void k_classify_degk(const int64_t *__restrict__ rp, int64_t n, uint3
         if (valid) h = (rp[v + 1] - rp[v]) > (int64_t)k;
         unsigned word = __ballot_sync(FULL, h);
         if (lane_id() == 0 && valid) hbits[v >> 5] = word;
-        if (vlist) {  // one reservation per CTA and class (the list order is immaterial)
-            __shared__ uint32_t wl[32], wh[32], bl, bh;
-            const unsigned mL = __ballot_sync(FULL, valid && !h), mH = word;
-            const int wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
-            if (lane_id() == 0) {
-                wl[wid] = __popc(mL);
-                wh[wid] = __popc(mH);
-            }
-            __syncthreads();
-            if (threadIdx.x == 0) {
-                uint32_t tl = 0, th = 0;
-                for (int q = 0; q < nw; q++) {
-                    const uint32_t a0 = wl[q], a1 = wh[q];
-                    wl[q] = tl;
-                    wh[q] = th;
-                    tl += a0;
-                    th += a1;
-                }
-                bl = tl ? atomicAdd(cnt_front, tl) : 0u;
-                bh = th ? atomicAdd(cnt_back, th) : 0u;
-            }
-            __syncthreads();
-            const unsigned lt = (1u << lane_id()) - 1u;
-            if (valid && !h) vlist[bl + wl[wid] + __popc(mL & lt)] = (int32_t)v;
-            if (valid && h) vlist[n - 1 - (int64_t)(bh + wh[wid] + __popc(mH & lt))] = (int32_t)v;
-            __syncthreads();
-        }
+        if (vlist) cta_append2(valid && !h, h, (int32_t)v, n, vlist, cnt_front, cnt_back);
     }
 }
 
