@@ -34,10 +34,10 @@ METRIC = "MIS/MM/COLOR edges/s at 1/2/4/8 B200; % of HBM roofline; vs CPU oracle
 TRAFFIC = {
     "split": 4.51e9,       # k_split<DEGK> / <RAND> at R-MAT s24 (profiles/r1b_ncu.md): 2.22 GB read + 2.29 GB written
     "mm_round0": 0.719e9,  # k_round0<MM> on the RAND-4 intra CSR
-    # COLOR-Deg2 at R-MAT s24 (profiles/r1h_color_launches.csv): the build kernels
+    # COLOR-Deg2 at R-MAT s24 (profiles/r1i_color_launches.csv): the build kernels
     # (k_jpc_*: compact ids, counts, lists) and the early-commit rounds kernel
-    "jp_build": 8.45e9,
-    "jp_rounds": 17.24e9,  # k_jp_rounds: 14.82 GB read + 2.41 GB written (lists, meta, hot records)
+    "jp_build": 8.46e9,
+    "jp_rounds": 17.12e9,  # k_jp_rounds: 14.72 GB read + 2.40 GB written (lists, meta, hot records)
 }
 
 
