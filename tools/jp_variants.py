@@ -9,7 +9,9 @@ sys.path.insert(0, ROOT)
 OUT = os.path.join(ROOT, "build", "variants")
 VARIANTS = {  # the last comparison run (DESIGN §7 records the others)
     "base": [],
-    "filter0": ["-DSYM_JP_PUSH_FILTER0=1"],
+    "t256x4": ["-DSYM_JR_THREADS=256", "-DSYM_JR_MINB=4"],
+    "t1024x1": ["-DSYM_JR_THREADS=1024", "-DSYM_JR_MINB=1"],
+    "lc2": ["-DSYM_JP_LANE_CHECKS=2"],
 }
 
 if sys.argv[1] == "build":
