@@ -268,6 +268,48 @@ int sym_shard_mm_round(const sym_graph_shard *g, const sym_params *p, int round,
                        const int32_t *pick_prev, int32_t *pick_cur, const int32_t *frontier, const uint32_t *count,
                        int32_t *next, uint32_t *next_count, void *ws, size_t ws_bytes, sym_stream_t stream);
 
+/* ---- sharded COLOR (COLOR-NONE P:214, COLOR-Rand Alg 8, COLOR-Degk Alg 9
+   P:234; Jones-Plassmann rounds [18]) ----
+   Same shard layout as sharded MIS (v_begin a multiple of 32).  Every rank keeps a
+   full replica of the colour array, uint32[n_global] (0 = uncoloured), zeroed by the
+   caller.  p->kind / p->param / p->seed select the class function (NONE: one class;
+   RAND: the hash label with p parts, global id; DEGK: the all-gathered V_H bitmap
+   hbits of sym_shard_classify) and the vertex priorities (the single-GPU ones).
+   admit = 1 restricts every step to arcs whose endpoints share a class (the induced
+   subgraphs), admit = 0 uses every arc.  After each round the caller all-gathers the
+   owned colour segments and all-reduces *next_count; a phase ends at global count 0.
+     COLOR-NONE:  frontier; rounds with admit = 0.
+     COLOR-Degk:  frontier; rounds with admit = 1 (G_H and G_L at once); M = the
+                  all-reduced max of sym_shard_color_maxh; sym_shard_color_shift(M).
+     COLOR-Rand:  frontier; rounds with admit = 1; all-gather; conflicts (V', the
+                  owned endpoints of monochromatic cross arcs) -> list; clear;
+                  all-gather; rounds on that list with admit = 0.
+   The result equals sym_color() bit for bit (any schedule of the rounds gives the
+   greedy colouring in priority order).  All pointers are device pointers;
+   counts are device uint32. */
+
+/* owned vertices with color == 0 -> list, *count (set by the call) */
+int sym_shard_color_frontier(const sym_graph_shard *g, const uint32_t *color, int32_t *list, uint32_t *count,
+                             sym_stream_t stream);
+/* one JP round over the owned frontier: a vertex whose admitted higher-priority
+   neighbours are all coloured takes the smallest colour >= 1 not held by an admitted
+   neighbour; the others -> next, *next_count (set by the call) */
+int sym_shard_jp_round(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits, int admit,
+                       uint32_t *color, const int32_t *frontier, const uint32_t *count, int32_t *next,
+                       uint32_t *next_count, sym_stream_t stream);
+/* COLOR-Rand V' (Alg 8): owned v with a cross-class neighbour of the same colour -> list */
+int sym_shard_color_conflicts(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits,
+                              const uint32_t *color, int32_t *list, uint32_t *count, sym_stream_t stream);
+/* color[list[i]] = 0 for i < *count */
+int sym_shard_color_clear(const sym_graph_shard *g, uint32_t *color, const int32_t *list, const uint32_t *count,
+                          sym_stream_t stream);
+/* *max_out = max colour over owned V_H vertices (0 if none) */
+int sym_shard_color_maxh(const sym_graph_shard *g, const uint32_t *hbits, const uint32_t *color, uint32_t *max_out,
+                         sym_stream_t stream);
+/* color[v] += M for owned V_L vertices (COLOR-Degk's palette shift) */
+int sym_shard_color_shift(const sym_graph_shard *g, const uint32_t *hbits, uint32_t *color, uint32_t M,
+                          sym_stream_t stream);
+
 /* ---- kernel profiling hook (measurement only; off by default) ----
    sym_profile_enable(1) makes every later call record a CUDA event pair on its
    stream around each hot-kernel launch, grouped by kernel class ("split",

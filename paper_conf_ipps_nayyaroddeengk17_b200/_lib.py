@@ -23,6 +23,8 @@ EXPORTS = (
     "sym_shard_mis_kill", "sym_shard_mis_finish",
     "sym_shard_decompose_workspace_bytes", "sym_shard_decompose", "sym_shard_mm_workspace_bytes",
     "sym_shard_mm_frontier", "sym_shard_mm_round",
+    "sym_shard_color_frontier", "sym_shard_jp_round", "sym_shard_color_conflicts", "sym_shard_color_clear",
+    "sym_shard_color_maxh", "sym_shard_color_shift",
 )
 
 
@@ -110,6 +112,13 @@ def load(build_if_missing: bool = False):
         "sym_shard_mm_frontier": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P, P]),
         "sym_shard_mm_round": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, ctypes.c_int, P, P, P, P, P, P,
                                               P, P, ctypes.c_size_t, P]),
+        "sym_shard_color_frontier": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P, P]),
+        "sym_shard_jp_round": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, ctypes.c_int, P, P, P, P, P,
+                                              P]),
+        "sym_shard_color_conflicts": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, P, P, P, P]),
+        "sym_shard_color_clear": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P, P]),
+        "sym_shard_color_maxh": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P, P]),
+        "sym_shard_color_shift": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, ctypes.c_uint32, P]),
         "sym_profile_enable": (ctypes.c_int, [ctypes.c_int]),
         "sym_profile_collect": (ctypes.c_int, [ctypes.POINTER(SymKernelProfile), ctypes.c_int,
                                                ctypes.POINTER(ctypes.c_int)]),

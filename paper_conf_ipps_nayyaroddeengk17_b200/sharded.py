@@ -1,4 +1,4 @@
-"""Sharded MIS and MM over several GPUs (C-ABI: include/sym.h `sym_shard_*`).
+"""Sharded MIS, MM and COLOR over several GPUs (C-ABI: include/sym.h `sym_shard_*`).
 
 One process per GPU.  Rank r owns the 32-aligned vertex block [r*B, min(n, (r+1)*B))
 and holds those rows with global column ids; every rank keeps a full replica of the
@@ -16,6 +16,13 @@ buffers; per handshake round (`sym_shard_mm_round`) the owned segment
 the current picks and of mate are all-gathered.  MM-Rand decomposes the owned rows
 locally (`sym_shard_decompose`; labels hash the global id): phase 1 on the local
 intra CSR, phase 2 on the local cross CSR.  Results equal sym_mm() bit for bit.
+
+COLOR-NONE / COLOR-Degk / COLOR-Rand (Alg 9, Alg 8) keep a
+replica of the colour array; per Jones-Plassmann round (`sym_shard_jp_round`) the
+owned colour segments are all-gathered.  COLOR-Degk colours G_H and G_L at once
+(same-class arcs), all-reduces max C_H and shifts the V_L colours; COLOR-Rand colours
+the induced subgraphs, marks and clears V' (monochromatic cross arcs), all-gathers,
+and recolours V' against G.  Results equal sym_color() bit for bit.
 
 This module is orchestration only: every step of the method runs in libsym.so
 kernels (`GpuBackend`); the exchange is a `Transport`:
@@ -73,6 +80,8 @@ class Shard:
     mate: torch.Tensor = None    # MM: replica, int32[nranks * block]
     picks: list = None           # MM: two pick replicas (round r writes picks[r & 1])
     pick_cur: torch.Tensor = None
+    color: torch.Tensor = None   # COLOR: replica, int32 view of uint32[nranks * block]
+    cmax: torch.Tensor = None    # COLOR-Degk: owned max colour over V_H (1 element)
     extra: dict = field(default_factory=dict)
 
     def __post_init__(self):
@@ -108,6 +117,11 @@ class Shard:
         self.mate = torch.full((pad,), -1, dtype=torch.int32, device=dev)
         self.picks = [torch.full((pad,), -1, dtype=torch.int32, device=dev) for _ in range(2)]
 
+    def init_color(self):
+        dev = self.row_ptr.device
+        self.color = torch.zeros(self.nranks * self.block, dtype=torch.int32, device=dev)
+        self.cmax = torch.zeros(1, dtype=torch.int32, device=dev)
+
 
 @dataclass
 class PhaseView:
@@ -138,6 +152,9 @@ class LocalTransport:
     def allreduce_sum(self, shards, attr) -> int:
         return int(sum(int(getattr(s, attr)[0]) for s in shards))
 
+    def allreduce_max(self, shards, attr) -> int:
+        return int(max(int(getattr(s, attr)[0]) for s in shards))
+
 
 class DistTransport:
     """One shard per process; torch.distributed collectives (NCCL on GPUs)."""
@@ -158,6 +175,13 @@ class DistTransport:
         (s,) = shards
         t = getattr(s, attr).clone()
         dist.all_reduce(t, group=self.group)
+        return int(t[0])
+
+    def allreduce_max(self, shards, attr) -> int:
+        import torch.distributed as dist
+        (s,) = shards
+        t = getattr(s, attr).clone()
+        dist.all_reduce(t, op=dist.ReduceOp.MAX, group=self.group)
         return int(t[0])
 
 
@@ -245,6 +269,39 @@ class GpuBackend:
                                               sh.nxt_cnt.data_ptr(), ws.data_ptr(), ws.numel(), self._s(sh)),
                   "mm_round")
 
+    # ---- COLOR
+    def color_frontier(self, sh: Shard):
+        g = sh.c_struct()
+        self._chk(self.lib.sym_shard_color_frontier(ctypes.byref(g), sh.color.data_ptr(), sh.cur.data_ptr(),
+                                                    sh.cur_cnt.data_ptr(), self._s(sh)), "color_frontier")
+
+    def jp_round(self, sh: Shard, kind: int, param: int, seed: int, admit: int):
+        g = sh.c_struct()
+        p = L.SymParams(kind, int(param), seed & (2**64 - 1), 0, 0)
+        self._chk(self.lib.sym_shard_jp_round(ctypes.byref(g), ctypes.byref(p), sh.hbits.data_ptr(), admit,
+                                              sh.color.data_ptr(), sh.cur.data_ptr(), sh.cur_cnt.data_ptr(),
+                                              sh.nxt.data_ptr(), sh.nxt_cnt.data_ptr(), self._s(sh)), "jp_round")
+
+    def color_conflicts(self, sh: Shard, kind: int, param: int, seed: int):
+        g = sh.c_struct()
+        p = L.SymParams(kind, int(param), seed & (2**64 - 1), 0, 0)
+        self._chk(self.lib.sym_shard_color_conflicts(ctypes.byref(g), ctypes.byref(p), sh.hbits.data_ptr(),
+                                                     sh.color.data_ptr(), sh.cur.data_ptr(), sh.cur_cnt.data_ptr(),
+                                                     self._s(sh)), "color_conflicts")
+        g = sh.c_struct()
+        self._chk(self.lib.sym_shard_color_clear(ctypes.byref(g), sh.color.data_ptr(), sh.cur.data_ptr(),
+                                                 sh.cur_cnt.data_ptr(), self._s(sh)), "color_clear")
+
+    def color_maxh(self, sh: Shard):
+        g = sh.c_struct()
+        self._chk(self.lib.sym_shard_color_maxh(ctypes.byref(g), sh.hbits.data_ptr(), sh.color.data_ptr(),
+                                                sh.cmax.data_ptr(), self._s(sh)), "color_maxh")
+
+    def color_shift(self, sh: Shard, M: int):
+        g = sh.c_struct()
+        self._chk(self.lib.sym_shard_color_shift(ctypes.byref(g), sh.hbits.data_ptr(), sh.color.data_ptr(), int(M),
+                                                 self._s(sh)), "color_shift")
+
 
 # ------------------------------------------------------------------ the flow
 def sym_mis_sharded(shards, kind="none", param=0, seed=42, transport=None, backend=None, stats=None):
@@ -330,6 +387,63 @@ def sym_mm_sharded(shards, kind="none", param=0, seed=42, transport=None, backen
     if stats is not None:
         stats["rounds"] = rounds
     return [s.mate[s.v0:s.v1].clone() for s in shards]
+
+
+def sym_color_sharded(shards, kind="none", param=0, seed=42, transport=None, backend=None, stats=None):
+    """COLOR-NONE / COLOR-Degk / COLOR-Rand over the given shards (Jones-Plassmann
+    rounds; Alg 9; Alg 8).  Returns the owned colours (int32
+    view of uint32, >= 1) of every shard, in the order given; equal to sym_color()."""
+    kind = {"none": L.NONE, "rand": L.RAND, "degk": L.DEGK}.get(kind, kind) if isinstance(kind, str) else int(kind)
+    if kind not in (L.NONE, L.RAND, L.DEGK):
+        raise ValueError("unknown decomposition kind")
+    if kind == L.RAND and not 1 <= int(param) <= 65535:
+        raise ValueError("RAND needs 1 <= p <= 65535")
+    transport = transport or LocalTransport()
+    backend = backend or GpuBackend()
+    for s in shards:
+        s.init_color()
+    if kind == L.DEGK:
+        for s in shards:
+            s.hbits.zero_()
+            backend.classify(s, int(param))
+        transport.allgather(shards, "hbits")
+
+    def run_phase(admit, fresh):
+        if fresh:
+            for s in shards:
+                backend.color_frontier(s)
+        r = 0
+        while True:
+            for s in shards:
+                backend.jp_round(s, kind, param, seed, admit)
+            transport.allgather(shards, "color")
+            r += 1
+            left = transport.allreduce_sum(shards, "nxt_cnt")
+            for s in shards:
+                s.cur, s.nxt = s.nxt, s.cur
+                s.cur_cnt, s.nxt_cnt = s.nxt_cnt, s.cur_cnt
+            if left == 0:
+                return r
+
+    rounds = [run_phase(0 if kind == L.NONE else 1, True)]
+    conflicts = 0
+    if kind == L.DEGK:
+        for s in shards:
+            backend.color_maxh(s)
+        M = transport.allreduce_max(shards, "cmax")
+        for s in shards:
+            backend.color_shift(s, M)
+        transport.allgather(shards, "color")
+    elif kind == L.RAND:
+        for s in shards:
+            backend.color_conflicts(s, kind, param, seed)   # V' -> s.cur, then cleared
+        transport.allgather(shards, "color")
+        conflicts = transport.allreduce_sum(shards, "cur_cnt")
+        rounds.append(run_phase(0, False) if conflicts else 0)
+    if stats is not None:
+        stats["rounds"] = rounds
+        stats["conflicts"] = conflicts
+    return [s.color[s.v0:s.v1].clone() for s in shards]
 
 
 def make_shards(row_ptr, col_idx, nranks, ranks=None):

@@ -148,3 +148,65 @@ class CpuBackend:
         if nxt:
             sh.nxt[: len(nxt)] = torch.tensor(nxt, dtype=torch.int32)
         sh.nxt_cnt[0] = len(nxt)
+
+    # ---- COLOR (JP rounds P:214; Alg 8; Alg 9)
+    def _cls(self, kind, param, seed, hb, v):
+        if kind == 1:  # RAND
+            return O.label(seed, v, param)
+        if kind == 2:  # DEGK
+            return self._bit(hb, v)
+        return 0
+
+    def color_frontier(self, sh):
+        col = sh.color.numpy()
+        vs = [v for v in range(sh.v0, sh.v1) if col[v] == 0]
+        if vs:
+            sh.cur[: len(vs)] = torch.tensor(vs, dtype=torch.int32)
+        sh.cur_cnt[0] = len(vs)
+
+    def jp_round(self, sh, kind, param, seed, admit):
+        rp, ci = sh.row_ptr.numpy(), sh.col_idx.numpy()
+        col = sh.color.numpy()
+        hb = sh.hbits.numpy().view(np.uint32)
+        snap = col.copy()  # synchronous round (the kernel may see in-round colours: same result)
+        nxt = []
+        for v in sh.cur[: int(sh.cur_cnt[0])].tolist():
+            cv = self._cls(kind, param, seed, hb, v)
+            nb = [int(w) for w in ci[rp[v - sh.v0]: rp[v - sh.v0 + 1]]
+                  if admit == 0 or self._cls(kind, param, seed, hb, int(w)) == cv]
+            if any(self.key[w] > self.key[v] and snap[w] == 0 for w in nb):
+                nxt.append(v)
+                continue
+            used = {int(snap[w]) for w in nb}
+            c = 1
+            while c in used:
+                c += 1
+            col[v] = c
+        if nxt:
+            sh.nxt[: len(nxt)] = torch.tensor(nxt, dtype=torch.int32)
+        sh.nxt_cnt[0] = len(nxt)
+
+    def color_conflicts(self, sh, kind, param, seed):
+        rp, ci = sh.row_ptr.numpy(), sh.col_idx.numpy()
+        col = sh.color.numpy()
+        hb = sh.hbits.numpy().view(np.uint32)
+        vs = [v for v in range(sh.v0, sh.v1)
+              if any(self._cls(kind, param, seed, hb, int(w)) != self._cls(kind, param, seed, hb, v)
+                     and col[w] == col[v] for w in ci[rp[v - sh.v0]: rp[v - sh.v0 + 1]])]
+        for v in vs:
+            col[v] = 0
+        if vs:
+            sh.cur[: len(vs)] = torch.tensor(vs, dtype=torch.int32)
+        sh.cur_cnt[0] = len(vs)
+
+    def color_maxh(self, sh):
+        col = sh.color.numpy()
+        hb = sh.hbits.numpy().view(np.uint32)
+        sh.cmax[0] = max([int(col[v]) for v in range(sh.v0, sh.v1) if self._bit(hb, v)] or [0])
+
+    def color_shift(self, sh, M):
+        col = sh.color.numpy()
+        hb = sh.hbits.numpy().view(np.uint32)
+        for v in range(sh.v0, sh.v1):
+            if not self._bit(hb, v):
+                col[v] += M
