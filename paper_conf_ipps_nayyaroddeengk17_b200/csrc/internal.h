@@ -4,7 +4,13 @@
 #include <stddef.h>
 #include <stdint.h>
 
+#include <algorithm>
 #include <string>
+
+// round kernels (MIS, MM) launch one resident wave instead of 8 CTAs per SM
+#ifndef SYM_ROUND_ONE_WAVE
+#define SYM_ROUND_ONE_WAVE 1
+#endif
 
 #include "../../include/sym.h"
 #include "common.cuh"

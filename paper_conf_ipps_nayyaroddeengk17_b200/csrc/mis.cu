@@ -271,7 +271,22 @@ void carve_mis_ws(Arena &a, int64_t n, int64_t nnz, MisWs &w) {
     w.gmax = a.take<unsigned long long>((size_t)n + 1);
 }
 
-static int round_grid() { return num_sms() * (2048 / MIS_THREADS); }
+// One resident wave: the grid-stride round kernels lose ~20 % to a partial second wave
+// when the grid asks for more CTAs than fit (8 requested, 6 resident at 40 regs).
+static int round_grid() {
+#if SYM_ROUND_ONE_WAVE
+    static int g = 0;
+    if (!g) {
+        int per = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_mis_round, MIS_THREADS, 0) != cudaSuccess || per < 1)
+            per = 2048 / MIS_THREADS;
+        g = num_sms() * per;
+    }
+    return g;
+#else
+    return num_sms() * (2048 / MIS_THREADS);
+#endif
+}
 
 // Run Luby rounds of one phase until the frontier is empty.  Round 0 reads
 // (list0, rev0, cnt0) -- or the implicit range [0, implicit_n) when list0 == nullptr.

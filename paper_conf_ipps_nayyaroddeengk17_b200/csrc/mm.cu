@@ -300,13 +300,33 @@ struct MmPhase {
     int64_t nnz = -1;  // arcs of the phase CSR when known on the host (profiling only)
 };
 
+// One resident wave of the grid-stride round kernel (see mis.cu round_grid).
+static int mm_round_grid() {
+#if SYM_ROUND_ONE_WAVE
+    static int g = 0;
+    if (!g) {
+        int per = 2048 / MM_THREADS, x = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_mm_round<false, false>, MM_THREADS, 0) == cudaSuccess && x > 0)
+            per = std::min(per, x);
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_mm_round<false, true>, MM_THREADS, 0) == cudaSuccess && x > 0)
+            per = std::min(per, x);
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_mm_round<true, true>, MM_THREADS, 0) == cudaSuccess && x > 0)
+            per = std::min(per, x);
+        g = num_sms() * per;
+    }
+    return g;
+#else
+    return num_sms() * (2048 / MM_THREADS);
+#endif
+}
+
 static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph, int phase) {
     Ctl *ctl = f.ctl;
     cudaStream_t s = f.stream;
     SYM_CUDA(cudaMemsetAsync(ctl->ring, 0, sizeof(ctl->ring) + sizeof(ctl->huge), s));
     const Key k = stream_key(f.p.seed, TAG_EDGE, 0);
     const uint32_t maxr = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
-    const int full_grid = num_sms() * (2048 / MM_THREADS);
+    const int full_grid = mm_round_grid();
     int grid = full_grid;
     int r = 0;
     const int batch = 4;  // rounds launched per host poll of the frontier count
@@ -550,7 +570,7 @@ extern "C" int sym_shard_mm_round(const sym_graph_shard *g, const sym_params *p,
     A.k = stream_key(p->seed, TAG_EDGE, 0);
     A.prof = nullptr;
     A.row_base = g->v_begin;
-    const int grid = num_sms() * (2048 / MM_THREADS);
+    const int grid = mm_round_grid();
     if (round == 0) k_mm_round<false, true><<<grid, MM_THREADS, 0, s>>>(A);
     else k_mm_round<true, true><<<grid, MM_THREADS, 0, s>>>(A);
     SYM_LAUNCH_CHECK();
