@@ -80,11 +80,12 @@ constexpr uint64_t LB_AGG = 1ULL << 62, LB_INC = 2ULL << 62, LB_VAL = (1ULL << 6
 // of a tile is resident or finished when the tile looks back (as CUB's single-pass
 // scans rely on).
 template <int KIND, bool VEC>
-__global__ void __launch_bounds__(SPLIT_THREADS)
-    k_split(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, int64_t n, int64_t nnz,
-            const int64_t *__restrict__ first_row, int64_t ntiles, const uint32_t *__restrict__ hbits, Key kr,
-            uint32_t p, uint64_t *tile_state, int64_t *__restrict__ rp_in, int32_t *__restrict__ ci_in,
-            int64_t *__restrict__ rp_x, int32_t *__restrict__ ci_x, int64_t row_base) {
+__device__ __forceinline__ void split_tile(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, int64_t n,
+                                           int64_t nnz, const int64_t *__restrict__ first_row, int64_t ntiles,
+                                           const uint32_t *__restrict__ hbits, Key kr, uint32_t p,
+                                           uint64_t *tile_state, int64_t *__restrict__ rp_in,
+                                           int32_t *__restrict__ ci_in, int64_t *__restrict__ rp_x,
+                                           int32_t *__restrict__ ci_x, int64_t row_base) {
     constexpr int T = SPLIT_TILE, V = SPLIT_PER_THREAD, NT = SPLIT_THREADS, NW = NT / 32;
     static_assert(V % 4 == 0 && T < 32768, "tile layout");
     __shared__ __align__(16) int16_t s_head[T];   // head position of the row owning each arc, or -1
@@ -300,6 +301,25 @@ __global__ void __launch_bounds__(SPLIT_THREADS)
     }
 }
 
+#define SPLIT_PARAMS                                                                                             \
+    const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, int64_t n, int64_t nnz,                      \
+        const int64_t *__restrict__ first_row, int64_t ntiles, const uint32_t *__restrict__ hbits, Key kr,       \
+        uint32_t p, uint64_t *tile_state, int64_t *__restrict__ rp_in, int32_t *__restrict__ ci_in,              \
+        int64_t *__restrict__ rp_x, int32_t *__restrict__ ci_x, int64_t row_base
+#define SPLIT_FWD rp, ci, n, nnz, first_row, ntiles, hbits, kr, p, tile_state, rp_in, ci_in, rp_x, ci_x, row_base
+
+// DEGk / NONE: 4 CTAs/SM at the compiler's register choice.  RAND (hash labels, no
+// class gathers) gains from a 5th CTA per SM (<= 51 regs, 40 KB smem each): 2.0 ->
+// 1.8 ms at R-MAT s24 p = 4; the same bound made the DEGk split slower (3.4 -> 5.0 ms).
+template <int KIND, bool VEC>
+__global__ void __launch_bounds__(SPLIT_THREADS) k_split(SPLIT_PARAMS) {
+    split_tile<KIND, VEC>(SPLIT_FWD);
+}
+template <bool VEC>
+__global__ void __launch_bounds__(SPLIT_THREADS, 5) k_split_rand(SPLIT_PARAMS) {
+    split_tile<KIND_RAND, VEC>(SPLIT_FWD);
+}
+
 // ------------------------------------------------------------------ host side
 void carve_split_ws(Arena &a, int64_t n, int64_t nnz, SplitWs &w) {
     int64_t ntiles = (nnz + SPLIT_TILE - 1) / SPLIT_TILE;
@@ -347,8 +367,8 @@ int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const Spl
     g.rp, g.ci, g.n, g.nnz, w.first_row, w.ntiles, w.hbits, kr, param, w.tile_state, rp_in, \
         ci_in, rp_x, ci_x, row_base
     if (kind == KIND_RAND) {
-        if (vec) k_split<KIND_RAND, true><<<grid, SPLIT_THREADS, 0, s>>>(SPLIT_ARGS);
-        else k_split<KIND_RAND, false><<<grid, SPLIT_THREADS, 0, s>>>(SPLIT_ARGS);
+        if (vec) k_split_rand<true><<<grid, SPLIT_THREADS, 0, s>>>(SPLIT_ARGS);
+        else k_split_rand<false><<<grid, SPLIT_THREADS, 0, s>>>(SPLIT_ARGS);
     } else if (kind == KIND_DEGK) {
         if (vec) k_split<KIND_DEGK, true><<<grid, SPLIT_THREADS, 0, s>>>(SPLIT_ARGS);
         else k_split<KIND_DEGK, false><<<grid, SPLIT_THREADS, 0, s>>>(SPLIT_ARGS);
