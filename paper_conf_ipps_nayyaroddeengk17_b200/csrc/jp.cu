@@ -539,7 +539,15 @@ __device__ __forceinline__ void jp_fixed(const JpArgs &A, int64_t h, uint32_t R,
 // fill pass: higher and lower lists (list ids, CSR order); fixed colours of
 // neighbours outside S.  Columns and lists stream (evict-first) so the id map stays
 // in L2 for the gathers.
+// 5 CTAs/SM (48 regs, no spills; 59 without the bound -> 4): more rank lookups in flight
+#ifndef SYM_FILL_MINB
+#define SYM_FILL_MINB 5
+#endif
+#if SYM_FILL_MINB > 0
+__global__ void __launch_bounds__(JP_THREADS, SYM_FILL_MINB) k_jpc_fill(JpArgs A) {
+#else
 __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
+#endif
     const uint32_t cnt = A.nc[0];
     const int lane = lane_id();
     const int64_t warp_g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -1287,7 +1295,16 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
         k_jpc_place<<<tiles_c, JP_THREADS, 0, s>>>(A);
         SYM_LAUNCH_CHECK();
     }
-    k_jpc_fill<<<num_sms() * (2048 / JP_THREADS), JP_THREADS, 0, s>>>(A);
+    {
+        // one resident wave of the grid-stride fill (see mis.cu round_grid)
+        int per = 2048 / JP_THREADS;
+#if SYM_ROUND_ONE_WAVE
+        int x = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_jpc_fill, JP_THREADS, 0) == cudaSuccess && x > 0)
+            per = std::min(per, x);
+#endif
+        k_jpc_fill<<<num_sms() * per, JP_THREADS, 0, s>>>(A);
+    }
     SYM_LAUNCH_CHECK();
     k_jpc_fill_huge<<<num_sms() * 4, JP_HUGE_THREADS, 0, s>>>(A);
     SYM_LAUNCH_CHECK();
