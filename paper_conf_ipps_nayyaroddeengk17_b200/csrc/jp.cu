@@ -1306,7 +1306,17 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
         k_jpc_fill<<<num_sms() * per, JP_THREADS, 0, s>>>(A);
     }
     SYM_LAUNCH_CHECK();
-    k_jpc_fill_huge<<<num_sms() * 4, JP_HUGE_THREADS, 0, s>>>(A);
+    {
+        // block-strided pieces: one resident wave (40 regs x 512 threads -> 3 CTAs/SM, not 4)
+        int per = 4;
+#if SYM_ROUND_ONE_WAVE
+        int x = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_jpc_fill_huge, JP_HUGE_THREADS, 0) == cudaSuccess &&
+            x > 0)
+            per = std::min(per, x);
+#endif
+        k_jpc_fill_huge<<<num_sms() * per, JP_HUGE_THREADS, 0, s>>>(A);
+    }
     SYM_LAUNCH_CHECK();
     prof_end_dev(s, ctr);
     A.prof = nullptr;
