@@ -250,7 +250,8 @@ __global__ void __launch_bounds__(MM_HUGE_THREADS) k_mm_huge(MmRoundArgs A) {
     }
 }
 
-// phase-2 frontier: unmatched vertices that have phase-2 arcs
+// phase-2 frontier: unmatched vertices that have phase-2 arcs (CTA-aggregated appends:
+// per-warp appends serialised at the counter, 0.38 ms at R-MAT s24)
 __global__ void k_mm_phase2_list(const int64_t *__restrict__ rp, const int64_t *__restrict__ rp2,
                                  const uint32_t *__restrict__ hbits, int dual, int64_t n, const int32_t *mate,
                                  int32_t *list, uint32_t *cnt) {
@@ -263,8 +264,7 @@ __global__ void k_mm_phase2_list(const int64_t *__restrict__ rp, const int64_t *
             const int64_t *r = useX ? rp2 : rp;
             take = r[v + 1] > r[v];
         }
-        int64_t s = warp_append(take, cnt);
-        if (s >= 0) list[s] = (int32_t)v;
+        cta_append2(take, false, (int32_t)v, n, list, cnt, cnt);  // one atomic per CTA (order immaterial)
     }
 }
 
