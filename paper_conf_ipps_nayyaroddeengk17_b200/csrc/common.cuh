@@ -115,6 +115,36 @@ __device__ __forceinline__ void cta_append2(bool c0, bool c1, int32_t v, int64_t
     __syncthreads();  // the scratch is reused by the next call
 }
 
+// Same, into two separate lists (list0 / cnt0, list1 / cnt1), u32 entries.
+__device__ __forceinline__ void cta_append2x(bool c0, bool c1, uint32_t v, uint32_t *list0, uint32_t *cnt0,
+                                             uint32_t *list1, uint32_t *cnt1) {
+    __shared__ uint32_t x0[32], x1[32], xb0, xb1;
+    const unsigned m0 = __ballot_sync(FULL, c0), m1 = __ballot_sync(FULL, c1);
+    const int wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+    if (lane_id() == 0) {
+        x0[wid] = __popc(m0);
+        x1[wid] = __popc(m1);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t t0 = 0, t1 = 0;
+        for (int q = 0; q < nw; q++) {
+            const uint32_t a0 = x0[q], a1 = x1[q];
+            x0[q] = t0;
+            x1[q] = t1;
+            t0 += a0;
+            t1 += a1;
+        }
+        xb0 = t0 ? atomicAdd(cnt0, t0) : 0u;
+        xb1 = t1 ? atomicAdd(cnt1, t1) : 0u;
+    }
+    __syncthreads();
+    const unsigned lt = (1u << lane_id()) - 1u;
+    if (c0) list0[xb0 + x0[wid] + __popc(m0 & lt)] = v;
+    if (c1) list1[xb1 + x1[wid] + __popc(m1 & lt)] = v;
+    __syncthreads();
+}
+
 __device__ __forceinline__ uint64_t ld_volatile_u64(const uint64_t *p) {
     uint64_t v;
     asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");

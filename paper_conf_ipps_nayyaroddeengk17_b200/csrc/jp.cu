@@ -507,7 +507,8 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
         const bool ready = active && hd == 0, later = active && hd > 0 && hd <= JP_WATCH;
         const bool r0 = ready || (later && A.in_list != nullptr);
         const bool first = r0 || later;
-        const int64_t s0 = warp_append(r0, A.ucnt), s1 = warp_append(first && !r0, A.ucnt + 1);
+        // CTA-aggregated list appends (one atomic per CTA and list; order immaterial)
+        cta_append2x(r0, first && !r0, (uint32_t)h, A.ul[0], A.ucnt, A.ul[1], A.ucnt + 1);
         if (active) {
             const unsigned long long off = o0 + p0;
             const uint32_t x0 = (uint32_t)(o1 + p1);
@@ -515,8 +516,6 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
             A.meta[2 * h + 1] = make_uint4(0u, 0u, (uint32_t)off, (uint32_t)(off >> 32));
             A.hot[h] = make_uint4(0u, hd, 0u, (x0 & JP_HMASK) | (min(R, JP_R5) << JP_HBITS));
             for (uint32_t q = 1; q < R; q++) A.xb[x0 + q - 1] = 0u;
-            if (r0) A.ul[0][s0] = (uint32_t)h;
-            else if (first) A.ul[1][s1] = (uint32_t)h;
             A.hdeg[h] = 0;  // fill cursors of the huge rows
             A.ldeg[h] = 0;
         }
