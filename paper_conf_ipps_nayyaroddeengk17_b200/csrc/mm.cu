@@ -66,8 +66,17 @@ __device__ __forceinline__ void mm_row(const MmRoundArgs &A, int32_t u, int64_t 
     }
 }
 
+// 6 CTAs/SM (<= 40 regs, no spills; 47 without the bound -> 5): more mate gathers in flight
+#ifndef SYM_MM_MINB
+#define SYM_MM_MINB 6
+#endif
+#if SYM_MM_MINB > 0
+#define MM_ROUND_BOUNDS __launch_bounds__(MM_THREADS, SYM_MM_MINB)
+#else
+#define MM_ROUND_BOUNDS __launch_bounds__(MM_THREADS)
+#endif
 template <bool RESOLVE, bool MATE>
-__global__ void __launch_bounds__(MM_THREADS) k_mm_round(MmRoundArgs A) {
+__global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
     const uint32_t cnt = A.in_list ? *A.in_cnt : (uint32_t)A.implicit_n;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         *A.clear_cnt = 0;
