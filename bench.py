@@ -345,6 +345,7 @@ def main():
             sc.wait_event(consumed[cur])
             with torch.cuda.stream(sc):
                 for h, d in zip(out_h, (I, C, M)):
+                    d.record_stream(sc)  # keep the block alive until sc's copy has run
                     h.copy_(d, non_blocking=True)
         stream.wait_stream(sc)
         e1.record(stream)

@@ -319,7 +319,7 @@ int sym_shard_color_shift(const sym_graph_shard *g, const uint32_t *hbits, uint3
    bytes those launches had to move when the library knows them exactly from host
    sizes (split = 8 B/arc + 24 B/vertex; first MM round = 4 B/arc + 24
    B/vertex of its phase graph), else -1.  Collect resets the accumulators.
-   Not thread-safe: profile one host thread at a time. */
+   Thread-safe: begin/end pairs nest per stream; the state is mutex-guarded. */
 typedef struct {
     char name[24];
     int64_t launches;

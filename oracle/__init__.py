@@ -66,6 +66,7 @@ _SIGS = {
     "or_cert_mis": (_I64, [_I64, _P, _P, _P, _U64, _P]),
     "or_cert_mm": (_I64, [_I64, _P, _P, _P, _INT, _P, _U64, _P]),
     "or_cert_col": (_I64, [_I64, _P, _P, _P, _P, _INT, _U64, _P]),
+    "or_cert_col_rand": (_I64, [_I64, _P, _P, _U32, _U64, _P, _P]),
 }
 
 
@@ -221,6 +222,15 @@ def cert_col(rp, ci, C, seed, inS=None, cls=None, admit=ADMIT_ALL):
     return lib().or_cert_col(n, _ptr(rp), _ptr(ci), _ptr(S), _ptr(c), admit, seed & (2**64 - 1), _ptr(Cc))
 
 
+def cert_col_rand(rp, ci, C, p, seed):
+    """COLOR-Rand certificate in O(m + n) -> (violations, |V'|)."""
+    n, rp, ci = _graph(rp, ci)
+    Cc = _np(C, np.uint32)
+    nconf = ctypes.c_int64(0)
+    bad = lib().or_cert_col_rand(n, _ptr(rp), _ptr(ci), int(p), seed & (2**64 - 1), _ptr(Cc), ctypes.byref(nconf))
+    return int(bad), int(nconf.value)
+
+
 def cert_flow(problem, rp, ci, kind, param, seed, result):
     """O(m) exact check that `result` equals the oracle flow's output, phase by phase
     (used at full sizes where the sequential run or its sort is too slow).
@@ -288,8 +298,7 @@ def cert_flow(problem, rp, ci, kind, param, seed, result):
             bad += int(((~H) & ((CL < 1) | (CL > 0xFFFFFFFF))).sum())
             CL = np.clip(CL, 0, None).astype(np.uint32)
             return bad + cert_col(rp, ci, CL, seed, inS=(~H).astype(np.uint8), cls=cls, admit=ADMIT_SAME)
-        # RAND: recompute C_IS from the oracle itself is the slow part; instead check
-        # phase-2 certificate given the conflict set derived from a phase-1 colouring
-        # computed by the oracle (LF-COL on intra arcs is O(m log n)).
-        raise NotImplementedError("use color() for COLOR-RAND parity")
+        # RAND: C1 by a topological sweep of the intra priority DAG, V' from C1, then
+        # C = C1 off V' and the first-fit certificate on V' (oracle.c or_cert_col_rand)
+        return cert_col_rand(rp, ci, C, param, seed)[0]
     raise ValueError(problem)

@@ -579,3 +579,72 @@ int64_t or_cert_col(int64_t n, const int64_t *rp, const int32_t *ci, const uint8
     free(mark);
     return bad;
 }
+
+/* COLOR-Rand certificate (Alg 8; reading C3 of DESIGN §3), O(m + n):
+     1. C1 = LF-COL(V, E_intra) computed by a topological sweep of the priority DAG
+        over the intra arcs: a vertex is coloured (first fit over its higher intra
+        neighbours) once all of them are coloured.  First-fit colour of v depends only
+        on the colours of its higher neighbours, so any topological order gives the
+        colours of the sorted order -- without the O(n log n) sort.
+     2. V' = both endpoints of every cross edge whose endpoints share a C1 colour.
+     3. C must equal C1 off V'; on V', C must be LF-COL(V', E, C1 off V'): checked by
+        or_cert_col over S = V' with all arcs admitted (non-V' neighbours count as
+        pre-coloured with C = C1).
+   Returns the number of violated vertices (0 = C is the oracle's COLOR-Rand output);
+   *nconf (nullable) receives |V'|. */
+int64_t or_cert_col_rand(int64_t n, const int64_t *rp, const int32_t *ci, uint32_t p, uint64_t seed,
+                         const uint32_t *C, int64_t *nconf) {
+    uint64_t key = or_stream_key(seed, OR_TAG_VERTEX, 0);
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+    uint32_t *C1 = (uint32_t *)calloc(nn, sizeof(uint32_t));
+    int64_t *pend = (int64_t *)malloc(sizeof(int64_t) * nn); /* uncoloured higher intra neighbours */
+    int32_t *queue = (int32_t *)malloc(sizeof(int32_t) * nn);
+    uint8_t *S = (uint8_t *)calloc(nn, 1);
+    int64_t maxd = 0, head = 0, tail = 0, bad = 0, conf = 0;
+    or_classes(n, rp, OR_RAND, p, seed, cls);
+    for (int64_t v = 0; v < n; v++) {
+        if (rp[v + 1] - rp[v] > maxd) maxd = rp[v + 1] - rp[v];
+        pend[v] = 0;
+        for (int64_t e = rp[v]; e < rp[v + 1]; e++)
+            if (cls[ci[e]] == cls[v] && vgreater(key, ci[e], (int32_t)v)) pend[v]++;
+        if (pend[v] == 0) queue[tail++] = (int32_t)v;
+    }
+    uint8_t *mark = (uint8_t *)malloc((size_t)maxd + 2);
+    while (head < tail) { /* step 1 */
+        int32_t v = queue[head++];
+        int64_t d = rp[v + 1] - rp[v];
+        memset(mark, 0, (size_t)d + 2);
+        for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+            int32_t w = ci[e];
+            if (cls[w] == cls[v] && vgreater(key, w, v) && (int64_t)C1[w] <= d + 1) mark[C1[w]] = 1;
+        }
+        uint32_t c = 1;
+        while (mark[c]) c++;
+        C1[v] = c;
+        for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+            int32_t w = ci[e];
+            if (cls[w] == cls[v] && vgreater(key, v, w) && --pend[w] == 0) queue[tail++] = w;
+        }
+    }
+    if (tail != n) bad += n - tail; /* unreachable for a DAG; defensive */
+    for (int64_t v = 0; v < n; v++) { /* step 2 */
+        for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+            int32_t w = ci[e];
+            if (cls[w] != cls[v] && C1[w] == C1[v]) { S[v] = 1; break; }
+        }
+        conf += S[v];
+        if (!S[v] && C[v] != C1[v]) bad++; /* step 3, off V' */
+    }
+    uint32_t *zero = (uint32_t *)calloc(nn, sizeof(uint32_t));
+    bad += or_cert_col(n, rp, ci, S, zero, 0, seed, C); /* step 3, on V' */
+    if (nconf) *nconf = conf;
+    free(zero);
+    free(mark);
+    free(S);
+    free(queue);
+    free(pend);
+    free(C1);
+    free(cls);
+    return bad;
+}

@@ -126,7 +126,9 @@ def sym_decompose(row_ptr, col_idx, kind, param, seed=42, label=False, flags=0) 
     ws_n = lib.sym_workspace_bytes(ctypes.byref(g), ctypes.byref(p), L.PROBLEM_DECOMPOSE)
     ws = _workspace(ws_n, dev)
     d = out.c_struct()
-    rc = lib.sym_decompose(ctypes.byref(g), ctypes.byref(p), ws.data_ptr(), ws.numel(), ctypes.byref(d), _stream_ptr(dev))
+    with torch.cuda.device(dev):  # the library launches on the current device
+        rc = lib.sym_decompose(ctypes.byref(g), ctypes.byref(p), ws.data_ptr(), ws.numel(), ctypes.byref(d),
+                               _stream_ptr(dev))
     if rc != L.SYM_OK:
         raise SymError(rc, "sym_decompose")
     out.nnz_in, out.nnz_x = int(d.nnz_in), int(d.nnz_x)
@@ -152,8 +154,9 @@ def _flow(name, problem, out_dtype, row_ptr, col_idx, kind, param, seed, decomp,
     st = L.SymStats()
     dptr = ctypes.byref(decomp.c_struct()) if decomp is not None else None
     fn = getattr(lib, name)
-    rc = fn(ctypes.byref(g), ctypes.byref(p), dptr, ws.data_ptr(), ws.numel(), out.data_ptr(),
-            ctypes.byref(st) if stats else None, _stream_ptr(dev))
+    with torch.cuda.device(dev):  # the library launches on the current device
+        rc = fn(ctypes.byref(g), ctypes.byref(p), dptr, ws.data_ptr(), ws.numel(), out.data_ptr(),
+                ctypes.byref(st) if stats else None, _stream_ptr(dev))
     if rc != L.SYM_OK:
         raise SymError(rc, name)
     out = out[: g.n]
@@ -207,7 +210,9 @@ def sym_validate(row_ptr, col_idx) -> int:
     ws_n = lib.sym_workspace_bytes(ctypes.byref(g), None, L.PROBLEM_VALIDATE)
     ws = _workspace(ws_n, row_ptr.device)
     bad = ctypes.c_int64(0)
-    rc = lib.sym_validate(ctypes.byref(g), ws.data_ptr(), ws.numel(), ctypes.byref(bad), _stream_ptr(row_ptr.device))
+    with torch.cuda.device(row_ptr.device):
+        rc = lib.sym_validate(ctypes.byref(g), ws.data_ptr(), ws.numel(), ctypes.byref(bad),
+                              _stream_ptr(row_ptr.device))
     if rc not in (L.SYM_OK, L.SYM_EGRAPH):
         raise SymError(rc, "sym_validate")
     return int(bad.value)

@@ -21,17 +21,20 @@ int cuda_fail(cudaError_t e, const char *what, const char *file, int line) {
     return SYM_ECUDA;
 }
 
+int current_device() {
+    int dev = -1;
+    return cudaGetDevice(&dev) == cudaSuccess ? dev : -1;
+}
+
 int num_sms() {
-    static int cached = 0;
-    if (!cached) {
-        int dev = 0, v = 0;
-        if (cudaGetDevice(&dev) == cudaSuccess &&
-            cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && v > 0)
-            cached = v;
-        else
-            cached = 148;
-    }
-    return cached;
+    static std::atomic<int> slots[SYM_MAX_DEVICES];
+    return dev_cached(slots, [] {
+        int v = 0;
+        const int dev = current_device();
+        if (dev >= 0 && cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && v > 0)
+            return v;
+        return 148;
+    });
 }
 
 int read_u32(const uint32_t *dev, uint32_t *host, cudaStream_t s) {

@@ -5,6 +5,7 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <atomic>
 #include <string>
 
 // round kernels (MIS, MM) launch one resident wave instead of 8 CTAs per SM
@@ -133,6 +134,24 @@ __device__ __forceinline__ void prof_add(unsigned long long *ctr, unsigned long 
 int read_u32(const uint32_t *dev, uint32_t *host, cudaStream_t s);
 int read_u64(const uint64_t *dev, uint64_t *host, cudaStream_t s);
 int num_sms();
+int current_device();
+
+// A value cached per CUDA device (grid sizes from occupancy queries, function
+// attributes): computed lazily by `compute` on the first call on each device.  A
+// process may drive several GPUs from several host threads; the slots are atomics
+// (a racing first call computes the same value twice, which is harmless).
+constexpr int SYM_MAX_DEVICES = 64;
+template <class F>
+int dev_cached(std::atomic<int> *slots, F compute) {
+    const int d = current_device();
+    if (d < 0 || d >= SYM_MAX_DEVICES) return compute();
+    int v = slots[d].load(std::memory_order_relaxed);
+    if (v == 0) {
+        v = compute();
+        slots[d].store(v, std::memory_order_relaxed);
+    }
+    return v;
+}
 
 // ------------------------------------------------------------------ flows
 struct FlowArgs {

@@ -1328,21 +1328,21 @@ static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t 
     Ctl *ctl = f.ctl;
     cudaStream_t s = f.stream;
     if (f.g.n == 0) return SYM_OK;
-    static int grid = 0;
-    if (grid == 0) {
-        int dev = 0, coop = 0, per_sm = 0;
-        SYM_CUDA(cudaGetDevice(&dev));
-        SYM_CUDA(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev));
-        if (!coop) {
-            set_error("JP needs cooperative launch (persistent rounds kernel), unsupported on this device");
-            return SYM_ECUDA;
-        }
-        SYM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_jp_rounds, JR_THREADS, 0));
-        if (per_sm < 1) {
-            set_error("k_jp_rounds does not fit on an SM");
-            return SYM_ECUDA;
-        }
-        grid = num_sms() * per_sm;
+    // one resident wave of the cooperative rounds kernel, per device (-1: unsupported)
+    static std::atomic<int> grid_slots[SYM_MAX_DEVICES];
+    const int grid = dev_cached(grid_slots, [] {
+        int coop = 0, per_sm = 0;
+        const int dev = current_device();
+        if (dev < 0 || cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev) != cudaSuccess || !coop)
+            return -1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_jp_rounds, JR_THREADS, 0) != cudaSuccess ||
+            per_sm < 1)
+            return -1;
+        return num_sms() * per_sm;
+    });
+    if (grid < 0) {
+        set_error("JP needs a cooperative launch of k_jp_rounds (persistent rounds kernel) on this device");
+        return SYM_ECUDA;
     }
     JpArgs A;
     SYM_TRY(jp_build(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n));

@@ -275,14 +275,13 @@ void carve_mis_ws(Arena &a, int64_t n, int64_t nnz, MisWs &w) {
 // when the grid asks for more CTAs than fit (8 requested, 6 resident at 40 regs).
 static int round_grid() {
 #if SYM_ROUND_ONE_WAVE
-    static int g = 0;
-    if (!g) {
+    static std::atomic<int> slots[SYM_MAX_DEVICES];
+    return dev_cached(slots, [] {
         int per = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_mis_round, MIS_THREADS, 0) != cudaSuccess || per < 1)
             per = 2048 / MIS_THREADS;
-        g = num_sms() * per;
-    }
-    return g;
+        return num_sms() * per;
+    });
 #else
     return num_sms() * (2048 / MIS_THREADS);
 #endif
@@ -313,7 +312,7 @@ static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp
     int r = 0;
     const int batch = 4;  // rounds launched per host poll of the frontier count
     for (;;) {
-        for (int b = 0; b < batch; b++, r++) {
+        for (int b = 0; b < batch && (uint32_t)r < maxr; b++, r++) {  // never past the cap
             MisRoundArgs A;
             A.rp = rp;
             A.ci = ci;

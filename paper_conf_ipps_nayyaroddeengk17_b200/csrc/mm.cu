@@ -312,8 +312,8 @@ struct MmPhase {
 // One resident wave of the grid-stride round kernel (see mis.cu round_grid).
 static int mm_round_grid() {
 #if SYM_ROUND_ONE_WAVE
-    static int g = 0;
-    if (!g) {
+    static std::atomic<int> slots[SYM_MAX_DEVICES];
+    return dev_cached(slots, [] {
         int per = 2048 / MM_THREADS, x = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_mm_round<false, false>, MM_THREADS, 0) == cudaSuccess && x > 0)
             per = std::min(per, x);
@@ -321,9 +321,8 @@ static int mm_round_grid() {
             per = std::min(per, x);
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_mm_round<true, true>, MM_THREADS, 0) == cudaSuccess && x > 0)
             per = std::min(per, x);
-        g = num_sms() * per;
-    }
-    return g;
+        return num_sms() * per;
+    });
 #else
     return num_sms() * (2048 / MM_THREADS);
 #endif
@@ -351,7 +350,7 @@ static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph
         }
     }
     for (;;) {
-        for (int bb = 0; bb < batch; bb++, r++) {
+        for (int bb = 0; bb < batch && (uint32_t)r < maxr; bb++, r++) {  // never past the cap
             MmRoundArgs A;
             A.rp = ph.rp;
             A.rp2 = ph.rp2;

@@ -3,6 +3,7 @@
 // collection synchronises them after the caller's timed region.
 #include <cstring>
 #include <map>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -17,7 +18,7 @@ struct Rec {
     double bytes;
     int slot;  // device byte counter slot, or -1
 };
-bool g_on = false;
+std::atomic<bool> g_on{false};
 // device byte counters for launches whose algorithmic bytes depend on the frontier
 // (measurement mode only; the one allocation the library makes, lazily, when
 // profiling is enabled)
@@ -26,8 +27,10 @@ unsigned long long *g_dev = nullptr;
 int g_dev_next = 0;
 std::vector<Rec> g_recs;
 std::vector<cudaEvent_t> g_pool;
-std::vector<std::pair<std::string, double>> g_open;  // pending begin (class, bytes)
-std::vector<cudaEvent_t> g_open_ev;
+// pending begins, a LIFO per stream (calls on different streams / host threads nest
+// independently); every global here is guarded by g_mu
+std::map<cudaStream_t, std::vector<std::pair<std::string, cudaEvent_t>>> g_open;
+std::mutex g_mu;
 
 cudaEvent_t get_event() {
     if (!g_pool.empty()) {
@@ -45,24 +48,32 @@ bool prof_on() { return g_on; }
 
 void prof_begin(const char *cls, cudaStream_t s) {
     if (!g_on) return;
+    std::lock_guard<std::mutex> lk(g_mu);
     cudaEvent_t e = get_event();
     cudaEventRecord(e, s);
-    g_open.emplace_back(cls, 0.0);
-    g_open_ev.push_back(e);
+    g_open[s].emplace_back(cls, e);
+}
+
+// closes the innermost pending begin of stream s
+static void close_rec(cudaStream_t s, double bytes, int slot) {
+    auto it = g_open.find(s);
+    if (it == g_open.end() || it->second.empty()) return;
+    cudaEvent_t e = get_event();
+    cudaEventRecord(e, s);
+    Rec r{it->second.back().first, it->second.back().second, e, bytes, slot};
+    it->second.pop_back();
+    g_recs.push_back(r);
 }
 
 void prof_end(cudaStream_t s, double bytes) {
-    if (!g_on || g_open.empty()) return;
-    cudaEvent_t e = get_event();
-    cudaEventRecord(e, s);
-    Rec r{g_open.back().first, g_open_ev.back(), e, bytes, -1};
-    g_open.pop_back();
-    g_open_ev.pop_back();
-    g_recs.push_back(r);
+    if (!g_on) return;
+    std::lock_guard<std::mutex> lk(g_mu);
+    close_rec(s, bytes, -1);
 }
 
 unsigned long long *prof_counter(cudaStream_t s) {
     if (!g_on) return nullptr;
+    std::lock_guard<std::mutex> lk(g_mu);
     if (!g_dev && cudaMalloc(&g_dev, sizeof(unsigned long long) * DEV_SLOTS) != cudaSuccess) {
         g_dev = nullptr;
         return nullptr;
@@ -74,13 +85,9 @@ unsigned long long *prof_counter(cudaStream_t s) {
 }
 
 void prof_end_dev(cudaStream_t s, unsigned long long *ctr) {
-    if (!g_on || g_open.empty()) return;
-    cudaEvent_t e = get_event();
-    cudaEventRecord(e, s);
-    Rec r{g_open.back().first, g_open_ev.back(), e, ctr ? 0.0 : -1.0, ctr ? (int)(ctr - g_dev) : -1};
-    g_open.pop_back();
-    g_open_ev.pop_back();
-    g_recs.push_back(r);
+    if (!g_on) return;
+    std::lock_guard<std::mutex> lk(g_mu);
+    close_rec(s, ctr ? 0.0 : -1.0, ctr ? (int)(ctr - g_dev) : -1);
 }
 
 }  // namespace sym
@@ -88,6 +95,7 @@ void prof_end_dev(cudaStream_t s, unsigned long long *ctr) {
 using namespace sym;
 
 extern "C" int sym_profile_enable(int on) {
+    std::lock_guard<std::mutex> lk(g_mu);
     g_on = on != 0;
     return SYM_OK;
 }
@@ -98,6 +106,7 @@ extern "C" int sym_profile_collect(sym_kernel_profile *out, int max_entries, int
         double ms = 0, bytes = 0;
         bool known = true;
     };
+    std::lock_guard<std::mutex> lk(g_mu);
     std::map<std::string, Acc> acc;
     std::vector<std::string> order;
     std::vector<unsigned long long> dev(g_dev_next);

@@ -265,21 +265,30 @@ int run_round0(int mode, const Graph &g, const int64_t *first_row, int64_t ntile
     A.hfilter = hfilter;
     A.out_list = out_list;
     A.out_cnt = out_cnt;
-    static bool attr = false;
-    if (!attr) {
-        SYM_CUDA(cudaFuncSetAttribute(k_round0<R0_MIS>, cudaFuncAttributeMaxDynamicSharedMemorySize, R0_SMEM));
-        SYM_CUDA(cudaFuncSetAttribute(k_round0<R0_MM>, cudaFuncAttributeMaxDynamicSharedMemorySize, R0_SMEM));
-        attr = true;
-    }
+    // function attributes are per device context: set once per device
+    static std::atomic<int> attr[SYM_MAX_DEVICES];
+    const int ok = dev_cached(attr, [] {
+        if (cudaFuncSetAttribute(k_round0<R0_MIS>, cudaFuncAttributeMaxDynamicSharedMemorySize, R0_SMEM) !=
+                cudaSuccess ||
+            cudaFuncSetAttribute(k_round0<R0_MM>, cudaFuncAttributeMaxDynamicSharedMemorySize, R0_SMEM) != cudaSuccess)
+            return -1;
+        return 1;
+    });
+    if (ok != 1) SYM_CUDA(cudaGetLastError());
     if (g.nnz <= 0 || ntiles <= 0) return SYM_EINVAL;  // caller uses the frontier kernel instead
     SYM_TRY(launch_first_row(g, ntiles, const_cast<int64_t *>(first_row), s));
     if (ntiles > 1) {
         k_r0_span_init<<<(unsigned)((ntiles + 255) / 256), 256, 0, s>>>(A);
         SYM_LAUNCH_CHECK();
     }
-    int per_sm = 0;
-    SYM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round0<R0_MM>, SPLIT_THREADS, R0_SMEM));
-    const int64_t want = (int64_t)num_sms() * (per_sm > 0 ? per_sm : 1);
+    static std::atomic<int> per_slots[SYM_MAX_DEVICES];
+    const int per_sm = dev_cached(per_slots, [] {
+        int x = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_round0<R0_MM>, SPLIT_THREADS, R0_SMEM) != cudaSuccess)
+            return 1;
+        return x > 0 ? x : 1;
+    });
+    const int64_t want = (int64_t)num_sms() * per_sm;
     const unsigned grid = (unsigned)(want < ntiles ? want : ntiles);
     prof_begin(mode == R0_MIS ? "mis_round0" : "mm_round0", s);
     if (mode == R0_MIS) k_round0<R0_MIS><<<grid, SPLIT_THREADS, R0_SMEM, s>>>(A);

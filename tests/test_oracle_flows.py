@@ -206,12 +206,43 @@ def test_certificates_accept_oracle_and_reject_perturbations(rmat14, kind, p):
     M2[M2[u]] = -1
     M2[u] = -1
     assert O.cert_flow("mm", rp, ci, kind, p, 42, M2) > 0
-    if kind != "rand":
-        C = O.color(rp, ci, kind, p, 42)
-        assert O.cert_flow("color", rp, ci, kind, p, 42, C) == 0
-        C2 = C.copy()
-        C2[int(np.argmax(np.diff(rp)))] += 1
-        assert O.cert_flow("color", rp, ci, kind, p, 42, C2) > 0
+    C = O.color(rp, ci, kind, p, 42)
+    assert O.cert_flow("color", rp, ci, kind, p, 42, C) == 0
+    C2 = C.copy()
+    C2[int(np.argmax(np.diff(rp)))] += 1
+    assert O.cert_flow("color", rp, ci, kind, p, 42, C2) > 0
+
+
+@pytest.mark.parametrize("seed", SEEDS)
+@pytest.mark.parametrize("p", [1, 2, 4, 64])
+def test_color_rand_certificate(rmat14, road, seed, p):
+    """The O(m) COLOR-Rand certificate (Alg 8; C1 by a topological sweep
+    instead of the sort) accepts exactly the oracle's output: every single-vertex
+    change -- in V' or outside it, up or down -- is rejected; p = 1 (no cross edges,
+    V' empty) reduces it to the JP/greedy certificate of COLOR-NONE; |V'| is the
+    fraction the paper reports the recolouring works on (~45 % at p = 2 on its
+    graphs; [sim] 25-37 % for R-MAT at p = 2..4)."""
+    for rp, ci in (rmat14, road):
+        n = rp.size - 1
+        C = O.color(rp, ci, "rand", p, seed)
+        bad, nconf = O.cert_col_rand(rp, ci, C, p, seed)
+        assert bad == 0
+        if p == 1:
+            assert nconf == 0
+            assert np.array_equal(C, O.color(rp, ci, "none", 0, seed))
+        elif (rp, ci) is rmat14 and p <= 4:
+            assert 0.15 < nconf / n < 0.5
+        rng = np.random.default_rng(seed & 0xFFFF)
+        for v in rng.choice(n, 12, replace=False):
+            for d in (1, -1):
+                if int(C[v]) + d < 1:
+                    continue
+                C2 = C.copy()
+                C2[v] = int(C[v]) + d
+                assert O.cert_col_rand(rp, ci, C2, p, seed)[0] > 0
+    # the NONE colouring is rejected as a COLOR-Rand result once cross edges exist
+    rp, ci = rmat14
+    assert O.cert_col_rand(rp, ci, O.color(rp, ci, "none", 0, seed), 4, seed)[0] > 0
 
 
 def test_round_counts_are_logarithmic(rmat14):
