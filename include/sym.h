@@ -312,19 +312,26 @@ int sym_shard_color_shift(const sym_graph_shard *g, const uint32_t *hbits, uint3
 
 /* ---- kernel profiling hook (measurement only; off by default) ----
    sym_profile_enable(1) makes every later call record a CUDA event pair on its
-   stream around each hot-kernel launch, grouped by kernel class ("split",
-   "mis_round", "mis_huge", "mm_round0", "mm_round", "mm_huge", "jp_build",
-   "jp_rounds", ...).  sym_profile_collect() synchronises those events and
-   returns, per class: launches, summed device milliseconds, and the algorithmic
-   bytes those launches had to move when the library knows them exactly from host
-   sizes (split = 8 B/arc + 24 B/vertex; first MM round = 4 B/arc + 24
-   B/vertex of its phase graph), else -1.  Collect resets the accumulators.
-   Thread-safe: begin/end pairs nest per stream; the state is mutex-guarded. */
+   stream around each hot-kernel launch, grouped by kernel class ("split_degk",
+   "split_rand", "mis_round", "mis_huge", "mm_round0", "mm_round", "mm_huge",
+   "jp_build", "jp_rounds", ...).  sym_profile_collect() synchronises those
+   events and returns, per class: launches, summed device milliseconds and two byte
+   counts of those launches (exact: counted by the kernels on device or known on the
+   host; -1 if unknown):
+     alg_bytes  = SURVEY §8(d)'s algorithmic bytes: a round moves 4 B per scanned arc
+                  + 9 B per active vertex (row_ptr pair + status); the split 8 B/arc +
+                  24 B per row pointer; JP 8 B/arc + 12 B/vertex of its phase graph
+                  (charged to "jp_rounds"; the build reports 0);
+     impl_bytes = the words this implementation's kernels load and store (lists,
+                  records, counters), i.e. alg plus the implementation's overheads.
+   Collect resets the accumulators.  Thread-safe: begin/end pairs nest per stream; the
+   state is mutex-guarded. */
 typedef struct {
     char name[24];
     int64_t launches;
     double ms;
     double alg_bytes;
+    double impl_bytes;
 } sym_kernel_profile;
 
 int sym_profile_enable(int on);

@@ -33,13 +33,45 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
 
+_SRC_OMP = os.path.join(_HERE, "oracle_omp.c")
+_LIB_OMP = os.path.join(_HERE, "liboracle_omp.so")
+_lib_omp = None
+
+
 def build(force: bool = False) -> str:
-    """Compile oracle.c with gcc (plain -O2, single-threaded)."""
+    """Compile oracle.c with gcc (plain -O2, single-threaded) -> liboracle.so, and the
+    round-based all-core forms (oracle_omp.c + oracle.c, -fopenmp) -> liboracle_omp.so."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-o", tmp, _SRC])
         os.replace(tmp, _LIB)
+    t_omp = os.path.getmtime(_LIB_OMP) if os.path.exists(_LIB_OMP) else -1
+    if force or t_omp < max(os.path.getmtime(_SRC), os.path.getmtime(_SRC_OMP)):
+        tmp = _LIB_OMP + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fopenmp", "-fPIC", "-shared", "-o", tmp, _SRC_OMP, _SRC])
+        os.replace(tmp, _LIB_OMP)
     return _LIB
+
+
+def lib_omp():
+    """liboracle_omp.so: LubyMIS / LMAX / JP as synchronous rounds on all host cores."""
+    global _lib_omp
+    if _lib_omp is None:
+        build()
+        l = ctypes.CDLL(_LIB_OMP)
+        for name in ("oro_mis", "oro_mm", "oro_color"):
+            f = getattr(l, name)
+            f.restype = None
+            f.argtypes = [_I64, _P, _P, _INT, _U32, _U64, _P]
+        l.oro_threads.restype = _INT
+        l.oro_threads.argtypes = []
+        _lib_omp = l
+    return _lib_omp
+
+
+def omp_threads() -> int:
+    """Threads the OpenMP round oracle uses (OMP_NUM_THREADS, else every host core)."""
+    return int(lib_omp().oro_threads())
 
 
 _P = ctypes.c_void_p
@@ -67,6 +99,7 @@ _SIGS = {
     "or_cert_mm": (_I64, [_I64, _P, _P, _P, _INT, _P, _U64, _P]),
     "or_cert_col": (_I64, [_I64, _P, _P, _P, _P, _INT, _U64, _P]),
     "or_cert_col_rand": (_I64, [_I64, _P, _P, _U32, _U64, _P, _P]),
+    "or_cert_flow": (_I64, [_INT, _I64, _P, _P, _INT, _U32, _U64, _P]),
 }
 
 
@@ -172,6 +205,30 @@ def color(rp, ci, kind="none", param=0, seed=42):
     return out[:n]
 
 
+def omp_mis(rp, ci, kind="none", param=0, seed=42):
+    """MIS flows as synchronous LubyMIS rounds on all cores (oracle_omp.c)."""
+    n, rp, ci = _graph(rp, ci)
+    out = np.zeros(max(n, 1), np.uint8)
+    lib_omp().oro_mis(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), _ptr(out))
+    return out[:n]
+
+
+def omp_mm(rp, ci, kind="none", param=0, seed=42):
+    """MM flows as synchronous LMAX rounds on all cores (oracle_omp.c)."""
+    n, rp, ci = _graph(rp, ci)
+    out = np.zeros(max(n, 1), np.int32)
+    lib_omp().oro_mm(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), _ptr(out))
+    return out[:n]
+
+
+def omp_color(rp, ci, kind="none", param=0, seed=42):
+    """COLOR flows as JP levels on all cores (oracle_omp.c)."""
+    n, rp, ci = _graph(rp, ci)
+    out = np.zeros(max(n, 1), np.uint32)
+    lib_omp().oro_color(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), _ptr(out))
+    return out[:n]
+
+
 # ---------------------------------------------------------------- round forms
 def luby_rounds(rp, ci, seed=42, inS=None, status=None):
     n, rp, ci = _graph(rp, ci)
@@ -232,73 +289,11 @@ def cert_col_rand(rp, ci, C, p, seed):
 
 
 def cert_flow(problem, rp, ci, kind, param, seed, result):
-    """O(m) exact check that `result` equals the oracle flow's output, phase by phase
-    (used at full sizes where the sequential run or its sort is too slow).
-    Returns the number of violations (0 = identical to the oracle)."""
-    kind = _kind(kind)
+    """O(m)-time, O(n)-memory exact check that `result` equals the oracle flow's output,
+    phase by phase (oracle.c or_cert_flow; used at full sizes -- up to R-MAT scale 27
+    -- where the sequential run's sort is too slow).  Returns the number of violations
+    (0 = identical to the oracle)."""
     n, rp, ci = _graph(rp, ci)
-    cls = classes(rp, ci, kind, param, seed)
-    deg = np.diff(rp)
-    src = np.repeat(np.arange(n, dtype=np.int64), deg)
-    if problem == "mis":
-        I = _np(result, np.uint8)
-        if kind == NONE:
-            return cert_mis(rp, ci, I, seed)
-        if kind == DEGK:
-            L = (cls == 0).astype(np.uint8)
-            bad = cert_mis(rp, ci, I * L, seed, inS=L)
-            killed = np.zeros(n, bool)
-            hit = (cls[src] == 1) & (L[ci] == 1) & (I[ci] == 1)
-            killed[src[hit]] = True
-            X = ((cls == 1) & ~killed).astype(np.uint8)
-            bad += int(((cls == 1) & killed & (I == 1)).sum())
-            return bad + cert_mis(rp, ci, I * X, seed, inS=X)
-        # RAND
-        cross = cls[src] != cls[ci]
-        B = np.zeros(n, bool)
-        B[src[cross]] = True
-        H = (~B).astype(np.uint8)
-        bad = cert_mis(rp, ci, I * H, seed, inS=H)
-        killed = np.zeros(n, bool)
-        hit = B[src] & (H[ci] == 1) & (I[ci] == 1)
-        killed[src[hit]] = True
-        X = (B & ~killed).astype(np.uint8)
-        bad += int((B & killed & (I == 1)).sum())
-        return bad + cert_mis(rp, ci, I * X, seed, inS=X)
-    if problem == "mm":
-        M = _np(result, np.int32)
-        if kind == NONE:
-            return cert_mm(rp, ci, M, seed)
-        a1, a2 = (ADMIT_SAME, ADMIT_DIFF) if kind == RAND else (ADMIT_HH, ADMIT_LX)
-        # phase-1 matching = M restricted to admitted phase-1 edges
-        M1 = M.copy()
-        has = M >= 0
-        c_self = cls
-        c_mate = np.where(has, cls[np.where(has, M, 0)], 0)
-        if kind == RAND:
-            in1 = has & (c_self == c_mate)
-        else:
-            in1 = has & (c_self == 1) & (c_mate == 1)
-        M1[~in1] = -1
-        bad = cert_mm(rp, ci, M1, seed, cls=cls, admit=a1)
-        free = (~in1).astype(np.uint8)
-        M2 = M.copy()
-        M2[in1] = -1
-        return bad + cert_mm(rp, ci, M2, seed, cls=cls, admit=a2, elig=free)
-    if problem == "color":
-        C = _np(result, np.uint32)
-        if kind == NONE:
-            return cert_col(rp, ci, C, seed)
-        if kind == DEGK:
-            H = (cls == 1)
-            CH = np.where(H, C, 0).astype(np.uint32)
-            bad = cert_col(rp, ci, CH, seed, inS=H.astype(np.uint8), cls=cls, admit=ADMIT_SAME)
-            M = int(CH.max()) if n and H.any() else 0
-            CL = np.where(~H, C.astype(np.int64) - M, 0)
-            bad += int(((~H) & ((CL < 1) | (CL > 0xFFFFFFFF))).sum())
-            CL = np.clip(CL, 0, None).astype(np.uint32)
-            return bad + cert_col(rp, ci, CL, seed, inS=(~H).astype(np.uint8), cls=cls, admit=ADMIT_SAME)
-        # RAND: C1 by a topological sweep of the intra priority DAG, V' from C1, then
-        # C = C1 off V' and the first-fit certificate on V' (oracle.c or_cert_col_rand)
-        return cert_col_rand(rp, ci, C, param, seed)[0]
-    raise ValueError(problem)
+    code, dt = {"mis": (1, np.uint8), "mm": (2, np.int32), "color": (3, np.uint32)}[problem]
+    R = _np(result, dt)
+    return int(lib().or_cert_flow(code, n, _ptr(rp), _ptr(ci), _kind(kind), int(param), seed & (2**64 - 1), _ptr(R)))

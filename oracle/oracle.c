@@ -648,3 +648,99 @@ int64_t or_cert_col_rand(int64_t n, const int64_t *rp, const int32_t *ci, uint32
     free(cls);
     return bad;
 }
+
+/* Flow certificates with O(n) extra memory (no arc-sized arrays, so they run at
+   R-MAT scale 27 on the host): the result of each problem/decomposition flow is
+   checked phase by phase against the definitions in or_mis / or_mm / or_color,
+   using the single-phase certificates above.  problem: 1 MIS (uint8 in_set), 2 MM
+   (int32 mate), 3 COLOR (uint32 colour).  Returns the number of violations. */
+int64_t or_cert_flow(int problem, int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t param,
+                     uint64_t seed, const void *result) {
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    int64_t bad = 0;
+    if (problem == 3 && kind == OR_RAND) return or_cert_col_rand(n, rp, ci, param, seed, (const uint32_t *)result, 0);
+    uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+    uint8_t *S = (uint8_t *)malloc(nn);
+    or_classes(n, rp, kind, param, seed, cls);
+    if (problem == 1) { /* MIS: M1 NONE, M2 DEGk, M3 RAND */
+        const uint8_t *I = (const uint8_t *)result;
+        if (kind == OR_NONE) {
+            memset(S, 1, nn);
+            bad = or_cert_mis(n, rp, ci, S, seed, I);
+        } else {
+            /* first set: V_L (DEGk) / interior vertices V \ B (RAND) */
+            for (int64_t v = 0; v < n; v++) {
+                if (kind == OR_DEGK) {
+                    S[v] = cls[v] == 0;
+                } else {
+                    S[v] = 1;
+                    for (int64_t e = rp[v]; e < rp[v + 1]; e++)
+                        if (cls[ci[e]] != cls[v]) { S[v] = 0; break; }
+                }
+            }
+            bad = or_cert_mis(n, rp, ci, S, seed, I);
+            /* the rest: removed if a first-set neighbour is In, else the second phase */
+            uint8_t *X = (uint8_t *)malloc(nn);
+            for (int64_t v = 0; v < n; v++) {
+                X[v] = 0;
+                if (S[v]) continue;
+                int killed = 0;
+                for (int64_t e = rp[v]; e < rp[v + 1] && !killed; e++) killed = S[ci[e]] && I[ci[e]];
+                if (killed) bad += I[v] != 0;
+                else X[v] = 1;
+            }
+            bad += or_cert_mis(n, rp, ci, X, seed, I);
+            free(X);
+        }
+    } else if (problem == 2) { /* MM: MM1 NONE, MM2 RAND (Alg 5), MM3 DEGk (Alg 6) */
+        const int32_t *M = (const int32_t *)result;
+        if (kind == OR_NONE) {
+            memset(S, 1, nn);
+            bad = or_cert_mm(n, rp, ci, cls, 0, S, seed, M);
+        } else {
+            int a1 = kind == OR_RAND ? 1 : 3, a2 = kind == OR_RAND ? 2 : 4;
+            int32_t *M1 = (int32_t *)malloc(sizeof(int32_t) * nn), *M2 = (int32_t *)malloc(sizeof(int32_t) * nn);
+            for (int64_t v = 0; v < n; v++) {
+                int32_t w = M[v];
+                int in1 = w >= 0 && w < n && admitted(a1, cls[v], cls[w]);
+                M1[v] = in1 ? w : -1;
+                M2[v] = in1 ? -1 : w;
+                S[v] = !in1; /* free after phase 1 */
+            }
+            uint8_t *all = (uint8_t *)malloc(nn);
+            memset(all, 1, nn);
+            bad = or_cert_mm(n, rp, ci, cls, a1, all, seed, M1);
+            bad += or_cert_mm(n, rp, ci, cls, a2, S, seed, M2);
+            free(all);
+            free(M1);
+            free(M2);
+        }
+    } else { /* COLOR: C1 NONE, C2 DEGk (Alg 9) */
+        const uint32_t *C = (const uint32_t *)result;
+        if (kind == OR_NONE) {
+            memset(S, 1, nn);
+            bad = or_cert_col(n, rp, ci, S, cls, 0, seed, C);
+        } else {
+            uint32_t M = 0;
+            for (int64_t v = 0; v < n; v++) {
+                S[v] = cls[v] == 1;
+                if (S[v] && C[v] > M) M = C[v];
+            }
+            bad = or_cert_col(n, rp, ci, S, cls, 1, seed, C); /* C_H on G_H */
+            uint32_t *CL = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+            for (int64_t v = 0; v < n; v++) {
+                S[v] = cls[v] == 0;
+                CL[v] = 0;
+                if (S[v]) {
+                    if (C[v] <= M) bad++; /* L colours start above max C_H */
+                    else CL[v] = C[v] - M;
+                }
+            }
+            bad += or_cert_col(n, rp, ci, S, cls, 1, seed, CL); /* C_L on G_L */
+            free(CL);
+        }
+    }
+    free(S);
+    free(cls);
+    return bad;
+}

@@ -192,7 +192,8 @@ def sym_profile_enable(on: bool = True) -> None:
 
 
 def sym_profile_collect() -> dict:
-    """{class: {"launches", "ms", "alg_bytes"}} accumulated since the last collect."""
+    """{class: {"launches", "ms", "alg_bytes", "impl_bytes"}} accumulated since the last collect
+    (alg = SURVEY §8(d) algorithmic bytes, impl = the implementation's own words)."""
     lib = L.load()
     buf = (L.SymKernelProfile * 64)()
     cnt = ctypes.c_int(0)
@@ -200,7 +201,8 @@ def sym_profile_collect() -> dict:
     if rc != L.SYM_OK:
         raise SymError(rc, "sym_profile_collect")
     return {buf[i].name.decode(): {"launches": int(buf[i].launches), "ms": float(buf[i].ms),
-                                   "alg_bytes": float(buf[i].alg_bytes)} for i in range(min(cnt.value, 64))}
+                                   "alg_bytes": float(buf[i].alg_bytes), "impl_bytes": float(buf[i].impl_bytes)}
+            for i in range(min(cnt.value, 64))}
 
 
 def sym_validate(row_ptr, col_idx) -> int:

@@ -35,7 +35,7 @@ class SymGraphShard(ctypes.Structure):
 
 class SymKernelProfile(ctypes.Structure):
     _fields_ = [("name", ctypes.c_char * 24), ("launches", ctypes.c_int64), ("ms", ctypes.c_double),
-                ("alg_bytes", ctypes.c_double)]
+                ("alg_bytes", ctypes.c_double), ("impl_bytes", ctypes.c_double)]
 
 
 class SymGraph(ctypes.Structure):

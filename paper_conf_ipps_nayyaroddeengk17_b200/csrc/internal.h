@@ -115,19 +115,31 @@ int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const Spl
               int64_t row_base = 0);
 
 // ------------------------------------------------------------------ profiling hook (profile.cu)
+// Every hot launch may record a CUDA event pair on its stream plus two byte counts:
+// alg  = SURVEY §8(d)'s algorithmic bytes (what the method must move: rounds 4 B per
+//        scanned arc + 9 B per active vertex; split 8 B/arc + 24 B/row pointer; JP
+//        8 B/arc + 12 B/vertex), and
+// impl = what this implementation's kernel moves (its own HBM/L2 words: lists,
+//        records, counters).
 bool prof_on();
 void prof_begin(const char *cls, cudaStream_t s);
-void prof_end(cudaStream_t s, double alg_bytes);  // alg_bytes < 0: unknown on the host
-// a zeroed device counter (nullptr unless profiling) that a kernel accumulates its
-// algorithmic bytes into; prof_end_dev closes the event pair and reads it at collect
+void prof_end(cudaStream_t s, double alg_bytes, double impl_bytes);  // < 0: unknown on the host
+// a zeroed device counter pair {alg, impl} (nullptr unless profiling) that kernels
+// accumulate into; prof_end_dev closes the event pair and reads it at collect
 unsigned long long *prof_counter(cudaStream_t s);
 void prof_end_dev(cudaStream_t s, unsigned long long *ctr);
 
-// warp-aggregated add of per-lane byte counts into a profiling counter (nullable)
-__device__ __forceinline__ void prof_add(unsigned long long *ctr, unsigned long long lane_bytes) {
+// warp-aggregated add of per-lane byte counts into a profiling counter pair (nullable)
+__device__ __forceinline__ void prof_add(unsigned long long *ctr, unsigned long long alg, unsigned long long impl) {
     if (ctr == nullptr) return;
-    for (int d = 16; d; d >>= 1) lane_bytes += __shfl_xor_sync(0xffffffffu, lane_bytes, d);
-    if ((threadIdx.x & 31) == 0 && lane_bytes) atomicAdd(ctr, lane_bytes);
+    for (int d = 16; d; d >>= 1) {
+        alg += __shfl_xor_sync(0xffffffffu, alg, d);
+        impl += __shfl_xor_sync(0xffffffffu, impl, d);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        if (alg) atomicAdd(ctr, alg);
+        if (impl) atomicAdd(ctr + 1, impl);
+    }
 }
 
 // ------------------------------------------------------------------ helpers (api.cu)

@@ -121,7 +121,8 @@ struct JpArgs {
     uint32_t *err;       // 1 = timeout / max rounds, 2 = offsets overflow
     uint32_t *hist;
     uint32_t *trace;     // nullable: per-round diagnostics (SYM_JP_TRACE)
-    unsigned long long *prof;  // algorithmic bytes of the rounds pass (nullable)
+    unsigned long long *prof;  // profiling counter pair {alg, impl} of the current launch (nullable)
+    unsigned long long *prof_jp;  // the rounds launch's pair: the count pass adds §8(d)'s JP bytes
     Key k;
 };
 
@@ -355,7 +356,10 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_count(JpArgs A) {
         }
         // algorithmic bytes: the row's columns (huge rows: k_jpc_count_huge), row pair,
         // id map entry, the two counts
-        prof_add(A.prof, active ? (huge ? 0ull : 4ull * (uint64_t)(e - b)) + 28ull : 0ull);
+        prof_add(A.prof, 0ull, active ? (huge ? 0ull : 4ull * (uint64_t)(e - b)) + 28ull : 0ull);
+        // §8(d) JP (push form): 8 B per phase arc + 12 B per vertex, charged to the rounds
+        // (huge rows: their pieces add the arcs in k_jpc_count_huge)
+        prof_add(A.prof_jp, active ? 8ull * (uint64_t)(hi + lo) + 12ull : 0ull, 0ull);
         const uint32_t np = huge ? (uint32_t)((e - b + JP_PIECE - 1) / JP_PIECE) : 0u;
         const int64_t ps = warp_reserve(np, A.huge_cnt);
         for (uint32_t q = 0; q < np; q++) A.huge[ps + q] = ((int64_t)q << 32) | (uint32_t)h;
@@ -388,7 +392,8 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_count_huge(JpArgs A) {
             if (lh) atomicAdd(A.hdeg + h, lh);
             if (ll) atomicAdd(A.ldeg + h, ll);
         }
-        prof_add(A.prof, threadIdx.x == 0 ? 4ull * (uint64_t)(pe_ - pb) : 0ull);
+        prof_add(A.prof, 0ull, threadIdx.x == 0 ? 4ull * (uint64_t)(pe_ - pb) : 0ull);
+        prof_add(A.prof_jp, 8ull * (uint64_t)(lh + ll), 0ull);
     }
 }
 
@@ -520,7 +525,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
             A.ldeg[h] = 0;
         }
         // algorithmic bytes: counts read, meta + hot record + zeroed extra words written
-        prof_add(A.prof, active ? 8ull + 48ull + 4ull * (R - 1u) : 0ull);
+        prof_add(A.prof, 0ull, active ? 8ull + 48ull + 4ull * (R - 1u) : 0ull);
         o0 += t0;
         o1 += t1;
     }
@@ -631,7 +636,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
         }
         // algorithmic bytes: the row's columns read + list ids written (huge rows:
         // k_jpc_fill_huge), row pair, id map, meta + hot record read
-        prof_add(A.prof, active ? (e - b > JP_BUDGET ? 0ull : 8ull * (uint64_t)(e - b)) + 68ull : 0ull);
+        prof_add(A.prof, 0ull, active ? (e - b > JP_BUDGET ? 0ull : 8ull * (uint64_t)(e - b)) + 68ull : 0ull);
     }
 }
 
@@ -698,7 +703,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
                 pd += __popc(md);
             }
         }
-        prof_add(A.prof, lane == 0 && se > sb0 ? 8ull * (uint64_t)(se - sb0) : 0ull);
+        prof_add(A.prof, 0ull, lane == 0 && se > sb0 ? 8ull * (uint64_t)(se - sb0) : 0ull);
     }
 }
 
@@ -1136,7 +1141,7 @@ __global__ void __launch_bounds__(JR_THREADS, SYM_JR_MINB) k_jp_rounds(JpArgs A,
         grid_sync(C, k, A.ucnt + (r + 1) % 3, nullptr, nullptr, s_val);
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *C.levels = r;
-    prof_add(A.prof, bytes);
+    prof_add(A.prof, 0ull, bytes);
 }
 
 // ---------------------------------------------------------------- fix-up kernels
@@ -1223,7 +1228,7 @@ void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
 // rounds, [40..41] compact counts.
 static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, const int64_t *rp,
                     const int32_t *ci, const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0,
-                    int64_t implicit_n) {
+                    int64_t implicit_n, unsigned long long *rounds_ctr) {
     Ctl *ctl = f.ctl;
     cudaStream_t s = f.stream;
     const int64_t n = f.g.n;
@@ -1260,6 +1265,7 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     A.hist = nullptr;
     A.trace = nullptr;
     A.prof = nullptr;
+    A.prof_jp = rounds_ctr;
     A.k = stream_key(f.p.seed, TAG_VERTEX, 0);
     const int64_t nwords = (n + 31) / 32;
     const unsigned tiles_w = (unsigned)((nwords + JP_TILE - 1) / JP_TILE);
@@ -1319,6 +1325,7 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     SYM_LAUNCH_CHECK();
     prof_end_dev(s, ctr);
     A.prof = nullptr;
+    A.prof_jp = nullptr;
     return SYM_OK;
 }
 
@@ -1345,7 +1352,8 @@ static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t 
         return SYM_ECUDA;
     }
     JpArgs A;
-    SYM_TRY(jp_build(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n));
+    unsigned long long *rounds_ctr = prof_counter(s);  // profiling: the rounds launch's byte pair
+    SYM_TRY(jp_build(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n, rounds_ctr));
     JrCtl C;
     C.arr = w.sync;
     C.gen = w.sync + 1;
@@ -1357,7 +1365,7 @@ static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t 
     static const bool jp_trace = getenv("SYM_JP_TRACE") != nullptr;
     A.trace = jp_trace && f.stats && phase == 0 ? ctl->hist + 2048 : nullptr;
     if (A.trace) SYM_CUDA(cudaMemsetAsync(A.trace, 0, 2048 * sizeof(uint32_t), s));
-    A.prof = prof_counter(s);
+    A.prof = rounds_ctr;
     void *args[] = {&A, &C};
     prof_begin("jp_rounds", s);
     SYM_CUDA(cudaLaunchCooperativeKernel((const void *)k_jp_rounds, dim3(grid), dim3(JR_THREADS), args, 0, s));

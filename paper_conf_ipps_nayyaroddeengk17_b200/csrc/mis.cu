@@ -58,9 +58,10 @@ __device__ __forceinline__ bool mis_in_phase(const MisRoundArgs &A, uint32_t w) 
     return A.ncls < 0 || (int)((A.nfilter[w >> 5] >> (w & 31)) & 1u) == A.ncls;
 }
 
-// algorithmic bytes: 4 B per column word the kernel loads, 16 B for the
-// row_ptr pair + 1 B status per active vertex, 1 B per decided status write;
-// neighbour-status gathers hit the L2-resident status array and count 0 HBM bytes.
+// bytes: §8(d) algorithmic = 4 B per column word the kernel loads + 9 B
+// per active vertex (row_ptr pair + status); the implementation's own count adds the
+// list entry and status read (5 B more per active vertex) and 1 B per decided status
+// write.  Neighbour-status gathers hit the L2-resident status array: 0 HBM bytes.
 // A short row (<= MIS_SMALL arcs, one sector) is decided by one lane: all column
 // loads, then all status gathers, then the rule (the order of the arcs does not
 // matter: any In neighbour -> Out, else any higher undecided neighbour -> blocked).
@@ -107,7 +108,7 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
         }
         int res = R_NONE;
         int64_t resume = 0;
-        unsigned long long lb = active ? 17 : 0;
+        unsigned long long lb = 0;  // column words loaded (4 B each)
         if (active && e - b <= MIS_SMALL) res = mis_scan_small(A, b, e, kv, lb);
         unsigned longm = __ballot_sync(FULL, active && e - b > MIS_SMALL);
         while (longm) {
@@ -147,7 +148,9 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
         }
         if (res == R_IN) A.st[v] = ST_IN;
         else if (res == R_OUT) A.st[v] = ST_OUT;
-        prof_add(A.prof, lb + ((res == R_IN || res == R_OUT) ? 1 : 0));
+        // §8(d): 4 B per scanned arc + 9 B per active vertex; the implementation also
+        // reads the list entry and the status (5 B) and writes decided statuses
+        prof_add(A.prof, lb + (active ? 9 : 0), lb + (active ? 17 : 0) + ((res == R_IN || res == R_OUT) ? 1 : 0));
         int64_t slot = warp_append(res == R_BLK, A.out_cnt);
         if (slot >= 0) A.out_list[slot] = v;
         int64_t hs = warp_append(res == R_DEFER, A.huge_cnt);
@@ -166,7 +169,7 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
         const int64_t b = A.huge[2 * h + 1], e = A.rp[v - A.row_base + 1];
         const uint64_t kv = vkey(A.k, (uint32_t)v);
         int r = R_IN;
-        unsigned long long lb = threadIdx.x == 0 ? 9 : 0;  // row end + status write
+        unsigned long long lb = 0;  // column words (the vertex was counted active by k_mis_round)
         for (int64_t x = b; x < e; x += 4 * MIS_HUGE_THREADS) {
             bool fin = false, fblk = false;
             uint32_t w[4];
@@ -197,7 +200,7 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
                 A.out_list[slot] = v;
             }
         }
-        prof_add(A.prof, lb);
+        prof_add(A.prof, lb, lb + (threadIdx.x == 0 ? 9 : 0));  // impl: + row end + status write
         __syncthreads();
     }
 }

@@ -91,7 +91,8 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
         int32_t u = -1;
         if (i < cnt) u = A.in_list ? (A.in_rev ? A.in_list[-1 - i] : A.in_list[i]) : (int32_t)i;
         bool active = u >= 0;
-        unsigned long long nb = 0;  // algorithmic bytes of this lane
+        const bool listed = active;
+        unsigned long long nb = 0, colb = 0;  // implementation bytes beyond the column words; column words
         int32_t p = -1;
         bool reuse = false;
         if (RESOLVE && active) {
@@ -127,7 +128,7 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
         if (scan && d <= MM_SMALL) {
             // short row by one lane: all column loads (streamed, evict-first so the
             // gathered mate array stays in L2), then all mate gathers, then the argmax
-            nb += 4 * (unsigned long long)d;
+            colb += 4 * (unsigned long long)d;
             uint32_t w[MM_SMALL];
             bool live[MM_SMALL];
 #pragma unroll
@@ -161,7 +162,7 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
                     int64_t y = x + q * 32 + lane;
                     ok[q] = y < we;
                     w[q] = ok[q] ? (uint32_t)__ldcs(wci + y) : 0u;
-                    nb += ok[q] ? 4 : 0;
+                    colb += ok[q] ? 4 : 0;
                 }
 #pragma unroll
                 for (int q = 0; q < 4; q++) {
@@ -190,7 +191,8 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
         if (slot >= 0) A.out_list[slot] = u;
         int64_t hs = warp_append(defer, A.huge_cnt);
         if (hs >= 0) A.huge[hs] = u;
-        prof_add(A.prof, nb);
+        // §8(d): 4 B per scanned arc + 9 B per active vertex (row_ptr pair, pick)
+        prof_add(A.prof, colb + (listed ? 9 : 0), colb + nb);
     }
 }
 
@@ -234,7 +236,7 @@ __global__ void __launch_bounds__(MM_HUGE_THREADS) k_mm_huge(MmRoundArgs A) {
             lb = o > lb ? o : lb;
         }
         bool wh = __any_sync(FULL, lh);
-        prof_add(A.prof, nb);
+        prof_add(A.prof, nb, nb);
         if (lane == 0) {
             s_best[warp] = lb;
             s_has[warp] = wh;

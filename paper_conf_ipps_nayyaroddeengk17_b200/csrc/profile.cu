@@ -15,8 +15,8 @@ namespace {
 struct Rec {
     std::string cls;
     cudaEvent_t a, b;
-    double bytes;
-    int slot;  // device byte counter slot, or -1
+    double alg, impl;
+    int slot;  // device byte counter pair slot, or -1
 };
 std::atomic<bool> g_on{false};
 // device byte counters for launches whose algorithmic bytes depend on the frontier
@@ -55,39 +55,39 @@ void prof_begin(const char *cls, cudaStream_t s) {
 }
 
 // closes the innermost pending begin of stream s
-static void close_rec(cudaStream_t s, double bytes, int slot) {
+static void close_rec(cudaStream_t s, double alg, double impl, int slot) {
     auto it = g_open.find(s);
     if (it == g_open.end() || it->second.empty()) return;
     cudaEvent_t e = get_event();
     cudaEventRecord(e, s);
-    Rec r{it->second.back().first, it->second.back().second, e, bytes, slot};
+    Rec r{it->second.back().first, it->second.back().second, e, alg, impl, slot};
     it->second.pop_back();
     g_recs.push_back(r);
 }
 
-void prof_end(cudaStream_t s, double bytes) {
+void prof_end(cudaStream_t s, double alg, double impl) {
     if (!g_on) return;
     std::lock_guard<std::mutex> lk(g_mu);
-    close_rec(s, bytes, -1);
+    close_rec(s, alg, impl, -1);
 }
 
 unsigned long long *prof_counter(cudaStream_t s) {
     if (!g_on) return nullptr;
     std::lock_guard<std::mutex> lk(g_mu);
-    if (!g_dev && cudaMalloc(&g_dev, sizeof(unsigned long long) * DEV_SLOTS) != cudaSuccess) {
+    if (!g_dev && cudaMalloc(&g_dev, 2 * sizeof(unsigned long long) * DEV_SLOTS) != cudaSuccess) {
         g_dev = nullptr;
         return nullptr;
     }
     if (g_dev_next >= DEV_SLOTS) return nullptr;
-    unsigned long long *p = g_dev + g_dev_next++;
-    cudaMemsetAsync(p, 0, sizeof(unsigned long long), s);
+    unsigned long long *p = g_dev + 2 * g_dev_next++;
+    cudaMemsetAsync(p, 0, 2 * sizeof(unsigned long long), s);
     return p;
 }
 
 void prof_end_dev(cudaStream_t s, unsigned long long *ctr) {
     if (!g_on) return;
     std::lock_guard<std::mutex> lk(g_mu);
-    close_rec(s, ctr ? 0.0 : -1.0, ctr ? (int)(ctr - g_dev) : -1);
+    close_rec(s, ctr ? 0.0 : -1.0, ctr ? 0.0 : -1.0, ctr ? (int)((ctr - g_dev) / 2) : -1);
 }
 
 }  // namespace sym
@@ -103,19 +103,19 @@ extern "C" int sym_profile_enable(int on) {
 extern "C" int sym_profile_collect(sym_kernel_profile *out, int max_entries, int *count) {
     struct Acc {
         int64_t n = 0;
-        double ms = 0, bytes = 0;
-        bool known = true;
+        double ms = 0, alg = 0, impl = 0;
+        bool alg_known = true, impl_known = true;
     };
     std::lock_guard<std::mutex> lk(g_mu);
     std::map<std::string, Acc> acc;
     std::vector<std::string> order;
-    std::vector<unsigned long long> dev(g_dev_next);
+    std::vector<unsigned long long> dev(2 * (size_t)g_dev_next);
     if (!g_recs.empty()) {
         cudaError_t e = cudaEventSynchronize(g_recs.back().b);
         if (e != cudaSuccess) return cuda_fail(e, "cudaEventSynchronize", __FILE__, __LINE__);
     }
     if (g_dev_next > 0) {
-        cudaError_t e = cudaMemcpy(dev.data(), g_dev, sizeof(unsigned long long) * g_dev_next, cudaMemcpyDeviceToHost);
+        cudaError_t e = cudaMemcpy(dev.data(), g_dev, 2 * sizeof(unsigned long long) * g_dev_next, cudaMemcpyDeviceToHost);
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy(profile counters)", __FILE__, __LINE__);
     }
     for (auto &r : g_recs) {
@@ -127,9 +127,12 @@ extern "C" int sym_profile_collect(sym_kernel_profile *out, int max_entries, int
         Acc &x = acc[r.cls];
         x.n++;
         x.ms += ms;
-        double bytes = r.slot >= 0 ? (double)dev[r.slot] : r.bytes;
-        if (bytes < 0) x.known = false;
-        else x.bytes += bytes;
+        const double alg = r.slot >= 0 ? (double)dev[2 * r.slot] : r.alg;
+        const double impl = r.slot >= 0 ? (double)dev[2 * r.slot + 1] : r.impl;
+        if (alg < 0) x.alg_known = false;
+        else x.alg += alg;
+        if (impl < 0) x.impl_known = false;
+        else x.impl += impl;
         g_pool.push_back(r.a);
         g_pool.push_back(r.b);
     }
@@ -143,7 +146,8 @@ extern "C" int sym_profile_collect(sym_kernel_profile *out, int max_entries, int
             strncpy(out[c].name, name.c_str(), sizeof(out[c].name) - 1);
             out[c].launches = x.n;
             out[c].ms = x.ms;
-            out[c].alg_bytes = x.known ? x.bytes : -1.0;
+            out[c].alg_bytes = x.alg_known ? x.alg : -1.0;
+            out[c].impl_bytes = x.impl_known ? x.impl : -1.0;
         }
         c++;
     }

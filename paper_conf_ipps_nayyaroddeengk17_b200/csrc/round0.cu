@@ -293,8 +293,11 @@ int run_round0(int mode, const Graph &g, const int64_t *first_row, int64_t ntile
     prof_begin(mode == R0_MIS ? "mis_round0" : "mm_round0", s);
     if (mode == R0_MIS) k_round0<R0_MIS><<<grid, SPLIT_THREADS, R0_SMEM, s>>>(A);
     else k_round0<R0_MM><<<grid, SPLIT_THREADS, R0_SMEM, s>>>(A);
-    // algorithmic bytes: 4 B/arc + 16 B/row read, plus the decision writes
-    prof_end(s, 4.0 * (double)g.nnz + 16.0 * (double)g.n + (mode == R0_MIS ? 1.0 : 8.0) * (double)g.n);
+    // §8(d): 4 B/arc + 9 B/vertex (every row is active in round 0); the kernel reads
+    // 4 B/arc + 16 B/row (row pointers) and writes the decision (1 B status / 4 B pick +
+    // 4 B frontier entry)
+    prof_end(s, 4.0 * (double)g.nnz + 9.0 * (double)g.n,
+             4.0 * (double)g.nnz + 16.0 * (double)g.n + (mode == R0_MIS ? 1.0 : 8.0) * (double)g.n);
     SYM_LAUNCH_CHECK();
     if (ntiles > 1) {
         if (mode == R0_MIS) k_r0_span_emit<R0_MIS><<<(unsigned)((ntiles + 255) / 256), 256, 0, s>>>(A);

@@ -362,7 +362,7 @@ int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const Spl
     SYM_LAUNCH_CHECK();
     bool vec = ((uintptr_t)g.ci & 15) == 0;
     dim3 grid((unsigned)w.ntiles);
-    prof_begin("split", s);
+    prof_begin(kind == SYM_DECOMP_DEGK ? "split_degk" : (kind == SYM_DECOMP_RAND ? "split_rand" : "split_none"), s);
 #define SPLIT_ARGS                                                                                          \
     g.rp, g.ci, g.n, g.nnz, w.first_row, w.ntiles, w.hbits, kr, param, w.tile_state, rp_in, \
         ci_in, rp_x, ci_x, row_base
@@ -379,7 +379,8 @@ int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const Spl
 #undef SPLIT_ARGS
     // algorithmic bytes: read + write every arc (8 B), read row_ptr, write both row
     // pointer arrays (24 B per row pointer)
-    prof_end(s, 8.0 * (double)g.nnz + 24.0 * (double)(g.n + 1));
+    // 8 B/arc (column read + written) + 24 B/row pointer (read + two written)
+    prof_end(s, 8.0 * (double)g.nnz + 24.0 * (double)(g.n + 1), 8.0 * (double)g.nnz + 24.0 * (double)(g.n + 1));
     SYM_LAUNCH_CHECK();
     return SYM_OK;
 }

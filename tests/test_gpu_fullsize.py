@@ -8,7 +8,10 @@
   certificate, which holds iff the matching equals LF-MM phase by phase
   (oracle/oracle.c §CRT; exact, not a sample).
 * C2  road-like grid 2048^2 (keep 0.6), MM-Rand p=64: every mate vs the oracle.
-* C1  R-MAT scale 14, MIS-Rand p=4 is in test_gpu_parity.py.
+* the DEG2 and RAND-4 decompositions at scale 24: all four CSR arrays, every element.
+* MM-NONE and COLOR-NONE (the undecomposed baselines) at scale 24: O(m) certificates.
+* C1  R-MAT scale 14, MIS-Rand p=4 is in test_gpu_parity.py; C5 (scale 27) in
+  test_gpu_scale27.py.
 Graphs are generated on the GPU (graphgen, bit-identical to the CPU generator,
 checked in test_gpu_parity.py) and copied to the host for the oracle.
 """
@@ -54,6 +57,18 @@ def test_c4_color_deg2_and_rand_scale24(rmat24):
         d = sb.sym_decompose(rp, ci, kind, p, SEED)
         C = sb.sym_color(rp, ci, kind, p, SEED, decomp=d)
         assert _mismatch(C, O.color(hrp, hci, kind, p, SEED)) == 0, kind
+        # and the O(m) certificate agrees (it is what the scale-27 test relies on)
+        assert O.cert_flow("color", hrp, hci, kind, p, SEED, C.cpu().numpy()) == 0, kind
+
+
+def test_c4_mm_none_and_color_none_scale24(rmat24):
+    """The undecomposed baselines the bench reports beside C3/C4 (MM-NONE = LMAX,
+    COLOR-NONE = JP): exact O(m) certificates."""
+    (rp, ci), (hrp, hci) = rmat24
+    M = sb.sym_mm(rp, ci, "none", 0, SEED).cpu().numpy()
+    assert O.cert_flow("mm", hrp, hci, "none", 0, SEED, M) == 0
+    C = sb.sym_color(rp, ci, "none", 0, SEED).cpu().numpy()
+    assert O.cert_flow("color", hrp, hci, "none", 0, SEED, C) == 0
 
 
 def test_mm_rand4_scale24_certificate(rmat24):
@@ -71,23 +86,17 @@ def test_c2_road_grid_mm_rand64():
     assert _mismatch(M, ref) == 0
 
 
-def test_decomposition_scale24_sampled_rows(rmat24):
-    """sym_decompose at full size vs the oracle's split of sampled rows (plus the
-    global totals)."""
+def test_decomposition_scale24_full(rmat24):
+    """sym_decompose at full size vs the oracle's split (Alg 2 / Alg 3):
+    all four arrays (row_ptr_in, col_in, row_ptr_x, col_x) compared element by
+    element -- 2 x 520.8 M column entries and 2 x 16.8 M row offsets."""
     (rp, ci), (hrp, hci) = rmat24
     for kind, p in (("degk", 2), ("rand", 4)):
         d = sb.sym_decompose(rp, ci, kind, p, SEED)
-        cls = O.classes(hrp, hci, kind, p, SEED)
-        rin, cin = d.row_ptr_in.cpu().numpy(), d.col_in.cpu().numpy()
-        rx, cx = d.row_ptr_x.cpu().numpy(), d.col_x.cpu().numpy()
-        src = np.repeat(np.arange(hrp.size - 1), np.diff(hrp))
-        n_intra = int((cls[src] == cls[hci]).sum())
-        assert d.nnz_in == n_intra and d.nnz_x == hci.size - n_intra
-        rng = np.random.default_rng(0)
-        deg = np.diff(hrp)
-        rows = np.concatenate([rng.integers(0, hrp.size - 1, 20000), np.argsort(-deg)[:50]])
-        for v in rows:
-            row = hci[hrp[v]:hrp[v + 1]]
-            same = cls[row] == cls[v]
-            assert np.array_equal(cin[rin[v]:rin[v + 1]], row[same])
-            assert np.array_equal(cx[rx[v]:rx[v + 1]], row[~same])
+        rin, cin, rx, cx = O.decompose(hrp, hci, kind, p, SEED)
+        assert d.nnz_in == cin.size and d.nnz_x == cx.size
+        assert np.array_equal(d.row_ptr_in.cpu().numpy(), rin), kind
+        assert np.array_equal(d.row_ptr_x.cpu().numpy(), rx), kind
+        assert np.array_equal(d.col_in[: d.nnz_in].cpu().numpy(), cin), kind
+        assert np.array_equal(d.col_x[: d.nnz_x].cpu().numpy(), cx), kind
+        del d

@@ -190,6 +190,16 @@ def test_closed_forms(seed):
     assert (O.mm(rp, ci, "none", 0, seed) == -1).all()
 
 
+@pytest.mark.parametrize("seed", SEEDS)
+@pytest.mark.parametrize("kind,p", [("none", 0), ("degk", 2), ("rand", 4), ("rand", 64)])
+def test_flow_certificates_accept_oracle_outputs(rmat14, road, kind, p, seed):
+    """or_cert_flow (O(n) memory, used up to scale 27) returns 0 on the oracle's own
+    output of every flow, on R-MAT and on the road grid."""
+    for rp, ci in (rmat14, road):
+        for prob, fn in (("mis", O.mis), ("mm", O.mm), ("color", O.color)):
+            assert O.cert_flow(prob, rp, ci, kind, p, seed, fn(rp, ci, kind, p, seed)) == 0, prob
+
+
 @pytest.mark.parametrize("kind,p", [("none", 0), ("degk", 2), ("rand", 4)])
 def test_certificates_accept_oracle_and_reject_perturbations(rmat14, kind, p):
     rp, ci = rmat14
