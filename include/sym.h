@@ -54,7 +54,7 @@ enum {
     SYM_EWORKSPACE = 2, /* ws_bytes smaller than sym_workspace_bytes() */
     SYM_EGRAPH = 3,     /* sym_validate / SYM_F_VALIDATE found an invalid graph */
     SYM_ECUDA = 4,      /* a CUDA runtime call or kernel launch failed */
-    SYM_ENCCL = 5,      /* reserved for the sharded path */
+    SYM_ENCCL = 5,      /* an NCCL call of the sharded path failed */
     SYM_EROUNDS = 6     /* params->max_rounds reached before the phase converged */
 };
 
@@ -195,120 +195,65 @@ const char *sym_last_error(void);
 /* Library version string ("symbreak-b200 <semver> sm_100a"). */
 const char *sym_version(void);
 
-/* ---- sharded MIS (multi-GPU; one process per GPU) ----
-   A rank owns the contiguous vertex range [v_begin, v_end) (v_begin a multiple of
-   32) and holds those rows as a local CSR with GLOBAL column ids:
+/* ---- multi-GPU: sharded MIS / MM / COLOR ----
+   One process (or host thread) per rank, each with a communicator.  A rank owns the
+   vertex block [v_begin, v_end) = [rank*B, min(n, (rank+1)*B)), B = ceil(n/N) rounded
+   up to a multiple of 32 (SYM_EINVAL otherwise), and passes those rows as a local CSR
+   with GLOBAL column ids:
      row_ptr int64[v_end - v_begin + 1] (row_ptr[0] = 0, local arc offsets),
      col_idx int32[nnz] (global ids).
-   Every rank keeps a full replica of the MIS status array, uint8[n_global] (0 =
-   undecided, 1 = In, 2 = Out), zero-initialised by the caller.  The exchange is the
-   caller's (bindings: torch.distributed all_gather over NCCL/NVLink): after each round
-   and after the fix-up, the owned segments of the status replicas are all-gathered
-   and the next-frontier counts all-reduced; the phase ends when the global count is
-   0.  Priorities are the single-GPU ones, so the result equals sym_mis() bit for bit
-   (FIXED mode is schedule-independent).  MIS-Deg2: phase L =
-   rounds on V_L with cls = 0, sym_shard_mis_kill, phase R = rounds on V_H with
-   cls = 1.  MIS-NONE: rounds with cls = -1.  All pointers are device pointers. */
+   Each call runs the whole flow -- decomposition of the owned rows, every round and
+   every fix-up -- inside the library; the only data exchanged are, after each round,
+   the state changes of the rank's BOUNDARY vertices (owned vertices with a neighbour
+   owned elsewhere): one 8-B all-gather of {delta count, next-frontier count} and one
+   all-gather of the delta lists padded to the largest count (4 B per MIS status change,
+   8 B per MM pick/match or colour), applied by a scatter kernel.  The result for the
+   owned rows equals the single-GPU call (sym_mis / sym_mm / sym_color with the same
+   params) bit for bit.  Supported: MIS NONE / DEGK / RAND, MM NONE / RAND, COLOR NONE /
+   DEGK / RAND (COLOR runs plain Jones-Plassmann rounds).  n_global < 2^30.
+   Calls synchronise the stream once per round (the host reads the gathered counts). */
 typedef struct {
     int64_t n_global, v_begin, v_end, nnz;
     const int64_t *row_ptr;
     const int32_t *col_idx;
 } sym_graph_shard;
 
-/* workspace for sym_shard_mis_round (host only; 0 on invalid arguments) */
-size_t sym_shard_workspace_bytes(const sym_graph_shard *g);
-/* DEGk class bits (deg > k, Alg 3) of the owned rows into hbits (uint32
-   words, n_global bits; words v_begin/32 .. written, the rest untouched) */
-int sym_shard_classify(const sym_graph_shard *g, uint32_t k, uint32_t *hbits, sym_stream_t stream);
-/* owned undecided vertices of class cls (-1: any) -> list (int32), *count (device u32) */
-int sym_shard_frontier(const sym_graph_shard *g, const uint32_t *hbits, int cls, const uint8_t *status,
-                       int32_t *list, uint32_t *count, sym_stream_t stream);
-/* one Luby round over the owned frontier (list, *count on the device);
-   neighbours whose class differs from cls are outside the phase (cls = -1: none);
-   still-undecided vertices -> next, *next_count (device u32, set by the call) */
-int sym_shard_mis_round(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits, int cls,
-                        uint8_t *status, const int32_t *frontier, const uint32_t *count, int32_t *next,
-                        uint32_t *next_count, void *ws, size_t ws_bytes, sym_stream_t stream);
-/* MIS-Deg2 fix-up: owned undecided V_H vertices with an In V_L neighbour -> Out */
-int sym_shard_mis_kill(const sym_graph_shard *g, const uint32_t *hbits, uint8_t *status, sym_stream_t stream);
-/* in_set_owned[v - v_begin] = (status[v] == In) for the owned range */
-int sym_shard_mis_finish(const sym_graph_shard *g, const uint8_t *status, uint8_t *in_set_owned,
-                         sym_stream_t stream);
+/* communicator: NCCL (one per GPU; rank 0 makes the id with sym_comm_unique_id, the
+   caller broadcasts its 128 bytes, every rank calls sym_comm_create on its device), or
+   local (N ranks driven by N host threads of one process, any devices; ranks that pass
+   the same `group` key join the same group). */
+typedef struct sym_comm sym_comm;
+#define SYM_COMM_ID_BYTES 128
+int sym_comm_unique_id(void *id /* host, SYM_COMM_ID_BYTES */);
+int sym_comm_create(sym_comm **out, int nranks, int rank, const void *id);
+int sym_comm_create_local(sym_comm **out, int nranks, int rank, uint64_t group);
+int sym_comm_destroy(sym_comm *c);
+int sym_comm_size(const sym_comm *c, int *nranks, int *rank);
 
-/* ---- sharded MM (MM-NONE / MM-Rand, Alg 5; handshake rounds P:152-154) ----
-   Same shard layout as above (v_begin need not be 32-aligned here).  Every rank keeps
-   full replicas of mate int32[n_global] (caller-initialised to -1) and of two pick
-   buffers int32[n_global] (contents arbitrary before round 0).  Round r writes
-   pick_cur = picks[r & 1] and reads pick_prev = picks[(r + 1) & 1] (round 0 reads no
-   picks).  After each round the caller all-gathers the owned segments of pick_cur
-   and mate and all-reduces *next_count; the phase ends when the global count is 0.
-   MM-Rand: decompose the owned rows with sym_shard_decompose (labels hash the GLOBAL
-   id, so the parts equal the single-GPU ones), phase 1 = rounds on the local intra
-   CSR, phase 2 = rounds on the local cross CSR starting from the vertices still
-   unmatched.  Priorities are the single-GPU ones, so the result equals sym_mm() bit
-   for bit.  All pointers are device pointers. */
+/* per-rank statistics of a sharded call (host struct) */
+typedef struct {
+    uint32_t rounds[3];         /* rounds of each phase */
+    uint32_t exchanges;         /* exchange steps (each: 2 all-gathers) */
+    int64_t boundary;           /* owned vertices with a remote neighbour */
+    int64_t sent_bytes;         /* delta bytes this rank contributed (sum over exchanges) */
+    int64_t gathered_bytes;     /* bytes the padded delta all-gathers delivered to this rank */
+    int64_t max_exchange_bytes; /* largest single delta all-gather */
+} sym_shard_stats;
 
-/* workspace for sym_shard_decompose (host only; 0 on invalid arguments) */
-size_t sym_shard_decompose_workspace_bytes(const sym_graph_shard *g);
-/* RAND decomposition (Alg 2) of the owned rows: local intra / cross CSRs
-   row_ptr_* int64[v_end - v_begin + 1], col_idx_* int32[nnz] (capacity; global ids),
-   the intra arcs first in the same order as sym_decompose.  p->kind RAND or NONE. */
-int sym_shard_decompose(const sym_graph_shard *g, const sym_params *p, void *ws, size_t ws_bytes,
-                        int64_t *row_ptr_in, int32_t *col_idx_in, int64_t *row_ptr_x, int32_t *col_idx_x,
-                        sym_stream_t stream);
-/* workspace for sym_shard_mm_round (host only; 0 on invalid arguments) */
-size_t sym_shard_mm_workspace_bytes(const sym_graph_shard *g);
-/* owned vertices with mate < 0 and at least one arc in g -> list, *count (device u32) */
-int sym_shard_mm_frontier(const sym_graph_shard *g, const int32_t *mate, int32_t *list, uint32_t *count,
-                          sym_stream_t stream);
-/* one handshake round over the owned frontier: resolve round-(r-1) mutual picks
-   (r > 0), then pick the heaviest edge to a neighbour with mate < 0; vertices with a
-   pick -> next, *next_count (device u32, set by the call) */
-int sym_shard_mm_round(const sym_graph_shard *g, const sym_params *p, int round, int32_t *mate,
-                       const int32_t *pick_prev, int32_t *pick_cur, const int32_t *frontier, const uint32_t *count,
-                       int32_t *next, uint32_t *next_count, void *ws, size_t ws_bytes, sym_stream_t stream);
-
-/* ---- sharded COLOR (COLOR-NONE P:214, COLOR-Rand Alg 8, COLOR-Degk Alg 9
-   P:234; Jones-Plassmann rounds [18]) ----
-   Same shard layout as sharded MIS (v_begin a multiple of 32).  Every rank keeps a
-   full replica of the colour array, uint32[n_global] (0 = uncoloured), zeroed by the
-   caller.  p->kind / p->param / p->seed select the class function (NONE: one class;
-   RAND: the hash label with p parts, global id; DEGK: the all-gathered V_H bitmap
-   hbits of sym_shard_classify) and the vertex priorities (the single-GPU ones).
-   admit = 1 restricts every step to arcs whose endpoints share a class (the induced
-   subgraphs), admit = 0 uses every arc.  After each round the caller all-gathers the
-   owned colour segments and all-reduces *next_count; a phase ends at global count 0.
-     COLOR-NONE:  frontier; rounds with admit = 0.
-     COLOR-Degk:  frontier; rounds with admit = 1 (G_H and G_L at once); M = the
-                  all-reduced max of sym_shard_color_maxh; sym_shard_color_shift(M).
-     COLOR-Rand:  frontier; rounds with admit = 1; all-gather; conflicts (V', the
-                  owned endpoints of monochromatic cross arcs) -> list; clear;
-                  all-gather; rounds on that list with admit = 0.
-   The result equals sym_color() bit for bit (any schedule of the rounds gives the
-   greedy colouring in priority order).  All pointers are device pointers;
-   counts are device uint32. */
-
-/* owned vertices with color == 0 -> list, *count (set by the call) */
-int sym_shard_color_frontier(const sym_graph_shard *g, const uint32_t *color, int32_t *list, uint32_t *count,
-                             sym_stream_t stream);
-/* one JP round over the owned frontier: a vertex whose admitted higher-priority
-   neighbours are all coloured takes the smallest colour >= 1 not held by an admitted
-   neighbour; the others -> next, *next_count (set by the call) */
-int sym_shard_jp_round(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits, int admit,
-                       uint32_t *color, const int32_t *frontier, const uint32_t *count, int32_t *next,
-                       uint32_t *next_count, sym_stream_t stream);
-/* COLOR-Rand V' (Alg 8): owned v with a cross-class neighbour of the same colour -> list */
-int sym_shard_color_conflicts(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits,
-                              const uint32_t *color, int32_t *list, uint32_t *count, sym_stream_t stream);
-/* color[list[i]] = 0 for i < *count */
-int sym_shard_color_clear(const sym_graph_shard *g, uint32_t *color, const int32_t *list, const uint32_t *count,
-                          sym_stream_t stream);
-/* *max_out = max colour over owned V_H vertices (0 if none) */
-int sym_shard_color_maxh(const sym_graph_shard *g, const uint32_t *hbits, const uint32_t *color, uint32_t *max_out,
-                         sym_stream_t stream);
-/* color[v] += M for owned V_L vertices (COLOR-Degk's palette shift) */
-int sym_shard_color_shift(const sym_graph_shard *g, const uint32_t *hbits, uint32_t *color, uint32_t M,
-                          sym_stream_t stream);
+/* device workspace of a sharded call (problem = SYM_PROBLEM_MIS / MM / COLOR); host
+   only; 0 on invalid arguments */
+size_t sym_sharded_workspace_bytes(const sym_graph_shard *g, const sym_params *p, const sym_comm *c, int problem);
+/* in_set uint8[v_end - v_begin]: MIS flows as in sym_mis */
+int sym_mis_sharded(const sym_graph_shard *g, const sym_params *p, sym_comm *c, void *ws, size_t ws_bytes,
+                    uint8_t *in_set, sym_shard_stats *stats, sym_stream_t stream);
+/* mate int32[v_end - v_begin] (global partner id or -1): MM flows as in sym_mm
+   (Alg 5) */
+int sym_mm_sharded(const sym_graph_shard *g, const sym_params *p, sym_comm *c, void *ws, size_t ws_bytes,
+                   int32_t *mate, sym_shard_stats *stats, sym_stream_t stream);
+/* color uint32[v_end - v_begin] (>= 1): COLOR flows as in sym_color (Alg 8
+   P:226/232, Alg 9) */
+int sym_color_sharded(const sym_graph_shard *g, const sym_params *p, sym_comm *c, void *ws, size_t ws_bytes,
+                      uint32_t *color, sym_shard_stats *stats, sym_stream_t stream);
 
 /* ---- kernel profiling hook (measurement only; off by default) ----
    sym_profile_enable(1) makes every later call record a CUDA event pair on its

@@ -19,13 +19,21 @@ F_VALIDATE, F_STATS, F_EXT_DECOMP = 0x1, 0x2, 0x4
 EXPORTS = (
     "sym_workspace_bytes", "sym_decompose", "sym_mis", "sym_mm", "sym_color", "sym_validate",
     "sym_error_string", "sym_last_error", "sym_version", "sym_profile_enable", "sym_profile_collect",
-    "sym_shard_workspace_bytes", "sym_shard_classify", "sym_shard_frontier", "sym_shard_mis_round",
-    "sym_shard_mis_kill", "sym_shard_mis_finish",
-    "sym_shard_decompose_workspace_bytes", "sym_shard_decompose", "sym_shard_mm_workspace_bytes",
-    "sym_shard_mm_frontier", "sym_shard_mm_round",
-    "sym_shard_color_frontier", "sym_shard_jp_round", "sym_shard_color_conflicts", "sym_shard_color_clear",
-    "sym_shard_color_maxh", "sym_shard_color_shift",
+    "sym_comm_unique_id", "sym_comm_create", "sym_comm_create_local", "sym_comm_destroy", "sym_comm_size",
+    "sym_sharded_workspace_bytes", "sym_mis_sharded", "sym_mm_sharded", "sym_color_sharded",
 )
+COMM_ID_BYTES = 128
+
+
+class SymShardStats(ctypes.Structure):
+    _fields_ = [("rounds", ctypes.c_uint32 * 3), ("exchanges", ctypes.c_uint32), ("boundary", ctypes.c_int64),
+                ("sent_bytes", ctypes.c_int64), ("gathered_bytes", ctypes.c_int64),
+                ("max_exchange_bytes", ctypes.c_int64)]
+
+    def as_dict(self):
+        return {"rounds": list(self.rounds), "exchanges": self.exchanges, "boundary": self.boundary,
+                "sent_bytes": self.sent_bytes, "gathered_bytes": self.gathered_bytes,
+                "max_exchange_bytes": self.max_exchange_bytes}
 
 
 class SymGraphShard(ctypes.Structure):
@@ -98,27 +106,18 @@ def load(build_if_missing: bool = False):
         "sym_error_string": (ctypes.c_char_p, [ctypes.c_int]),
         "sym_last_error": (ctypes.c_char_p, []),
         "sym_version": (ctypes.c_char_p, []),
-        "sym_shard_workspace_bytes": (ctypes.c_size_t, [ctypes.POINTER(SymGraphShard)]),
-        "sym_shard_classify": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), ctypes.c_uint32, P, P]),
-        "sym_shard_frontier": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, ctypes.c_int, P, P, P, P]),
-        "sym_shard_mis_round": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, ctypes.c_int, P, P, P, P, P,
-                                               P, ctypes.c_size_t, P]),
-        "sym_shard_mis_kill": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P]),
-        "sym_shard_mis_finish": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P]),
-        "sym_shard_decompose_workspace_bytes": (ctypes.c_size_t, [ctypes.POINTER(SymGraphShard)]),
-        "sym_shard_decompose": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, ctypes.c_size_t, P, P, P, P,
-                                               P]),
-        "sym_shard_mm_workspace_bytes": (ctypes.c_size_t, [ctypes.POINTER(SymGraphShard)]),
-        "sym_shard_mm_frontier": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P, P]),
-        "sym_shard_mm_round": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, ctypes.c_int, P, P, P, P, P, P,
-                                              P, P, ctypes.c_size_t, P]),
-        "sym_shard_color_frontier": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P, P]),
-        "sym_shard_jp_round": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, ctypes.c_int, P, P, P, P, P,
-                                              P]),
-        "sym_shard_color_conflicts": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, P, P, P, P]),
-        "sym_shard_color_clear": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P, P]),
-        "sym_shard_color_maxh": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, P, P]),
-        "sym_shard_color_shift": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), P, P, ctypes.c_uint32, P]),
+        "sym_comm_unique_id": (ctypes.c_int, [P]),
+        "sym_comm_create": (ctypes.c_int, [ctypes.POINTER(P), ctypes.c_int, ctypes.c_int, P]),
+        "sym_comm_create_local": (ctypes.c_int, [ctypes.POINTER(P), ctypes.c_int, ctypes.c_int, ctypes.c_uint64]),
+        "sym_comm_destroy": (ctypes.c_int, [P]),
+        "sym_comm_size": (ctypes.c_int, [P, ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.c_int)]),
+        "sym_sharded_workspace_bytes": (ctypes.c_size_t, [ctypes.POINTER(SymGraphShard), PR, P, ctypes.c_int]),
+        "sym_mis_sharded": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, P, ctypes.c_size_t, P,
+                                           ctypes.POINTER(SymShardStats), P]),
+        "sym_mm_sharded": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, P, ctypes.c_size_t, P,
+                                          ctypes.POINTER(SymShardStats), P]),
+        "sym_color_sharded": (ctypes.c_int, [ctypes.POINTER(SymGraphShard), PR, P, P, ctypes.c_size_t, P,
+                                             ctypes.POINTER(SymShardStats), P]),
         "sym_profile_enable": (ctypes.c_int, [ctypes.c_int]),
         "sym_profile_collect": (ctypes.c_int, [ctypes.POINTER(SymKernelProfile), ctypes.c_int,
                                                ctypes.POINTER(ctypes.c_int)]),

@@ -159,128 +159,182 @@ __global__ void k_shard_color_shift(const uint32_t *__restrict__ hbits, uint32_t
         if (!((hbits[v >> 5] >> (v & 31)) & 1u)) color[v] += M;
 }
 
+// ---- deltas of the sharded flow (shard.cu): {id, colour} of owned boundary vertices
+// coloured in this round (the round's input list entries, uncoloured at its start)
+__global__ void k_sh_delta_col(const int32_t *__restrict__ list, const uint32_t *cnt, const uint32_t *color,
+                               const uint32_t *__restrict__ bnd, int64_t v0, uint2 *send, uint32_t *dcnt) {
+    const int64_t c = *cnt, stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < c; base += stride) {
+        const int64_t i = base + threadIdx.x;
+        const int32_t v = i < c ? list[i] : -1;
+        const uint32_t cv = v >= 0 ? color[v] : 0u;
+        const bool b = cv != 0 && ((bnd[(v - v0) >> 5] >> ((v - v0) & 31)) & 1u);
+        const int64_t slot = warp_append(b, dcnt);
+        if (slot >= 0) send[slot] = make_uint2((uint32_t)v, cv);
+    }
+}
+
+// COLOR-Rand fix-up, step 2: uncolour V' (the conflicts list), boundary ones as deltas
+__global__ void k_sh_clear_col(const int32_t *__restrict__ list, const uint32_t *cnt, uint32_t *color,
+                               const uint32_t *__restrict__ bnd, int64_t v0, uint2 *send, uint32_t *dcnt) {
+    const int64_t c = *cnt, stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < c; base += stride) {
+        const int64_t i = base + threadIdx.x;
+        const int32_t v = i < c ? list[i] : -1;
+        if (v >= 0) color[v] = 0u;
+        const bool b = v >= 0 && ((bnd[(v - v0) >> 5] >> ((v - v0) & 31)) & 1u);
+        const int64_t slot = warp_append(b, dcnt);
+        if (slot >= 0) send[slot] = make_uint2((uint32_t)v, 0u);
+    }
+}
+
+__global__ void k_sh_col_out(const uint32_t *color, int64_t v0, int64_t v1, uint32_t *out) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = v0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < v1; v += stride) out[v - v0] = color[v];
+}
+
+// DEGk class bits of the owned rows (deg > k, Alg 3), mis.cu
+__global__ void k_shard_classify(const int64_t *__restrict__ rp, int64_t v0, int64_t v1, uint32_t k,
+                                 uint32_t *__restrict__ hbits);
+
 }  // namespace sym
 
 using namespace sym;
 
-static int cs_check(const sym_graph_shard *g) {
-    if (!g) { set_error("shard is NULL"); return SYM_EINVAL; }
-    if (g->n_global < 0 || g->n_global >= ((int64_t)1 << 31) - 1 || g->v_begin < 0 || g->v_end < g->v_begin ||
-        g->v_end > g->n_global || g->nnz < 0) {
-        set_error("bad shard range: need 0 <= v_begin <= v_end <= n_global < 2^31 - 1, nnz >= 0");
-        return SYM_EINVAL;
-    }
-    if (g->v_end > g->v_begin && !g->row_ptr) { set_error("row_ptr is NULL"); return SYM_EINVAL; }
-    if (g->nnz > 0 && !g->col_idx) { set_error("col_idx is NULL"); return SYM_EINVAL; }
-    return SYM_OK;
-}
-
-static int cs_args(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits, int admit,
-                   ShardColorArgs *A) {
-    if (!p) { set_error("params is NULL"); return SYM_EINVAL; }
-    if (p->kind != SYM_DECOMP_NONE && p->kind != SYM_DECOMP_RAND && p->kind != SYM_DECOMP_DEGK) {
-        set_error("unknown decomposition kind");
-        return SYM_EINVAL;
-    }
-    if (p->kind == SYM_DECOMP_RAND && (p->param == 0 || p->param > 65535)) {
-        set_error("RAND needs 1 <= p <= 65535");
-        return SYM_EINVAL;
-    }
-    if (p->kind == SYM_DECOMP_DEGK && !hbits) { set_error("DEGk needs hbits"); return SYM_EINVAL; }
-    if (admit != 0 && admit != 1) { set_error("admit must be 0 or 1"); return SYM_EINVAL; }
-    A->rp = g->row_ptr;
-    A->ci = g->col_idx;
-    A->v0 = g->v_begin;
-    A->v1 = g->v_end;
-    A->kind = (int)p->kind;
-    A->param = p->param;
-    A->kr = stream_key(p->seed, TAG_RAND, 0);
-    A->kv = stream_key(p->seed, TAG_VERTEX, 0);
-    A->hbits = hbits;
-    A->admit = admit;
-    return SYM_OK;
-}
-
+// ------------------------------------------------------------------ sharded COLOR (C-ABI)
 static int cs_grid(int64_t items, int per_cta) {
     int64_t want = (items + per_cta - 1) / per_cta;
     int64_t cap = (int64_t)num_sms() * 8;
     return (int)(want < 1 ? 1 : (want < cap ? want : cap));
 }
 
-extern "C" int sym_shard_color_frontier(const sym_graph_shard *g, const uint32_t *color, int32_t *list,
-                                        uint32_t *count, sym_stream_t stream) {
-    SYM_TRY(cs_check(g));
-    if (!color || !list || !count) { set_error("NULL argument"); return SYM_EINVAL; }
-    cudaStream_t s = (cudaStream_t)stream;
-    SYM_CUDA(cudaMemsetAsync(count, 0, sizeof(uint32_t), s));
-    if (g->v_end == g->v_begin) return SYM_OK;
-    if (g->v_begin % 32) { set_error("v_begin must be a multiple of 32"); return SYM_EINVAL; }
-    k_shard_color_frontier<<<cs_grid(g->v_end - g->v_begin, 256), 256, 0, s>>>(color, g->v_begin, g->v_end, list,
-                                                                               count);
-    SYM_LAUNCH_CHECK();
-    return SYM_OK;
+static void carve_color_sharded(Arena &a, const ShardPlan &P, ShardCtx &x, uint32_t *&color) {
+    carve_shard_common(a, P, sizeof(uint2), x);
+    color = a.take<uint32_t>((size_t)P.N * (size_t)P.B);
 }
 
-extern "C" int sym_shard_jp_round(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits, int admit,
-                                  uint32_t *color, const int32_t *frontier, const uint32_t *count, int32_t *next,
-                                  uint32_t *next_count, sym_stream_t stream) {
-    SYM_TRY(cs_check(g));
-    if (!color || !frontier || !count || !next || !next_count) { set_error("NULL argument"); return SYM_EINVAL; }
+namespace sym {
+void carve_color_sharded_dry(Arena &a, const ShardPlan &P, ShardCtx &x) {
+    uint32_t *c;
+    carve_color_sharded(a, P, x, c);
+}
+}  // namespace sym
+
+// Jones-Plassmann rounds over the owned list fr[0] / pair[3] (filled by the
+// caller), exchanging the boundary colours after every round
+static int color_sharded_phase(const ShardPlan &P, ShardCtx &x, const sym_params *p, const ShardColorArgs &A,
+                               uint32_t *color, uint32_t *rounds) {
+    cudaStream_t s = x.s;
+    const uint32_t maxr = p->max_rounds ? p->max_rounds : 0xffffffffu;
+    int64_t local = P.nl;
+    for (int r = 0;; r++) {
+        if ((uint32_t)r >= maxr) {
+            set_error("sharded COLOR phase did not converge within max_rounds");
+            return SYM_EROUNDS;
+        }
+        SYM_CUDA(cudaMemsetAsync(x.dcnt(r), 0, 2 * sizeof(uint32_t), s));
+        if (local > 0) {
+            k_shard_jp_round<<<cs_grid(local, CS_WARPS), CS_THREADS, 0, s>>>(A, color, x.list_in(r), x.cnt_in(r),
+                                                                            x.list_out(r), x.cnt_out(r));
+            SYM_LAUNCH_CHECK();
+            k_sh_delta_col<<<cs_grid(local, 256), 256, 0, s>>>(x.list_in(r), x.cnt_in(r), color, x.bnd, P.v0,
+                                                               (uint2 *)x.send, x.dcnt(r));
+            SYM_LAUNCH_CHECK();
+        }
+        uint64_t front = 0;
+        SYM_TRY(shard_exchange(P, x, r & 1, SH_COLOR, nullptr, nullptr, nullptr, color, &front));
+        local = x.host_all[2 * P.rank + 1];
+        if (front == 0) {
+            *rounds = (uint32_t)(r + 1);
+            return SYM_OK;
+        }
+    }
+}
+
+extern "C" int sym_color_sharded(const sym_graph_shard *g, const sym_params *p, sym_comm *c, void *ws,
+                                 size_t ws_bytes, uint32_t *color_out, sym_shard_stats *stats, sym_stream_t stream) {
+    ShardPlan P;
+    SYM_TRY(shard_check(g, p, c, &P));
+    if (P.nl > 0 && !color_out) { set_error("color is NULL"); return SYM_EINVAL; }
+    ShardCtx x;
+    uint32_t *color = nullptr;
+    SYM_TRY(shard_carve_ws(ws, ws_bytes, [&](Arena &a) {
+        x = ShardCtx();
+        carve_color_sharded(a, P, x, color);
+    }));
+    x.c = c;
+    x.s = (cudaStream_t)stream;
+    cudaStream_t s = x.s;
+    if (stats) memset(stats, 0, sizeof(*stats));
+    SYM_CUDA(cudaMemsetAsync(color, 0, sizeof(uint32_t) * (size_t)P.N * (size_t)P.B, s));
+    SYM_CUDA(cudaMemsetAsync(x.pair, 0, 8 * sizeof(uint32_t), s));
+    SYM_TRY(shard_boundary(P, x, s));
     ShardColorArgs A;
-    SYM_TRY(cs_args(g, p, hbits, admit, &A));
-    cudaStream_t s = (cudaStream_t)stream;
-    SYM_CUDA(cudaMemsetAsync(next_count, 0, sizeof(uint32_t), s));
-    if (g->v_end == g->v_begin) return SYM_OK;
-    k_shard_jp_round<<<cs_grid(g->v_end - g->v_begin, CS_WARPS), CS_THREADS, 0, s>>>(A, color, frontier, count, next,
-                                                                                     next_count);
-    SYM_LAUNCH_CHECK();
-    return SYM_OK;
-}
-
-extern "C" int sym_shard_color_conflicts(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits,
-                                         const uint32_t *color, int32_t *list, uint32_t *count, sym_stream_t stream) {
-    SYM_TRY(cs_check(g));
-    if (!color || !list || !count) { set_error("NULL argument"); return SYM_EINVAL; }
-    ShardColorArgs A;
-    SYM_TRY(cs_args(g, p, hbits, 1, &A));
-    cudaStream_t s = (cudaStream_t)stream;
-    SYM_CUDA(cudaMemsetAsync(count, 0, sizeof(uint32_t), s));
-    if (g->v_end == g->v_begin) return SYM_OK;
-    k_shard_color_conflicts<<<cs_grid(g->v_end - g->v_begin, CS_WARPS), CS_THREADS, 0, s>>>(A, color, list, count);
-    SYM_LAUNCH_CHECK();
-    return SYM_OK;
-}
-
-extern "C" int sym_shard_color_clear(const sym_graph_shard *g, uint32_t *color, const int32_t *list,
-                                     const uint32_t *count, sym_stream_t stream) {
-    SYM_TRY(cs_check(g));
-    if (!color || !list || !count) { set_error("NULL argument"); return SYM_EINVAL; }
-    if (g->v_end == g->v_begin) return SYM_OK;
-    k_shard_color_clear<<<cs_grid(g->v_end - g->v_begin, 256), 256, 0, (cudaStream_t)stream>>>(color, list, count);
-    SYM_LAUNCH_CHECK();
-    return SYM_OK;
-}
-
-extern "C" int sym_shard_color_maxh(const sym_graph_shard *g, const uint32_t *hbits, const uint32_t *color,
-                                    uint32_t *max_out, sym_stream_t stream) {
-    SYM_TRY(cs_check(g));
-    if (!hbits || !color || !max_out) { set_error("NULL argument"); return SYM_EINVAL; }
-    cudaStream_t s = (cudaStream_t)stream;
-    SYM_CUDA(cudaMemsetAsync(max_out, 0, sizeof(uint32_t), s));
-    if (g->v_end == g->v_begin) return SYM_OK;
-    k_shard_color_maxh<<<cs_grid(g->v_end - g->v_begin, 256), 256, 0, s>>>(hbits, color, g->v_begin, g->v_end,
-                                                                           max_out);
-    SYM_LAUNCH_CHECK();
-    return SYM_OK;
-}
-
-extern "C" int sym_shard_color_shift(const sym_graph_shard *g, const uint32_t *hbits, uint32_t *color, uint32_t M,
-                                     sym_stream_t stream) {
-    SYM_TRY(cs_check(g));
-    if (!hbits || !color) { set_error("NULL argument"); return SYM_EINVAL; }
-    if (g->v_end == g->v_begin) return SYM_OK;
-    k_shard_color_shift<<<cs_grid(g->v_end - g->v_begin, 256), 256, 0, (cudaStream_t)stream>>>(hbits, color,
-                                                                                               g->v_begin, g->v_end, M);
-    SYM_LAUNCH_CHECK();
+    A.rp = P.rp;
+    A.ci = P.ci;
+    A.v0 = P.v0;
+    A.v1 = P.v1;
+    A.kind = p->kind;
+    A.param = p->param;
+    A.kr = stream_key(p->seed, TAG_RAND, 0);
+    A.kv = stream_key(p->seed, TAG_VERTEX, 0);
+    A.hbits = x.hbits;
+    A.admit = p->kind == SYM_DECOMP_NONE ? 0 : 1;
+    if (p->kind == SYM_DECOMP_DEGK) {
+        if (P.nl > 0) {
+            k_shard_classify<<<cs_grid(P.nl, 256), 256, 0, s>>>(P.rp, P.v0, P.v1, p->param, x.hbits);
+            SYM_LAUNCH_CHECK();
+        }
+        SYM_TRY(shard_gather_hbits(P, x));
+    }
+    uint32_t rounds[3] = {0, 0, 0};
+    // phase 1: every owned vertex (NONE: on G; DEGk: G_H and G_L at once; RAND: the parts)
+    SYM_CUDA(cudaMemsetAsync(x.cnt_in(0), 0, sizeof(uint32_t), s));
+    if (P.nl > 0) {
+        k_shard_color_frontier<<<cs_grid(P.nl, 256), 256, 0, s>>>(color, P.v0, P.v1, x.list_in(0), x.cnt_in(0));
+        SYM_LAUNCH_CHECK();
+    }
+    SYM_TRY(color_sharded_phase(P, x, p, A, color, &rounds[0]));
+    uint64_t front = 0;
+    if (p->kind == SYM_DECOMP_DEGK) {
+        // Alg 9: M = max C_H over all ranks; V_L colours += M (owned only: nothing
+        // reads a remote colour after this)
+        SYM_CUDA(cudaMemsetAsync(x.pair + 4, 0, sizeof(uint32_t), s));
+        if (P.nl > 0) {
+            k_shard_color_maxh<<<cs_grid(P.nl, 256), 256, 0, s>>>(x.hbits, color, P.v0, P.v1, x.pair + 4);
+            SYM_LAUNCH_CHECK();
+        }
+        uint32_t M = 0;
+        SYM_TRY(shard_allmax(P, x, &M));
+        if (P.nl > 0) {
+            k_shard_color_shift<<<cs_grid(P.nl, 256), 256, 0, s>>>(x.hbits, color, P.v0, P.v1, M);
+            SYM_LAUNCH_CHECK();
+        }
+    } else if (p->kind == SYM_DECOMP_RAND) {
+        // Alg 8: V' = owned endpoints of monochromatic cross arcs -> fr[0] /
+        // pair[3]; uncolour them (boundary ones exchanged); recolour V' against G
+        SYM_CUDA(cudaMemsetAsync(x.pair, 0, 4 * sizeof(uint32_t), s));
+        if (P.nl > 0) {
+            k_shard_color_conflicts<<<cs_grid(P.nl, CS_WARPS), CS_THREADS, 0, s>>>(A, color, x.list_in(0),
+                                                                                   x.cnt_in(0));
+            SYM_LAUNCH_CHECK();
+            k_sh_clear_col<<<cs_grid(P.nl, 256), 256, 0, s>>>(x.list_in(0), x.cnt_in(0), color, x.bnd, P.v0,
+                                                              (uint2 *)x.send, x.pair);
+            SYM_LAUNCH_CHECK();
+        }
+        SYM_TRY(shard_exchange(P, x, 0, SH_COLOR, nullptr, nullptr, nullptr, color, &front));
+        ShardColorArgs A2 = A;
+        A2.admit = 0;
+        SYM_TRY(color_sharded_phase(P, x, p, A2, color, &rounds[1]));
+    }
+    if (P.nl > 0) {
+        k_sh_col_out<<<cs_grid(P.nl, 256), 256, 0, s>>>(color, P.v0, P.v1, color_out);
+        SYM_LAUNCH_CHECK();
+    }
+    if (stats) {
+        memcpy(stats->rounds, rounds, sizeof(rounds));
+        shard_stats_out(x, stats);
+        SYM_TRY(shard_count_boundary(P, x, &stats->boundary));
+    }
     return SYM_OK;
 }

@@ -7,6 +7,7 @@
 #include <algorithm>
 #include <atomic>
 #include <string>
+#include <vector>
 
 // round kernels (MIS, MM) launch one resident wave instead of 8 CTAs per SM
 #ifndef SYM_ROUND_ONE_WAVE
@@ -232,5 +233,72 @@ int run_mm(const FlowArgs &f, MmWs &w, int32_t *mate);
 
 void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w);
 int run_color(const FlowArgs &f, ColorWs &w, uint32_t *color);
+
+// ------------------------------------------------------------------ multi-GPU (shard.cu)
+enum { SH_MIS = 0, SH_MM = 1, SH_COLOR = 2 };
+
+// a rank's block of the shard plan (shard.cu header): rows [v0, v1) with global ids
+struct ShardPlan {
+    int N = 1, rank = 0;
+    int64_t B = 0, n = 0, v0 = 0, v1 = 0, nl = 0, nnz = 0;
+    const int64_t *rp = nullptr;
+    const int32_t *ci = nullptr;
+};
+
+// per-call state of a sharded flow (device buffers carved from the workspace)
+struct ShardCtx {
+    sym_comm *c = nullptr;
+    cudaStream_t s = nullptr;
+    uint32_t *pair = nullptr;     // [2 parities] x {delta count, frontier count}, [4] all-max value
+    uint32_t *all = nullptr;      // gathered pairs [2N]
+    uint32_t *scratch = nullptr;  // round-kernel counters (zeroed per round)
+    uint32_t *bnd = nullptr;      // owned boundary bitmap
+    uint32_t *hbits = nullptr;    // DEGk class bitmap replica [N*B/32]
+    int32_t *fr[2] = {nullptr, nullptr};
+    size_t entry = 0;             // delta entry bytes
+    void *send = nullptr, *recv = nullptr;
+    std::vector<uint32_t> host_all;
+    uint32_t exchanges = 0;
+    int64_t sent_bytes = 0, gathered_bytes = 0, max_exchange = 0;
+    // round r reads list fr[r & 1] with its count in pair[2 ((r + 1) & 1) + 1] and
+    // writes the next list fr[(r + 1) & 1], its count pair[2 (r & 1) + 1] and its
+    // delta count pair[2 (r & 1)]; a phase's frontier kernel fills fr[0] / pair[3]
+    int32_t *list_in(int r) const { return fr[r & 1]; }
+    int32_t *list_out(int r) const { return fr[(r + 1) & 1]; }
+    uint32_t *cnt_in(int r) const { return pair + 2 * ((r + 1) & 1) + 1; }
+    uint32_t *cnt_out(int r) const { return pair + 2 * (r & 1) + 1; }
+    uint32_t *dcnt(int r) const { return pair + 2 * (r & 1); }
+};
+
+int64_t shard_block(int64_t n, int nranks);
+int shard_check(const sym_graph_shard *g, const sym_params *p, const sym_comm *c, ShardPlan *plan);
+void carve_shard_common(Arena &a, const ShardPlan &P, size_t entry, ShardCtx &x);
+int shard_boundary(const ShardPlan &P, ShardCtx &x, cudaStream_t s);
+int shard_exchange(const ShardPlan &P, ShardCtx &x, int par, int problem, uint8_t *st, int32_t *mate, int32_t *pick,
+                   uint32_t *color, uint64_t *front);
+int shard_gather_hbits(const ShardPlan &P, ShardCtx &x);
+int shard_allmax(const ShardPlan &P, ShardCtx &x, uint32_t *out);
+int shard_count_boundary(const ShardPlan &P, const ShardCtx &x, int64_t *out);
+void shard_stats_out(const ShardCtx &x, sym_shard_stats *st);
+// workspace layouts of the sharded MM / COLOR calls (mm.cu, color_shard.cu)
+void carve_mm_sharded_dry(Arena &a, const ShardPlan &P, const sym_params *p, ShardCtx &x);
+void carve_color_sharded_dry(Arena &a, const ShardPlan &P, ShardCtx &x);
+
+// the workspace of a sharded call: carve into a dry arena (sizes) or the real one
+template <class F>
+int shard_carve_ws(void *ws, size_t ws_bytes, F carve) {
+    Arena dry;
+    carve(dry);
+    const size_t need = dry.used + 256;
+    if (!ws || ws_bytes < need) {
+        set_error("sharded workspace too small: need " + std::to_string(need) + " bytes");
+        return SYM_EWORKSPACE;
+    }
+    Arena a;
+    a.base = (char *)(((uintptr_t)ws + 255) & ~(uintptr_t)255);
+    a.cap = ws_bytes;
+    carve(a);
+    return SYM_OK;
+}
 
 }  // namespace sym

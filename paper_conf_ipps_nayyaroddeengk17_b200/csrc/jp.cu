@@ -393,7 +393,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_count_huge(JpArgs A) {
             if (ll) atomicAdd(A.ldeg + h, ll);
         }
         prof_add(A.prof, 0ull, threadIdx.x == 0 ? 4ull * (uint64_t)(pe_ - pb) : 0ull);
-        prof_add(A.prof_jp, 8ull * (uint64_t)(lh + ll), 0ull);
+        prof_add(A.prof_jp, lane_id() == 0 ? 8ull * (uint64_t)(lh + ll) : 0ull, 0ull);  // lh, ll: warp totals
     }
 }
 

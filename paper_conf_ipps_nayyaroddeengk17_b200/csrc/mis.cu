@@ -459,10 +459,35 @@ __global__ void k_shard_frontier(const uint32_t *__restrict__ hbits, int cls, co
     }
 }
 
-// MIS-Deg2 fix-up, pull form: an owned undecided V_H vertex with an In V_L neighbour
-// leaves the remaining graph (warp per vertex, ballot early exit)
-__global__ void k_shard_kill(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci,
-                             const uint32_t *__restrict__ hbits, uint8_t *st, int64_t v0, int64_t v1) {
+__global__ void k_shard_finish(const uint8_t *__restrict__ st, int64_t v0, int64_t v1, uint8_t *__restrict__ out) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = v0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < v1; v += stride)
+        out[v - v0] = st[v] == ST_IN ? 1 : 0;
+}
+
+// ---- deltas of the sharded flow (shard.cu): owned boundary vertices whose status
+// changed, packed id << 2 | status (4 B)
+__device__ __forceinline__ bool sh_bnd(const uint32_t *bnd, int64_t i) { return (bnd[i >> 5] >> (i & 31)) & 1u; }
+
+// decided in this round: the round's input list entries (all undecided at its start)
+// that are now In / Out
+__global__ void k_sh_delta_mis(const int32_t *__restrict__ list, const uint32_t *cnt, const uint8_t *st,
+                               const uint32_t *__restrict__ bnd, int64_t v0, uint32_t *send, uint32_t *dcnt) {
+    const int64_t c = *cnt, stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < c; base += stride) {
+        const int64_t i = base + threadIdx.x;
+        const int32_t v = i < c ? list[i] : -1;
+        const uint8_t sv = v >= 0 ? st[v] : (uint8_t)ST_UNDEC;
+        const int64_t slot = warp_append(v >= 0 && sv != ST_UNDEC && sh_bnd(bnd, v - v0), dcnt);
+        if (slot >= 0) send[slot] = ((uint32_t)v << 2) | sv;
+    }
+}
+
+// MIS-Deg2 fix-up, pull form with deltas: an owned undecided V_H vertex with
+// an In V_L neighbour leaves the remaining graph (warp per vertex)
+__global__ void k_sh_kill_degk(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci,
+                               const uint32_t *__restrict__ hbits, uint8_t *st, int64_t v0, int64_t v1,
+                               const uint32_t *__restrict__ bnd, uint32_t *send, uint32_t *dcnt) {
     const int lane = lane_id();
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t v = v0 + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); v < v1; v += nw) {
@@ -477,132 +502,223 @@ __global__ void k_shard_kill(const int64_t *__restrict__ rp, const int32_t *__re
             }
             hit = __any_sync(FULL, h);
         }
-        if (hit && lane == 0) st[v] = ST_OUT;
+        if (hit && lane == 0) {
+            st[v] = ST_OUT;
+            if (sh_bnd(bnd, v - v0)) send[atomicAdd(dcnt, 1u)] = ((uint32_t)v << 2) | ST_OUT;
+        }
     }
 }
 
-__global__ void k_shard_finish(const uint8_t *__restrict__ st, int64_t v0, int64_t v1, uint8_t *__restrict__ out) {
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t v = v0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < v1; v += stride)
-        out[v - v0] = st[v] == ST_IN ? 1 : 0;
+// MIS-Rand (reading G10): B = owned vertices with a cross arc (RAND labels
+// differ) are not in phase A: INACTIVE (warp per vertex)
+__global__ void k_sh_rand_inactive(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, Key kr,
+                                   uint32_t p, uint8_t *st, int64_t v0, int64_t v1, const uint32_t *__restrict__ bnd,
+                                   uint32_t *send, uint32_t *dcnt) {
+    const int lane = lane_id();
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = v0 + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); v < v1; v += nw) {
+        const uint32_t lv = rand_label(kr, (uint32_t)v, p);
+        const int64_t b = rp[v - v0], e = rp[v - v0 + 1];
+        bool hit = false;
+        for (int64_t x = b; x < e && !hit; x += 32) {
+            const bool h = x + lane < e && rand_label(kr, (uint32_t)ci[x + lane], p) != lv;
+            hit = __any_sync(FULL, h);
+        }
+        if (hit && lane == 0) {
+            st[v] = ST_INACTIVE;
+            if (sh_bnd(bnd, v - v0)) send[atomicAdd(dcnt, 1u)] = ((uint32_t)v << 2) | ST_INACTIVE;
+        }
+    }
+}
+
+// MIS-Rand fix-up: an owned B vertex with an In neighbour (an interior vertex of I_A)
+// is removed (Out); the others enter phase B (undecided)
+__global__ void k_sh_rand_release(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, uint8_t *st,
+                                  int64_t v0, int64_t v1, const uint32_t *__restrict__ bnd, uint32_t *send,
+                                  uint32_t *dcnt) {
+    const int lane = lane_id();
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = v0 + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); v < v1; v += nw) {
+        if (st[v] != ST_INACTIVE) continue;
+        const int64_t b = rp[v - v0], e = rp[v - v0 + 1];
+        bool hit = false;
+        for (int64_t x = b; x < e && !hit; x += 32) {
+            const bool h = x + lane < e && st[ci[x + lane]] == ST_IN;
+            hit = __any_sync(FULL, h);
+        }
+        if (lane == 0) {
+            const uint8_t ns = hit ? ST_OUT : ST_UNDEC;
+            st[v] = ns;
+            if (sh_bnd(bnd, v - v0)) send[atomicAdd(dcnt, 1u)] = ((uint32_t)v << 2) | ns;
+        }
+    }
 }
 
 }  // namespace sym
 
 using namespace sym;
 
-static int check_shard(const sym_graph_shard *g) {
-    if (!g) { set_error("shard is NULL"); return SYM_EINVAL; }
-    if (g->n_global < 0 || g->n_global >= ((int64_t)1 << 31) - 1 || g->v_begin < 0 || g->v_end < g->v_begin ||
-        g->v_end > g->n_global || g->nnz < 0) {
-        set_error("bad shard range: need 0 <= v_begin <= v_end <= n_global < 2^31 - 1, nnz >= 0");
-        return SYM_EINVAL;
-    }
-    if (g->v_begin % 32 && g->v_end > g->v_begin) {
-        set_error("v_begin must be a multiple of 32");
-        return SYM_EINVAL;
-    }
-    if (g->v_end > g->v_begin && !g->row_ptr) { set_error("row_ptr is NULL"); return SYM_EINVAL; }
-    if (g->nnz > 0 && !g->col_idx) { set_error("col_idx is NULL"); return SYM_EINVAL; }
-    return SYM_OK;
+// ------------------------------------------------------------------ sharded MIS (C-ABI)
+static void carve_mis_sharded(Arena &a, const ShardPlan &P, ShardCtx &x, uint8_t *&st, int64_t *&huge) {
+    carve_shard_common(a, P, sizeof(uint32_t), x);
+    st = a.take<uint8_t>((size_t)P.N * (size_t)P.B);
+    huge = a.take<int64_t>(2 * (size_t)(P.nnz / MIS_BUDGET + 2));
 }
 
 static int shard_grid(int64_t items) {
-    int64_t want = (items + 255) / 256;
-    int64_t cap = (int64_t)num_sms() * 8;
+    int64_t want = (items + 255) / 256, cap = (int64_t)num_sms() * 8;
     return (int)(want < 1 ? 1 : (want < cap ? want : cap));
 }
 
-extern "C" size_t sym_shard_workspace_bytes(const sym_graph_shard *g) {
-    if (check_shard(g) != SYM_OK) return 0;
-    return 256 + 64 + sizeof(int64_t) * 2 * (size_t)(g->nnz / MIS_BUDGET + 2) + 256;
-}
-
-extern "C" int sym_shard_classify(const sym_graph_shard *g, uint32_t k, uint32_t *hbits, sym_stream_t stream) {
-    SYM_TRY(check_shard(g));
-    if (g->v_end == g->v_begin) return SYM_OK;
-    if (!hbits) { set_error("hbits is NULL"); return SYM_EINVAL; }
-    k_shard_classify<<<shard_grid(g->v_end - g->v_begin), 256, 0, (cudaStream_t)stream>>>(g->row_ptr, g->v_begin,
-                                                                                           g->v_end, k, hbits);
-    SYM_LAUNCH_CHECK();
-    return SYM_OK;
-}
-
-extern "C" int sym_shard_frontier(const sym_graph_shard *g, const uint32_t *hbits, int cls, const uint8_t *status,
-                                  int32_t *list, uint32_t *count, sym_stream_t stream) {
-    SYM_TRY(check_shard(g));
-    if (!status || !list || !count || (cls >= 0 && !hbits)) { set_error("NULL argument"); return SYM_EINVAL; }
-    cudaStream_t s = (cudaStream_t)stream;
-    SYM_CUDA(cudaMemsetAsync(count, 0, sizeof(uint32_t), s));
-    if (g->v_end == g->v_begin) return SYM_OK;
-    k_shard_frontier<<<shard_grid(g->v_end - g->v_begin), 256, 0, s>>>(hbits, cls, status, g->v_begin, g->v_end, list,
-                                                                       count);
-    SYM_LAUNCH_CHECK();
-    return SYM_OK;
-}
-
-extern "C" int sym_shard_mis_round(const sym_graph_shard *g, const sym_params *p, const uint32_t *hbits, int cls,
-                                   uint8_t *status, const int32_t *frontier, const uint32_t *count, int32_t *next,
-                                   uint32_t *next_count, void *ws, size_t ws_bytes, sym_stream_t stream) {
-    SYM_TRY(check_shard(g));
-    if (!p || !status || !frontier || !count || !next || !next_count || (cls >= 0 && !hbits)) {
-        set_error("NULL argument");
-        return SYM_EINVAL;
+// Luby rounds of one phase over the owned frontier (class cls of the DEGk bitmap, -1:
+// all), exchanging the boundary decisions after every round.  *rounds = rounds run.
+static int mis_sharded_phase(const ShardPlan &P, ShardCtx &x, const sym_params *p, uint8_t *st, int64_t *huge, int cls,
+                             uint32_t *rounds) {
+    cudaStream_t s = x.s;
+    SYM_CUDA(cudaMemsetAsync(x.cnt_in(0), 0, sizeof(uint32_t), s));
+    if (P.nl > 0) {
+        k_shard_frontier<<<shard_grid(P.nl), 256, 0, s>>>(x.hbits, cls, st, P.v0, P.v1, x.list_in(0), x.cnt_in(0));
+        SYM_LAUNCH_CHECK();
     }
-    const size_t need = sym_shard_workspace_bytes(g);
-    if (!ws || ws_bytes < need) { set_error("shard workspace too small"); return SYM_EWORKSPACE; }
-    cudaStream_t s = (cudaStream_t)stream;
-    char *base = (char *)(((uintptr_t)ws + 255) & ~(uintptr_t)255);
-    uint32_t *ctr = reinterpret_cast<uint32_t *>(base);               // [0] huge count, [1..3] scratch
-    int64_t *huge = reinterpret_cast<int64_t *>(base + 64);
-    SYM_CUDA(cudaMemsetAsync(ctr, 0, 64, s));
-    SYM_CUDA(cudaMemsetAsync(next_count, 0, sizeof(uint32_t), s));
-    MisRoundArgs A;
-    A.rp = g->row_ptr;
-    A.ci = g->col_idx;
-    A.st = status;
-    A.in_list = frontier;
-    A.in_rev = 0;
-    A.in_cnt = count;
-    A.implicit_n = 0;
-    A.out_list = next;
-    A.out_cnt = next_count;
-    A.clear_cnt = ctr + 1;
-    A.huge = huge;
-    A.huge_cnt = ctr;
-    A.huge_clear = ctr + 2;
-    A.hist = nullptr;
-    A.round = 0;
-    A.k = stream_key(p->seed, TAG_VERTEX, 0);
-    A.prof = nullptr;
-    A.row_base = g->v_begin;
-    A.nfilter = hbits;
-    A.ncls = cls;
-    k_mis_round<<<round_grid(), MIS_THREADS, 0, s>>>(A);
-    SYM_LAUNCH_CHECK();
-    k_mis_huge<<<num_sms() * 2, MIS_HUGE_THREADS, 0, s>>>(A);
-    SYM_LAUNCH_CHECK();
+    const uint32_t maxr = p->max_rounds ? p->max_rounds : 0xffffffffu;
+    const Key k = stream_key(p->seed, TAG_VERTEX, 0);
+    int64_t local = P.nl;  // this rank's frontier length (host view, sizes the grid)
+    for (int r = 0;; r++) {
+        if ((uint32_t)r >= maxr) {
+            set_error("sharded MIS phase did not converge within max_rounds");
+            return SYM_EROUNDS;
+        }
+        SYM_CUDA(cudaMemsetAsync(x.dcnt(r), 0, 2 * sizeof(uint32_t), s));
+        SYM_CUDA(cudaMemsetAsync(x.scratch, 0, 4 * sizeof(uint32_t), s));
+        if (local > 0) {
+            MisRoundArgs A;
+            A.rp = P.rp;
+            A.ci = P.ci;
+            A.st = st;
+            A.in_list = x.list_in(r);
+            A.in_rev = 0;
+            A.in_cnt = x.cnt_in(r);
+            A.implicit_n = 0;
+            A.out_list = x.list_out(r);
+            A.out_cnt = x.cnt_out(r);
+            A.clear_cnt = x.scratch + 1;
+            A.huge = huge;
+            A.huge_cnt = x.scratch;
+            A.huge_clear = x.scratch + 2;
+            A.hist = nullptr;
+            A.round = 0;
+            A.k = k;
+            A.prof = nullptr;
+            A.row_base = P.v0;
+            A.nfilter = x.hbits;
+            A.ncls = cls;
+            k_mis_round<<<std::min<int64_t>(round_grid(), shard_grid(local)), MIS_THREADS, 0, s>>>(A);
+            SYM_LAUNCH_CHECK();
+            k_mis_huge<<<num_sms() * 2, MIS_HUGE_THREADS, 0, s>>>(A);
+            SYM_LAUNCH_CHECK();
+            k_sh_delta_mis<<<shard_grid(local), 256, 0, s>>>(x.list_in(r), x.cnt_in(r), st, x.bnd, P.v0,
+                                                             (uint32_t *)x.send, x.dcnt(r));
+            SYM_LAUNCH_CHECK();
+        }
+        uint64_t front = 0;
+        SYM_TRY(shard_exchange(P, x, r & 1, SH_MIS, st, nullptr, nullptr, nullptr, &front));
+        local = x.host_all[2 * P.rank + 1];
+        if (front == 0) {
+            *rounds = (uint32_t)(r + 1);
+            return SYM_OK;
+        }
+    }
+}
+
+extern "C" {
+
+size_t sym_sharded_workspace_bytes(const sym_graph_shard *g, const sym_params *p, const sym_comm *c, int problem) {
+    ShardPlan P;
+    if (shard_check(g, p, c, &P) != SYM_OK) return 0;
+    Arena a;
+    ShardCtx x;
+    if (problem == SYM_PROBLEM_MIS) {
+        uint8_t *st;
+        int64_t *huge;
+        carve_mis_sharded(a, P, x, st, huge);
+    } else if (problem == SYM_PROBLEM_MM) {
+        carve_mm_sharded_dry(a, P, p, x);
+    } else if (problem == SYM_PROBLEM_COLOR) {
+        carve_color_sharded_dry(a, P, x);
+    } else {
+        return 0;
+    }
+    return a.used + 256;
+}
+
+int sym_mis_sharded(const sym_graph_shard *g, const sym_params *p, sym_comm *c, void *ws, size_t ws_bytes,
+                    uint8_t *in_set, sym_shard_stats *stats, sym_stream_t stream) {
+    ShardPlan P;
+    SYM_TRY(shard_check(g, p, c, &P));
+    if (P.nl > 0 && !in_set) { set_error("in_set is NULL"); return SYM_EINVAL; }
+    ShardCtx x;
+    uint8_t *st = nullptr;
+    int64_t *huge = nullptr;
+    SYM_TRY(shard_carve_ws(ws, ws_bytes, [&](Arena &a) {
+        x = ShardCtx();
+        carve_mis_sharded(a, P, x, st, huge);
+    }));
+    x.c = c;
+    x.s = (cudaStream_t)stream;
+    cudaStream_t s = x.s;
+    if (stats) memset(stats, 0, sizeof(*stats));
+    SYM_CUDA(cudaMemsetAsync(st, ST_UNDEC, (size_t)P.N * (size_t)P.B, s));
+    SYM_CUDA(cudaMemsetAsync(x.pair, 0, 8 * sizeof(uint32_t), s));
+    SYM_TRY(shard_boundary(P, x, s));
+    uint32_t rounds[3] = {0, 0, 0};
+    uint64_t front = 0;
+    if (p->kind == SYM_DECOMP_NONE) {
+        SYM_TRY(mis_sharded_phase(P, x, p, st, huge, -1, &rounds[0]));
+    } else if (p->kind == SYM_DECOMP_DEGK) {
+        // V_H bitmap: owned words, then all-gathered once
+        if (P.nl > 0) {
+            k_shard_classify<<<shard_grid(P.nl), 256, 0, s>>>(P.rp, P.v0, P.v1, p->param, x.hbits);
+            SYM_LAUNCH_CHECK();
+        }
+        SYM_TRY(shard_gather_hbits(P, x));
+        SYM_TRY(mis_sharded_phase(P, x, p, st, huge, 0, &rounds[0]));  // I_L = MIS(G_L)
+        SYM_CUDA(cudaMemsetAsync(x.pair, 0, 2 * sizeof(uint32_t), s));
+        if (P.nl > 0) {
+            k_sh_kill_degk<<<num_sms() * 8, 256, 0, s>>>(P.rp, P.ci, x.hbits, st, P.v0, P.v1, x.bnd,
+                                                         (uint32_t *)x.send, x.pair);
+            SYM_LAUNCH_CHECK();
+        }
+        SYM_TRY(shard_exchange(P, x, 0, SH_MIS, st, nullptr, nullptr, nullptr, &front));
+        SYM_TRY(mis_sharded_phase(P, x, p, st, huge, 1, &rounds[1]));  // I_R on the remaining V_H
+    } else {
+        const Key kr = stream_key(p->seed, TAG_RAND, 0);
+        SYM_CUDA(cudaMemsetAsync(x.pair, 0, 2 * sizeof(uint32_t), s));
+        if (P.nl > 0) {
+            k_sh_rand_inactive<<<num_sms() * 8, 256, 0, s>>>(P.rp, P.ci, kr, p->param, st, P.v0, P.v1, x.bnd,
+                                                             (uint32_t *)x.send, x.pair);
+            SYM_LAUNCH_CHECK();
+        }
+        SYM_TRY(shard_exchange(P, x, 0, SH_MIS, st, nullptr, nullptr, nullptr, &front));
+        SYM_TRY(mis_sharded_phase(P, x, p, st, huge, -1, &rounds[0]));  // I_A on the interiors
+        SYM_CUDA(cudaMemsetAsync(x.pair, 0, 2 * sizeof(uint32_t), s));
+        if (P.nl > 0) {
+            k_sh_rand_release<<<num_sms() * 8, 256, 0, s>>>(P.rp, P.ci, st, P.v0, P.v1, x.bnd, (uint32_t *)x.send,
+                                                            x.pair);
+            SYM_LAUNCH_CHECK();
+        }
+        SYM_TRY(shard_exchange(P, x, 0, SH_MIS, st, nullptr, nullptr, nullptr, &front));
+        SYM_TRY(mis_sharded_phase(P, x, p, st, huge, -1, &rounds[1]));  // I_B on G - N[I_A]
+    }
+    if (P.nl > 0) {
+        k_shard_finish<<<shard_grid(P.nl), 256, 0, s>>>(st, P.v0, P.v1, in_set);
+        SYM_LAUNCH_CHECK();
+    }
+    if (stats) {
+        memcpy(stats->rounds, rounds, sizeof(rounds));
+        shard_stats_out(x, stats);
+        SYM_TRY(shard_count_boundary(P, x, &stats->boundary));
+    }
     return SYM_OK;
 }
 
-extern "C" int sym_shard_mis_kill(const sym_graph_shard *g, const uint32_t *hbits, uint8_t *status,
-                                  sym_stream_t stream) {
-    SYM_TRY(check_shard(g));
-    if (!hbits || !status) { set_error("NULL argument"); return SYM_EINVAL; }
-    if (g->v_end == g->v_begin) return SYM_OK;
-    k_shard_kill<<<num_sms() * 8, 256, 0, (cudaStream_t)stream>>>(g->row_ptr, g->col_idx, hbits, status, g->v_begin,
-                                                                   g->v_end);
-    SYM_LAUNCH_CHECK();
-    return SYM_OK;
-}
-
-extern "C" int sym_shard_mis_finish(const sym_graph_shard *g, const uint8_t *status, uint8_t *in_set_owned,
-                                    sym_stream_t stream) {
-    SYM_TRY(check_shard(g));
-    if (!status || (g->v_end > g->v_begin && !in_set_owned)) { set_error("NULL argument"); return SYM_EINVAL; }
-    if (g->v_end == g->v_begin) return SYM_OK;
-    k_shard_finish<<<shard_grid(g->v_end - g->v_begin), 256, 0, (cudaStream_t)stream>>>(status, g->v_begin, g->v_end,
-                                                                                        in_set_owned);
-    SYM_LAUNCH_CHECK();
-    return SYM_OK;
-}
+}  // extern "C"

@@ -502,89 +502,176 @@ __global__ void k_shard_mm_frontier(const int64_t *__restrict__ rp, int64_t v0, 
     }
 }
 
+// ---- deltas of the sharded flow (shard.cu): every pick / match an owned boundary
+// vertex wrote in this round, {id | matched << 31, pick} (8 B)
+__global__ void k_sh_delta_mm(const int32_t *__restrict__ list, const uint32_t *cnt, const int32_t *mate,
+                              const int32_t *pick_cur, const uint32_t *__restrict__ bnd, int64_t v0, uint2 *send,
+                              uint32_t *dcnt) {
+    const int64_t c = *cnt, stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < c; base += stride) {
+        const int64_t i = base + threadIdx.x;
+        const int32_t u = i < c ? list[i] : -1;
+        const bool b = u >= 0 && ((bnd[(u - v0) >> 5] >> ((u - v0) & 31)) & 1u);
+        const int64_t slot = warp_append(b, dcnt);
+        if (slot >= 0) send[slot] = make_uint2((uint32_t)u | (mate[u] >= 0 ? 0x80000000u : 0u), (uint32_t)pick_cur[u]);
+    }
+}
+
+// the owned mates (global ids) -> the caller's output
+__global__ void k_sh_mm_out(const int32_t *mate, int64_t v0, int64_t v1, int32_t *out) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = v0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < v1; v += stride) out[v - v0] = mate[v];
+}
+
 }  // namespace sym
 
 using namespace sym;
 
-static int check_mm_shard(const sym_graph_shard *g) {
-    if (!g) { set_error("shard is NULL"); return SYM_EINVAL; }
-    if (g->n_global < 0 || g->n_global >= ((int64_t)1 << 31) - 1 || g->v_begin < 0 || g->v_end < g->v_begin ||
-        g->v_end > g->n_global || g->nnz < 0) {
-        set_error("bad shard range: need 0 <= v_begin <= v_end <= n_global < 2^31 - 1, nnz >= 0");
+// ------------------------------------------------------------------ sharded MM (C-ABI)
+struct MmShardWs {
+    int32_t *mate = nullptr, *pick[2] = {nullptr, nullptr}, *huge = nullptr;
+    SplitWs sw;
+    int64_t *rp_in = nullptr, *rp_x = nullptr;
+    int32_t *ci_in = nullptr, *ci_x = nullptr;
+};
+
+static void carve_mm_sharded(Arena &a, const ShardPlan &P, const sym_params *p, ShardCtx &x, MmShardWs &w) {
+    carve_shard_common(a, P, sizeof(uint2), x);
+    const size_t pad = (size_t)P.N * (size_t)P.B;
+    w.mate = a.take<int32_t>(pad);
+    w.pick[0] = a.take<int32_t>(pad);
+    w.pick[1] = a.take<int32_t>(pad);
+    w.huge = a.take<int32_t>((size_t)(P.nnz / MM_BUDGET + 2));
+    if (p->kind == SYM_DECOMP_RAND) {  // the owned rows' RAND decomposition (Alg 2, local)
+        carve_split_ws(a, P.nl, P.nnz, w.sw);
+        w.rp_in = a.take<int64_t>((size_t)P.nl + 1);
+        w.rp_x = a.take<int64_t>((size_t)P.nl + 1);
+        w.ci_in = a.take<int32_t>((size_t)P.nnz + 1);
+        w.ci_x = a.take<int32_t>((size_t)P.nnz + 1);
+    }
+}
+
+namespace sym {
+void carve_mm_sharded_dry(Arena &a, const ShardPlan &P, const sym_params *p, ShardCtx &x) {
+    MmShardWs w;
+    carve_mm_sharded(a, P, p, x, w);
+}
+}  // namespace sym
+
+static int mm_shard_grid(int64_t items) {
+    int64_t want = (items + 255) / 256, cap = (int64_t)num_sms() * 8;
+    return (int)(want < 1 ? 1 : (want < cap ? want : cap));
+}
+
+// handshake rounds of one phase (phase CSR rp/ci over the owned rows, global ids)
+static int mm_sharded_phase(const ShardPlan &P, ShardCtx &x, const sym_params *p, MmShardWs &w, const int64_t *rp,
+                            const int32_t *ci, uint32_t *rounds) {
+    cudaStream_t s = x.s;
+    SYM_CUDA(cudaMemsetAsync(x.cnt_in(0), 0, sizeof(uint32_t), s));
+    if (P.nl > 0) {
+        k_shard_mm_frontier<<<mm_shard_grid(P.nl), 256, 0, s>>>(rp, P.v0, P.v1, w.mate, x.list_in(0), x.cnt_in(0));
+        SYM_LAUNCH_CHECK();
+    }
+    const uint32_t maxr = p->max_rounds ? p->max_rounds : 0xffffffffu;
+    const Key k = stream_key(p->seed, TAG_EDGE, 0);
+    int64_t local = P.nl;
+    for (int r = 0;; r++) {
+        if ((uint32_t)r >= maxr) {
+            set_error("sharded MM phase did not converge within max_rounds");
+            return SYM_EROUNDS;
+        }
+        SYM_CUDA(cudaMemsetAsync(x.dcnt(r), 0, 2 * sizeof(uint32_t), s));
+        SYM_CUDA(cudaMemsetAsync(x.scratch, 0, 4 * sizeof(uint32_t), s));
+        if (local > 0) {
+            MmRoundArgs A;
+            A.rp = rp;
+            A.rp2 = nullptr;
+            A.ci = ci;
+            A.ci2 = nullptr;
+            A.hbits = nullptr;
+            A.dual = 0;
+            A.mate = w.mate;
+            A.pick_prev = w.pick[(r + 1) & 1];
+            A.pick_cur = w.pick[r & 1];
+            A.in_list = x.list_in(r);
+            A.in_rev = 0;
+            A.in_cnt = x.cnt_in(r);
+            A.implicit_n = 0;
+            A.out_list = x.list_out(r);
+            A.out_cnt = x.cnt_out(r);
+            A.clear_cnt = x.scratch + 1;
+            A.huge = w.huge;
+            A.huge_cnt = x.scratch;
+            A.huge_clear = x.scratch + 2;
+            A.hist = nullptr;
+            A.round = 0;
+            A.k = k;
+            A.prof = nullptr;
+            A.row_base = P.v0;
+            const int grid = (int)std::min<int64_t>(mm_round_grid(), mm_shard_grid(local));
+            if (r == 0) k_mm_round<false, true><<<grid, MM_THREADS, 0, s>>>(A);  // round 0: nothing to resolve
+            else k_mm_round<true, true><<<grid, MM_THREADS, 0, s>>>(A);
+            SYM_LAUNCH_CHECK();
+            k_mm_huge<true><<<num_sms() * 2, MM_HUGE_THREADS, 0, s>>>(A);
+            SYM_LAUNCH_CHECK();
+            k_sh_delta_mm<<<mm_shard_grid(local), 256, 0, s>>>(x.list_in(r), x.cnt_in(r), w.mate, A.pick_cur, x.bnd,
+                                                              P.v0, (uint2 *)x.send, x.dcnt(r));
+            SYM_LAUNCH_CHECK();
+        }
+        uint64_t front = 0;
+        SYM_TRY(shard_exchange(P, x, r & 1, SH_MM, nullptr, w.mate, w.pick[r & 1], nullptr, &front));
+        local = x.host_all[2 * P.rank + 1];
+        if (front == 0) {
+            *rounds = (uint32_t)(r + 1);
+            return SYM_OK;
+        }
+    }
+}
+
+extern "C" int sym_mm_sharded(const sym_graph_shard *g, const sym_params *p, sym_comm *c, void *ws, size_t ws_bytes,
+                              int32_t *mate, sym_shard_stats *stats, sym_stream_t stream) {
+    ShardPlan P;
+    SYM_TRY(shard_check(g, p, c, &P));
+    if (p->kind == SYM_DECOMP_DEGK) {
+        set_error("sharded MM supports the NONE and RAND decompositions");
         return SYM_EINVAL;
     }
-    if (g->v_end > g->v_begin && !g->row_ptr) { set_error("row_ptr is NULL"); return SYM_EINVAL; }
-    if (g->nnz > 0 && !g->col_idx) { set_error("col_idx is NULL"); return SYM_EINVAL; }
-    return SYM_OK;
-}
-
-extern "C" size_t sym_shard_mm_workspace_bytes(const sym_graph_shard *g) {
-    if (check_mm_shard(g) != SYM_OK) return 0;
-    return 256 + 64 + sizeof(int32_t) * (size_t)(g->nnz / MM_BUDGET + 2) + 256;
-}
-
-extern "C" int sym_shard_mm_frontier(const sym_graph_shard *g, const int32_t *mate, int32_t *list, uint32_t *count,
-                                     sym_stream_t stream) {
-    SYM_TRY(check_mm_shard(g));
-    if (!mate || !list || !count) { set_error("NULL argument"); return SYM_EINVAL; }
-    cudaStream_t s = (cudaStream_t)stream;
-    SYM_CUDA(cudaMemsetAsync(count, 0, sizeof(uint32_t), s));
-    const int64_t nl = g->v_end - g->v_begin;
-    if (nl == 0) return SYM_OK;
-    int64_t want = (nl + 255) / 256, cap = (int64_t)num_sms() * 8;
-    k_shard_mm_frontier<<<(int)(want < cap ? want : cap), 256, 0, s>>>(g->row_ptr, g->v_begin, g->v_end, mate, list,
-                                                                       count);
-    SYM_LAUNCH_CHECK();
-    return SYM_OK;
-}
-
-extern "C" int sym_shard_mm_round(const sym_graph_shard *g, const sym_params *p, int round, int32_t *mate,
-                                  const int32_t *pick_prev, int32_t *pick_cur, const int32_t *frontier,
-                                  const uint32_t *count, int32_t *next, uint32_t *next_count, void *ws,
-                                  size_t ws_bytes, sym_stream_t stream) {
-    SYM_TRY(check_mm_shard(g));
-    if (!p || !mate || !pick_cur || (round > 0 && !pick_prev) || !frontier || !count || !next || !next_count) {
-        set_error("NULL argument");
-        return SYM_EINVAL;
+    if (P.nl > 0 && !mate) { set_error("mate is NULL"); return SYM_EINVAL; }
+    ShardCtx x;
+    MmShardWs w;
+    SYM_TRY(shard_carve_ws(ws, ws_bytes, [&](Arena &a) {
+        x = ShardCtx();
+        w = MmShardWs();
+        carve_mm_sharded(a, P, p, x, w);
+    }));
+    x.c = c;
+    x.s = (cudaStream_t)stream;
+    cudaStream_t s = x.s;
+    if (stats) memset(stats, 0, sizeof(*stats));
+    const size_t pad = (size_t)P.N * (size_t)P.B;
+    SYM_CUDA(cudaMemsetAsync(w.mate, 0xff, sizeof(int32_t) * pad, s));
+    SYM_CUDA(cudaMemsetAsync(w.pick[0], 0xff, sizeof(int32_t) * pad, s));
+    SYM_CUDA(cudaMemsetAsync(w.pick[1], 0xff, sizeof(int32_t) * pad, s));
+    SYM_CUDA(cudaMemsetAsync(x.pair, 0, 8 * sizeof(uint32_t), s));
+    SYM_TRY(shard_boundary(P, x, s));
+    uint32_t rounds[3] = {0, 0, 0};
+    if (p->kind == SYM_DECOMP_NONE) {
+        SYM_TRY(mm_sharded_phase(P, x, p, w, P.rp, P.ci, &rounds[0]));  // LMAX on G
+    } else {
+        // labels hash the GLOBAL id (row_base), so the parts equal the single-GPU ones
+        SYM_TRY(run_split(Graph{P.nl, P.nnz, P.rp, P.ci}, p->kind, p->param, p->seed, w.sw, nullptr, w.rp_in, w.ci_in,
+                          w.rp_x, w.ci_x, nullptr, s, P.v0));
+        SYM_TRY(mm_sharded_phase(P, x, p, w, w.rp_in, w.ci_in, &rounds[0]));  // M_IS on the parts (Alg 5 l.5)
+        SYM_TRY(mm_sharded_phase(P, x, p, w, w.rp_x, w.ci_x, &rounds[1]));    // cross edges among unmatched (l.6-7)
     }
-    if (round < 0) { set_error("round must be >= 0"); return SYM_EINVAL; }
-    const size_t need = sym_shard_mm_workspace_bytes(g);
-    if (!ws || ws_bytes < need) { set_error("shard workspace too small"); return SYM_EWORKSPACE; }
-    cudaStream_t s = (cudaStream_t)stream;
-    char *base = (char *)(((uintptr_t)ws + 255) & ~(uintptr_t)255);
-    uint32_t *ctr = reinterpret_cast<uint32_t *>(base);  // [0] huge count, [1..3] scratch
-    SYM_CUDA(cudaMemsetAsync(ctr, 0, 64, s));
-    SYM_CUDA(cudaMemsetAsync(next_count, 0, sizeof(uint32_t), s));
-    MmRoundArgs A;
-    A.rp = g->row_ptr;
-    A.rp2 = nullptr;
-    A.ci = g->col_idx;
-    A.ci2 = nullptr;
-    A.hbits = nullptr;
-    A.dual = 0;
-    A.mate = mate;
-    A.pick_prev = pick_prev;
-    A.pick_cur = pick_cur;
-    A.in_list = frontier;
-    A.in_rev = 0;
-    A.in_cnt = count;
-    A.implicit_n = 0;
-    A.out_list = next;
-    A.out_cnt = next_count;
-    A.clear_cnt = ctr + 1;
-    A.huge = reinterpret_cast<int32_t *>(base + 64);
-    A.huge_cnt = ctr;
-    A.huge_clear = ctr + 2;
-    A.hist = nullptr;
-    A.round = 0;
-    A.k = stream_key(p->seed, TAG_EDGE, 0);
-    A.prof = nullptr;
-    A.row_base = g->v_begin;
-    const int grid = mm_round_grid();
-    if (round == 0) k_mm_round<false, true><<<grid, MM_THREADS, 0, s>>>(A);
-    else k_mm_round<true, true><<<grid, MM_THREADS, 0, s>>>(A);
-    SYM_LAUNCH_CHECK();
-    k_mm_huge<true><<<num_sms() * 2, MM_HUGE_THREADS, 0, s>>>(A);
-    SYM_LAUNCH_CHECK();
+    if (P.nl > 0) {
+        k_sh_mm_out<<<mm_shard_grid(P.nl), 256, 0, s>>>(w.mate, P.v0, P.v1, mate);
+        SYM_LAUNCH_CHECK();
+    }
+    if (stats) {
+        memcpy(stats->rounds, rounds, sizeof(rounds));
+        shard_stats_out(x, stats);
+        SYM_TRY(shard_count_boundary(P, x, &stats->boundary));
+    }
     return SYM_OK;
 }

@@ -387,54 +387,3 @@ int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const Spl
 
 }  // namespace sym
 
-// ------------------------------------------------------------------ sharded decomposition (C-ABI)
-using namespace sym;
-
-static int check_split_shard(const sym_graph_shard *g) {
-    if (!g) { set_error("shard is NULL"); return SYM_EINVAL; }
-    if (g->n_global < 0 || g->n_global >= ((int64_t)1 << 31) - 1 || g->v_begin < 0 || g->v_end < g->v_begin ||
-        g->v_end > g->n_global || g->nnz < 0) {
-        set_error("bad shard range: need 0 <= v_begin <= v_end <= n_global < 2^31 - 1, nnz >= 0");
-        return SYM_EINVAL;
-    }
-    if (g->v_end > g->v_begin && !g->row_ptr) { set_error("row_ptr is NULL"); return SYM_EINVAL; }
-    if (g->nnz > 0 && !g->col_idx) { set_error("col_idx is NULL"); return SYM_EINVAL; }
-    return SYM_OK;
-}
-
-extern "C" size_t sym_shard_decompose_workspace_bytes(const sym_graph_shard *g) {
-    if (check_split_shard(g) != SYM_OK) return 0;
-    Arena a;
-    SplitWs w;
-    carve_split_ws(a, g->v_end - g->v_begin, g->nnz, w);
-    return a.used + 256;
-}
-
-extern "C" int sym_shard_decompose(const sym_graph_shard *g, const sym_params *p, void *ws, size_t ws_bytes,
-                                   int64_t *row_ptr_in, int32_t *col_idx_in, int64_t *row_ptr_x, int32_t *col_idx_x,
-                                   sym_stream_t stream) {
-    SYM_TRY(check_split_shard(g));
-    if (!p) { set_error("params is NULL"); return SYM_EINVAL; }
-    if (p->kind != SYM_DECOMP_RAND && p->kind != SYM_DECOMP_NONE) {
-        set_error("sharded decomposition supports RAND (and NONE) only");
-        return SYM_EINVAL;
-    }
-    if (p->kind == SYM_DECOMP_RAND && (p->param < 1 || p->param > 65535)) {
-        set_error("RAND needs 1 <= p <= 65535");
-        return SYM_EINVAL;
-    }
-    if (!row_ptr_in || !row_ptr_x || (g->nnz > 0 && (!col_idx_in || !col_idx_x))) {
-        set_error("NULL output buffer");
-        return SYM_EINVAL;
-    }
-    const size_t need = sym_shard_decompose_workspace_bytes(g);
-    if (!ws || ws_bytes < need) { set_error("shard workspace too small"); return SYM_EWORKSPACE; }
-    Arena a;
-    a.base = (char *)(((uintptr_t)ws + 255) & ~(uintptr_t)255);
-    a.cap = ws_bytes - 256;
-    SplitWs w;
-    const int64_t nl = g->v_end - g->v_begin;
-    carve_split_ws(a, nl, g->nnz, w);
-    return run_split(Graph{nl, g->nnz, g->row_ptr, g->col_idx}, p->kind, p->param, p->seed, w, nullptr, row_ptr_in,
-                     col_idx_in, row_ptr_x, col_idx_x, nullptr, (cudaStream_t)stream, g->v_begin);
-}

@@ -73,19 +73,20 @@ def test_c5_rand8_mm_color(rmat27):
 
 
 def test_c5_sharded8_equals_single_gpu(rmat27):
-    """8 shards (the C5 multi-GPU layout) through the sharded kernels, exchanged in
-    process: bit-identical to the single-GPU calls (FIXED priorities are
-    schedule-independent)."""
+    """8 ranks (the C5 multi-GPU layout) through the library's sharded calls, one host
+    thread and local communicator per rank on this GPU: bit-identical to the
+    single-GPU calls (FIXED priorities are schedule-independent)."""
     from paper_conf_ipps_nayyaroddeengk17_b200 import sharded as S
     (rp, ci), _ = rmat27
     ref_I = sb.sym_mis(rp, ci, "degk", 2, SEED)
     ref_M = sb.sym_mm(rp, ci, "rand", 8, SEED)
     _free()
     shards = S.make_shards(rp, ci, 8)
-    out = S.sym_mis_sharded(shards, "degk", 2, SEED)
+    out = S.run_local(shards, "mis", "degk", 2, SEED)
     assert torch.equal(torch.cat(out), ref_I)
     del out
-    out = S.sym_mm_sharded(shards, "rand", 8, SEED)
+    _free()
+    out = S.run_local(shards, "mm", "rand", 8, SEED)
     assert torch.equal(torch.cat(out), ref_M)
     del out, shards
     _free()

@@ -68,9 +68,10 @@ def main():
            "note": "DRAM bytes = dram__bytes_read.sum + dram__bytes_write.sum per kernel class over the measured "
                    "step (the second of two); serialised replay, no cache flush: compare shares and bytes, "
                    "not absolute times", "classes": classes}
-    dst = os.path.join(ROOT, "profiles", f"{tag}_traffic.json")
-    with open(dst, "w") as f:
-        json.dump(res, f, indent=1)
+    for dst in (os.path.join(ROOT, "profiles", f"{tag}_traffic.json"),
+                os.path.join(ROOT, "gpurun_out", f"{tag}_traffic.json")):
+        with open(dst, "w") as f:
+            json.dump(res, f, indent=1)
     print(json.dumps(res, indent=1))
 
 

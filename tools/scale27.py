@@ -58,7 +58,7 @@ def main():
     del dR
     torch.cuda.empty_cache()
     shards = S.make_shards(rp, ci, 8)
-    out, ms_sh = timed(lambda: S.sym_mis_sharded(shards, "degk", 2, seed))
+    out, ms_sh = timed(lambda: S.run_local(shards, "mis", "degk", 2, seed))
     sh_equal = bool(torch.equal(torch.cat(out), I))
     del shards, out
     rec["ms"] = {"decompose_deg2": ms_dec, "mis_deg2": ms_mis, "color_deg2": ms_col, "decompose_rand8": ms_decr,
