@@ -24,6 +24,8 @@ import subprocess
 import numpy as np
 
 NONE, RAND, DEGK = 0, 1, 2
+# f1 variant flags (the same numbers as SYM_F_* in include/sym.h)
+F_PER_ROUND, F_CONFLICT_DROP, F_SPARSER_FIRST, F_LOWER_ONLY = 0x10, 0x20, 0x40, 0x80
 KINDS = {"none": NONE, "rand": RAND, "degk": DEGK}
 TAG_VERTEX, TAG_EDGE, TAG_RAND = 1, 2, 3
 
@@ -100,6 +102,8 @@ _SIGS = {
     "or_cert_col": (_I64, [_I64, _P, _P, _P, _P, _INT, _U64, _P]),
     "or_cert_col_rand": (_I64, [_I64, _P, _P, _U32, _U64, _P, _P]),
     "or_cert_flow": (_I64, [_INT, _I64, _P, _P, _INT, _U32, _U64, _P]),
+    "or_mis_ex": (None, [_I64, _P, _P, _INT, _U32, _U64, _U32, _P]),
+    "or_color_ex": (None, [_I64, _P, _P, _INT, _U32, _U64, _U32, _P]),
 }
 
 
@@ -184,10 +188,14 @@ def decompose(rp, ci, kind, param, seed):
 
 
 # ---------------------------------------------------------------- flows
-def mis(rp, ci, kind="none", param=0, seed=42):
+def mis(rp, ci, kind="none", param=0, seed=42, flags=0):
+    """MIS flows (or_mis); flags: the f1 variants (or_mis_ex)."""
     n, rp, ci = _graph(rp, ci)
     out = np.zeros(max(n, 1), np.uint8)
-    lib().or_mis(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), _ptr(out))
+    if flags:
+        lib().or_mis_ex(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), flags, _ptr(out))
+    else:
+        lib().or_mis(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), _ptr(out))
     return out[:n]
 
 
@@ -198,10 +206,14 @@ def mm(rp, ci, kind="none", param=0, seed=42):
     return out[:n]
 
 
-def color(rp, ci, kind="none", param=0, seed=42):
+def color(rp, ci, kind="none", param=0, seed=42, flags=0):
+    """COLOR flows (or_color); flags: the f1 variants (or_color_ex)."""
     n, rp, ci = _graph(rp, ci)
     out = np.zeros(max(n, 1), np.uint32)
-    lib().or_color(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), _ptr(out))
+    if flags:
+        lib().or_color_ex(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), flags, _ptr(out))
+    else:
+        lib().or_color(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), _ptr(out))
     return out[:n]
 
 

@@ -744,3 +744,187 @@ int64_t or_cert_flow(int problem, int64_t n, const int64_t *rp, const int32_t *c
     free(cls);
     return bad;
 }
+
+/* ------------------------------------------------------------------ §VAR variants */
+/* flag values of the variant contract (the same numbers as SYM_F_* in the C-ABI) */
+#define OR_F_PER_ROUND 0x10u      /* MIS: classic Luby -- priorities re-drawn every round */
+#define OR_F_CONFLICT_DROP 0x20u  /* MIS-RAND: MIS of the parts, drop the lower In end of In-In cross arcs */
+#define OR_F_SPARSER_FIRST 0x40u  /* MIS-RAND: the sparser of E[V\B], E[B] first */
+#define OR_F_LOWER_ONLY 0x80u     /* COLOR-RAND: V' = lower-priority endpoints only */
+
+/* LubyMIS as Luby states it ("uses randomization to break symmetry"), the
+   two-step synchronous round with FRESH priorities every round: in round r (0, 1, ..
+   within the phase) every undecided v of S draws pv_r(v) (stream key K(seed, VERTEX,
+   r)); the undecided local maxima of (pv_r, id) over their undecided S-neighbours join
+   I; then every undecided vertex with a neighbour that just joined I leaves.  st[]:
+   OR_UNDEC on S on entry. */
+static void luby_per_round(int64_t n, const int64_t *rp, const int32_t *ci, const uint8_t *inS, uint64_t seed,
+                           uint8_t *st) {
+    uint8_t *sel = (uint8_t *)calloc((size_t)(n > 0 ? n : 1), 1);
+    for (uint32_t r = 0;; r++) {
+        uint64_t key = or_stream_key(seed, OR_TAG_VERTEX, r);
+        int64_t undec = 0;
+        for (int64_t v = 0; v < n; v++) {        /* step 1: local maxima of the round's draw */
+            sel[v] = 0;
+            if (!inS[v] || st[v] != OR_UNDEC) continue;
+            undec++;
+            int best = 1;
+            for (int64_t e = rp[v]; e < rp[v + 1] && best; e++) {
+                int32_t w = ci[e];
+                if (inS[w] && st[w] == OR_UNDEC && vgreater(key, w, (int32_t)v)) best = 0;
+            }
+            sel[v] = (uint8_t)best;
+        }
+        if (!undec) break;
+        for (int64_t v = 0; v < n; v++)          /* they join I ... */
+            if (sel[v]) st[v] = OR_IN;
+        for (int64_t v = 0; v < n; v++) {        /* step 2: ... and their neighbours leave */
+            if (!inS[v] || st[v] != OR_UNDEC) continue;
+            for (int64_t e = rp[v]; e < rp[v + 1]; e++)
+                if (inS[ci[e]] && sel[ci[e]]) { st[v] = OR_OUT; break; }
+        }
+    }
+    free(sel);
+}
+
+/* the MIS of G[S] a flow step computes: LF-MIS (FIXED priorities) or per-round Luby */
+static void mis_step(int64_t n, const int64_t *rp, const int32_t *ci, const uint8_t *inS, uint64_t seed,
+                     uint32_t flags, uint8_t *st) {
+    if (flags & OR_F_PER_ROUND) luby_per_round(n, rp, ci, inS, seed, st);
+    else lf_mis(n, rp, ci, inS, or_stream_key(seed, OR_TAG_VERTEX, 0), st);
+}
+
+/* X = the vertices of `from` none of whose neighbours in `by` is In (the others are
+   removed: Out) -- "remove from G vertices that are in I or have a neighbour in I" */
+static void reduce(int64_t n, const int64_t *rp, const int32_t *ci, const uint8_t *from, const uint8_t *by,
+                   uint8_t *st, uint8_t *X) {
+    for (int64_t v = 0; v < n; v++) {
+        X[v] = 0;
+        if (!from[v]) continue;
+        int hit = 0;
+        for (int64_t e = rp[v]; e < rp[v + 1] && !hit; e++) hit = by[ci[e]] && st[ci[e]] == OR_IN;
+        if (hit) st[v] = OR_OUT;
+        else X[v] = 1;
+    }
+}
+
+/* MIS flows with the f1 variants (flags 0: exactly or_mis).
+   PER_ROUND: every MIS step of the flow (NONE; DEGK's I_L, I_R; RAND's I_A, I_B) is
+     per-round Luby instead of LF-MIS; the flow is unchanged.
+   RAND + CONFLICT_DROP (reading G10 (i)): I_P = MIS of the induced subgraphs (every
+     intra arc, all vertices); D = the In vertices with a higher-priority In cross
+     neighbour; I' = I_P \ D (independent in G); X = V \ N[I'] (the vertices not in I'
+     without a neighbour in I'); I_B = MIS(X, E[X]); I = I' u I_B.
+   RAND + SPARSER_FIRST ("I_A and I_B can be computed in any order. We
+     base our decision on which of the two graphs U G_i or G_{k+1} is sparser";
+     reading G10 (ii)): B = vertices with a cross arc; if G_{k+1} has fewer arcs than
+     U G_i, the boundary goes first -- I_1 = MIS(B, E[B]) (all arcs among B, so that
+     I_1 is independent in G), X = interior vertices without a neighbour in I_1,
+     I_2 = MIS(X, E[X]), I = I_1 u I_2 -- else the standard order. */
+void or_mis_ex(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t param, uint64_t seed,
+               uint32_t flags, uint8_t *in_set) {
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    uint8_t *st = (uint8_t *)calloc(nn, 1), *S = (uint8_t *)calloc(nn, 1), *X = (uint8_t *)calloc(nn, 1);
+    uint8_t *B = (uint8_t *)calloc(nn, 1);
+    uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+    or_classes(n, rp, kind, param, seed, cls);
+    if (kind == OR_NONE) {
+        for (int64_t v = 0; v < n; v++) S[v] = 1;
+        mis_step(n, rp, ci, S, seed, flags, st);
+    } else if (kind == OR_DEGK) {
+        uint8_t *H = (uint8_t *)calloc(nn, 1);
+        for (int64_t v = 0; v < n; v++) {
+            S[v] = cls[v] == 0;
+            H[v] = cls[v] == 1;
+        }
+        mis_step(n, rp, ci, S, seed, flags, st);  /* I_L */
+        reduce(n, rp, ci, H, S, st, X);           /* X = V_H \ N(I_L) */
+        mis_step(n, rp, ci, X, seed, flags, st);  /* I_R */
+        free(H);
+    } else if (flags & OR_F_CONFLICT_DROP) {
+        uint8_t *ip = (uint8_t *)calloc(nn, 1);
+        /* I_P: the MIS of each part G[V_i] = the MIS of the union of the induced
+           subgraphs; computed part by part (every part is an S of its own) */
+        for (uint32_t part = 0; part < param; part++) {
+            int any = 0;
+            for (int64_t v = 0; v < n; v++) any |= (S[v] = cls[v] == part);
+            if (any) mis_step(n, rp, ci, S, seed, flags, st);
+        }
+        for (int64_t v = 0; v < n; v++) {         /* D: lower In end of an In-In cross arc */
+            ip[v] = st[v] == OR_IN;
+            for (int64_t e = rp[v]; e < rp[v + 1] && ip[v]; e++) {
+                int32_t w = ci[e];
+                if (cls[w] != cls[v] && st[w] == OR_IN && vgreater(or_stream_key(seed, OR_TAG_VERTEX, 0), w, (int32_t)v))
+                    ip[v] = 0;
+            }
+        }
+        for (int64_t v = 0; v < n; v++) {
+            st[v] = ip[v] ? OR_IN : OR_UNDEC;
+            S[v] = !ip[v];
+        }
+        reduce(n, rp, ci, S, ip, st, X);          /* X = V \ N[I'] */
+        mis_step(n, rp, ci, X, seed, flags, st);  /* I_B */
+        free(ip);
+    } else {
+        for (int64_t v = 0; v < n; v++)
+            for (int64_t e = rp[v]; e < rp[v + 1]; e++)
+                if (cls[ci[e]] != cls[v]) { B[v] = 1; break; }
+        int64_t a_intra = 0, a_cross = 0;  /* arcs of U G_i and of G_{k+1} */
+        for (int64_t v = 0; v < n; v++)
+            for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+                a_intra += cls[ci[e]] == cls[v];
+                a_cross += cls[ci[e]] != cls[v];
+            }
+        int bfirst = (flags & OR_F_SPARSER_FIRST) && a_cross < a_intra;
+        uint8_t *first = (uint8_t *)calloc(nn, 1), *rest = (uint8_t *)calloc(nn, 1);
+        for (int64_t v = 0; v < n; v++) {
+            first[v] = bfirst ? B[v] : !B[v];
+            rest[v] = !first[v];
+        }
+        mis_step(n, rp, ci, first, seed, flags, st);  /* I_A (or I_1 = MIS(G[B])) */
+        reduce(n, rp, ci, rest, first, st, X);
+        mis_step(n, rp, ci, X, seed, flags, st);      /* I_B on the reduced graph */
+        free(first);
+        free(rest);
+    }
+    for (int64_t v = 0; v < n; v++) in_set[v] = st[v] == OR_IN;
+    free(st);
+    free(S);
+    free(X);
+    free(B);
+    free(cls);
+}
+
+/* COLOR flows with the f1 variant (flags 0: exactly or_color).
+   RAND + LOWER_ONLY: V' = the LOWER-priority endpoint of every cross edge whose ends
+   share a C_IS colour (instead of both, reading C3); V' is recoloured first-fit in
+   priority order against all of G, as in or_color. */
+void or_color_ex(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t param, uint64_t seed,
+                 uint32_t flags, uint32_t *colour) {
+    if (!(kind == OR_RAND && (flags & OR_F_LOWER_ONLY))) {
+        or_color(n, rp, ci, kind, param, seed, colour);
+        return;
+    }
+    uint64_t key = or_stream_key(seed, OR_TAG_VERTEX, 0);
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+    uint8_t *S = (uint8_t *)calloc(nn, 1);
+    or_classes(n, rp, kind, param, seed, cls);
+    for (int64_t v = 0; v < n; v++) {
+        colour[v] = 0;
+        S[v] = 1;
+    }
+    lf_col(n, rp, ci, S, cls, 1, key, colour);           /* C_IS on the induced subgraphs */
+    for (int64_t v = 0; v < n; v++) {                    /* V' = lower ends of conflicts */
+        S[v] = 0;
+        for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+            int32_t w = ci[e];
+            if (cls[w] != cls[v] && colour[w] == colour[v] && vgreater(key, w, (int32_t)v)) { S[v] = 1; break; }
+        }
+    }
+    for (int64_t v = 0; v < n; v++)
+        if (S[v]) colour[v] = 0;
+    lf_col(n, rp, ci, S, cls, 0, key, colour);           /* recolour V' against G */
+    free(cls);
+    free(S);
+}

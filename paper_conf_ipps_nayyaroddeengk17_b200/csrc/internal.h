@@ -196,6 +196,7 @@ struct MmWs {
     unsigned long long *huge_best = nullptr;
     int64_t huge_cap = 0;
     unsigned long long *gmax = nullptr;  // round 0: maxima of rows crossing tiles
+    uint32_t *mbits = nullptr;           // matched bitmap
 };
 
 struct ColorWs {
@@ -274,6 +275,7 @@ int64_t shard_block(int64_t n, int nranks);
 int shard_check(const sym_graph_shard *g, const sym_params *p, const sym_comm *c, ShardPlan *plan);
 void carve_shard_common(Arena &a, const ShardPlan &P, size_t entry, ShardCtx &x);
 int shard_boundary(const ShardPlan &P, ShardCtx &x, cudaStream_t s);
+// (SH_MIS: st; SH_MM: mate, pick and, in `color`, the matched bitmap; SH_COLOR: color)
 int shard_exchange(const ShardPlan &P, ShardCtx &x, int par, int problem, uint8_t *st, int32_t *mate, int32_t *pick,
                    uint32_t *color, uint64_t *front);
 int shard_gather_hbits(const ShardPlan &P, ShardCtx &x);

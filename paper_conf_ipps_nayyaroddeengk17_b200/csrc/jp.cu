@@ -78,12 +78,6 @@ constexpr uint32_t JP_NOTBUILT = 0xffffffffu;
 #ifndef SYM_JP_PUSH_FILTER0
 #define SYM_JP_PUSH_FILTER0 0  // 1: also filter colours 1..32 (a load on the chain; 26.3 vs 26.05 ms)
 #endif
-#ifndef SYM_JR_POLL
-#define SYM_JR_POLL 0
-#endif
-#ifndef SYM_JR_BARRIER_RED
-#define SYM_JR_BARRIER_RED 1  // grid barrier: 1 = release-RED arrival + polling the counter (29.5 vs 30.9 ms)
-#endif
 constexpr int JP_BUILD = 256;    // phase B: higher entries per watch-list build task
 constexpr uint32_t JP_HBITS = 27;  // hot.w = offset of the extra bitmap words | min(R, 31) << 27
 constexpr uint32_t JP_HMASK = (1u << JP_HBITS) - 1u;
@@ -727,7 +721,6 @@ __device__ __forceinline__ void st_release_u32(uint32_t *p, uint32_t v) {
 
 struct JrCtl {
     uint32_t *arr;     // barrier arrivals (monotone)
-    uint32_t *gen;     // index of the last completed barrier, published by its last arriver
     uint32_t *levels;  // out: rounds run
     uint32_t max_rounds;
 };
@@ -743,28 +736,12 @@ __device__ __forceinline__ void grid_sync(const JrCtl &C, uint32_t &k, const uin
     __syncthreads();
     k++;
     if (threadIdx.x == 0) {
-#if SYM_JR_BARRIER_RED
-        // arrival = one release reduction (no return); every CTA polls the counter
+        // arrival = one release reduction (no return); every CTA polls the counter (a
+        // polling back-off of 100-1000 ns changed nothing: profiles/r2h_jp_async_sweep.json)
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(C.arr) : "memory");
         const uint32_t target = k * gridDim.x;
-#if SYM_JR_POLL == 1  // relaxed polling, one acquire fence at the end
-        while (ld_volatile_u32(C.arr) < target) {
-        }
-        asm volatile("fence.acq_rel.gpu;" ::: "memory");
-#elif SYM_JR_POLL == 2  // acquire polling with a short back-off
-        while (ld_acquire_u32(C.arr) < target) __nanosleep(40);
-#else
         while (ld_acquire_u32(C.arr) < target) {
         }
-#endif
-#else
-        __threadfence();
-        const uint32_t old = atomicAdd(C.arr, 1u);
-        if (old + 1u == k * gridDim.x) st_release_u32(C.gen, k);
-        else
-            while (ld_acquire_u32(C.gen) < k) {
-            }
-#endif
         if (p0) sm[0] = __ldcg(p0);
         if (p1) sm[1] = __ldcg(p1);
         if (p2) sm[2] = __ldcg(p2);
@@ -795,9 +772,144 @@ __device__ __forceinline__ void nb_load(const JpArgs &A, uint32_t e, uint32_t q,
     w = q == 0u ? s.z : (q < R5 ? (s.w & JP_HMASK) : 0u);
 }
 
-// Phase A of round r: every active vertex (count <= JP_WATCH) checks its watch list
-// (the higher neighbours that were uncoloured when the list was built; every other
-// higher neighbour's colour is already in v's bitmap, so it cannot equal m).  A
+// One check of vertex h (compact id; act = the lane holds a vertex): the early-commit
+// rule over its watch list (the higher neighbours that were uncoloured -- or, in the
+// asynchronous tail, not yet fully pushed -- when the list was built; every other
+// higher neighbour's colour is already in h's bitmap, so it cannot equal m).  The
+// first JP_LANE_CHECKS entries are checked by the lane (all loads in flight), the rest
+// by the whole warp, 32 per step, resuming at the last blocker when m is unchanged.
+// Must be called by all lanes of the warp.
+struct JpLane {
+    uint32_t h, R, hd, ld, wc, pos, lm, m;
+    uint64_t off;
+    int state;  // 0 checking, 1 passed, 2 failed (memo pos/lm), 3 idle, 5 watch list not built
+};
+
+__device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_in, JpLane &L,
+                                         unsigned long long &bytes) {
+    const int lane = lane_id();
+    uint32_t h = h_in, R = 1, hd = 0, ld = 0, wc = 0, pos = 0, lm = 0, m = 1;
+    uint64_t off = 0;
+    int state = 3;
+    if (act) {
+        const uint4 m0 = __ldcg(A.meta + 2 * h), m1 = __ldcg(A.meta + 2 * h + 1);
+        R = m0.x;
+        hd = m0.y;
+        ld = m0.z;
+        wc = m0.w;
+        pos = m1.x;
+        lm = m1.y;
+        off = meta_off(m1);
+        bytes += 40;
+        if (wc == JP_NOTBUILT) {
+            state = 5;
+        } else {
+            state = 0;
+            const uint4 hs = __ldcg(A.hot + h);
+            const uint32_t z0 = ~hs.z;
+            if (z0) {
+                m = __ffs(z0);
+            } else {  // colours > 32
+                const uint32_t *xw = A.xb + (hs.w & JP_HMASK);
+                for (uint32_t k = 1; k < R; k++) {
+                    const uint32_t z = ~__ldcg(xw + k - 1);
+                    if (z) {
+                        m = k * 32 + __ffs(z);
+                        break;
+                    }
+                }
+                if (m == 1) m = R * 32 + 1;  // unreachable: a zero lies within cap bits
+            }
+        }
+    }
+    const uint32_t q = (m - 1) >> 5, bit = (m - 1) & 31;
+    uint32_t j = (lm == m && pos < wc) ? pos : 0u;  // m unchanged: resume at the last blocker
+    // ---- lane: the first JP_LANE_CHECKS entries (all loads of a stage in flight)
+    if (state == 0) {
+        uint32_t e[JP_LANE_CHECKS], c[JP_LANE_CHECKS], w[JP_LANE_CHECKS], r5[JP_LANE_CHECKS];
+#pragma unroll
+        for (int u = 0; u < JP_LANE_CHECKS; u++) e[u] = j + u < wc ? __ldcg(A.lst + off + j + u) : 0u;
+#pragma unroll
+        for (int u = 0; u < JP_LANE_CHECKS; u++) {
+            c[u] = 1u;
+            w[u] = 0u;
+            r5[u] = 0u;
+            if (j + u < wc) nb_load(A, e[u], q, c[u], w[u], r5[u]);
+        }
+        if (q > 0) {
+#pragma unroll
+            for (int u = 0; u < JP_LANE_CHECKS; u++)
+                if (j + u < wc && c[u] == 0u && q < r5[u]) w[u] = __ldcg(A.xb + w[u] + q - 1);
+        }
+#pragma unroll
+        for (int u = 0; u < JP_LANE_CHECKS; u++) {
+            if (state == 0) {
+                if (j >= wc) {
+                    state = 1;
+                } else if (!nb_ok(A, e[u], c[u], w[u], r5[u], m, q, bit)) {
+                    state = 2;
+                    pos = j;
+                    lm = m;
+                } else {
+                    j++;
+                }
+            }
+        }
+        if (state == 0 && j >= wc) state = 1;
+        bytes += 12ull * min(wc, (uint32_t)JP_LANE_CHECKS);
+    }
+    // ---- warp: the rest of a list (<= JP_WLIST entries: at most two steps)
+    unsigned need = __ballot_sync(FULL, state == 0);
+    while (need) {
+        const int src = __ffs(need) - 1;
+        need &= need - 1;
+        uint32_t wj = __shfl_sync(FULL, j, src);
+        const uint32_t wwc = __shfl_sync(FULL, wc, src), wm = __shfl_sync(FULL, m, src);
+        const uint64_t woff = __shfl_sync(FULL, off, src);
+        const uint32_t wq = (wm - 1) >> 5, wbit = (wm - 1) & 31;
+        int wstate = 0;
+        uint32_t wpos = 0;
+        while (wstate == 0) {
+            const uint32_t jj = wj + lane;
+            bool ok = true;
+            if (jj < wwc) {
+                const uint32_t eu = __ldcg(A.lst + woff + jj);
+                uint32_t cu, wu, ru;
+                nb_load(A, eu, wq, cu, wu, ru);
+                if (wq > 0 && cu == 0u && wq < ru) wu = __ldcg(A.xb + wu + wq - 1);
+                ok = nb_ok(A, eu, cu, wu, ru, wm, wq, wbit);
+            }
+            const unsigned fails = __ballot_sync(FULL, !ok);
+            if (fails) {
+                wstate = 2;
+                wpos = wj + __ffs(fails) - 1;
+            } else {
+                wj += 32;
+                if (wj >= wwc) wstate = 1;
+            }
+            bytes += lane == 0 ? 384ull : 0ull;
+        }
+        if (lane == src) {
+            state = wstate;
+            if (wstate == 2) {
+                pos = wpos;
+                lm = m;
+            }
+        }
+    }
+    L.h = h;
+    L.R = R;
+    L.hd = hd;
+    L.ld = ld;
+    L.wc = wc;
+    L.pos = pos;
+    L.lm = lm;
+    L.m = m;
+    L.off = off;
+    L.state = state;
+}
+
+// Phase A of round r: every active vertex (count <= JP_WATCH) is checked (jp_check); a
 // vertex whose higher list is longer than JP_WLIST asks phase B for its watch list
 // first.
 __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t cnt, int64_t warp_g,
@@ -812,116 +924,11 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
     for (int64_t it = 0; it < cnt; it += nwarps * 32) {
         const int64_t i = it + (spread ? (int64_t)lane * nwarps + warp_g : warp_g * 32 + lane);
         const bool act = i < cnt;
-        uint32_t h = 0, R = 1, hd = 0, ld = 0, wc = 0, pos = 0, lm = 0, m = 1;
-        uint64_t off = 0;
-        int state = 3;  // 0 checking, 1 passed, 2 failed (memo), 3 idle, 5 build request
-        if (act) {
-            h = __ldcg(U + i);
-            const uint4 m0 = __ldcg(A.meta + 2 * h), m1 = __ldcg(A.meta + 2 * h + 1);
-            R = m0.x;
-            hd = m0.y;
-            ld = m0.z;
-            wc = m0.w;
-            pos = m1.x;
-            lm = m1.y;
-            off = meta_off(m1);
-            bytes += 40;
-            if (wc == JP_NOTBUILT) {
-                state = 5;
-            } else {
-                state = 0;
-                const uint4 hs = __ldcg(A.hot + h);
-                const uint32_t z0 = ~hs.z;
-                if (z0) {
-                    m = __ffs(z0);
-                } else {  // colours > 32
-                    const uint32_t *xw = A.xb + (hs.w & JP_HMASK);
-                    for (uint32_t k = 1; k < R; k++) {
-                        const uint32_t z = ~__ldcg(xw + k - 1);
-                        if (z) {
-                            m = k * 32 + __ffs(z);
-                            break;
-                        }
-                    }
-                    if (m == 1) m = R * 32 + 1;  // unreachable: a zero lies within cap bits
-                }
-            }
-        }
-        const uint32_t q = (m - 1) >> 5, bit = (m - 1) & 31;
-        uint32_t j = (lm == m && pos < wc) ? pos : 0u;  // m unchanged: resume at the last blocker
-        // ---- lane: the first JP_LANE_CHECKS entries (all loads of a stage in flight)
-        if (state == 0) {
-            uint32_t e[JP_LANE_CHECKS], c[JP_LANE_CHECKS], w[JP_LANE_CHECKS], r5[JP_LANE_CHECKS];
-#pragma unroll
-            for (int u = 0; u < JP_LANE_CHECKS; u++) e[u] = j + u < wc ? __ldcg(A.lst + off + j + u) : 0u;
-#pragma unroll
-            for (int u = 0; u < JP_LANE_CHECKS; u++) {
-                c[u] = 1u;
-                w[u] = 0u;
-                r5[u] = 0u;
-                if (j + u < wc) nb_load(A, e[u], q, c[u], w[u], r5[u]);
-            }
-            if (q > 0) {
-#pragma unroll
-                for (int u = 0; u < JP_LANE_CHECKS; u++)
-                    if (j + u < wc && c[u] == 0u && q < r5[u]) w[u] = __ldcg(A.xb + w[u] + q - 1);
-            }
-#pragma unroll
-            for (int u = 0; u < JP_LANE_CHECKS; u++) {
-                if (state == 0) {
-                    if (j >= wc) {
-                        state = 1;
-                    } else if (!nb_ok(A, e[u], c[u], w[u], r5[u], m, q, bit)) {
-                        state = 2;
-                        pos = j;
-                        lm = m;
-                    } else {
-                        j++;
-                    }
-                }
-            }
-            if (state == 0 && j >= wc) state = 1;
-            bytes += 12ull * min(wc, (uint32_t)JP_LANE_CHECKS);
-        }
-        // ---- warp: the rest of a list (<= JP_WLIST entries: at most two steps)
-        unsigned need = __ballot_sync(FULL, state == 0);
-        while (need) {
-            const int src = __ffs(need) - 1;
-            need &= need - 1;
-            uint32_t wj = __shfl_sync(FULL, j, src);
-            const uint32_t wwc = __shfl_sync(FULL, wc, src), wm = __shfl_sync(FULL, m, src);
-            const uint64_t woff = __shfl_sync(FULL, off, src);
-            const uint32_t wq = (wm - 1) >> 5, wbit = (wm - 1) & 31;
-            int wstate = 0;
-            uint32_t wpos = 0;
-            while (wstate == 0) {
-                const uint32_t jj = wj + lane;
-                bool ok = true;
-                if (jj < wwc) {
-                    const uint32_t eu = __ldcg(A.lst + woff + jj);
-                    uint32_t cu, wu, ru;
-                    nb_load(A, eu, wq, cu, wu, ru);
-                    if (wq > 0 && cu == 0u && wq < ru) wu = __ldcg(A.xb + wu + wq - 1);
-                    ok = nb_ok(A, eu, cu, wu, ru, wm, wq, wbit);
-                }
-                const unsigned fails = __ballot_sync(FULL, !ok);
-                if (fails) {
-                    wstate = 2;
-                    wpos = wj + __ffs(fails) - 1;
-                } else {
-                    wj += 32;
-                    if (wj >= wwc) wstate = 1;
-                }
-                bytes += lane == 0 ? 384ull : 0ull;
-            }
-            if (lane == src) {
-                state = wstate;
-                if (wstate == 2) {
-                    pos = wpos;
-                    lm = m;
-                }
-            }
-        }
+        JpLane L;
+        jp_check(A, act, act ? __ldcg(U + i) : 0u, L, bytes);
+        const uint32_t h = L.h, hd = L.hd, ld = L.ld, pos = L.pos, lm = L.lm, m = L.m;
+        const uint64_t off = L.off;
+        const int state = L.state;
         // ---- outcome
         const bool pass = state == 1, stay = state == 2 || state == 5;
         if (pass) A.hot[h].x = m;
@@ -973,9 +980,9 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
 // bit and one higher neighbour less to wait for.  The push that brings a count to
 // JP_WATCH activates the neighbour (next round's list).  Each stage's loads/atomics
 // are in flight together.
-template <int K>
-__device__ __forceinline__ void jp_push(const JpArgs &A, uint32_t r, const uint32_t (&e)[K], bool (&act)[K],
-                                        uint32_t q, uint32_t bit) {
+template <int K, class Activate>
+__device__ __forceinline__ void jp_push(const JpArgs &A, const uint32_t (&e)[K], bool (&act)[K], uint32_t q,
+                                        uint32_t bit, const Activate &activate) {
     uint32_t old[K], x[K];
 #pragma unroll
     for (int u = 0; u < K; u++) {  // colour, R field and extra-word offset in one 16-B load
@@ -1009,13 +1016,19 @@ __device__ __forceinline__ void jp_push(const JpArgs &A, uint32_t r, const uint3
             if (x[u] != 0xffffffffu) atomicOr(A.xb + x[u] + q - 1, 1u << bit);
     }
 #pragma unroll
-    for (int u = 0; u < K; u++) {
-        if (act[u] && old[u] == JP_WATCH + 1u) {
-            const uint32_t slot = atomicAdd(A.ucnt + (r + 1) % 3, 1u);
-            A.ul[(r + 1) & 1][slot] = e[u];
-        }
-    }
+    for (int u = 0; u < K; u++)
+        if (act[u] && old[u] == JP_WATCH + 1u) activate(e[u]);
 }
+
+// round mode: an activated vertex joins round r+1's list
+struct JpNextList {
+    const JpArgs &A;
+    uint32_t r;
+    __device__ __forceinline__ void operator()(uint32_t e) const {
+        const uint32_t slot = atomicAdd(A.ucnt + (r + 1) % 3, 1u);
+        A.ul[(r + 1) & 1][slot] = e;
+    }
+};
 
 // Phase B of round r: push the new colours; build the requested watch lists
 __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, uint32_t cnt, uint32_t nbt,
@@ -1036,7 +1049,7 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, uint32_t
                 act[u] = u < (int)tk.z;
                 e[u] = act[u] ? __ldcs(A.lst + s0 + u) : 0u;
             }
-            jp_push<JP_PUSH_LANE>(A, r, e, act, q, bit);
+            jp_push<JP_PUSH_LANE>(A, e, act, q, bit, JpNextList{A, r});
             bytes += 4ull * tk.z;
         }
         unsigned bigm = __ballot_sync(FULL, tk.z > JP_PUSH_LANE);
@@ -1054,7 +1067,7 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, uint32_t
                 act[u] = u * 32 + lane < (int)wn;
                 e[u] = act[u] ? __ldcs(A.lst + ws + u * 32 + lane) : 0u;
             }
-            jp_push<K>(A, r, e, act, q, bit);
+            jp_push<K>(A, e, act, q, bit, JpNextList{A, r});
             bytes += lane == 0 ? 4ull * wn : 0ull;
         }
     }
@@ -1356,7 +1369,6 @@ static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t 
     SYM_TRY(jp_build(f, w, A, color, rp, ci, inS, list0, cnt0, implicit_n, rounds_ctr));
     JrCtl C;
     C.arr = w.sync;
-    C.gen = w.sync + 1;
     C.levels = w.sync + 33;
     C.max_rounds = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
     // barriers (2 per round) x grid must not overflow the arrival word

@@ -4,6 +4,9 @@
 //   -> OUT  if some phase neighbour is IN,
 //   -> IN   if no undecided phase neighbour has a larger (pv, id) key,
 //   else stays undecided and is appended to the next frontier.
+// Only HIGHER neighbours' statuses are gathered: a lower neighbour w turns In only when
+// every higher neighbour of w -- v among them -- is Out, so none is In while v is
+// undecided (this halves the status gathers).
 // Status moves only UNDEC -> {IN, OUT}, and v turns IN only when every higher
 // neighbour is final-OUT, so decisions may be taken in place and read by other
 // threads of the same round: any interleaving yields the lexicographically-first
@@ -72,13 +75,16 @@ __device__ __forceinline__ int mis_scan_small(const MisRoundArgs &A, int64_t b, 
     uint8_t s[MIS_SMALL];
 #pragma unroll
     for (int u = 0; u < MIS_SMALL; u++) w[u] = (b + u < e) ? (uint32_t)__ldcs(A.ci + b + u) : 0u;
+    // only higher neighbours can decide v: a lower neighbour turns In only once every
+    // higher neighbour of it -- v included -- is Out, so while v is undecided none is In
 #pragma unroll
-    for (int u = 0; u < MIS_SMALL; u++) s[u] = (b + u < e && mis_in_phase(A, w[u])) ? A.st[w[u]] : ST_OUT;
+    for (int u = 0; u < MIS_SMALL; u++)
+        s[u] = (b + u < e && vkey(A.k, w[u]) > kv && mis_in_phase(A, w[u])) ? A.st[w[u]] : ST_OUT;
     bool in = false, blk = false;
 #pragma unroll
     for (int u = 0; u < MIS_SMALL; u++) {
         in |= s[u] == ST_IN;
-        blk |= (s[u] == ST_UNDEC) && (vkey(A.k, w[u]) > kv);
+        blk |= s[u] == ST_UNDEC;
     }
     lb += 4 * (unsigned long long)(e - b);
     return in ? R_OUT : (blk ? R_BLK : R_IN);
@@ -131,10 +137,10 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
                 bool fin = false, fblk = false;
 #pragma unroll
                 for (int u = 0; u < 4; u++) {
-                    if (ok[u] && mis_in_phase(A, w[u])) {
+                    if (ok[u] && vkey(A.k, w[u]) > wk && mis_in_phase(A, w[u])) {  // higher neighbours only
                         uint8_t sw = A.st[w[u]];
                         fin |= sw == ST_IN;
-                        fblk |= (sw == ST_UNDEC) && (vkey(A.k, w[u]) > wk);
+                        fblk |= sw == ST_UNDEC;
                     }
                 }
                 if (__any_sync(FULL, fin)) { r = R_OUT; break; }
@@ -183,10 +189,10 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
             }
 #pragma unroll
             for (int u = 0; u < 4; u++) {
-                if (ok[u] && mis_in_phase(A, w[u])) {
+                if (ok[u] && vkey(A.k, w[u]) > kv && mis_in_phase(A, w[u])) {  // higher neighbours only
                     uint8_t sw = A.st[w[u]];
                     fin |= sw == ST_IN;
-                    fblk |= (sw == ST_UNDEC) && (vkey(A.k, w[u]) > kv);
+                    fblk |= sw == ST_UNDEC;
                 }
             }
             if (__syncthreads_or(fin)) { r = R_OUT; break; }

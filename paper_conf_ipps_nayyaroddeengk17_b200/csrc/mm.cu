@@ -31,6 +31,7 @@ struct MmRoundArgs {
     const uint32_t *hbits;
     int dual;
     int32_t *mate;
+    uint32_t *mbits;  // matched bitmap (1 bit per vertex, L2-resident): the liveness gathers
     const int32_t *pick_prev;
     int32_t *pick_cur;
     const int32_t *in_list;
@@ -51,8 +52,12 @@ struct MmRoundArgs {
 };
 // algorithmic bytes: 4 B per column word loaded; per active vertex the
 // row_ptr pair (16 B) and the pick write (4 B); per resolved vertex the two pick
-// reads (8 B) and, if matched, the mate write (4 B).  Neighbour mate gathers hit the
-// L2-resident mate array and count 0 HBM bytes.
+// reads (8 B) and, if matched, the mate write (4 B).  Neighbour liveness is one bit of
+// the matched bitmap (n/8 bytes: 2 MB at R-MAT s24, L2-resident; the 4-B mate array is
+// 67 MB) and counts 0 HBM bytes.
+
+__device__ __forceinline__ bool mm_matched(const uint32_t *mbits, uint32_t v) { return (mbits[v >> 5] >> (v & 31)) & 1u; }
+__device__ __forceinline__ void mm_set_matched(uint32_t *mbits, uint32_t v) { atomicOr(mbits + (v >> 5), 1u << (v & 31)); }
 
 __device__ __forceinline__ void mm_row(const MmRoundArgs &A, int32_t u, int64_t &b, int64_t &e, const int32_t *&ci) {
     if (A.dual && ((A.hbits[u >> 5] >> (u & 31)) & 1u)) {
@@ -100,13 +105,14 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
             nb += 8;
             if (p >= 0 && A.pick_prev[p] == u) {
                 A.mate[u] = p;
+                mm_set_matched(A.mbits, (uint32_t)u);
                 A.pick_cur[u] = -1;
                 active = false;
                 nb += 4;
             } else if (A.mate[u] >= 0) {  // defensive: never re-pick a matched vertex
                 A.pick_cur[u] = -1;
                 active = false;
-            } else if (MATE && p >= 0 && A.mate[p] < 0) {
+            } else if (MATE && p >= 0 && !mm_matched(A.mbits, (uint32_t)p)) {
                 // u's pick is still unmatched: the live set only shrinks and the keys are
                 // fixed, so it is still u's heaviest live edge -- no rescan.  A stale read
                 // (p matched in this very round) keeps a dead pick one more round, as a
@@ -134,7 +140,7 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
 #pragma unroll
             for (int q = 0; q < MM_SMALL; q++) w[q] = (q < d) ? (uint32_t)__ldcs(ci + b + q) : 0u;
 #pragma unroll
-            for (int q = 0; q < MM_SMALL; q++) live[q] = (q < d) && (!MATE || A.mate[w[q]] < 0);
+            for (int q = 0; q < MM_SMALL; q++) live[q] = (q < d) && (!MATE || !mm_matched(A.mbits, w[q]));
 #pragma unroll
             for (int q = 0; q < MM_SMALL; q++) {
                 if (live[q]) {
@@ -166,7 +172,7 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
                 }
 #pragma unroll
                 for (int q = 0; q < 4; q++) {
-                    if (ok[q] && (!MATE || A.mate[w[q]] < 0)) {
+                    if (ok[q] && (!MATE || !mm_matched(A.mbits, w[q]))) {
                         uint64_t kk = ekey(A.k, (uint32_t)wu, w[q]);
                         if (!lh || kk > lb) lb = kk;
                         lh = true;
@@ -223,7 +229,7 @@ __global__ void __launch_bounds__(MM_HUGE_THREADS) k_mm_huge(MmRoundArgs A) {
             }
 #pragma unroll
             for (int q = 0; q < 4; q++) {
-                if (ok[q] && (!MATE || A.mate[w[q]] < 0)) {
+                if (ok[q] && (!MATE || !mm_matched(A.mbits, w[q]))) {
                     uint64_t kk = ekey(A.k, (uint32_t)u, w[q]);
                     if (!lh || kk > lb) lb = kk;
                     lh = true;
@@ -297,6 +303,7 @@ void carve_mm_ws(Arena &a, int64_t n, int64_t nnz, MmWs &w) {
     w.huge_cap = nnz / MM_BUDGET + 2;
     w.huge = reinterpret_cast<int64_t *>(a.take<int32_t>((size_t)w.huge_cap));
     w.gmax = a.take<unsigned long long>((size_t)n + 1);
+    w.mbits = a.take<uint32_t>((size_t)(n + 31) / 32 + 1);
 }
 
 struct MmPhase {
@@ -361,6 +368,7 @@ static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph
             A.hbits = f.hbits;
             A.dual = ph.dual;
             A.mate = mate;
+            A.mbits = w.mbits;
             A.pick_prev = w.pick[(r + 1) & 1];
             A.pick_cur = w.pick[r & 1];
             if (r == 0) {
@@ -439,6 +447,7 @@ int run_mm(const FlowArgs &f, MmWs &w, int32_t *mate) {
     cudaStream_t s = f.stream;
     Ctl *ctl = f.ctl;
     SYM_CUDA(cudaMemsetAsync(mate, 0xff, sizeof(int32_t) * (size_t)g.n, s));
+    SYM_CUDA(cudaMemsetAsync(w.mbits, 0, sizeof(uint32_t) * ((size_t)(g.n + 31) / 32 + 1), s));
     const int kind = f.p.kind;
     MmPhase ph{};
     if (kind == SYM_DECOMP_NONE) {
@@ -530,6 +539,7 @@ using namespace sym;
 // ------------------------------------------------------------------ sharded MM (C-ABI)
 struct MmShardWs {
     int32_t *mate = nullptr, *pick[2] = {nullptr, nullptr}, *huge = nullptr;
+    uint32_t *mbits = nullptr;
     SplitWs sw;
     int64_t *rp_in = nullptr, *rp_x = nullptr;
     int32_t *ci_in = nullptr, *ci_x = nullptr;
@@ -542,6 +552,7 @@ static void carve_mm_sharded(Arena &a, const ShardPlan &P, const sym_params *p, 
     w.pick[0] = a.take<int32_t>(pad);
     w.pick[1] = a.take<int32_t>(pad);
     w.huge = a.take<int32_t>((size_t)(P.nnz / MM_BUDGET + 2));
+    w.mbits = a.take<uint32_t>(pad / 32 + 1);
     if (p->kind == SYM_DECOMP_RAND) {  // the owned rows' RAND decomposition (Alg 2, local)
         carve_split_ws(a, P.nl, P.nnz, w.sw);
         w.rp_in = a.take<int64_t>((size_t)P.nl + 1);
@@ -591,6 +602,7 @@ static int mm_sharded_phase(const ShardPlan &P, ShardCtx &x, const sym_params *p
             A.hbits = nullptr;
             A.dual = 0;
             A.mate = w.mate;
+            A.mbits = w.mbits;
             A.pick_prev = w.pick[(r + 1) & 1];
             A.pick_cur = w.pick[r & 1];
             A.in_list = x.list_in(r);
@@ -619,7 +631,7 @@ static int mm_sharded_phase(const ShardPlan &P, ShardCtx &x, const sym_params *p
             SYM_LAUNCH_CHECK();
         }
         uint64_t front = 0;
-        SYM_TRY(shard_exchange(P, x, r & 1, SH_MM, nullptr, w.mate, w.pick[r & 1], nullptr, &front));
+        SYM_TRY(shard_exchange(P, x, r & 1, SH_MM, nullptr, w.mate, w.pick[r & 1], w.mbits, &front));
         local = x.host_all[2 * P.rank + 1];
         if (front == 0) {
             *rounds = (uint32_t)(r + 1);
@@ -650,6 +662,7 @@ extern "C" int sym_mm_sharded(const sym_graph_shard *g, const sym_params *p, sym
     if (stats) memset(stats, 0, sizeof(*stats));
     const size_t pad = (size_t)P.N * (size_t)P.B;
     SYM_CUDA(cudaMemsetAsync(w.mate, 0xff, sizeof(int32_t) * pad, s));
+    SYM_CUDA(cudaMemsetAsync(w.mbits, 0, sizeof(uint32_t) * (pad / 32 + 1), s));
     SYM_CUDA(cudaMemsetAsync(w.pick[0], 0xff, sizeof(int32_t) * pad, s));
     SYM_CUDA(cudaMemsetAsync(w.pick[1], 0xff, sizeof(int32_t) * pad, s));
     SYM_CUDA(cudaMemsetAsync(x.pair, 0, 8 * sizeof(uint32_t), s));

@@ -223,7 +223,10 @@ __global__ void k_sh_scatter(const void *recv, const uint32_t *__restrict__ all,
             const uint2 e = static_cast<const uint2 *>(recv)[idx];
             const uint32_t u = e.x & 0x7fffffffu;
             pick[u] = (int32_t)e.y;
-            if (e.x >> 31) mate[u] = (int32_t)u;  // remote entries: only the sign is read
+            if (e.x >> 31) {  // remote entries: only "matched" is read (sign / bitmap)
+                mate[u] = (int32_t)u;
+                atomicOr(color + (u >> 5), 1u << (u & 31));  // SH_MM: `color` is the matched bitmap
+            }
         } else {
             const uint2 e = static_cast<const uint2 *>(recv)[idx];
             color[e.x] = e.y;
