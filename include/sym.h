@@ -75,6 +75,18 @@ typedef enum {
 #define SYM_F_EXT_DECOMP 0x4u /* a sym_decompose() result will be passed in: the workspace
                                  (query and call) then excludes the internal decomposition,
                                  and sym_mis/mm/color require decomp != NULL */
+/* variants: single-GPU calls only (SYM_EINVAL in the
+   sharded calls) */
+#define SYM_F_PER_ROUND 0x10u     /* sym_mis: classic LubyMIS -- priorities re-drawn
+                                     every round from K(seed, VERTEX, round), two-step
+                                     synchronous rounds (local maxima join I, then their
+                                     neighbours leave); every flow's MIS steps */
+#define SYM_F_CONFLICT_DROP 0x20u /* sym_mis RAND: MIS of the parts, the lower In end of every
+                                     In-In cross arc dropped, then the MIS of the rest (G10 i) */
+#define SYM_F_SPARSER_FIRST 0x40u /* sym_mis RAND: when G_{k+1} has fewer arcs than the parts,
+                                     the boundary's MIS first (G10 ii) */
+#define SYM_F_LOWER_ONLY 0x80u    /* sym_color RAND: V' = the lower-priority end of each
+                                     monochromatic cross edge only (P:232 variant) */
 
 /* Symmetric simple graph in CSR (directed edges symmetrised, self-loops
    dropped).  row_ptr int64[n+1] with row_ptr[0] = 0 and row_ptr[n] = nnz;

@@ -136,6 +136,10 @@ static int check_params(const sym_params *p) {
         set_error("RAND needs 1 <= p <= 65535");
         return SYM_EINVAL;
     }
+    if ((p->flags & SYM_F_CONFLICT_DROP) && (p->flags & SYM_F_SPARSER_FIRST)) {
+        set_error("SYM_F_CONFLICT_DROP and SYM_F_SPARSER_FIRST are alternative MIS-Rand flows");
+        return SYM_EINVAL;
+    }
     return SYM_OK;
 }
 

@@ -186,6 +186,7 @@ struct MisWs {
     int64_t *huge = nullptr;           // deferred (v, resume) pairs
     int64_t huge_cap = 0;
     unsigned long long *gmax = nullptr;  // round 0: maxima of rows crossing tiles
+    uint8_t *mark = nullptr;             // SYM_F_CONFLICT_DROP: dropped In vertices
 };
 
 struct MmWs {

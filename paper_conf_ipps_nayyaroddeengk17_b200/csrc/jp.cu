@@ -1175,16 +1175,20 @@ __global__ void k_color_shift_l(uint32_t *color, const uint32_t *hbits, int64_t 
         if (!((hbits[v >> 5] >> (v & 31)) & 1u)) color[v] += M;
 }
 
-// COLOR-Rand (Alg 8): V' = endpoints of monochromatic cross arcs
+// COLOR-Rand (Alg 8): V' = endpoints of monochromatic cross arcs (lower != 0,
+// SYM_F_LOWER_ONLY: only the lower-priority endpoint of each)
 __global__ void k_color_conflicts(const int64_t *__restrict__ rp_x, const int32_t *__restrict__ ci_x, int64_t n,
-                                  const uint32_t *color, uint8_t *mark, int32_t *list, uint32_t *cnt) {
+                                  const uint32_t *color, uint8_t *mark, int32_t *list, uint32_t *cnt, int lower,
+                                  Key k) {
     int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
         int64_t v = base + threadIdx.x;
         bool conf = false;
         if (v < n) {
             uint32_t cv = color[v];
-            for (int64_t x = rp_x[v]; x < rp_x[v + 1] && !conf; x++) conf = color[ci_x[x]] == cv;
+            const uint64_t kv = lower ? vkey(k, (uint32_t)v) : 0;
+            for (int64_t x = rp_x[v]; x < rp_x[v + 1] && !conf; x++)
+                conf = color[ci_x[x]] == cv && (!lower || vkey(k, (uint32_t)ci_x[x]) > kv);
             mark[v] = conf ? 1 : 0;
         }
         cta_append2(conf, false, (int32_t)v, n, list, cnt, cnt);  // one atomic per CTA
@@ -1426,7 +1430,8 @@ int run_color(const FlowArgs &f, ColorWs &w, uint32_t *color) {
         // V' = endpoints of monochromatic cross edges; uncolour them
         SYM_CUDA(cudaMemsetAsync(&ctl->conflicts, 0, sizeof(uint32_t), s));
         k_color_conflicts<<<num_sms() * 8, 256, 0, s>>>(f.split.rp_x, f.split.ci_x, g.n, color, w.mark, w.vlist,
-                                                          &ctl->conflicts);
+                                                          &ctl->conflicts, (f.p.flags & SYM_F_LOWER_ONLY) ? 1 : 0,
+                                                          stream_key(f.p.seed, TAG_VERTEX, 0));
         SYM_LAUNCH_CHECK();
         k_color_reset<<<num_sms() * 4, 256, 0, s>>>(w.vlist, &ctl->conflicts, color);
         SYM_LAUNCH_CHECK();

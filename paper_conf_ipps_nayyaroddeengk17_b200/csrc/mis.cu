@@ -270,6 +270,155 @@ __global__ void k_mis_finish(uint8_t *st, int64_t n, unsigned long long *count) 
     }
 }
 
+// ------------------------------------------------------------------ f1 variants
+// SYM_F_PER_ROUND -- LubyMIS as Luby states it: every round r draws fresh
+// priorities from K(seed, VERTEX, r) (phase-local r), and is two synchronous steps:
+// step 1, the undecided frontier vertices that beat every undecided phase neighbour
+// become candidates; step 2, candidates join I and undecided vertices with a candidate
+// (now In) neighbour leave.  With re-drawn priorities the result depends on the round
+// structure, so both steps run as separate kernels (warp per vertex).
+constexpr uint8_t ST_CAND = 4;
+
+__device__ __forceinline__ int32_t mis_list_at(const int32_t *list, int rev, int64_t i) {
+    return list ? (rev ? list[-1 - i] : list[i]) : (int32_t)i;
+}
+
+__global__ void k_luby_select(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, uint8_t *st,
+                              const int32_t *list, int rev, const uint32_t *cnt, int64_t implicit_n, Key k) {
+    const int lane = lane_id();
+    const int64_t c = list ? (int64_t)*cnt : implicit_n;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < c; i += nw) {
+        const int32_t v = mis_list_at(list, rev, i);
+        if (st[v] != ST_UNDEC) continue;
+        const uint64_t kv = vkey(k, (uint32_t)v);
+        const int64_t e = rp[v + 1];
+        bool beaten = false;
+        for (int64_t x = rp[v] + lane; x - lane < e && !beaten; x += 32) {
+            bool b = false;
+            if (x < e) {
+                const uint32_t w = (uint32_t)ci[x];
+                const uint8_t sw = st[w];
+                b = (sw == ST_UNDEC || sw == ST_CAND) && vkey(k, w) > kv;
+            }
+            beaten = __any_sync(FULL, b);
+        }
+        if (!beaten && lane == 0) st[v] = ST_CAND;
+    }
+}
+
+__global__ void k_luby_resolve(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, uint8_t *st,
+                               const int32_t *list, int rev, const uint32_t *cnt, int64_t implicit_n, int32_t *out,
+                               uint32_t *out_cnt) {
+    const int lane = lane_id();
+    const int64_t c = list ? (int64_t)*cnt : implicit_n;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < c; i += nw) {
+        const int32_t v = mis_list_at(list, rev, i);
+        const uint8_t sv = st[v];
+        if (sv == ST_CAND) {
+            if (lane == 0) st[v] = ST_IN;
+            continue;
+        }
+        if (sv != ST_UNDEC) continue;
+        const int64_t e = rp[v + 1];
+        bool hit = false;
+        for (int64_t x = rp[v] + lane; x - lane < e && !hit; x += 32) {
+            bool b = false;
+            if (x < e) {
+                const uint8_t sw = st[ci[x]];
+                b = sw == ST_CAND || sw == ST_IN;  // joined I in this round (no older In neighbour exists)
+            }
+            hit = __any_sync(FULL, b);
+        }
+        if (lane == 0) {
+            if (hit) st[v] = ST_OUT;
+            else out[atomicAdd(out_cnt, 1u)] = v;
+        }
+    }
+}
+
+// SYM_F_CONFLICT_DROP (MIS-Rand, reading G10 i): In vertices with a higher-priority In
+// cross neighbour are dropped (mark), then I' = In \ dropped and everything else is
+// undecided again (warp per vertex over the cross CSR)
+__global__ void k_mis_drop_mark(const int64_t *__restrict__ rp_x, const int32_t *__restrict__ ci_x, const uint8_t *st,
+                                int64_t n, Key k, uint8_t *mark) {
+    const int lane = lane_id();
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < n; v += nw) {
+        if (st[v] != ST_IN) {
+            if (lane == 0) mark[v] = 0;
+            continue;
+        }
+        const uint64_t kv = vkey(k, (uint32_t)v);
+        const int64_t e = rp_x[v + 1];
+        bool hit = false;
+        for (int64_t x = rp_x[v] + lane; x - lane < e && !hit; x += 32) {
+            const bool b = x < e && st[ci_x[x]] == ST_IN && vkey(k, (uint32_t)ci_x[x]) > kv;
+            hit = __any_sync(FULL, b);
+        }
+        if (lane == 0) mark[v] = hit ? 1 : 0;
+    }
+}
+
+__global__ void k_mis_drop_apply(uint8_t *st, const uint8_t *mark, int64_t n) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+        st[v] = (st[v] == ST_IN && !mark[v]) ? ST_IN : ST_UNDEC;
+}
+
+// undecided vertices with an In neighbour leave ("remove from G vertices that are in I
+// or have a neighbour in I"); the rest -> list (warp per vertex)
+__global__ void k_mis_kill_pull(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, uint8_t *st, int64_t n,
+                                int32_t *list, uint32_t *cnt) {
+    const int lane = lane_id();
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < n; v += nw) {
+        if (st[v] != ST_UNDEC) continue;
+        const int64_t e = rp[v + 1];
+        bool hit = false;
+        for (int64_t x = rp[v] + lane; x - lane < e && !hit; x += 32) hit = __any_sync(FULL, x < e && st[ci[x]] == ST_IN);
+        if (lane == 0) {
+            if (hit) st[v] = ST_OUT;
+            else list[atomicAdd(cnt, 1u)] = (int32_t)v;
+        }
+    }
+}
+
+// SYM_F_SPARSER_FIRST: the boundary first -- B undecided (back of vlist), the interior
+// INACTIVE (front)
+__global__ void k_mis_classify_bfirst(const int64_t *__restrict__ rp_x, int64_t n, uint8_t *st, int32_t *vlist,
+                                      uint32_t *cnt_front, uint32_t *cnt_back) {
+    int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
+        int64_t v = base + threadIdx.x;
+        bool valid = v < n;
+        bool bnd = valid && (rp_x[v + 1] > rp_x[v]);
+        if (valid) st[v] = bnd ? ST_UNDEC : ST_INACTIVE;
+        cta_append2(valid && !bnd, bnd, (int32_t)v, n, vlist, cnt_front, cnt_back);
+    }
+}
+
+// In vertices of a (possibly reversed) list remove their neighbours; then the
+// INACTIVE vertices of another list become undecided
+__global__ void k_mis_kill_list(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, const int32_t *list,
+                                int rev, const uint32_t *cnt, uint8_t *st) {
+    const uint32_t c = *cnt;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < c; i += gridDim.x * blockDim.x) {
+        const int32_t v = mis_list_at(list, rev, i);
+        if (st[v] != ST_IN) continue;
+        for (int64_t x = rp[v]; x < rp[v + 1]; x++) st[ci[x]] = ST_OUT;
+    }
+}
+
+__global__ void k_mis_wake_list(const int32_t *list, int rev, const uint32_t *cnt, uint8_t *st) {
+    const uint32_t c = *cnt;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < c; i += gridDim.x * blockDim.x) {
+        const int32_t v = mis_list_at(list, rev, i);
+        if (st[v] == ST_INACTIVE) st[v] = ST_UNDEC;
+    }
+}
+
 // ------------------------------------------------------------------ host side
 void carve_mis_ws(Arena &a, int64_t n, int64_t nnz, MisWs &w) {
     w.vlist = a.take<int32_t>((size_t)n + 1);
@@ -278,6 +427,7 @@ void carve_mis_ws(Arena &a, int64_t n, int64_t nnz, MisWs &w) {
     w.huge_cap = nnz / MIS_BUDGET + 2;
     w.huge = a.take<int64_t>((size_t)(2 * w.huge_cap));
     w.gmax = a.take<unsigned long long>((size_t)n + 1);
+    w.mark = a.take<uint8_t>((size_t)n + 1);
 }
 
 // One resident wave: the grid-stride round kernels lose ~20 % to a partial second wave
@@ -296,6 +446,44 @@ static int round_grid() {
 #endif
 }
 
+// SYM_F_PER_ROUND: classic Luby rounds of one phase (round r draws K(seed, VERTEX, r));
+// the host reads the frontier count after every round
+static int mis_phase_per_round(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp, const int32_t *ci,
+                               const int32_t *list0, int rev0, const uint32_t *cnt0, int64_t implicit_n, int phase) {
+    Ctl *ctl = f.ctl;
+    cudaStream_t s = f.stream;
+    const uint32_t maxr = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
+    const int32_t *list = list0;
+    int rev = rev0;
+    const uint32_t *cnt = cnt0;
+    int64_t len = list0 ? (int64_t)num_sms() * 8 * 8 : implicit_n;  // host view of the list length (grid size)
+    uint32_t r = 0;
+    for (;; r++) {
+        if (r >= maxr) {
+            set_error("MIS phase did not converge within max_rounds");
+            return SYM_EROUNDS;
+        }
+        const Key k = stream_key(f.p.seed, TAG_VERTEX, r);
+        uint32_t *out_cnt = &ctl->ring[(r + 1) % 2];
+        int32_t *out = w.fr[(r + 1) & 1];
+        SYM_CUDA(cudaMemsetAsync(out_cnt, 0, sizeof(uint32_t), s));
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 8, (len * 32 + 255) / 256));
+        k_luby_select<<<grid, 256, 0, s>>>(rp, ci, st, list, rev, cnt, implicit_n, k);
+        SYM_LAUNCH_CHECK();
+        k_luby_resolve<<<grid, 256, 0, s>>>(rp, ci, st, list, rev, cnt, implicit_n, out, out_cnt);
+        SYM_LAUNCH_CHECK();
+        uint32_t left = 0;
+        SYM_TRY(read_u32(out_cnt, &left, s));
+        if (f.stats && r < 2048) f.stats->rounds[phase] = r + 1;
+        if (left == 0) break;
+        list = out;
+        rev = 0;
+        cnt = out_cnt;
+        len = left;
+    }
+    return SYM_OK;
+}
+
 // Run Luby rounds of one phase until the frontier is empty.  Round 0 reads
 // (list0, rev0, cnt0) -- or the implicit range [0, implicit_n) when list0 == nullptr.
 static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp, const int32_t *ci,
@@ -304,6 +492,8 @@ static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp
     // stream_round0: round 0 as a gather-free streaming pass (round0.cu).  Measured at
     // R-MAT s24 it is slower than the early-exit frontier kernel, whose
     // round 0 reads only ~30 % of the arcs, so it is off by default for MIS.
+    if (f.p.flags & SYM_F_PER_ROUND)
+        return mis_phase_per_round(f, w, st, rp, ci, list0, rev0, cnt0, implicit_n, phase);
     Ctl *ctl = f.ctl;
     cudaStream_t s = f.stream;
     SYM_CUDA(cudaMemsetAsync(ctl->ring, 0, sizeof(ctl->ring) + sizeof(ctl->huge), s));
@@ -374,6 +564,13 @@ static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp
     return SYM_OK;
 }
 
+// SYM_F_SPARSER_FIRST: does G_{k+1} have fewer arcs than the union of the parts?
+static bool mis_cross_sparser(const FlowArgs &f) {
+    int64_t nin = 0;
+    if (phase_arcs(f, f.split.rp_in, &nin) != SYM_OK) return false;
+    return f.g.nnz - nin < nin;
+}
+
 int run_mis(const FlowArgs &f, MisWs &w, uint8_t *st) {
     const Graph &g = f.g;
     cudaStream_t s = f.stream;
@@ -396,6 +593,33 @@ int run_mis(const FlowArgs &f, MisWs &w, uint8_t *st) {
         SYM_LAUNCH_CHECK();
         // phase R: MIS of the remaining V_H on G_H
         SYM_TRY(mis_phase(f, w, st, f.split.rp_in, f.split.ci_in, w.vlist + g.n, 1, &ctl->cnt_back, 0, 1));
+    } else if (f.p.flags & SYM_F_CONFLICT_DROP) {
+        // reading G10 (i): I_P = MIS of the parts (every vertex, intra arcs); I' = I_P
+        // minus the lower In end of every In-In cross arc; then the MIS of V \ N[I'] on G
+        SYM_CUDA(cudaMemsetAsync(st, ST_UNDEC, (size_t)g.n, s));
+        SYM_TRY(mis_phase(f, w, st, f.split.rp_in, f.split.ci_in, nullptr, 0, nullptr, g.n, 0));
+        k_mis_drop_mark<<<num_sms() * 8, 256, 0, s>>>(f.split.rp_x, f.split.ci_x, st, g.n,
+                                                      stream_key(f.p.seed, TAG_VERTEX, 0), w.mark);
+        SYM_LAUNCH_CHECK();
+        k_mis_drop_apply<<<num_sms() * 8, 256, 0, s>>>(st, w.mark, g.n);
+        SYM_LAUNCH_CHECK();
+        SYM_CUDA(cudaMemsetAsync(&ctl->cnt_front, 0, sizeof(uint32_t), s));
+        k_mis_kill_pull<<<num_sms() * 8, 256, 0, s>>>(g.rp, g.ci, st, g.n, w.vlist, &ctl->cnt_front);
+        SYM_LAUNCH_CHECK();
+        SYM_TRY(mis_phase(f, w, st, g.rp, g.ci, w.vlist, 0, &ctl->cnt_front, 0, 1));
+    } else if ((f.p.flags & SYM_F_SPARSER_FIRST) && mis_cross_sparser(f)) {
+        // P:284/P:286 (reading G10 ii): G_{k+1} is sparser than the parts -> the
+        // boundary's MIS first (all arcs among B), then the interior not adjacent to it
+        SYM_CUDA(cudaMemsetAsync(&ctl->cnt_front, 0, 2 * sizeof(uint32_t), s));
+        k_mis_classify_bfirst<<<num_sms() * 8, 256, 0, s>>>(f.split.rp_x, g.n, st, w.vlist, &ctl->cnt_front,
+                                                            &ctl->cnt_back);
+        SYM_LAUNCH_CHECK();
+        SYM_TRY(mis_phase(f, w, st, g.rp, g.ci, w.vlist + g.n, 1, &ctl->cnt_back, 0, 0));  // I_1 = MIS(G[B])
+        k_mis_kill_list<<<num_sms() * 4, 256, 0, s>>>(g.rp, g.ci, w.vlist + g.n, 1, &ctl->cnt_back, st);
+        SYM_LAUNCH_CHECK();
+        k_mis_wake_list<<<num_sms() * 4, 256, 0, s>>>(w.vlist, 0, &ctl->cnt_front, st);
+        SYM_LAUNCH_CHECK();
+        SYM_TRY(mis_phase(f, w, st, g.rp, g.ci, w.vlist, 0, &ctl->cnt_front, 0, 1));  // I_2 on the interior
     } else {
         SYM_CUDA(cudaMemsetAsync(&ctl->cnt_front, 0, 2 * sizeof(uint32_t), s));
         k_mis_classify_cross<<<num_sms() * 8, 256, 0, s>>>(f.split.rp_x, g.n, st, w.vlist, &ctl->cnt_front,

@@ -160,6 +160,10 @@ int shard_check(const sym_graph_shard *g, const sym_params *p, const sym_comm *c
         set_error("RAND needs 1 <= p <= 65535");
         return SYM_EINVAL;
     }
+    if (p->flags & (SYM_F_PER_ROUND | SYM_F_CONFLICT_DROP | SYM_F_SPARSER_FIRST | SYM_F_LOWER_ONLY)) {
+        set_error("the f1 variant flags are single-GPU only");
+        return SYM_EINVAL;
+    }
     plan->N = c->nranks;
     plan->rank = c->rank;
     plan->B = B;
