@@ -48,8 +48,9 @@ def main():
     for x in r[1:]:
         name = re.sub(r"\(.*", "", x[ki]).replace("void ", "").replace("sym::", "").strip()
         per.setdefault(x[ii], {"name": name})[x[mi]] = float(x[vi].replace(",", "")) * scale.get(x[ui], 1.0)
-    launches = list(per.values())
-    # bench.py --profile-only --warmup 1 --steps 1: the second half of the launches is the measured step
+    # libsym's launches only (graph generation is torch's); bench.py --profile-only
+    # --warmup 1 --steps 1 runs the step twice: the second half is the measured step
+    launches = [k for k in per.values() if kclass(k["name"]) is not None]
     step = launches[len(launches) // 2:]
     agg = OrderedDict()
     for k in step:
