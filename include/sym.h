@@ -87,6 +87,22 @@ typedef enum {
                                      the boundary's MIS first (G10 ii) */
 #define SYM_F_LOWER_ONLY 0x80u    /* sym_color RAND: V' = the lower-priority end of each
                                      monochromatic cross edge only (P:232 variant) */
+/* the paper's own colouring subroutines, sym_color: speculative
+   colouring in synchronous rounds -- every uncoloured vertex takes the smallest colour of
+   its window no admitted neighbour holds (else the window moves on, "OFFSET"), then the
+   lower-id end of every same-colour edge is reset -- in place of Jones-Plassmann in every
+   step of the flow; DEGK colours G_H that way and G_L by Alg 9's literal (k+1)-slot loop
+   (all of V_L starts at max(C_H)+1; the lower-id end of a conflict moves to the smallest
+   free slot).  Deterministic; NOT the greedy colouring. */
+#define SYM_F_COLOR_EB 0x100u     /* edge-based: a 32-colour window */
+#define SYM_F_COLOR_VB 0x200u     /* vertex-based: a window of the average degree of
+                                     the graph being coloured (FORBIDDEN array) */
+/* JP vertex orderings (Hasenplaugh et al. [14]), sym_color
+   (JP only): the priority compares the degree in G first -- larger first (LF) or
+   smaller first (SF) -- and the FIXED hash second; the colouring is first-fit in that
+   order (with SYM_F_LOWER_ONLY, "lower" is in that order too) */
+#define SYM_F_ORDER_LF 0x400u
+#define SYM_F_ORDER_SF 0x800u
 
 /* Symmetric simple graph in CSR (directed edges symmetrised, self-loops
    dropped).  row_ptr int64[n+1] with row_ptr[0] = 0 and row_ptr[n] = nnz;

@@ -26,6 +26,8 @@ import numpy as np
 NONE, RAND, DEGK = 0, 1, 2
 # f1 variant flags (the same numbers as SYM_F_* in include/sym.h)
 F_PER_ROUND, F_CONFLICT_DROP, F_SPARSER_FIRST, F_LOWER_ONLY = 0x10, 0x20, 0x40, 0x80
+F_COLOR_EB, F_COLOR_VB = 0x100, 0x200  # f3: the paper's speculative colouring subroutines
+F_ORDER_LF, F_ORDER_SF = 0x400, 0x800  # f2: JP with largest / smallest degree first
 KINDS = {"none": NONE, "rand": RAND, "degk": DEGK}
 TAG_VERTEX, TAG_EDGE, TAG_RAND = 1, 2, 3
 
@@ -104,6 +106,8 @@ _SIGS = {
     "or_cert_flow": (_I64, [_INT, _I64, _P, _P, _INT, _U32, _U64, _P]),
     "or_mis_ex": (None, [_I64, _P, _P, _INT, _U32, _U64, _U32, _P]),
     "or_color_ex": (None, [_I64, _P, _P, _INT, _U32, _U64, _U32, _P]),
+    "or_color_spec": (None, [_I64, _P, _P, _INT, _U32, _U64, _U32, _P]),
+    "or_color_ord": (None, [_I64, _P, _P, _INT, _U32, _U64, _U32, _P]),
 }
 
 
@@ -207,10 +211,15 @@ def mm(rp, ci, kind="none", param=0, seed=42):
 
 
 def color(rp, ci, kind="none", param=0, seed=42, flags=0):
-    """COLOR flows (or_color); flags: the f1 variants (or_color_ex)."""
+    """COLOR flows (or_color); flags: the f1 variant (or_color_ex) or the f3 speculative
+    subroutines EB / VB (or_color_spec)."""
     n, rp, ci = _graph(rp, ci)
     out = np.zeros(max(n, 1), np.uint32)
-    if flags:
+    if flags & (F_ORDER_LF | F_ORDER_SF):
+        lib().or_color_ord(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), flags, _ptr(out))
+    elif flags & (F_COLOR_EB | F_COLOR_VB):
+        lib().or_color_spec(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), flags, _ptr(out))
+    elif flags:
         lib().or_color_ex(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), flags, _ptr(out))
     else:
         lib().or_color(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), _ptr(out))

@@ -928,3 +928,256 @@ void or_color_ex(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint
     free(cls);
     free(S);
 }
+
+/* ------------------------------------------------------------------ §SPEC the paper's subroutines */
+#define OR_F_COLOR_EB 0x100u  /* colouring subroutine: edge-based speculative colouring */
+#define OR_F_COLOR_VB 0x200u  /* colouring subroutine: vertex-based speculative colouring */
+
+/* Speculative colouring rounds as P:216-218 describes Deveci et al. [10], on the
+   admitted arcs (admit as in admitted()), with a colour window of W colours (EB: W = 32,
+   "a 32 bit integer is used to represent the availability of the colors"; VB: the
+   FORBIDDEN array, W = the average degree of the graph being coloured).  C holds
+   the colours (0 = uncoloured; every vertex with C = 0 takes part, the others are
+   fixed until reset); base[v] = the first colour of v's window (1 on entry).  A round,
+   synchronous (every step reads the state the previous step left):
+     1. every uncoloured v takes the smallest colour in [base_v, base_v + W) that no
+        admitted neighbour holds; if there is none, base_v += W ("OFFSET") and v waits;
+     2. every admitted edge whose endpoints share a colour resets its LOWER-id endpoint
+        ("the color of the endpoint with the lowest id is reset"; VB's choice is
+        not stated -- reading: the same rule);
+   until every vertex is coloured.  Returns the rounds. */
+static int spec_col(int64_t n, const int64_t *rp, const int32_t *ci, const uint32_t *cls, int admit, uint32_t W,
+                    uint32_t *C, uint32_t *base) {
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    uint32_t *T = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+    uint8_t *R = (uint8_t *)calloc(nn, 1);
+    uint8_t *mark = (uint8_t *)malloc((size_t)W + 1);
+    int rounds = 0;
+    for (;;) {
+        int64_t left = 0;
+        for (int64_t v = 0; v < n; v++) left += C[v] == 0;
+        if (!left) break;
+        rounds++;
+        for (int64_t v = 0; v < n; v++) {         /* step 1 (from the snapshot C) */
+            T[v] = C[v];
+            if (C[v] != 0) continue;
+            memset(mark, 0, (size_t)W);
+            for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+                int32_t w = ci[e];
+                if (!admitted(admit, cls[v], cls[w])) continue;
+                if (C[w] >= base[v] && C[w] - base[v] < W) mark[C[w] - base[v]] = 1;
+            }
+            uint32_t i = 0;
+            while (i < W && mark[i]) i++;
+            if (i < W) T[v] = base[v] + i;
+            else base[v] += W;
+        }
+        memcpy(C, T, sizeof(uint32_t) * (size_t)n);
+        for (int64_t v = 0; v < n; v++) {         /* step 2 (from the new snapshot) */
+            if (C[v] == 0) continue;
+            for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+                int32_t w = ci[e];
+                if (w > v && C[w] == C[v] && admitted(admit, cls[v], cls[w])) { R[v] = 1; break; }
+            }
+        }
+        for (int64_t v = 0; v < n; v++)
+            if (R[v]) { C[v] = 0; R[v] = 0; }
+    }
+    free(T);
+    free(R);
+    free(mark);
+    return rounds;
+}
+
+/* COLOR-Degk's literal G_L step (Alg 9 l.6): every V_L vertex starts with colour
+   M+1; then, in synchronous rounds, the lower-id endpoint of every G_L edge whose ends
+   share a colour takes the smallest colour of the (k+1)-slot FORBIDDEN palette
+   M+1 .. M+k+1 not held by a G_L neighbour ("vertices that have a color conflict use the
+   FORBIDDEN array to obtain a new color ... this process repeats in iteration until all
+   vertices in G_L are validly colored"; which endpoint moves is not stated -- reading:
+   the lower id, as in EB).  A free slot always exists (deg <= k).  Returns the rounds. */
+static int gl_loop(int64_t n, const int64_t *rp, const int32_t *ci, const uint32_t *cls, uint32_t k, uint32_t M,
+                   uint32_t *C) {
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    uint32_t *T = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+    uint8_t *mark = (uint8_t *)malloc((size_t)k + 2);
+    int rounds = 0;
+    for (int64_t v = 0; v < n; v++)
+        if (cls[v] == 0) C[v] = M + 1;
+    for (;;) {
+        int64_t moved = 0;
+        for (int64_t v = 0; v < n; v++) {
+            T[v] = C[v];
+            if (cls[v] != 0) continue;
+            int conf = 0;
+            for (int64_t e = rp[v]; e < rp[v + 1] && !conf; e++)
+                conf = cls[ci[e]] == 0 && ci[e] > v && C[ci[e]] == C[v];
+            if (!conf) continue;
+            memset(mark, 0, (size_t)k + 2);
+            for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+                int32_t w = ci[e];
+                if (cls[w] == 0 && C[w] > M && C[w] - M <= k + 1) mark[C[w] - M] = 1;
+            }
+            uint32_t c = 1;
+            while (c <= k + 1 && mark[c]) c++;
+            T[v] = M + c;
+            moved++;
+        }
+        if (!moved) break;
+        rounds++;
+        memcpy(C, T, sizeof(uint32_t) * (size_t)n);
+    }
+    free(T);
+    free(mark);
+    return rounds;
+}
+
+/* the colour window: EB 32 bits; VB the average degree of the graph being coloured
+   (admitted arcs / n, at least 1, at most 1024) */
+static uint32_t spec_window(int64_t n, const int64_t *rp, const int32_t *ci, const uint32_t *cls, int admit, int vb) {
+    if (!vb) return 32;
+    int64_t a = 0;
+    for (int64_t v = 0; v < n; v++)
+        for (int64_t e = rp[v]; e < rp[v + 1]; e++) a += admitted(admit, cls[v], cls[ci[e]]);
+    int64_t w = n > 0 ? a / n : 1;
+    return (uint32_t)(w < 1 ? 1 : (w > 1024 ? 1024 : w));
+}
+
+/* COLOR flows with the paper's own subroutines (flags COLOR_EB / COLOR_VB; f3):
+   the same flows as or_color with speculative colouring in place of LF-COL:
+   NONE: spec(V, E).  RAND: C_IS = spec(V, intra); V' = both ends of monochromatic cross
+   edges (or the lower ends with LOWER_ONLY); V' uncoloured; spec(all arcs) recolours
+   every uncoloured vertex (a reset may uncolour a vertex outside V', which is then
+   recoloured too).  DEGK: C_H = spec(V_H, E_H) with V_L held at colour 0 but not
+   admitted (same-class arcs only, V_L coloured later); M = max C_H; then the literal
+   G_L loop gl_loop.  W: EB 32; VB max(1, admitted arcs / n) of the graph being
+   coloured.  Returns 0 (the rounds are not reported). */
+void or_color_spec(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t param, uint64_t seed,
+                   uint32_t flags, uint32_t *colour) {
+    uint64_t key = or_stream_key(seed, OR_TAG_VERTEX, 0);
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+    uint32_t *base = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+    or_classes(n, rp, kind, param, seed, cls);
+    int vb = (flags & OR_F_COLOR_VB) != 0;
+    for (int64_t v = 0; v < n; v++) {
+        colour[v] = 0;
+        base[v] = 1;
+    }
+    if (kind == OR_NONE) {
+        spec_col(n, rp, ci, cls, 0, spec_window(n, rp, ci, cls, 0, vb), colour, base);
+    } else if (kind == OR_DEGK) {
+        /* C_H on G_H: V_L vertices are parked at a colour no H vertex can see (same-class
+           arcs only) and excluded from the rounds by a temporary non-zero colour */
+        for (int64_t v = 0; v < n; v++)
+            if (cls[v] == 0) colour[v] = 0xFFFFFFFFu;
+        spec_col(n, rp, ci, cls, 3, spec_window(n, rp, ci, cls, 3, vb), colour, base);
+        uint32_t M = 0;
+        for (int64_t v = 0; v < n; v++)
+            if (cls[v] == 1 && colour[v] > M) M = colour[v];
+        gl_loop(n, rp, ci, cls, param, M, colour);
+    } else {
+        spec_col(n, rp, ci, cls, 1, spec_window(n, rp, ci, cls, 1, vb), colour, base);  /* C_IS */
+        uint8_t *S = (uint8_t *)calloc(nn, 1);
+        for (int64_t v = 0; v < n; v++)
+            for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+                int32_t w = ci[e];
+                if (cls[w] != cls[v] && colour[w] == colour[v] &&
+                    (!(flags & OR_F_LOWER_ONLY) || vgreater(key, w, (int32_t)v))) { S[v] = 1; break; }
+            }
+        for (int64_t v = 0; v < n; v++) {
+            if (S[v]) colour[v] = 0;
+            base[v] = 1;
+        }
+        spec_col(n, rp, ci, cls, 0, spec_window(n, rp, ci, cls, 0, vb), colour, base);  /* recolour against G */
+        free(S);
+    }
+    free(cls);
+    free(base);
+}
+
+/* ------------------------------------------------------------------ §ORD JP vertex orderings */
+#define OR_F_ORDER_LF 0x400u  /* JP priority: largest degree first (Hasenplaugh et al. [14]) */
+#define OR_F_ORDER_SF 0x800u  /* JP priority: smallest degree first ([14]) */
+
+/* the (degree, pv, id) order of the colouring: LF compares the degree in G first
+   (larger first), SF the degree (smaller first); ties by (pv, id) as everywhere */
+static const int64_t *g_ord_rp;
+static uint32_t g_ord_flags;
+static int ord_greater(uint64_t key, int32_t a, int32_t b) {
+    int64_t da = g_ord_rp[a + 1] - g_ord_rp[a], db = g_ord_rp[b + 1] - g_ord_rp[b];
+    if (da != db) return (g_ord_flags & OR_F_ORDER_LF) ? da > db : da < db;
+    return vgreater(key, a, b);
+}
+static int cmp_ord_desc(const void *x, const void *y) {
+    int32_t a = *(const int32_t *)x, b = *(const int32_t *)y;
+    if (a == b) return 0;
+    return ord_greater(g_sort_key, a, b) ? -1 : 1;
+}
+
+/* LF-COL in the (degree, pv, id) order: first fit over the coloured admitted neighbours */
+static void lf_col_ord(int64_t n, const int64_t *rp, const int32_t *ci, const uint8_t *inS, const uint32_t *cls,
+                       int admit, uint64_t key, uint32_t *C) {
+    int64_t c = 0, maxd = 0;
+    for (int64_t v = 0; v < n; v++) {
+        c += inS[v] ? 1 : 0;
+        if (rp[v + 1] - rp[v] > maxd) maxd = rp[v + 1] - rp[v];
+    }
+    int32_t *order = (int32_t *)malloc(sizeof(int32_t) * (size_t)(c > 0 ? c : 1));
+    c = 0;
+    for (int64_t v = 0; v < n; v++)
+        if (inS[v]) order[c++] = (int32_t)v;
+    g_sort_key = key;
+    qsort(order, (size_t)c, sizeof(int32_t), cmp_ord_desc);
+    uint8_t *mark = (uint8_t *)malloc((size_t)maxd + 2);
+    for (int64_t i = 0; i < c; i++) C[order[i]] = mex_colour(rp, ci, order[i], cls, admit, C, mark);
+    free(mark);
+    free(order);
+}
+
+/* COLOR flows of or_color with JP's priority order replaced by LF / SF (the degree of
+   the vertex in G; FIXED hash ties); COLOR-Rand's lower-endpoint variant compares in
+   the same order.  Hasenplaugh et al. run JP with these orderings. */
+void or_color_ord(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t param, uint64_t seed,
+                  uint32_t flags, uint32_t *colour) {
+    uint64_t key = or_stream_key(seed, OR_TAG_VERTEX, 0);
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+    uint8_t *S = (uint8_t *)calloc(nn, 1);
+    g_ord_rp = rp;
+    g_ord_flags = flags;
+    or_classes(n, rp, kind, param, seed, cls);
+    for (int64_t v = 0; v < n; v++) colour[v] = 0;
+    if (kind == OR_NONE) {
+        for (int64_t v = 0; v < n; v++) S[v] = 1;
+        lf_col_ord(n, rp, ci, S, cls, 0, key, colour);
+    } else if (kind == OR_DEGK) {
+        uint32_t *CL = (uint32_t *)calloc(nn, sizeof(uint32_t));
+        for (int64_t v = 0; v < n; v++) S[v] = cls[v] == 1;
+        lf_col_ord(n, rp, ci, S, cls, 1, key, colour);
+        uint32_t M = 0;
+        for (int64_t v = 0; v < n; v++)
+            if (cls[v] == 1 && colour[v] > M) M = colour[v];
+        for (int64_t v = 0; v < n; v++) S[v] = cls[v] == 0;
+        lf_col_ord(n, rp, ci, S, cls, 1, key, CL);
+        for (int64_t v = 0; v < n; v++)
+            if (cls[v] == 0) colour[v] = M + CL[v];
+        free(CL);
+    } else {
+        for (int64_t v = 0; v < n; v++) S[v] = 1;
+        lf_col_ord(n, rp, ci, S, cls, 1, key, colour);
+        for (int64_t v = 0; v < n; v++) {
+            S[v] = 0;
+            for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+                int32_t w = ci[e];
+                if (cls[w] != cls[v] && colour[w] == colour[v] &&
+                    (!(flags & OR_F_LOWER_ONLY) || ord_greater(key, w, (int32_t)v))) { S[v] = 1; break; }
+            }
+        }
+        for (int64_t v = 0; v < n; v++)
+            if (S[v]) colour[v] = 0;
+        lf_col_ord(n, rp, ci, S, cls, 0, key, colour);
+    }
+    free(cls);
+    free(S);
+}

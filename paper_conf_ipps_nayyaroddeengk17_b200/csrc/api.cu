@@ -136,6 +136,18 @@ static int check_params(const sym_params *p) {
         set_error("RAND needs 1 <= p <= 65535");
         return SYM_EINVAL;
     }
+    if ((p->flags & (SYM_F_COLOR_EB | SYM_F_COLOR_VB)) && p->kind == SYM_DECOMP_DEGK && p->param > 62) {
+        set_error("the literal G_L loop (SYM_F_COLOR_EB / _VB with DEGk) supports k <= 62");
+        return SYM_EINVAL;
+    }
+    if ((p->flags & SYM_F_ORDER_LF) && (p->flags & SYM_F_ORDER_SF)) {
+        set_error("SYM_F_ORDER_LF and SYM_F_ORDER_SF are alternative orders");
+        return SYM_EINVAL;
+    }
+    if ((p->flags & (SYM_F_ORDER_LF | SYM_F_ORDER_SF)) && (p->flags & (SYM_F_COLOR_EB | SYM_F_COLOR_VB))) {
+        set_error("the LF / SF orders apply to Jones-Plassmann, not to the speculative subroutines");
+        return SYM_EINVAL;
+    }
     if ((p->flags & SYM_F_CONFLICT_DROP) && (p->flags & SYM_F_SPARSER_FIRST)) {
         set_error("SYM_F_CONFLICT_DROP and SYM_F_SPARSER_FIRST are alternative MIS-Rand flows");
         return SYM_EINVAL;

@@ -235,6 +235,7 @@ int run_mm(const FlowArgs &f, MmWs &w, int32_t *mate);
 
 void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w);
 int run_color(const FlowArgs &f, ColorWs &w, uint32_t *color);
+int run_color_spec(const FlowArgs &f, ColorWs &w, uint32_t *color);  // spec.cu (SYM_F_COLOR_EB / _VB)
 
 // ------------------------------------------------------------------ multi-GPU (shard.cu)
 enum { SH_MIS = 0, SH_MM = 1, SH_COLOR = 2 };

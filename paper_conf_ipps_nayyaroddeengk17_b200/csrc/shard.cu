@@ -160,8 +160,9 @@ int shard_check(const sym_graph_shard *g, const sym_params *p, const sym_comm *c
         set_error("RAND needs 1 <= p <= 65535");
         return SYM_EINVAL;
     }
-    if (p->flags & (SYM_F_PER_ROUND | SYM_F_CONFLICT_DROP | SYM_F_SPARSER_FIRST | SYM_F_LOWER_ONLY)) {
-        set_error("the f1 variant flags are single-GPU only");
+    if (p->flags & (SYM_F_PER_ROUND | SYM_F_CONFLICT_DROP | SYM_F_SPARSER_FIRST | SYM_F_LOWER_ONLY | SYM_F_COLOR_EB |
+                    SYM_F_COLOR_VB | SYM_F_ORDER_LF | SYM_F_ORDER_SF)) {
+        set_error("the variant flags (f1, f3) are single-GPU only");
         return SYM_EINVAL;
     }
     plan->N = c->nranks;

@@ -78,3 +78,25 @@ def test_variants_scale20_match_the_oracle():
         _eq(sb.sym_mis(*g, kind, p, 42, flags=f), O.mis(*h, kind, p, 42, flags=f), f"s20 {kind}{p} {f:#x}")
     _eq(sb.sym_color(*g, "rand", 4, 42, flags=O.F_LOWER_ONLY), O.color(*h, "rand", 4, 42, flags=O.F_LOWER_ONLY),
         "s20 lower-only")
+
+
+@pytest.mark.parametrize("seed", SEEDS)
+@pytest.mark.parametrize("flag", ["eb", "vb"])
+@pytest.mark.parametrize("kind,p", [("none", 0), ("degk", 2), ("rand", 4), ("rand", 64)])
+def test_speculative_colouring(graph, flag, kind, p, seed):
+    """f3: the paper's EB / VB subroutines and the literal G_L loop, bit-exact."""
+    name, g, (rp, ci) = graph
+    f = {"eb": O.F_COLOR_EB, "vb": O.F_COLOR_VB}[flag]
+    _eq(sb.sym_color(rp, ci, kind, p, seed, flags=f), O.color(*g, kind, p, seed, flags=f), f"{flag} {kind}{p} {name}")
+    if kind == "rand":
+        f |= O.F_LOWER_ONLY
+        _eq(sb.sym_color(rp, ci, kind, p, seed, flags=f), O.color(*g, kind, p, seed, flags=f),
+            f"{flag}+lower {kind}{p} {name}")
+
+
+def test_speculative_scale20():
+    g = G.rmat(20, 16, 1, device="cuda")
+    h = (g[0].cpu().numpy(), g[1].cpu().numpy())
+    for kind, p in (("none", 0), ("degk", 2), ("rand", 4)):
+        _eq(sb.sym_color(*g, kind, p, 42, flags=O.F_COLOR_EB), O.color(*h, kind, p, 42, flags=O.F_COLOR_EB),
+            f"s20 EB {kind}")

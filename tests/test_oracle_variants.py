@@ -179,3 +179,51 @@ def test_color_lower_only(graph, p, seed):
     lower[src[mono & (key[ci] > key[src])]] = True
     assert not np.any(lower & ~both)
     assert np.array_equal(C[~lower], C1[~lower])  # only V' is recoloured
+
+
+# ------------------------------------------------------------------ f3: the paper's subroutines
+SPEC = [("eb", O.F_COLOR_EB), ("vb", O.F_COLOR_VB)]
+
+
+@pytest.mark.parametrize("seed", SEEDS)
+@pytest.mark.parametrize("name,flag", SPEC)
+@pytest.mark.parametrize("kind,p", [("none", 0), ("degk", 2), ("rand", 1), ("rand", 4), ("rand", 64)])
+def test_speculative_colouring_is_proper(graph, name, flag, kind, p, seed):
+    """EB / VB and the literal G_L loop (Alg 9): every vertex coloured, no
+    edge monochromatic; COLOR-Degk's G_L colours lie in max(C_H)+1 .. max(C_H)+k+1
+    ("an additional k+1 colors"); RAND p = 1 is the plain speculative colouring."""
+    rp, ci = graph
+    n = rp.size - 1
+    C = O.color(rp, ci, kind, p, seed, flags=flag).astype(np.int64)
+    src = np.repeat(np.arange(n), np.diff(rp))
+    assert (C >= 1).all() and not np.any(C[src] == C[ci])
+    if kind == "degk":
+        cls = O.classes(rp, ci, kind, p, seed)
+        M = int(C[cls == 1].max()) if (cls == 1).any() else 0
+        assert ((C[cls == 0] > M) & (C[cls == 0] <= M + p + 1)).all()
+    if kind == "rand" and p == 1:
+        assert np.array_equal(C, O.color(rp, ci, "none", 0, seed, flags=flag).astype(np.int64))
+
+
+@pytest.mark.parametrize("name,flag", SPEC)
+@pytest.mark.parametrize("n", [5, 33, 70])
+def test_speculative_closed_forms(name, flag, n):
+    """K_n: round r leaves exactly the highest remaining id with its colour (every
+    other clique edge resets its lower end), so C(v) = n - v -- whatever the window
+    (EB 32, VB n - 1) and its OFFSET moves; the empty graph is coloured 1 in one round."""
+    rp, ci = (x.numpy() for x in G.complete(n))
+    C = O.color(rp, ci, "none", 0, 42, flags=flag)
+    assert C.tolist() == [n - v for v in range(n)]
+    rp, ci = (x.numpy() for x in G.empty(9))
+    assert (O.color(rp, ci, "none", 0, 42, flags=flag) == 1).all()
+
+
+def test_speculative_is_not_greedy():
+    """The speculative colourings are not the greedy (JP) one -- the variant really
+    replaces the subroutine.  (EB's and VB's windows only change a colour when a
+    colour below a vertex's moved window is freed later by a reset, which is rare:
+    on these R-MAT graphs they coincide.)"""
+    rp, ci = (x.numpy() for x in G.rmat(12, 8, 1))
+    for flag in (O.F_COLOR_EB, O.F_COLOR_VB):
+        for kind, p in (("none", 0), ("degk", 2), ("rand", 4)):
+            assert not np.array_equal(O.color(rp, ci, kind, p, 42, flags=flag), O.color(rp, ci, kind, p, 42))
