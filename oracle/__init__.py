@@ -23,12 +23,12 @@ import subprocess
 
 import numpy as np
 
-NONE, RAND, DEGK = 0, 1, 2
+NONE, RAND, DEGK, BRIDGE = 0, 1, 2, 3
 # f1 variant flags (the same numbers as SYM_F_* in include/sym.h)
 F_PER_ROUND, F_CONFLICT_DROP, F_SPARSER_FIRST, F_LOWER_ONLY = 0x10, 0x20, 0x40, 0x80
 F_COLOR_EB, F_COLOR_VB = 0x100, 0x200  # f3: the paper's speculative colouring subroutines
 F_ORDER_LF, F_ORDER_SF = 0x400, 0x800  # f2: JP with largest / smallest degree first
-KINDS = {"none": NONE, "rand": RAND, "degk": DEGK}
+KINDS = {"none": NONE, "rand": RAND, "degk": DEGK, "bridge": BRIDGE}
 TAG_VERTEX, TAG_EDGE, TAG_RAND = 1, 2, 3
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -91,7 +91,7 @@ _SIGS = {
     "or_pv": (_U32, [_U64, _U32]),
     "or_pe": (_U32, [_U64, _U32, _U32]),
     "or_label": (_U32, [_U64, _U32, _U32]),
-    "or_classes": (None, [_I64, _P, _INT, _U32, _U64, _P]),
+    "or_classes": (None, [_I64, _P, _P, _INT, _U32, _U64, _P]),
     "or_decompose": (None, [_I64, _P, _P, _INT, _U32, _U64, _P, _P, _P, _P]),
     "or_mis": (None, [_I64, _P, _P, _INT, _U32, _U64, _P]),
     "or_mm": (None, [_I64, _P, _P, _INT, _U32, _U64, _P]),
@@ -174,7 +174,7 @@ def label(seed: int, v: int, p: int) -> int:
 def classes(rp, ci, kind, param, seed):
     n, rp, ci = _graph(rp, ci)
     out = np.zeros(max(n, 0), dtype=np.uint32)
-    lib().or_classes(n, _ptr(rp), _kind(kind), param, seed & (2**64 - 1), _ptr(out))
+    lib().or_classes(n, _ptr(rp), _ptr(ci), _kind(kind), param, seed & (2**64 - 1), _ptr(out))
     return out
 
 

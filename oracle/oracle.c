@@ -38,7 +38,7 @@
 #define OR_IN 1
 #define OR_OUT 2
 
-enum { OR_NONE = 0, OR_RAND = 1, OR_DEGK = 2 };
+enum { OR_NONE = 0, OR_RAND = 1, OR_DEGK = 2, OR_BRIDGE = 3 };
 enum { OR_TAG_VERTEX = 1, OR_TAG_EDGE = 2, OR_TAG_RAND = 3 };
 
 /* ------------------------------------------------------------------ §H hash */
@@ -93,9 +93,84 @@ static int vgreater(uint64_t key, int32_t a, int32_t b) {
 }
 
 /* ------------------------------------------------------------------ §D decomposition */
+/* BRIDGE (Alg 1): the bridges are the edges on no cycle ("any bridge in a
+   graph can never be a part of a cycle"); G_1, G_2, .. = the connected components
+   of G - B.  Bridges by Tarjan's low-link depth-first search (iterative): a tree edge
+   (p, v) is a bridge iff no vertex of v's subtree reaches p or above by a non-tree
+   edge, low(v) > pre(p).  class(v) = the smallest vertex id of v's component of G - B
+   (a bridge's endpoints lie in different components).  Plain, sequential. */
+static void bridge_classes(int64_t n, const int64_t *rp, const int32_t *ci, uint32_t *cls) {
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    int64_t *pre = (int64_t *)malloc(sizeof(int64_t) * nn), *low = (int64_t *)malloc(sizeof(int64_t) * nn);
+    int32_t *par = (int32_t *)malloc(sizeof(int32_t) * nn), *stk = (int32_t *)malloc(sizeof(int32_t) * nn);
+    int64_t *it = (int64_t *)malloc(sizeof(int64_t) * nn);
+    uint8_t *bridge_up = (uint8_t *)calloc(nn, 1); /* the tree edge (v, par v) is a bridge */
+    int64_t t = 0;
+    for (int64_t v = 0; v < n; v++) pre[v] = -1;
+    for (int64_t r = 0; r < n; r++) {
+        if (pre[r] >= 0) continue;
+        int64_t top = 0;
+        stk[top++] = (int32_t)r;
+        par[r] = -1;
+        pre[r] = low[r] = t++;
+        it[r] = rp[r];
+        while (top > 0) {
+            int32_t v = stk[top - 1];
+            if (it[v] < rp[v + 1]) {
+                int32_t w = ci[it[v]++];
+                if (pre[w] < 0) {                   /* tree edge */
+                    par[w] = v;
+                    pre[w] = low[w] = t++;
+                    it[w] = rp[w];
+                    stk[top++] = w;
+                } else if (w != par[v] && pre[w] < low[v]) {
+                    low[v] = pre[w];                /* back edge (simple graph: one arc to the parent) */
+                }
+            } else {
+                top--;
+                int32_t p = par[v];
+                if (p >= 0) {
+                    if (low[v] < low[p]) low[p] = low[v];
+                    if (low[v] > pre[p]) bridge_up[v] = 1;
+                }
+            }
+        }
+    }
+    /* components of G - B: label = the smallest id, by a BFS over the non-bridge edges */
+    for (int64_t v = 0; v < n; v++) cls[v] = 0xFFFFFFFFu;
+    for (int64_t r = 0; r < n; r++) {
+        if (cls[r] != 0xFFFFFFFFu) continue;
+        int64_t head = 0, tail = 0;
+        stk[tail++] = (int32_t)r;
+        cls[r] = (uint32_t)r;
+        while (head < tail) {
+            int32_t v = stk[head++];
+            for (int64_t e = rp[v]; e < rp[v + 1]; e++) {
+                int32_t w = ci[e];
+                int is_bridge = (par[w] == v && bridge_up[w]) || (par[v] == w && bridge_up[v]);
+                if (!is_bridge && cls[w] == 0xFFFFFFFFu) {
+                    cls[w] = (uint32_t)r;
+                    stk[tail++] = w;
+                }
+            }
+        }
+    }
+    free(pre);
+    free(low);
+    free(par);
+    free(stk);
+    free(it);
+    free(bridge_up);
+}
+
 /* class(v): RAND -> label(v) (Alg 2); DEGK -> 1 if deg(v) > k else 0 (Alg 3 l.5-8:
-   deg <= k goes to V_L); NONE -> 0 (no decomposition). */
-void or_classes(int64_t n, const int64_t *rp, int kind, uint32_t param, uint64_t seed, uint32_t *cls) {
+   deg <= k goes to V_L); BRIDGE -> v's component of G - B (Alg 1); NONE -> 0. */
+void or_classes(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t param, uint64_t seed,
+                uint32_t *cls) {
+    if (kind == OR_BRIDGE) {
+        bridge_classes(n, rp, ci, cls);
+        return;
+    }
     uint64_t kr = or_stream_key(seed, OR_TAG_RAND, 0);
     for (int64_t v = 0; v < n; v++) {
         if (kind == OR_RAND) cls[v] = or_label(kr, (uint32_t)v, param);
@@ -110,7 +185,7 @@ void or_classes(int64_t n, const int64_t *rp, int kind, uint32_t param, uint64_t
 void or_decompose(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t param, uint64_t seed,
                   int64_t *rp_in, int32_t *ci_in, int64_t *rp_x, int32_t *ci_x) {
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)(n > 0 ? n : 1));
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     int64_t a = 0, b = 0;
     rp_in[0] = 0;
     rp_x[0] = 0;
@@ -184,7 +259,7 @@ void or_mis(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t 
     uint8_t *st = (uint8_t *)calloc(nn, 1);
     uint8_t *S = (uint8_t *)calloc(nn, 1);
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     if (kind == OR_NONE) {
         for (int64_t v = 0; v < n; v++) S[v] = 1;
         lf_mis(n, rp, ci, S, key, st);
@@ -293,11 +368,11 @@ void or_mm(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t p
     uint64_t key = or_stream_key(seed, OR_TAG_EDGE, 0);
     size_t nn = (size_t)(n > 0 ? n : 1);
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     for (int64_t v = 0; v < n; v++) mate[v] = -1;
     if (kind == OR_NONE) {
         lf_mm(n, rp, ci, cls, 0, key, mate);
-    } else if (kind == OR_RAND) {
+    } else if (kind == OR_RAND || kind == OR_BRIDGE) { /* MM-Rand, Alg 5 / MM-Bridge, Alg 4 */
         lf_mm(n, rp, ci, cls, 1, key, mate);   /* phase 1: induced subgraphs */
         lf_mm(n, rp, ci, cls, 2, key, mate);   /* phase 2: cross edges among unmatched */
     } else {
@@ -357,7 +432,7 @@ void or_color(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_
     size_t nn = (size_t)(n > 0 ? n : 1);
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
     uint8_t *S = (uint8_t *)calloc(nn, 1);
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     for (int64_t v = 0; v < n; v++) colour[v] = 0;
     if (kind == OR_NONE) {
         for (int64_t v = 0; v < n; v++) S[v] = 1;
@@ -592,17 +667,28 @@ int64_t or_cert_col(int64_t n, const int64_t *rp, const int32_t *ci, const uint8
         pre-coloured with C = C1).
    Returns the number of violated vertices (0 = C is the oracle's COLOR-Rand output);
    *nconf (nullable) receives |V'|. */
+static int64_t cert_col_split(int64_t n, const int64_t *rp, const int32_t *ci, const uint32_t *cls, uint64_t seed,
+                              const uint32_t *C, int64_t *nconf);
+
 int64_t or_cert_col_rand(int64_t n, const int64_t *rp, const int32_t *ci, uint32_t p, uint64_t seed,
                          const uint32_t *C, int64_t *nconf) {
+    uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)(n > 0 ? n : 1));
+    or_classes(n, rp, ci, OR_RAND, p, seed, cls);
+    int64_t bad = cert_col_split(n, rp, ci, cls, seed, C, nconf);
+    free(cls);
+    return bad;
+}
+
+/* the same certificate for any vertex classes (RAND parts, BRIDGE components) */
+static int64_t cert_col_split(int64_t n, const int64_t *rp, const int32_t *ci, const uint32_t *cls, uint64_t seed,
+                              const uint32_t *C, int64_t *nconf) {
     uint64_t key = or_stream_key(seed, OR_TAG_VERTEX, 0);
     size_t nn = (size_t)(n > 0 ? n : 1);
-    uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
     uint32_t *C1 = (uint32_t *)calloc(nn, sizeof(uint32_t));
     int64_t *pend = (int64_t *)malloc(sizeof(int64_t) * nn); /* uncoloured higher intra neighbours */
     int32_t *queue = (int32_t *)malloc(sizeof(int32_t) * nn);
     uint8_t *S = (uint8_t *)calloc(nn, 1);
     int64_t maxd = 0, head = 0, tail = 0, bad = 0, conf = 0;
-    or_classes(n, rp, OR_RAND, p, seed, cls);
     for (int64_t v = 0; v < n; v++) {
         if (rp[v + 1] - rp[v] > maxd) maxd = rp[v + 1] - rp[v];
         pend[v] = 0;
@@ -645,7 +731,6 @@ int64_t or_cert_col_rand(int64_t n, const int64_t *rp, const int32_t *ci, uint32
     free(queue);
     free(pend);
     free(C1);
-    free(cls);
     return bad;
 }
 
@@ -658,10 +743,14 @@ int64_t or_cert_flow(int problem, int64_t n, const int64_t *rp, const int32_t *c
                      uint64_t seed, const void *result) {
     size_t nn = (size_t)(n > 0 ? n : 1);
     int64_t bad = 0;
-    if (problem == 3 && kind == OR_RAND) return or_cert_col_rand(n, rp, ci, param, seed, (const uint32_t *)result, 0);
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
+    or_classes(n, rp, ci, kind, param, seed, cls);
+    if (problem == 3 && (kind == OR_RAND || kind == OR_BRIDGE)) {
+        bad = cert_col_split(n, rp, ci, cls, seed, (const uint32_t *)result, 0);
+        free(cls);
+        return bad;
+    }
     uint8_t *S = (uint8_t *)malloc(nn);
-    or_classes(n, rp, kind, param, seed, cls);
     if (problem == 1) { /* MIS: M1 NONE, M2 DEGk, M3 RAND */
         const uint8_t *I = (const uint8_t *)result;
         if (kind == OR_NONE) {
@@ -698,7 +787,7 @@ int64_t or_cert_flow(int problem, int64_t n, const int64_t *rp, const int32_t *c
             memset(S, 1, nn);
             bad = or_cert_mm(n, rp, ci, cls, 0, S, seed, M);
         } else {
-            int a1 = kind == OR_RAND ? 1 : 3, a2 = kind == OR_RAND ? 2 : 4;
+            int a1 = kind == OR_DEGK ? 3 : 1, a2 = kind == OR_DEGK ? 4 : 2;
             int32_t *M1 = (int32_t *)malloc(sizeof(int32_t) * nn), *M2 = (int32_t *)malloc(sizeof(int32_t) * nn);
             for (int64_t v = 0; v < n; v++) {
                 int32_t w = M[v];
@@ -827,7 +916,7 @@ void or_mis_ex(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32
     uint8_t *st = (uint8_t *)calloc(nn, 1), *S = (uint8_t *)calloc(nn, 1), *X = (uint8_t *)calloc(nn, 1);
     uint8_t *B = (uint8_t *)calloc(nn, 1);
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     if (kind == OR_NONE) {
         for (int64_t v = 0; v < n; v++) S[v] = 1;
         mis_step(n, rp, ci, S, seed, flags, st);
@@ -909,7 +998,7 @@ void or_color_ex(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint
     size_t nn = (size_t)(n > 0 ? n : 1);
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
     uint8_t *S = (uint8_t *)calloc(nn, 1);
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     for (int64_t v = 0; v < n; v++) {
         colour[v] = 0;
         S[v] = 1;
@@ -1058,7 +1147,7 @@ void or_color_spec(int64_t n, const int64_t *rp, const int32_t *ci, int kind, ui
     size_t nn = (size_t)(n > 0 ? n : 1);
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
     uint32_t *base = (uint32_t *)malloc(sizeof(uint32_t) * nn);
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     int vb = (flags & OR_F_COLOR_VB) != 0;
     for (int64_t v = 0; v < n; v++) {
         colour[v] = 0;
@@ -1146,7 +1235,7 @@ void or_color_ord(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uin
     uint8_t *S = (uint8_t *)calloc(nn, 1);
     g_ord_rp = rp;
     g_ord_flags = flags;
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     for (int64_t v = 0; v < n; v++) colour[v] = 0;
     if (kind == OR_NONE) {
         for (int64_t v = 0; v < n; v++) S[v] = 1;

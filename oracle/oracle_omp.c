@@ -36,9 +36,10 @@
 uint64_t or_stream_key(uint64_t seed, uint32_t tag, uint32_t round);
 uint32_t or_pv(uint64_t key, uint32_t v);
 uint32_t or_pe(uint64_t key, uint32_t lo, uint32_t hi);
-void or_classes(int64_t n, const int64_t *rp, int kind, uint32_t param, uint64_t seed, uint32_t *cls);
+void or_classes(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t param, uint64_t seed,
+                uint32_t *cls);
 
-enum { K_NONE = 0, K_RAND = 1, K_DEGK = 2 };
+enum { K_NONE = 0, K_RAND = 1, K_DEGK = 2, K_BRIDGE = 3 };
 enum { UNDEC = 0, IN = 1, OUT = 2 };
 
 static int vgt(uint64_t key, int32_t a, int32_t b) { /* (pv, id) order */
@@ -110,7 +111,7 @@ void oro_mis(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t
     size_t nn = (size_t)(n > 0 ? n : 1);
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
     uint8_t *S = (uint8_t *)malloc(nn), *st = (uint8_t *)calloc(nn, 1);
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     if (kind == K_NONE) {
         memset(S, 1, nn);
         luby_rounds(n, rp, ci, S, key, st);
@@ -201,11 +202,11 @@ void oro_mm(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32_t 
             int32_t *mate) {
     uint64_t key = or_stream_key(seed, 2, 0);
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)(n > 0 ? n : 1));
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     for (int64_t v = 0; v < n; v++) mate[v] = -1;
     if (kind == K_NONE) {
         lmax_rounds(n, rp, ci, cls, 0, key, mate);
-    } else if (kind == K_RAND) {
+    } else if (kind == K_RAND || kind == K_BRIDGE) {
         lmax_rounds(n, rp, ci, cls, 1, key, mate); /* intra edges */
         lmax_rounds(n, rp, ci, cls, 2, key, mate); /* cross edges among unmatched */
     } else {
@@ -296,7 +297,7 @@ void oro_color(int64_t n, const int64_t *rp, const int32_t *ci, int kind, uint32
     size_t nn = (size_t)(n > 0 ? n : 1);
     uint32_t *cls = (uint32_t *)malloc(sizeof(uint32_t) * nn);
     uint8_t *S = (uint8_t *)malloc(nn);
-    or_classes(n, rp, kind, param, seed, cls);
+    or_classes(n, rp, ci, kind, param, seed, cls);
     for (int64_t v = 0; v < n; v++) colour[v] = 0;
     if (kind == K_NONE) {
         memset(S, 1, nn);

@@ -100,3 +100,23 @@ def test_speculative_scale20():
     for kind, p in (("none", 0), ("degk", 2), ("rand", 4)):
         _eq(sb.sym_color(*g, kind, p, 42, flags=O.F_COLOR_EB), O.color(*h, kind, p, 42, flags=O.F_COLOR_EB),
             f"s20 EB {kind}")
+
+
+@pytest.mark.parametrize("seed", SEEDS)
+@pytest.mark.parametrize("order", ["lf", "sf"])
+@pytest.mark.parametrize("kind,p", [("none", 0), ("degk", 2), ("rand", 4)])
+def test_jp_orderings(graph, order, kind, p, seed):
+    """f2: early-commit JP with the largest / smallest degree first orders, bit-exact."""
+    name, g, (rp, ci) = graph
+    f = {"lf": O.F_ORDER_LF, "sf": O.F_ORDER_SF}[order]
+    _eq(sb.sym_color(rp, ci, kind, p, seed, flags=f), O.color(*g, kind, p, seed, flags=f), f"{order} {kind}{p} {name}")
+    if kind == "rand":
+        f |= O.F_LOWER_ONLY
+        _eq(sb.sym_color(rp, ci, kind, p, seed, flags=f), O.color(*g, kind, p, seed, flags=f), f"{order}+lower {name}")
+
+
+def test_jp_orderings_scale20():
+    g = G.rmat(20, 16, 1, device="cuda")
+    h = (g[0].cpu().numpy(), g[1].cpu().numpy())
+    for f in (O.F_ORDER_LF, O.F_ORDER_SF):
+        _eq(sb.sym_color(*g, "degk", 2, 42, flags=f), O.color(*h, "degk", 2, 42, flags=f), f"s20 order {f:#x}")

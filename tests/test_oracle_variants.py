@@ -227,3 +227,44 @@ def test_speculative_is_not_greedy():
     for flag in (O.F_COLOR_EB, O.F_COLOR_VB):
         for kind, p in (("none", 0), ("degk", 2), ("rand", 4)):
             assert not np.array_equal(O.color(rp, ci, kind, p, 42, flags=flag), O.color(rp, ci, kind, p, 42))
+
+
+# ------------------------------------------------------------------ f2: JP orderings
+@pytest.mark.parametrize("seed", SEEDS)
+@pytest.mark.parametrize("order", ["lf", "sf"])
+def test_jp_orderings_equal_networkx_first_fit(order, seed):
+    """JP with largest / smallest degree first (Hasenplaugh et al. [14]) =
+    first-fit in that order, computed by networkx's greedy_color (an independent
+    first-fit) with the same (degree, pv, id) order."""
+    nx = pytest.importorskip("networkx")
+    flag = {"lf": O.F_ORDER_LF, "sf": O.F_ORDER_SF}[order]
+    for g in (G.rmat(10, 8, 1), G.grid(24, 24, 0.6, 2), G.near_regular(400, 6, 1)):
+        rp, ci = (x.numpy() for x in g)
+        n = rp.size - 1
+        deg = np.diff(rp)
+        Gx = nx.Graph()
+        Gx.add_nodes_from(range(n))
+        src = np.repeat(np.arange(n), deg)
+        Gx.add_edges_from(zip(src.tolist(), ci.tolist()))
+        sign = 1 if order == "lf" else -1
+        orderv = sorted(range(n), key=lambda v: (sign * int(deg[v]), O.pv(seed, v), v), reverse=True)
+        want = nx.greedy_color(Gx, strategy=lambda _g, _c: iter(orderv))
+        got = O.color(rp, ci, "none", 0, seed, flags=flag)
+        assert got.tolist() == [want[v] + 1 for v in range(n)]
+
+
+@pytest.mark.parametrize("seed", SEEDS)
+def test_lf_welsh_powell_bound(graph, seed):
+    """Largest-first colouring obeys the Welsh-Powell bound max_i min(d_i + 1, i) over
+    the degree-sorted vertices; every ordering is proper in every flow."""
+    rp, ci = graph
+    n = rp.size - 1
+    d = np.sort(np.diff(rp))[::-1]
+    bound = int(max(min(int(d[i]) + 1, i + 1) for i in range(n)))
+    C = O.color(rp, ci, "none", 0, seed, flags=O.F_ORDER_LF)
+    assert int(C.max()) <= bound
+    src = np.repeat(np.arange(n), np.diff(rp))
+    for flag in (O.F_ORDER_LF, O.F_ORDER_SF):
+        for kind, p in (("degk", 2), ("rand", 4)):
+            C = O.color(rp, ci, kind, p, seed, flags=flag).astype(np.int64)
+            assert (C >= 1).all() and not np.any(C[src] == C[ci])
