@@ -58,8 +58,13 @@ enum {
     SYM_EROUNDS = 6     /* params->max_rounds reached before the phase converged */
 };
 
-/* decomposition kinds: NONE = no decomposition (the paper's baselines) */
-typedef enum { SYM_DECOMP_NONE = 0, SYM_DECOMP_RAND = 1, SYM_DECOMP_DEGK = 2 } sym_decomp_kind;
+/* decomposition kinds: NONE = no decomposition (the paper's baselines).
+   BRIDGE (Alg 1): the bridges of G (tree edges of a BFS
+   forest not covered by any non-tree edge's LCA walk) are the cross edges, the rest
+   (the 2-edge-connected components G_1, G_2, ..) the intra edges; MM-Bridge (Alg 4),
+   COLOR-Bridge (Alg 7) and MIS-Bridge (Alg 10) then run as the RAND flows.  param is
+   ignored; single-GPU; the optional label output is 1 for bridge endpoints. */
+typedef enum { SYM_DECOMP_NONE = 0, SYM_DECOMP_RAND = 1, SYM_DECOMP_DEGK = 2, SYM_DECOMP_BRIDGE = 3 } sym_decomp_kind;
 
 /* problem ids for sym_workspace_bytes */
 typedef enum {

@@ -25,7 +25,7 @@ from . import _lib as L
 __all__ = ["sym_workspace_bytes", "sym_decompose", "sym_mis", "sym_mm", "sym_color", "sym_validate",
            "sym_version", "Decomposition", "SymError", "KINDS"]
 
-KINDS = {"none": L.NONE, "rand": L.RAND, "degk": L.DEGK}
+KINDS = {"none": L.NONE, "rand": L.RAND, "degk": L.DEGK, "bridge": L.BRIDGE}
 
 
 class SymError(RuntimeError):

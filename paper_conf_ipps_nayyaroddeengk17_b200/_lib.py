@@ -11,7 +11,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("SYM_LIB") or os.path.join(HERE, "libsym.so")  # SYM_LIB: diagnostic builds
 
 SYM_OK, SYM_EINVAL, SYM_EWORKSPACE, SYM_EGRAPH, SYM_ECUDA, SYM_ENCCL, SYM_EROUNDS = range(7)
-NONE, RAND, DEGK = 0, 1, 2
+NONE, RAND, DEGK, BRIDGE = 0, 1, 2, 3
 PROBLEM_DECOMPOSE, PROBLEM_MIS, PROBLEM_MM, PROBLEM_COLOR, PROBLEM_VALIDATE = range(5)
 F_VALIDATE, F_STATS, F_EXT_DECOMP = 0x1, 0x2, 0x4
 

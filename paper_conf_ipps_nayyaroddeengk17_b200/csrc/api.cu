@@ -106,6 +106,8 @@ static void carve(Arena &a, int64_t n, int64_t nnz, const sym_params *p, int pro
     L.ctl = a.take<Ctl>(1);
     if (problem == SYM_PROBLEM_VALIDATE) return;
     carve_split_ws(a, n, nnz, L.sw);
+    if (p->kind == SYM_DECOMP_BRIDGE && (problem == SYM_PROBLEM_DECOMPOSE || !(p->flags & SYM_F_EXT_DECOMP)))
+        carve_bridge_ws(a, n, L.sw.br);
     if (problem == SYM_PROBLEM_DECOMPOSE) return;
     bool internal = p->kind != SYM_DECOMP_NONE && !(p->flags & SYM_F_EXT_DECOMP);
     if (internal) {
@@ -131,7 +133,12 @@ static int check_graph(const sym_graph *g) {
 
 static int check_params(const sym_params *p) {
     if (!p) { set_error("params is NULL"); return SYM_EINVAL; }
-    if (p->kind < SYM_DECOMP_NONE || p->kind > SYM_DECOMP_DEGK) { set_error("unknown decomposition kind"); return SYM_EINVAL; }
+    if (p->kind < SYM_DECOMP_NONE || p->kind > SYM_DECOMP_BRIDGE) { set_error("unknown decomposition kind"); return SYM_EINVAL; }
+    if (p->kind == SYM_DECOMP_BRIDGE && (p->flags & (SYM_F_CONFLICT_DROP | SYM_F_SPARSER_FIRST | SYM_F_LOWER_ONLY |
+                                                     SYM_F_COLOR_EB | SYM_F_COLOR_VB))) {
+        set_error("BRIDGE supports the FIXED flows, SYM_F_PER_ROUND and the LF / SF orders only");
+        return SYM_EINVAL;
+    }
     if (p->kind == SYM_DECOMP_RAND && (p->param < 1 || p->param > 65535)) {
         set_error("RAND needs 1 <= p <= 65535");
         return SYM_EINVAL;

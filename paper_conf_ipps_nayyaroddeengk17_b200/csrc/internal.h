@@ -87,11 +87,24 @@ constexpr int SPLIT_THREADS = 256;
 constexpr int SPLIT_PER_THREAD = 16;
 constexpr int SPLIT_TILE = SPLIT_THREADS * SPLIT_PER_THREAD;  // arcs per tile
 
+// BRIDGE decomposition scratch (bridge.cu; carved only for SYM_DECOMP_BRIDGE)
+struct BridgeWs {
+    int32_t *cc = nullptr, *level = nullptr, *par = nullptr;
+    uint8_t *mark = nullptr;
+    int32_t *fr[2] = {nullptr, nullptr};
+    int64_t *bsum = nullptr;
+    uint32_t *ctr = nullptr;
+};
+void carve_bridge_ws(Arena &a, int64_t n, BridgeWs &w);
+int run_bridge_split(const Graph &g, const BridgeWs &w, int64_t *rp_in, int32_t *ci_in, int64_t *rp_x, int32_t *ci_x,
+                     uint16_t *label, cudaStream_t s);
+
 struct SplitWs {
     uint32_t *hbits = nullptr;   // DEGk V_H bitmap [ceil(n/32)]
     int64_t *first_row = nullptr;
     uint64_t *tile_state = nullptr;
     int64_t ntiles = 0;
+    BridgeWs br;                 // SYM_DECOMP_BRIDGE only
 };
 void carve_split_ws(Arena &a, int64_t n, int64_t nnz, SplitWs &w);
 
@@ -222,6 +235,7 @@ struct ColorWs {
     int64_t *queue = nullptr;      // build: (piece << 32 | h) items of the huge rows
     int32_t *vlist = nullptr;
     uint8_t *mark = nullptr;       // COLOR-RAND V'
+    uint32_t *okey = nullptr;      // SYM_F_ORDER_LF / _SF order terms
     uint32_t *sync = nullptr;      // rounds kernel: barrier / counter / error words
 };
 

@@ -118,17 +118,26 @@ struct JpArgs {
     unsigned long long *prof;  // profiling counter pair {alg, impl} of the current launch (nullable)
     unsigned long long *prof_jp;  // the rounds launch's pair: the count pass adds §8(d)'s JP bytes
     Key k;
-    const int64_t *grp;  // the input graph's row_ptr (SYM_F_ORDER_LF / _SF: degree in G)
-    int ord;             // 0: (pv, id); 1: largest degree first; 2: smallest degree first
+    const uint32_t *okey;  // SYM_F_ORDER_LF / _SF: per-vertex order term (degree in G, or its
+                           // complement), 4 B per vertex: L2-resident for the per-arc gathers
+    int ord;               // 0: (pv, id); 1: largest degree first; 2: smallest degree first
 };
 
 // the vertex order of the colouring: (pv, id) -- or, with SYM_F_ORDER_LF / _SF
 // (Hasenplaugh et al. [14]), the degree in G first (pv is a bijection, so the
 // 64-bit key (degree term << 32 | pv) is unique)
-__device__ __forceinline__ uint64_t jp_okey(Key k, const int64_t *grp, int ord, uint32_t v) {
+__device__ __forceinline__ uint64_t jp_okey(Key k, const uint32_t *okey, int ord, uint32_t v) {
     if (ord == 0) return vkey(k, v);
-    const uint64_t d = (uint64_t)(grp[v + 1] - grp[v]);
-    return ((ord == 1 ? d : (0xffffffffull - d)) << 32) | pv(k, v);
+    return ((uint64_t)__ldg(okey + v) << 32) | pv(k, v);
+}
+
+// the order terms: degree (LF) or its complement (SF), degrees in G (< 2^31)
+__global__ void k_jp_okey(const int64_t *__restrict__ grp, int64_t n, int ord, uint32_t *okey) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+        const uint32_t d = (uint32_t)(grp[v + 1] - grp[v]);
+        okey[v] = ord == 1 ? d : ~d;
+    }
 }
 
 __device__ __forceinline__ uint64_t globaltimer_ns() {
@@ -309,7 +318,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_count(JpArgs A) {
             v = A.ov[h];
             b = A.rp[v];
             e = A.rp[v + 1];
-            kv = jp_okey(A.k, A.grp, A.ord, (uint32_t)v);
+            kv = jp_okey(A.k, A.okey, A.ord, (uint32_t)v);
         }
         uint32_t hi = 0, lo = 0;
         if (active && e - b <= JP_SMALL) {  // batches of 4 arcs: their loads in flight together
@@ -320,7 +329,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_count(JpArgs A) {
 #pragma unroll
                 for (int u = 0; u < 4; u++) {
                     if (xq + u < e && in_set(A.inS, w[u])) {
-                        const bool up = jp_okey(A.k, A.grp, A.ord, w[u]) > kv;
+                        const bool up = jp_okey(A.k, A.okey, A.ord, w[u]) > kv;
                         hi += up;
                         lo += !up;
                     }
@@ -341,7 +350,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_count(JpArgs A) {
 #pragma unroll
                 for (int u = 0; u < 4; u++) {
                     if (xb0 + u * 32 < we && in_set(A.inS, w[u])) {
-                        const bool up = jp_okey(A.k, A.grp, A.ord, w[u]) > wk;
+                        const bool up = jp_okey(A.k, A.okey, A.ord, w[u]) > wk;
                         lh += up;
                         ll += !up;
                     }
@@ -381,12 +390,12 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_count_huge(JpArgs A) {
         const int32_t v = A.ov[h];
         const int64_t b = A.rp[v], e = A.rp[v + 1];
         const int64_t pb = b + j * JP_PIECE, pe_ = min(e, pb + JP_PIECE);
-        const uint64_t kv = jp_okey(A.k, A.grp, A.ord, (uint32_t)v);
+        const uint64_t kv = jp_okey(A.k, A.okey, A.ord, (uint32_t)v);
         uint32_t lh = 0, ll = 0;
         for (int64_t x = pb + threadIdx.x; x < pe_; x += JP_HUGE_THREADS) {
             const uint32_t w = (uint32_t)__ldg(A.ci + x);
             if (in_set(A.inS, w)) {
-                const bool up = jp_okey(A.k, A.grp, A.ord, w) > kv;
+                const bool up = jp_okey(A.k, A.okey, A.ord, w) > kv;
                 lh += up;
                 ll += !up;
             }
@@ -572,7 +581,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
             v = A.ov[h];
             b = A.rp[v];
             e = A.rp[v + 1];
-            kv = jp_okey(A.k, A.grp, A.ord, (uint32_t)v);
+            kv = jp_okey(A.k, A.okey, A.ord, (uint32_t)v);
             const uint4 m0 = A.meta[2 * h], m1 = A.meta[2 * h + 1];
             R = m0.x;
             x0 = A.hot[h].w & JP_HMASK;
@@ -597,7 +606,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
                 for (int u = 0; u < 4; u++) {
                     if (!ok[u]) continue;
                     if (!sv[u]) jp_fixed(A, h, R, x0, w[u]);
-                    else if (jp_okey(A.k, A.grp, A.ord, w[u]) > kv) __stcs(A.lst + hl++, rk[u]);
+                    else if (jp_okey(A.k, A.okey, A.ord, w[u]) > kv) __stcs(A.lst + hl++, rk[u]);
                     else __stcs(A.lst + ll++, rk[u]);
                 }
             }
@@ -624,7 +633,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
                 for (int u = 0; u < 4; u++) {
                     const bool ok = xb0 + u * 32 + lane < we;
                     const bool sv = ok && in_set(A.inS, w[u]);
-                    up[u] = sv && jp_okey(A.k, A.grp, A.ord, w[u]) > wk;
+                    up[u] = sv && jp_okey(A.k, A.okey, A.ord, w[u]) > wk;
                     dn[u] = sv && !up[u];
                     rk[u] = sv ? jp_rank(A, w[u]) : 0u;
                     if (ok && !sv) jp_fixed(A, wh, wR, wx0, w[u]);
@@ -661,7 +670,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
         const int64_t b = A.rp[v], e = A.rp[v + 1];
         const int64_t sb0 = b + j * JP_PIECE + (int64_t)(threadIdx.x >> 5) * SLICE;
         const int64_t se = min(e, sb0 + SLICE);
-        const uint64_t kv = jp_okey(A.k, A.grp, A.ord, (uint32_t)v);
+        const uint64_t kv = jp_okey(A.k, A.okey, A.ord, (uint32_t)v);
         const uint4 m0 = A.meta[2 * h], m1 = A.meta[2 * h + 1];
         const uint32_t x0 = A.hot[h].w & JP_HMASK;
         const uint64_t hl = meta_off(m1) + watch_words(m0.y), ll = hl + m0.y;
@@ -671,7 +680,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
             if (x < se) {
                 const uint32_t w = (uint32_t)__ldg(A.ci + x);
                 if (in_set(A.inS, w)) {
-                    up = jp_okey(A.k, A.grp, A.ord, w) > kv;
+                    up = jp_okey(A.k, A.okey, A.ord, w) > kv;
                     dn = !up;
                 }
             }
@@ -694,7 +703,7 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
             for (int u = 0; u < 4; u++) {
                 const bool ok = xq + u * 32 < se;
                 const bool sv = ok && in_set(A.inS, w[u]);
-                up[u] = sv && jp_okey(A.k, A.grp, A.ord, w[u]) > kv;
+                up[u] = sv && jp_okey(A.k, A.okey, A.ord, w[u]) > kv;
                 dn[u] = sv && !up[u];
                 rk[u] = sv ? jp_rank(A, w[u]) : 0u;
                 if (ok && !sv) jp_fixed(A, h, m0.x, x0, w[u]);
@@ -1190,16 +1199,16 @@ __global__ void k_color_shift_l(uint32_t *color, const uint32_t *hbits, int64_t 
 // SYM_F_LOWER_ONLY: only the lower-priority endpoint of each)
 __global__ void k_color_conflicts(const int64_t *__restrict__ rp_x, const int32_t *__restrict__ ci_x, int64_t n,
                                   const uint32_t *color, uint8_t *mark, int32_t *list, uint32_t *cnt, int lower,
-                                  Key k, const int64_t *grp, int ord) {
+                                  Key k, const uint32_t *okey, int ord) {
     int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
         int64_t v = base + threadIdx.x;
         bool conf = false;
         if (v < n) {
             uint32_t cv = color[v];
-            const uint64_t kv = lower ? jp_okey(k, grp, ord, (uint32_t)v) : 0;
+            const uint64_t kv = lower ? jp_okey(k, okey, ord, (uint32_t)v) : 0;
             for (int64_t x = rp_x[v]; x < rp_x[v + 1] && !conf; x++)
-                conf = color[ci_x[x]] == cv && (!lower || jp_okey(k, grp, ord, (uint32_t)ci_x[x]) > kv);
+                conf = color[ci_x[x]] == cv && (!lower || jp_okey(k, okey, ord, (uint32_t)ci_x[x]) > kv);
             mark[v] = conf ? 1 : 0;
         }
         cta_append2(conf, false, (int32_t)v, n, list, cnt, cnt);  // one atomic per CTA
@@ -1246,6 +1255,7 @@ void carve_color_ws(Arena &a, int64_t n, int64_t nnz, ColorWs &w) {
     w.btask = a.take<uint4>((size_t)w.task_cap);
     w.vlist = a.take<int32_t>((size_t)n + 1);
     w.mark = a.take<uint8_t>((size_t)n + 1);
+    w.okey = a.take<uint32_t>((size_t)n + 1);
     w.queue = a.take<int64_t>((size_t)(nnz / JP_BUDGET + 2));  // huge-row pieces (<= nnz/JP_BUDGET)
     w.sync = a.take<uint32_t>(64);  // rounds kernel: barrier / counters / error words
 }
@@ -1300,7 +1310,7 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     A.prof = nullptr;
     A.prof_jp = rounds_ctr;
     A.k = stream_key(f.p.seed, TAG_VERTEX, 0);
-    A.grp = f.g.rp;
+    A.okey = w.okey;
     A.ord = jp_order(f);
     const int64_t nwords = (n + 31) / 32;
     const unsigned tiles_w = (unsigned)((nwords + JP_TILE - 1) / JP_TILE);
@@ -1432,6 +1442,10 @@ int run_color(const FlowArgs &f, ColorWs &w, uint32_t *color) {
     const int kind = f.p.kind;
     if (f.p.flags & (SYM_F_COLOR_EB | SYM_F_COLOR_VB)) return run_color_spec(f, w, color);  // the paper's subroutines
     SYM_CUDA(cudaMemsetAsync(color, 0, sizeof(uint32_t) * (size_t)g.n, s));
+    if (jp_order(f)) {
+        k_jp_okey<<<num_sms() * 8, 256, 0, s>>>(g.rp, g.n, jp_order(f), w.okey);
+        SYM_LAUNCH_CHECK();
+    }
     if (kind == SYM_DECOMP_NONE) {
         SYM_TRY(jp_run(f, w, color, g.rp, g.ci, nullptr, nullptr, nullptr, g.n, 0));
     } else if (kind == SYM_DECOMP_DEGK) {
@@ -1450,7 +1464,7 @@ int run_color(const FlowArgs &f, ColorWs &w, uint32_t *color) {
         SYM_CUDA(cudaMemsetAsync(&ctl->conflicts, 0, sizeof(uint32_t), s));
         k_color_conflicts<<<num_sms() * 8, 256, 0, s>>>(f.split.rp_x, f.split.ci_x, g.n, color, w.mark, w.vlist,
                                                           &ctl->conflicts, (f.p.flags & SYM_F_LOWER_ONLY) ? 1 : 0,
-                                                          stream_key(f.p.seed, TAG_VERTEX, 0), g.rp, jp_order(f));
+                                                          stream_key(f.p.seed, TAG_VERTEX, 0), w.okey, jp_order(f));
         SYM_LAUNCH_CHECK();
         k_color_reset<<<num_sms() * 4, 256, 0, s>>>(w.vlist, &ctl->conflicts, color);
         SYM_LAUNCH_CHECK();

@@ -455,8 +455,9 @@ int run_mm(const FlowArgs &f, MmWs &w, int32_t *mate) {
         ph.nnz = g.nnz;
         SYM_TRY(mm_phase(f, w, mate, ph, 0));
     } else {
-        // phase 1: M_IS = MM(union G_i) (RAND, Alg 5 l.5) / M_H = MM(G_H) (DEGk, Alg 6 l.5)
-        if (kind == SYM_DECOMP_RAND) {
+        // phase 1: M_IS = MM(union G_i) (RAND, Alg 5 l.5; BRIDGE, Alg 4: the 2-edge-connected
+        // components) / M_H = MM(G_H) (DEGk, Alg 6 l.5)
+        if (kind == SYM_DECOMP_RAND || kind == SYM_DECOMP_BRIDGE) {
             ph = MmPhase{f.split.rp_in, nullptr, f.split.ci_in, nullptr, 0, nullptr, 0, nullptr, g.n, true};
             ph.nnz = f.split.nnz_in;
         } else {

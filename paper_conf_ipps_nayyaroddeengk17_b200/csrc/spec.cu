@@ -243,7 +243,7 @@ __global__ void k_spec_arcs(SpecArgs A, int64_t n, unsigned long long *out) {
 __global__ void k_color_max_h(const uint32_t *color, const uint32_t *hbits, int64_t n, uint32_t *mx);
 __global__ void k_color_conflicts(const int64_t *__restrict__ rp_x, const int32_t *__restrict__ ci_x, int64_t n,
                                   const uint32_t *color, uint8_t *mark, int32_t *list, uint32_t *cnt, int lower,
-                                  Key k, const int64_t *grp, int ord);
+                                  Key k, const uint32_t *okey, int ord);
 __global__ void k_color_reset(const int32_t *list, const uint32_t *cnt, uint32_t *color);
 __global__ void k_color_max(const uint32_t *color, int64_t n, uint32_t *mx);
 
@@ -368,7 +368,7 @@ int run_color_spec(const FlowArgs &f, ColorWs &w, uint32_t *color) {
         SYM_CUDA(cudaMemsetAsync(&ctl->conflicts, 0, sizeof(uint32_t), s));
         k_color_conflicts<<<num_sms() * 8, 256, 0, s>>>(f.split.rp_x, f.split.ci_x, g.n, color, w.mark, w.vlist,
                                                           &ctl->conflicts, (f.p.flags & SYM_F_LOWER_ONLY) ? 1 : 0,
-                                                          stream_key(f.p.seed, TAG_VERTEX, 0), g.rp, 0);
+                                                          stream_key(f.p.seed, TAG_VERTEX, 0), nullptr, 0);
         SYM_LAUNCH_CHECK();
         k_color_reset<<<num_sms() * 4, 256, 0, s>>>(w.vlist, &ctl->conflicts, color);
         SYM_LAUNCH_CHECK();

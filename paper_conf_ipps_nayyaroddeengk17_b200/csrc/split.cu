@@ -346,6 +346,7 @@ int launch_classify_degk(const Graph &g, uint32_t k, uint32_t *hbits, int32_t *v
 
 int run_split(const Graph &g, int kind, uint32_t param, uint64_t seed, const SplitWs &w, Ctl *ctl, int64_t *rp_in,
               int32_t *ci_in, int64_t *rp_x, int32_t *ci_x, uint16_t *label, cudaStream_t s, int64_t row_base) {
+    if (kind == SYM_DECOMP_BRIDGE) return run_bridge_split(g, w.br, rp_in, ci_in, rp_x, ci_x, label, s);  // bridge.cu
     Key kr = stream_key(seed, TAG_RAND, 0);
     if (label && g.n > 0) {
         k_labels<<<grid_for(g.n, 256), 256, 0, s>>>(g.rp, g.n, kind, param, kr, label);
