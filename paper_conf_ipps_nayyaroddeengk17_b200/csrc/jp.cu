@@ -1390,6 +1390,10 @@ static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t 
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_jp_rounds, JR_THREADS, 0) != cudaSuccess ||
             per_sm < 1)
             return -1;
+        // SYM_JR_CTAS_PER_SM < the occupancy leaves SMs' register space to kernels of other
+        // streams (the latency-bound rounds barely use the GPU)
+        const char *e = getenv("SYM_JR_CTAS_PER_SM");
+        if (e && atoi(e) > 0) per_sm = std::min(per_sm, atoi(e));
         return num_sms() * per_sm;
     });
     if (grid < 0) {

@@ -18,6 +18,8 @@
 namespace sym {
 
 constexpr int SP_THREADS = 256, SP_WARPS = SP_THREADS / 32, SP_WIN = 1024;
+constexpr int SP_BUDGET = 2048;       // rows longer than this are scanned by a whole CTA
+constexpr int SP_HUGE_THREADS = 512;
 enum { SP_ALL = 0, SP_SAME = 1, SP_HH = 3 };
 
 struct SpecArgs {
@@ -49,12 +51,16 @@ __device__ __forceinline__ bool sp_admitted(const SpecArgs &A, uint32_t cv, uint
 
 // step 1 (warp per listed uncoloured vertex): T[v] = smallest free colour of the window
 __global__ void __launch_bounds__(SP_THREADS) k_spec_assign(SpecArgs A, const uint32_t *__restrict__ list,
-                                                            const uint32_t *cnt) {
+                                                            const uint32_t *cnt, uint32_t *hlist, uint32_t *hcnt) {
     __shared__ uint32_t s_mask[SP_WARPS][SP_WIN / 32];
     const int lane = lane_id(), wib = threadIdx.x >> 5;
     const int64_t c = *cnt, nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < c; i += nw) {
         const uint32_t v = list[i];
+        if (A.rp[v + 1] - A.rp[v] > SP_BUDGET) {  // a hub: k_spec_assign_huge
+            if (lane == 0) hlist[atomicAdd(hcnt, 1u)] = v;
+            continue;
+        }
         const uint32_t b0 = A.base[v], cv = sp_class(A, v);
         for (int q = lane; q < SP_WIN / 32; q += 32) s_mask[wib][q] = 0u;
         __syncwarp();
@@ -83,6 +89,44 @@ __global__ void __launch_bounds__(SP_THREADS) k_spec_assign(SpecArgs A, const ui
             }
         }
         __syncwarp();
+    }
+}
+
+// step 1 for the hubs (one CTA per vertex, the window mask in shared memory)
+__global__ void __launch_bounds__(SP_HUGE_THREADS) k_spec_assign_huge(SpecArgs A, const uint32_t *__restrict__ hlist,
+                                                                      const uint32_t *hcnt) {
+    __shared__ uint32_t s_mask[SP_WIN / 32];
+    __shared__ uint32_t s_first;
+    const uint32_t c = *hcnt;
+    for (uint32_t h = blockIdx.x; h < c; h += gridDim.x) {
+        const uint32_t v = hlist[h];
+        const uint32_t b0 = A.base[v], cv = sp_class(A, v);
+        if (threadIdx.x < SP_WIN / 32) s_mask[threadIdx.x] = 0u;
+        if (threadIdx.x == 0) s_first = 0xffffffffu;
+        __syncthreads();
+        for (int64_t x = A.rp[v] + threadIdx.x; x < A.rp[v + 1]; x += blockDim.x) {
+            const uint32_t w = (uint32_t)A.ci[x];
+            if (!sp_admitted(A, cv, w)) continue;
+            const uint32_t cw = A.C[w];
+            if (cw >= b0 && cw - b0 < A.W) atomicOr(&s_mask[(cw - b0) >> 5], 1u << ((cw - b0) & 31));
+        }
+        __syncthreads();
+        if (threadIdx.x < SP_WIN / 32 && threadIdx.x * 32 < A.W) {
+            uint32_t free = ~s_mask[threadIdx.x];
+            const uint32_t lim = A.W - threadIdx.x * 32;
+            if (lim < 32) free &= (1u << lim) - 1u;
+            if (free) atomicMin(&s_first, threadIdx.x * 32 + (uint32_t)(__ffs(free) - 1));
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            if (s_first != 0xffffffffu) {
+                A.T[v] = b0 + s_first;
+            } else {
+                A.T[v] = 0u;
+                A.base[v] = b0 + A.W;
+            }
+        }
+        __syncthreads();
     }
 }
 
@@ -121,6 +165,7 @@ __global__ void __launch_bounds__(SP_THREADS) k_spec_detect(SpecArgs A, const ui
         const uint32_t v = list[i];
         const uint32_t col = A.C[v];
         if (col == 0u) continue;  // waited (window full)
+        if (A.rp[v + 1] - A.rp[v] > SP_BUDGET) continue;  // a hub: k_spec_detect_huge
         const uint32_t cv = sp_class(A, v);
         bool self = false;
         for (int64_t x = A.rp[v] + lane; x < A.rp[v + 1]; x += 32) {
@@ -130,6 +175,27 @@ __global__ void __launch_bounds__(SP_THREADS) k_spec_detect(SpecArgs A, const ui
             else sp_flag(A, w, rlist, rcnt);  // a lower (maybe older) end
         }
         if (__any_sync(FULL, self) && lane == 0) sp_flag(A, v, rlist, rcnt);
+    }
+}
+
+// step 2 for the hubs (one CTA per vertex of the hub list)
+__global__ void __launch_bounds__(SP_HUGE_THREADS) k_spec_detect_huge(SpecArgs A, const uint32_t *__restrict__ hlist,
+                                                                      const uint32_t *hcnt, uint32_t *rlist,
+                                                                      uint32_t *rcnt) {
+    const uint32_t c = *hcnt;
+    for (uint32_t h = blockIdx.x; h < c; h += gridDim.x) {
+        const uint32_t v = hlist[h];
+        const uint32_t col = A.C[v];
+        if (col == 0u) continue;  // uniform across the CTA
+        const uint32_t cv = sp_class(A, v);
+        bool self = false;
+        for (int64_t x = A.rp[v] + threadIdx.x; x < A.rp[v + 1]; x += blockDim.x) {
+            const uint32_t w = (uint32_t)A.ci[x];
+            if (A.C[w] != col || !sp_admitted(A, cv, w)) continue;
+            if (w > v) self = true;
+            else sp_flag(A, w, rlist, rcnt);
+        }
+        if (__syncthreads_or(self) && threadIdx.x == 0) sp_flag(A, v, rlist, rcnt);
     }
 }
 
@@ -287,12 +353,19 @@ static int spec_phase(const FlowArgs &f, ColorWs &w, SpecArgs A, int vb, int pha
         uint32_t *list = w.ul[r & 1], *next = w.ul[(r + 1) & 1];
         SYM_CUDA(cudaMemsetAsync(cnt[(r + 1) & 1], 0, sizeof(uint32_t), s));
         SYM_CUDA(cudaMemsetAsync(rcnt, 0, sizeof(uint32_t), s));
-        k_spec_assign<<<sp_grid(left, SP_WARPS), SP_THREADS, 0, s>>>(A, list, cnt[r & 1]);
+        uint32_t *hlist = reinterpret_cast<uint32_t *>(w.queue), *hcnt = &ctl->huge[0];
+        SYM_CUDA(cudaMemsetAsync(hcnt, 0, sizeof(uint32_t), s));
+        k_spec_assign<<<sp_grid(left, SP_WARPS), SP_THREADS, 0, s>>>(A, list, cnt[r & 1], hlist, hcnt);
+        SYM_LAUNCH_CHECK();
+        k_spec_assign_huge<<<num_sms() * 2, SP_HUGE_THREADS, 0, s>>>(A, hlist, hcnt);
         SYM_LAUNCH_CHECK();
         k_spec_commit<<<sp_grid(left, 256), 256, 0, s>>>(A, list, cnt[r & 1]);
         SYM_LAUNCH_CHECK();
         k_spec_detect<<<sp_grid(left, SP_WARPS), SP_THREADS, 0, s>>>(A, list, cnt[r & 1],
                                                                      reinterpret_cast<uint32_t *>(w.ov), rcnt);
+        SYM_LAUNCH_CHECK();
+        k_spec_detect_huge<<<num_sms() * 2, SP_HUGE_THREADS, 0, s>>>(A, hlist, hcnt, reinterpret_cast<uint32_t *>(w.ov),
+                                                                    rcnt);
         SYM_LAUNCH_CHECK();
         k_spec_next_wait<<<sp_grid(left, 256), 256, 0, s>>>(A, list, cnt[r & 1], next, cnt[(r + 1) & 1]);
         SYM_LAUNCH_CHECK();

@@ -23,16 +23,28 @@ RUNS = [("mis", "none", 0, "default"), ("mis", "none", 0, "per_round"), ("mis", 
         ("mis", "rand", 2, "sparser_first"), ("color", "none", 0, "default"), ("color", "none", 0, "eb"),
         ("color", "none", 0, "vb"), ("color", "none", 0, "lf"), ("color", "none", 0, "sf"),
         ("color", "degk", 2, "default"), ("color", "degk", 2, "eb"), ("color", "degk", 2, "lf"),
-        ("color", "rand", 4, "default"), ("color", "rand", 4, "lower_only"), ("color", "rand", 4, "eb")]
+        ("color", "rand", 4, "default"), ("color", "rand", 4, "lower_only"), ("color", "rand", 4, "eb"),
+        ("mis", "bridge", 0, "default"), ("mm", "bridge", 0, "default"), ("color", "bridge", 0, "default"),
+        ("mm", "rand", 4, "default"), ("mm", "none", 0, "default")]
 
 
 def main():
     rp, ci = G.rmat(24, 16, 1, device="cuda")
     m = ci.numel() // 2
-    fns = {"mis": sb.sym_mis, "color": sb.sym_color}
+    fns = {"mis": sb.sym_mis, "mm": sb.sym_mm, "color": sb.sym_color}
     out = {}
     for prob, kind, p, var in RUNS:
-        d = sb.sym_decompose(rp, ci, kind, p, 42) if kind != "none" else None
+        dms = None
+        if kind != "none":
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            sb.sym_decompose(rp, ci, kind, p, 42)
+            a.record()
+            d = sb.sym_decompose(rp, ci, kind, p, 42)
+            b.record()
+            torch.cuda.synchronize()
+            dms = a.elapsed_time(b)
+        else:
+            d = None
         call = lambda: fns[prob](rp, ci, kind, p, 42, decomp=d, flags=F[var])  # noqa: E731
         call()
         ts = []
@@ -45,7 +57,7 @@ def main():
             ts.append(a.elapsed_time(b))
         res, st = fns[prob](rp, ci, kind, p, 42, decomp=d, stats=True, flags=F[var] | 2)
         key = f"{prob}_{kind}{p}_{var}"
-        out[key] = {"ms": statistics.median(ts), "edges_per_s": m / statistics.median(ts) * 1e3,
+        out[key] = {"ms": statistics.median(ts), "decompose_ms": dms, "edges_per_s": m / statistics.median(ts) * 1e3,
                     "rounds": st["rounds"], "result_size": st["result_size"]}
         print(key, out[key], flush=True)
         del d
