@@ -48,7 +48,16 @@ int main(int argc,char**argv){ TH=atol(getenv("TH")); NP=atoi(getenv("NP"));
     }
     for(long i=start;i<nl;i++){ long v=list[i]; col[v]=newc[v]; }
     }
-    for(long i=0;i<nl;i++){ long v=list[i]; int c=col[v]; for(long j=lp[v];j<lp[v+1];j++){int w=lc[j]; forb[(size_t)w*W+c/64]|=1ull<<(c%64); cnt[w]--;}}
+    long big[4]={0,0,0,0}, lact=0, maxld=0; static long rbig[4], rounds_t, lact_t, rnobig;
+    static const long TB[4]={8,256,2048,8192};
+    for(long i=0;i<nl;i++){ long v=list[i]; int c=col[v]; long ld=lp[v+1]-lp[v]; if(ld>maxld) maxld=ld;
+      for(int t=0;t<4;t++) if(ld>TB[t]) big[t]++;
+      for(long j=lp[v];j<lp[v+1];j++){int w=lc[j]; forb[(size_t)w*W+c/64]|=1ull<<(c%64); cnt[w]--;
+        if(cnt[w]==TH && hp[w+1]-hp[w]>TH) lact++;}}
+    if(round>=20){ rounds_t++; lact_t+=lact; for(int t=0;t<4;t++) if(big[t]) rbig[t]++; if(!big[1]&&!lact) rnobig++;
+      if(getenv("TAILSTATS")&&round%20==0) printf("R %d commits %ld ld>8 %ld ld>256 %ld ld>2048 %ld maxld %ld longact %ld\n",round,nl,big[0],big[1],big[2],maxld,lact); }
+    if(left-nl<=0&&getenv("TAILSTATS")) printf("tail rounds %ld: with ld>8 %ld >256 %ld >2048 %ld >8192 %ld; long-row activations %ld; rounds with neither ld>256 nor long activation %ld\n",
+      rounds_t,rbig[0],rbig[1],rbig[2],rbig[3],lact_t,rnobig);
     left-=nl; round++;
     if(round<4||round%100==0) printf("round %d coloured %ld (early %ld) left %ld work %ld\n",round,nl,early,left,work);
   }
