@@ -42,7 +42,9 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and up_to_date():
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, *ARCH, *FLAGS, "-I", os.path.join(ROOT, "include"), "-o", tmp, *sources(), "-lnccl"]
+    # SYM_NVCC_DEFS: extra -D knobs for experiments (tools/jp_variants.sh); unset for the product
+    extra = os.environ.get("SYM_NVCC_DEFS", "").split()
+    cmd = [NVCC, *ARCH, *FLAGS, *extra, "-I", os.path.join(ROOT, "include"), "-o", tmp, *sources(), "-lnccl"]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd))

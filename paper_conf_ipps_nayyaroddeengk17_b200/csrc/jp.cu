@@ -61,23 +61,20 @@ constexpr int JP_TPT = JP_TILE / JP_THREADS;
 #define SYM_JP_LANE_CHECKS 4
 #endif
 constexpr int JP_LANE_CHECKS = SYM_JP_LANE_CHECKS;  // phase A: entries a lane checks before the warp takes over
-#ifndef SYM_JP_PUSH
-#define SYM_JP_PUSH 256
-#endif
 #ifndef SYM_JP_WATCH
 #define SYM_JP_WATCH 64
 #endif
 #ifndef SYM_JP_WLIST
 #define SYM_JP_WLIST 64
 #endif
-constexpr int JP_PUSH = SYM_JP_PUSH;  // phase B: lower entries per push task
-constexpr int JP_PUSH_LANE = 8;  // phase B: tasks of <= JP_PUSH_LANE entries are a lane's
+#ifndef SYM_JP_PUSH_LANE
+#define SYM_JP_PUSH_LANE 4
+#endif
+constexpr int JP_PUSH_LANE = SYM_JP_PUSH_LANE;  // phase B: tasks of <= JP_PUSH_LANE entries are a lane's
+constexpr int JP_PUSH = 32 * JP_PUSH_LANE;  // phase B: lower entries per push task (one warp step)
 constexpr uint32_t JP_WATCH = SYM_JP_WATCH;  // a vertex checks once <= JP_WATCH higher neighbours are unpushed
 constexpr uint32_t JP_WLIST = SYM_JP_WLIST;  // higher lists up to JP_WLIST entries are their own watch list
 constexpr uint32_t JP_NOTBUILT = 0xffffffffu;
-#ifndef SYM_JP_PUSH_FILTER0
-#define SYM_JP_PUSH_FILTER0 0  // 1: also filter colours 1..32 (a load on the chain; 26.3 vs 26.05 ms)
-#endif
 constexpr int JP_BUILD = 256;    // phase B: higher entries per watch-list build task
 constexpr uint32_t JP_HBITS = 27;  // hot.w = offset of the extra bitmap words | min(R, 31) << 27
 constexpr uint32_t JP_HMASK = (1u << JP_HBITS) - 1u;
@@ -115,6 +112,8 @@ struct JpArgs {
     uint32_t *err;       // 1 = timeout / max rounds, 2 = offsets overflow
     uint32_t *hist;
     uint32_t *trace;     // nullable: per-round diagnostics (SYM_JP_TRACE)
+    int trace2;          // SYM_JP_TRACE=2: slots 512.. / 1024.. hold the slowest warp's push /
+                         //   build span of phase B instead of the task counts
     unsigned long long *prof;  // profiling counter pair {alg, impl} of the current launch (nullable)
     unsigned long long *prof_jp;  // the rounds launch's pair: the count pass adds §8(d)'s JP bytes
     Key k;
@@ -805,10 +804,16 @@ struct JpLane {
     int state;  // 0 checking, 1 passed, 2 failed (memo pos/lm), 3 idle, 5 watch list not built
 };
 
+// SPARSE (a round with at most one vertex per warp -- the latency-bound tail): every
+// step is warp-wide instead -- the extra bitmap words 32 at a time, the list 64
+// entries per step (a watch list holds <= JP_WATCH = 64), no lane stage -- so a check
+// is ~4 dependent loads instead of ~10.
+template <bool SPARSE>
 __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_in, JpLane &L,
                                          unsigned long long &bytes) {
     const int lane = lane_id();
     uint32_t h = h_in, R = 1, hd = 0, ld = 0, wc = 0, pos = 0, lm = 0, m = 1;
+    uint32_t xwo = 0;  // SPARSE: offset of h's extra bitmap words
     uint64_t off = 0;
     int state = 3;
     if (act) {
@@ -829,23 +834,49 @@ __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_i
             const uint32_t z0 = ~hs.z;
             if (z0) {
                 m = __ffs(z0);
-            } else {  // colours > 32
+            } else if (SPARSE) {
+                m = 0;  // the warp scans the extra words below
+                xwo = hs.w & JP_HMASK;
+            } else {  // colours > 32: bits are only ever set, so m >= the m of the last
+                      // failed check (lm) -- the scan starts at lm's word, 4 words in flight
                 const uint32_t *xw = A.xb + (hs.w & JP_HMASK);
-                for (uint32_t k = 1; k < R; k++) {
-                    const uint32_t z = ~__ldcg(xw + k - 1);
-                    if (z) {
-                        m = k * 32 + __ffs(z);
-                        break;
-                    }
+                uint32_t k = lm > 32u ? (lm - 1) >> 5 : 1u;
+                for (m = 0; m == 0 && k < R; k += 4) {
+                    uint32_t z[4];
+#pragma unroll
+                    for (int u = 0; u < 4; u++) z[u] = k + u < R ? ~__ldcg(xw + k + u - 1) : 0u;
+#pragma unroll
+                    for (int u = 3; u >= 0; u--)
+                        if (z[u]) m = (k + u) * 32 + __ffs(z[u]);
                 }
-                if (m == 1) m = R * 32 + 1;  // unreachable: a zero lies within cap bits
+                if (m == 0) m = R * 32 + 1;  // unreachable: a zero lies within cap bits
             }
+        }
+    }
+    if (SPARSE) {  // warp-wide mex over the extra bitmap words, 32 words per step
+        unsigned need = __ballot_sync(FULL, state == 0 && m == 0);
+        while (need) {
+            const int src = __ffs(need) - 1;
+            need &= need - 1;
+            const uint32_t sR = __shfl_sync(FULL, R, src), slm = __shfl_sync(FULL, lm, src);
+            const uint32_t *xw = A.xb + __shfl_sync(FULL, xwo, src);
+            uint32_t k = slm > 32u ? (slm - 1) >> 5 : 1u, mm = sR * 32 + 1;  // fallback unreachable
+            for (; k < sR; k += 32) {
+                const uint32_t z = k + lane < sR ? ~__ldcg(xw + k + lane - 1) : 0u;
+                const unsigned b = __ballot_sync(FULL, z != 0u);
+                if (b) {
+                    const int f = __ffs(b) - 1;
+                    mm = (k + f) * 32 + __ffs(__shfl_sync(FULL, z, f));
+                    break;
+                }
+            }
+            if (lane == src) m = mm;
         }
     }
     const uint32_t q = (m - 1) >> 5, bit = (m - 1) & 31;
     uint32_t j = (lm == m && pos < wc) ? pos : 0u;  // m unchanged: resume at the last blocker
     // ---- lane: the first JP_LANE_CHECKS entries (all loads of a stage in flight)
-    if (state == 0) {
+    if (!SPARSE && state == 0) {
         uint32_t e[JP_LANE_CHECKS], c[JP_LANE_CHECKS], w[JP_LANE_CHECKS], r5[JP_LANE_CHECKS];
 #pragma unroll
         for (int u = 0; u < JP_LANE_CHECKS; u++) e[u] = j + u < wc ? __ldcg(A.lst + off + j + u) : 0u;
@@ -887,27 +918,38 @@ __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_i
         const uint32_t wwc = __shfl_sync(FULL, wc, src), wm = __shfl_sync(FULL, m, src);
         const uint64_t woff = __shfl_sync(FULL, off, src);
         const uint32_t wq = (wm - 1) >> 5, wbit = (wm - 1) & 31;
-        int wstate = 0;
+        int wstate = wj >= wwc ? 1 : 0;
         uint32_t wpos = 0;
+        constexpr int S = SPARSE ? 2 : 1;  // entries per lane per step
         while (wstate == 0) {
-            const uint32_t jj = wj + lane;
-            bool ok = true;
-            if (jj < wwc) {
-                const uint32_t eu = __ldcg(A.lst + woff + jj);
-                uint32_t cu, wu, ru;
-                nb_load(A, eu, wq, cu, wu, ru);
-                if (wq > 0 && cu == 0u && wq < ru) wu = __ldcg(A.xb + wu + wq - 1);
-                ok = nb_ok(A, eu, cu, wu, ru, wm, wq, wbit);
+            bool ok[S];
+            uint32_t eu[S], cu[S], wu[S], ru[S];
+#pragma unroll
+            for (int u = 0; u < S; u++) eu[u] = wj + u * 32 + lane < wwc ? __ldcg(A.lst + woff + wj + u * 32 + lane) : 0u;
+#pragma unroll
+            for (int u = 0; u < S; u++) {
+                ok[u] = true;
+                if (wj + u * 32 + lane < wwc) {
+                    nb_load(A, eu[u], wq, cu[u], wu[u], ru[u]);
+                    if (wq > 0 && cu[u] == 0u && wq < ru[u]) wu[u] = __ldcg(A.xb + wu[u] + wq - 1);
+                }
             }
-            const unsigned fails = __ballot_sync(FULL, !ok);
-            if (fails) {
-                wstate = 2;
-                wpos = wj + __ffs(fails) - 1;
-            } else {
-                wj += 32;
+#pragma unroll
+            for (int u = 0; u < S; u++)
+                if (wj + u * 32 + lane < wwc) ok[u] = nb_ok(A, eu[u], cu[u], wu[u], ru[u], wm, wq, wbit);
+#pragma unroll
+            for (int u = 0; u < S; u++) {
+                const unsigned fails = __ballot_sync(FULL, !ok[u]);
+                if (wstate == 0 && fails) {
+                    wstate = 2;
+                    wpos = wj + u * 32 + __ffs(fails) - 1;
+                }
+            }
+            if (wstate == 0) {
+                wj += 32 * S;
                 if (wj >= wwc) wstate = 1;
             }
-            bytes += lane == 0 ? 384ull : 0ull;
+            bytes += lane == 0 ? 384ull * S : 0ull;
         }
         if (lane == src) {
             state = wstate;
@@ -945,7 +987,8 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
         const int64_t i = it + (spread ? (int64_t)lane * nwarps + warp_g : warp_g * 32 + lane);
         const bool act = i < cnt;
         JpLane L;
-        jp_check(A, act, act ? __ldcg(U + i) : 0u, L, bytes);
+        if (cnt <= nwarps) jp_check<true>(A, act, act ? __ldcg(U + i) : 0u, L, bytes);
+        else jp_check<false>(A, act, act ? __ldcg(U + i) : 0u, L, bytes);
         const uint32_t h = L.h, hd = L.hd, ld = L.ld, pos = L.pos, lm = L.lm, m = L.m;
         const uint64_t off = L.off;
         const int state = L.state;
@@ -1000,99 +1043,188 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
 // bit and one higher neighbour less to wait for.  The push that brings a count to
 // JP_WATCH activates the neighbour (next round's list).  Each stage's loads/atomics
 // are in flight together.
+// 4-B L2 load under a predicate (0xffffffff when !p), no branch
+__device__ __forceinline__ uint32_t ld_cg_pred(const uint32_t *addr, bool p) {
+    uint32_t v = 0xffffffffu;
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q ld.global.cg.u32 %0, [%1];\n\t}"
+                 : "+r"(v)
+                 : "l"(addr), "r"((uint32_t)p)
+                 : "memory");
+    return v;
+}
+
+// returning atomic decrement under a predicate (0 when !p), no branch
+__device__ __forceinline__ uint32_t atom_dec_pred(uint32_t *addr, bool p) {
+    uint32_t old = 0u;
+    asm volatile(
+        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q atom.global.add.u32 %0, [%1], %3;\n\t}"
+        : "+r"(old)
+        : "l"(addr), "r"((uint32_t)p), "r"(0xffffffffu)
+        : "memory");
+    return old;
+}
+
+#ifndef SYM_JP_DIAG
+#define SYM_JP_DIAG 0  // 1: compile the SYM_JP_TRACE=3/4 sub-step timers (they cost registers)
+#endif
+// diagnostics (SYM_JP_TRACE=4): wait for v, then read the timer
+__device__ __forceinline__ uint64_t jp_stamp_after(uint32_t v, uint32_t *sink) {
+    if (__ballot_sync(FULL, v == 0x7fffffe1u) == 0xffffffffu) *sink = 0u;
+    return globaltimer_ns();
+}
+
 template <int K, class Activate>
 __device__ __forceinline__ void jp_push(const JpArgs &A, const uint32_t (&e)[K], bool (&act)[K], uint32_t q,
-                                        uint32_t bit, const Activate &activate) {
-    uint32_t old[K], x[K];
-#pragma unroll
-    for (int u = 0; u < K; u++) {  // colour, R field and extra-word offset in one 16-B load
-        x[u] = 0xffffffffu;
-#if SYM_JP_PUSH_FILTER0
-        if (act[u]) {
-#else
-        if (act[u] && q > 0) {  // colours 1..32: no filter load, the atomics go straight out
+                                        uint32_t bit, const Activate &activate, uint32_t *tr4 = nullptr) {
+#if SYM_JP_DIAG
+    const uint64_t tq0 = tr4 ? globaltimer_ns() : 0;
 #endif
-            const uint4 s = __ldcg(A.hot + e[u]);
-            act[u] = s.x == 0u;
-            x[u] = s.w;
-        }
-    }
+    uint32_t old[K], x[K];
+    // the count decrement needs no filter: a coloured neighbour was activated before its
+    // check (count <= JP_WATCH), so its decrement can never be the activating one -- the
+    // atomics go out together with the filter loads (colours > 32: the extra-word offset)
+    // (predicated PTX atomics: with `act ? atomicSub(..) : 0` the compiler branched around
+    // each atomic and tested its result inside the branch, so the K returning atomics ran
+    // one after another -- ~1 us each in the tail)
 #pragma unroll
-    for (int u = 0; u < K; u++) old[u] = act[u] ? atomicSub(&A.hot[e[u]].y, 1u) : 0u;
+    for (int u = 0; u < K; u++) old[u] = atom_dec_pred(&A.hot[e[u]].y, act[u]);
+    // colours > 32: the R field and extra-word offset (hot.w) of every target, loads in
+    // flight together (predicated PTX again).  No colour filter: a bit in the bitmap of
+    // an already coloured vertex is never read (nb_ok tests its colour first).
+#pragma unroll
+    for (int u = 0; u < K; u++) x[u] = ld_cg_pred(&A.hot[e[u]].w, act[u] && q > 0);
+#if SYM_JP_DIAG
+    uint64_t tq1 = 0, tq2 = 0, tq3 = 0;
+    if (tr4) {
+        uint32_t y = 0, z = 0;
+#pragma unroll
+        for (int u = 0; u < K; u++) y ^= old[u], z ^= x[u];
+        tq1 = jp_stamp_after(y, tr4 + 3);
+        tq2 = jp_stamp_after(z, tr4 + 3);
+    }
+#endif
     if (q == 0) {
 #pragma unroll
         for (int u = 0; u < K; u++)
             if (act[u]) atomicOr(&A.hot[e[u]].z, 1u << bit);
     } else {
+        uint32_t Rf[K];  // saturated R field (>= 31 words): the full count from meta
+#pragma unroll
+        for (int u = 0; u < K; u++)
+            Rf[u] = ld_cg_pred(&A.meta[2 * e[u]].x, act[u] && (x[u] >> JP_HBITS) == JP_R5 && q >= JP_R5);
 #pragma unroll
         for (int u = 0; u < K; u++) {
             const uint32_t R5 = x[u] >> JP_HBITS;
-            bool go = act[u] && q < R5;
-            if (act[u] && !go && R5 == JP_R5) go = q < __ldg(&A.meta[2 * e[u]].x);
+            const bool go = act[u] && (q < R5 || (R5 == JP_R5 && q < Rf[u]));
             x[u] = go ? (x[u] & JP_HMASK) : 0xffffffffu;
         }
 #pragma unroll
         for (int u = 0; u < K; u++)
             if (x[u] != 0xffffffffu) atomicOr(A.xb + x[u] + q - 1, 1u << bit);
     }
+#if SYM_JP_DIAG
+    if (tr4) {
+        uint32_t z = 0;
 #pragma unroll
-    for (int u = 0; u < K; u++)
-        if (act[u] && old[u] == JP_WATCH + 1u) activate(e[u]);
+        for (int u = 0; u < K; u++) z ^= x[u];
+        tq3 = jp_stamp_after(z, tr4 + 3);
+    }
+#endif
+    // activations: one warp-aggregated reservation on the next list (all lanes call)
+    uint32_t na = 0;
+#pragma unroll
+    for (int u = 0; u < K; u++) na += (act[u] && old[u] == JP_WATCH + 1u) ? 1u : 0u;
+    if (__any_sync(FULL, na != 0)) {
+        const int lane = lane_id();
+        uint32_t incl = na;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(FULL, incl, d);
+            if (lane >= d) incl += y;
+        }
+        uint32_t base = 0;
+        if (lane == 31) base = atomicAdd(activate.cnt, incl);
+        uint32_t slot = __shfl_sync(FULL, base, 31) + incl - na;
+#pragma unroll
+        for (int u = 0; u < K; u++)
+            if (act[u] && old[u] == JP_WATCH + 1u) activate.list[slot++] = e[u];
+    }
+#if SYM_JP_DIAG
+    if (tr4) {
+        __syncwarp();
+        const uint64_t tq4 = globaltimer_ns();
+        if (lane_id() == 0) {  // slowest: atomics returned, hot loads, saturated-R loads + REDs, activations
+            atomicMax(tr4 + 512, (uint32_t)((tq1 - tq0) >> 5));
+            atomicMax(tr4 + 1024, (uint32_t)((tq2 - tq1) >> 5));
+            atomicMax(tr4 + 1536, (uint32_t)((tq4 - tq3) >> 5));
+        }
+    }
+#endif
 }
 
 // round mode: an activated vertex joins round r+1's list
 struct JpNextList {
-    const JpArgs &A;
-    uint32_t r;
-    __device__ __forceinline__ void operator()(uint32_t e) const {
-        const uint32_t slot = atomicAdd(A.ucnt + (r + 1) % 3, 1u);
-        A.ul[(r + 1) & 1][slot] = e;
-    }
+    uint32_t *cnt, *list;
+    __device__ __forceinline__ JpNextList(const JpArgs &A, uint32_t r)
+        : cnt(A.ucnt + (r + 1) % 3), list(A.ul[(r + 1) & 1]) {}
 };
 
 // Phase B of round r: push the new colours; build the requested watch lists
 __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, uint32_t cnt, uint32_t nbt,
                                            int64_t warp_g, int64_t nwarps, unsigned long long &bytes) {
     const int lane = lane_id();
+    const bool tr = A.trace2 && A.trace && r < 512;
+    const uint64_t tp0 = tr ? globaltimer_ns() : 0;
     for (int64_t base = warp_g; base - warp_g < cnt; base += nwarps * 32) {
         const int64_t i = base + (int64_t)lane * nwarps;  // tasks spread over all warps
         uint4 tk = make_uint4(0u, 0u, 0u, 0u);
         if (i < cnt) tk = __ldcg(A.task + i);
         const uint64_t s0 = (uint64_t)tk.x | ((uint64_t)tk.y << 32);
-        const bool small = tk.z > 0 && tk.z <= JP_PUSH_LANE;
-        if (small) {
-            const uint32_t q = (tk.w - 1) >> 5, bit = (tk.w - 1) & 31;
+        // one jp_push shape for both kinds: first every lane's own small task (<=
+        // JP_PUSH_LANE entries), then each big task with its entries spread over the warp
+        static_assert(JP_PUSH == 32 * JP_PUSH_LANE, "a big task is one warp step");
+        bool small = tk.z > 0 && tk.z <= JP_PUSH_LANE;
+        unsigned bigm = __ballot_sync(FULL, tk.z > JP_PUSH_LANE);
+        bool pend = __any_sync(FULL, small);
+        while (pend || bigm) {
+            uint64_t ws;
+            uint32_t wn, wc, stride, first;
+            if (pend) {  // own small tasks
+                ws = s0;
+                wn = small ? tk.z : 0u;
+                wc = tk.w;
+                stride = 1;
+                first = 0;
+                pend = false;
+                bytes += 4ull * wn;
+            } else {
+                const int src = __ffs(bigm) - 1;
+                bigm &= bigm - 1;
+                ws = __shfl_sync(FULL, s0, src);
+                wn = __shfl_sync(FULL, tk.z, src);
+                wc = __shfl_sync(FULL, tk.w, src);
+                stride = 32;
+                first = lane;
+                bytes += lane == 0 ? 4ull * wn : 0ull;
+            }
+            const uint32_t q = (wc - 1) >> 5, bit = (wc - 1) & 31;
             uint32_t e[JP_PUSH_LANE];
             bool act[JP_PUSH_LANE];
 #pragma unroll
             for (int u = 0; u < JP_PUSH_LANE; u++) {
-                act[u] = u < (int)tk.z;
-                e[u] = act[u] ? __ldcs(A.lst + s0 + u) : 0u;
+                const uint32_t j = first + u * stride;
+                act[u] = j < wn;
+                e[u] = act[u] ? __ldcs(A.lst + ws + j) : 0u;
             }
-            jp_push<JP_PUSH_LANE>(A, e, act, q, bit, JpNextList{A, r});
-            bytes += 4ull * tk.z;
-        }
-        unsigned bigm = __ballot_sync(FULL, tk.z > JP_PUSH_LANE);
-        while (bigm) {
-            const int src = __ffs(bigm) - 1;
-            bigm &= bigm - 1;
-            const uint64_t ws = __shfl_sync(FULL, s0, src);
-            const uint32_t wn = __shfl_sync(FULL, tk.z, src), wc = __shfl_sync(FULL, tk.w, src);
-            const uint32_t q = (wc - 1) >> 5, bit = (wc - 1) & 31;
-            constexpr int K = JP_PUSH / 32;
-            uint32_t e[K];
-            bool act[K];
-#pragma unroll
-            for (int u = 0; u < K; u++) {
-                act[u] = u * 32 + lane < (int)wn;
-                e[u] = act[u] ? __ldcs(A.lst + ws + u * 32 + lane) : 0u;
-            }
-            jp_push<K>(A, e, act, q, bit, JpNextList{A, r});
-            bytes += lane == 0 ? 4ull * wn : 0ull;
+            jp_push<JP_PUSH_LANE>(A, e, act, q, bit, JpNextList(A, r),
+                                  SYM_JP_DIAG && tr && A.trace2 == 4 ? A.trace + r : nullptr);
         }
     }
-    // watch lists: a warp per task filters JP_BUILD higher entries (uncoloured ones kept)
-    for (int64_t t = warp_g; t < nbt; t += nwarps) {
+    const uint64_t tp1 = tr ? globaltimer_ns() : 0;
+    if (tr && A.trace2 == 2 && lane == 0 && warp_g < cnt) atomicMax(A.trace + 512 + r, (uint32_t)((tp1 - tp0) >> 5));
+    // (the last warps first: in a tail round the push tasks sit on the first warps, so a
+    // warp holds a push OR a build and phase B is one dependent chain, not two)
+    for (int64_t t = nwarps - 1 - warp_g; t < nbt; t += nwarps) {
         const uint4 bt = __ldcg(A.btask + t);
         const uint64_t wl = ((uint64_t)(bt.y >> 24) << 32) | bt.w, hl = wl + watch_words(bt.z);
         uint32_t *wcp = reinterpret_cast<uint32_t *>(A.meta + 2 * bt.x) + 3;
@@ -1121,6 +1253,8 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, uint32_t
         }
         bytes += lane == 0 ? 8ull * (j1 - j0) : 0ull;
     }
+    if (tr && A.trace2 == 2 && lane == 0 && nwarps - 1 - warp_g < nbt)
+        atomicMax(A.trace + 1024 + r, (uint32_t)((globaltimer_ns() - tp1) >> 5));
 }
 
 #ifndef SYM_JR_THREADS
@@ -1162,12 +1296,14 @@ __global__ void __launch_bounds__(JR_THREADS, SYM_JR_MINB) k_jp_rounds(JpArgs A,
         const uint32_t pc = s_val[0], bc = s_val[1];
         if (A.trace && blockIdx.x == 0 && threadIdx.x == 0 && r < 512) {  // diagnostics
             A.trace[r] = (uint32_t)((globaltimer_ns() - t0) >> 5);
-            A.trace[512 + r] = __ldcg(A.pcnt + r % 3);
-            A.trace[1024 + r] = __ldcg(A.bcnt + r % 3);
+            if (!A.trace2) {
+                A.trace[512 + r] = __ldcg(A.pcnt + r % 3);
+                A.trace[1024 + r] = __ldcg(A.bcnt + r % 3);
+            }
         }
         const uint64_t tb = A.trace ? globaltimer_ns() : 0;
         jp_phase_b(A, r, pc, bc, warp_g, nwarps, bytes);
-        if (A.trace && r < 512) {  // diagnostics: slowest CTA's phase-B work span
+        if (A.trace && A.trace2 < 3 && r < 512) {  // diagnostics: slowest CTA's phase-B work span
             __syncthreads();
             if (threadIdx.x == 0) atomicMax(A.trace + 1536 + r, (uint32_t)((globaltimer_ns() - tb) >> 5));
         }
@@ -1307,6 +1443,7 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     A.err = w.sync + 32;
     A.hist = nullptr;
     A.trace = nullptr;
+    A.trace2 = 0;
     A.prof = nullptr;
     A.prof_jp = rounds_ctr;
     A.k = stream_key(f.p.seed, TAG_VERTEX, 0);
@@ -1412,6 +1549,8 @@ static int jp_run(const FlowArgs &f, ColorWs &w, uint32_t *color, const int64_t 
     A.hist = f.stats ? ctl->hist + phase * 2048 : nullptr;
     static const bool jp_trace = getenv("SYM_JP_TRACE") != nullptr;
     A.trace = jp_trace && f.stats && phase == 0 ? ctl->hist + 2048 : nullptr;
+    static const int jp_trace2 = jp_trace ? atoi(getenv("SYM_JP_TRACE")) : 0;
+    A.trace2 = jp_trace2 >= 2 ? jp_trace2 : 0;  // 2: push / build spans, 3: push sub-steps
     if (A.trace) SYM_CUDA(cudaMemsetAsync(A.trace, 0, 2048 * sizeof(uint32_t), s));
     A.prof = rounds_ctr;
     void *args[] = {&A, &C};

@@ -32,7 +32,14 @@ print("rounds", st["rounds"])
 dt = np.diff(t[:min(R, 1024)])
 for r in list(range(0, 16)) + list(range(20, min(R, 1023), 40)):
     if r < len(dt):
-        extra = f" A {pa[r]-t[r]:7.2f} us pushT {tr[512+r]:7d} buildT {tr[1024+r]:7d} Bwork {tr[1536+r]*0.032:7.2f}" if r < 512 else ""
+        if os.environ.get("SYM_JP_TRACE") == "4":  # slowest big push: atomics returned, hot loads, activations
+            extra = (f" A {pa[r]-t[r]:7.2f} us atom {tr[512+r]*0.032:6.2f} hot {tr[1024+r]*0.032:6.2f}"
+                     f" activ {tr[1536+r]*0.032:7.2f}") if r < 512 else ""
+        elif os.environ.get("SYM_JP_TRACE") == "2":  # slowest warp's push / build span of phase B
+            extra = (f" A {pa[r]-t[r]:7.2f} us push {tr[512+r]*0.032:6.2f} build {tr[1024+r]*0.032:6.2f}"
+                     f" Bwork {tr[1536+r]*0.032:7.2f}") if r < 512 else ""
+        else:
+            extra = f" A {pa[r]-t[r]:7.2f} us pushT {tr[512+r]:7d} buildT {tr[1024+r]:7d} Bwork {tr[1536+r]*0.032:7.2f}" if r < 512 else ""
         print(f"R{r:5d} |U| {cnt[r]:9d} t {t[r]:9.1f} us  dt {dt[r]:7.2f} us" + extra)
 if len(dt) > 40:
     print("median dt (rounds >= 20)", np.median(dt[20:]), "mean", dt[20:].mean())
