@@ -728,6 +728,38 @@ __global__ void k_jpc_scatter(JpArgs A) {
 }
 
 // ---------------------------------------------------------------- rounds
+// Predicated PTX loads/atomics (no branch per element): with `p ? load : default` the
+// compiler branched around each access and, short of registers, consumed its result
+// inside the branch, so K independent accesses ran one after another (~1 us each).
+__device__ __forceinline__ uint32_t ld_cg_pred(const uint32_t *addr, bool p) {  // 0xffffffff if !p
+    uint32_t v = 0xffffffffu;
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q ld.global.cg.u32 %0, [%1];\n\t}"
+                 : "+r"(v)
+                 : "l"(addr), "r"((uint32_t)p)
+                 : "memory");
+    return v;
+}
+
+__device__ __forceinline__ uint4 ld_cg_v4_pred(const uint4 *addr, bool p) {  // {1,0,0,0} if !p
+    uint4 v = make_uint4(1u, 0u, 0u, 0u);
+    asm volatile(
+        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %5, 0;\n\t@q ld.global.cg.v4.u32 {%0, %1, %2, %3}, [%4];\n\t}"
+        : "+r"(v.x), "+r"(v.y), "+r"(v.z), "+r"(v.w)
+        : "l"(addr), "r"((uint32_t)p)
+        : "memory");
+    return v;
+}
+
+__device__ __forceinline__ uint32_t atom_add_pred(uint32_t *addr, uint32_t val, bool p) {  // 0 if !p
+    uint32_t old = 0u;
+    asm volatile(
+        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q atom.global.add.u32 %0, [%1], %3;\n\t}"
+        : "+r"(old)
+        : "l"(addr), "r"((uint32_t)p), "r"(val)
+        : "memory");
+    return old;
+}
+
 __device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *p) {
     uint32_t v;
     asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -761,34 +793,44 @@ __device__ __forceinline__ void grid_sync(const JrCtl &C, uint32_t &k, const uin
         const uint32_t target = k * gridDim.x;
         while (ld_acquire_u32(C.arr) < target) {
         }
-        if (p0) sm[0] = __ldcg(p0);
-        if (p1) sm[1] = __ldcg(p1);
-        if (p2) sm[2] = __ldcg(p2);
+        // the three counter loads in flight together (predicated, see ld_cg_pred)
+        const uint32_t v0 = ld_cg_pred(p0, p0 != nullptr), v1 = ld_cg_pred(p1, p1 != nullptr),
+                       v2 = ld_cg_pred(p2, p2 != nullptr);
+        if (p0) sm[0] = v0;
+        if (p1) sm[1] = v1;
+        if (p2) sm[2] = v2;
     }
     __syncthreads();
 }
 
-// Can higher neighbour e (list id) not take colour m (word q, bit)?  Coloured: its
-// colour differs; uncoloured: m is forbidden for it, or m > cap (q >= R).  c = its
-// colour, w = its bitmap word q when q < R (loaded by the caller).
-__device__ __forceinline__ bool nb_ok(const JpArgs &A, uint32_t e, uint32_t c, uint32_t w, uint32_t R5, uint32_t m,
-                                      uint32_t q, uint32_t bit) {
-    if (c != 0u) return c != m;
-    if (q == 0u || q < R5) return (w >> bit) & 1u;
-    if (R5 < JP_R5) return true;  // m > 32 R >= cap: the neighbour's colour is below m
-    const uint32_t R = __ldg(&A.meta[2 * e].x);  // saturated R field: the full count
-    return q >= R || ((__ldcg(A.xb + (__ldcg(&A.hot[e].w) & JP_HMASK) + q - 1) >> bit) & 1u);
-}
-
-// a neighbour's colour c, R field and bitmap word q (q == 0: bm0; q < R: offset of
-// its words in xb, resolved by the caller; else unused) from ONE 16-B load of its
-// hot record
-__device__ __forceinline__ void nb_load(const JpArgs &A, uint32_t e, uint32_t q, uint32_t &c, uint32_t &w,
-                                        uint32_t &R5) {
-    const uint4 s = __ldcg(A.hot + e);
-    c = s.x;
-    R5 = s.w >> JP_HBITS;
-    w = q == 0u ? s.z : (q < R5 ? (s.w & JP_HMASK) : 0u);
+// One check stage over N watch-list entries e[u] (valid[u]): can higher neighbour e
+// not take colour m (word q, bit)?  Coloured: its colour differs; uncoloured: m is
+// forbidden for it, or m > cap (q >= R).  Three batched load steps: the 16-B hot
+// records; the full R of saturated R fields (>= 31 words, from meta); the bitmap words
+// q of the uncoloured ones.
+template <int N>
+__device__ __forceinline__ void jp_nb_stage(const JpArgs &A, const uint32_t (&e)[N], const bool (&valid)[N],
+                                            uint32_t m, uint32_t q, uint32_t bit, bool (&ok)[N]) {
+    uint4 s[N];
+    uint32_t Rf[N], wd[N];
+#pragma unroll
+    for (int u = 0; u < N; u++) s[u] = ld_cg_v4_pred(A.hot + e[u], valid[u]);
+#pragma unroll
+    for (int u = 0; u < N; u++)
+        Rf[u] = ld_cg_pred(&A.meta[2 * e[u]].x, valid[u] && s[u].x == 0u && q >= JP_R5 && (s[u].w >> JP_HBITS) == JP_R5);
+#pragma unroll
+    for (int u = 0; u < N; u++) {
+        const uint32_t R5 = s[u].w >> JP_HBITS, R = R5 < JP_R5 ? R5 : (q >= JP_R5 ? Rf[u] : JP_R5);
+        wd[u] = ld_cg_pred(A.xb + (s[u].w & JP_HMASK) + q - 1, valid[u] && s[u].x == 0u && q > 0u && q < R);
+        Rf[u] = R;
+    }
+#pragma unroll
+    for (int u = 0; u < N; u++) {
+        if (!valid[u]) ok[u] = true;
+        else if (s[u].x != 0u) ok[u] = s[u].x != m;
+        else if (q == 0u) ok[u] = (s[u].z >> bit) & 1u;
+        else ok[u] = q >= Rf[u] || ((wd[u] >> bit) & 1u);  // q >= R: m > cap
+    }
 }
 
 // One check of vertex h (compact id; act = the lane holds a vertex): the early-commit
@@ -877,27 +919,20 @@ __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_i
     uint32_t j = (lm == m && pos < wc) ? pos : 0u;  // m unchanged: resume at the last blocker
     // ---- lane: the first JP_LANE_CHECKS entries (all loads of a stage in flight)
     if (!SPARSE && state == 0) {
-        uint32_t e[JP_LANE_CHECKS], c[JP_LANE_CHECKS], w[JP_LANE_CHECKS], r5[JP_LANE_CHECKS];
-#pragma unroll
-        for (int u = 0; u < JP_LANE_CHECKS; u++) e[u] = j + u < wc ? __ldcg(A.lst + off + j + u) : 0u;
+        uint32_t e[JP_LANE_CHECKS];
+        bool valid[JP_LANE_CHECKS], ok[JP_LANE_CHECKS];
 #pragma unroll
         for (int u = 0; u < JP_LANE_CHECKS; u++) {
-            c[u] = 1u;
-            w[u] = 0u;
-            r5[u] = 0u;
-            if (j + u < wc) nb_load(A, e[u], q, c[u], w[u], r5[u]);
+            valid[u] = j + u < wc;
+            e[u] = ld_cg_pred(A.lst + off + j + u, valid[u]);
         }
-        if (q > 0) {
-#pragma unroll
-            for (int u = 0; u < JP_LANE_CHECKS; u++)
-                if (j + u < wc && c[u] == 0u && q < r5[u]) w[u] = __ldcg(A.xb + w[u] + q - 1);
-        }
+        jp_nb_stage<JP_LANE_CHECKS>(A, e, valid, m, q, bit, ok);
 #pragma unroll
         for (int u = 0; u < JP_LANE_CHECKS; u++) {
             if (state == 0) {
                 if (j >= wc) {
                     state = 1;
-                } else if (!nb_ok(A, e[u], c[u], w[u], r5[u], m, q, bit)) {
+                } else if (!ok[u]) {
                     state = 2;
                     pos = j;
                     lm = m;
@@ -922,21 +957,14 @@ __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_i
         uint32_t wpos = 0;
         constexpr int S = SPARSE ? 2 : 1;  // entries per lane per step
         while (wstate == 0) {
-            bool ok[S];
-            uint32_t eu[S], cu[S], wu[S], ru[S];
-#pragma unroll
-            for (int u = 0; u < S; u++) eu[u] = wj + u * 32 + lane < wwc ? __ldcg(A.lst + woff + wj + u * 32 + lane) : 0u;
+            bool ok[S], valid[S];
+            uint32_t eu[S];
 #pragma unroll
             for (int u = 0; u < S; u++) {
-                ok[u] = true;
-                if (wj + u * 32 + lane < wwc) {
-                    nb_load(A, eu[u], wq, cu[u], wu[u], ru[u]);
-                    if (wq > 0 && cu[u] == 0u && wq < ru[u]) wu[u] = __ldcg(A.xb + wu[u] + wq - 1);
-                }
+                valid[u] = wj + u * 32 + lane < wwc;
+                eu[u] = ld_cg_pred(A.lst + woff + wj + u * 32 + lane, valid[u]);
             }
-#pragma unroll
-            for (int u = 0; u < S; u++)
-                if (wj + u * 32 + lane < wwc) ok[u] = nb_ok(A, eu[u], cu[u], wu[u], ru[u], wm, wq, wbit);
+            jp_nb_stage<S>(A, eu, valid, wm, wq, wbit, ok);
 #pragma unroll
             for (int u = 0; u < S; u++) {
                 const unsigned fails = __ballot_sync(FULL, !ok[u]);
@@ -1013,15 +1041,14 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
             }
         }
         const uint32_t Ts = __shfl_sync(FULL, xs, 31), Tt = __shfl_sync(FULL, xt, 31), Tb = __shfl_sync(FULL, xb_, 31);
-        uint32_t bsv = 0, btv = 0, bbv = 0;
-        if (lane == 0) {
-            if (Ts) bsv = atomicAdd(A.ucnt + (r + 1) % 3, Ts);
-            if (Tt) btv = atomicAdd(A.pcnt + r % 3, Tt);
-            if (Tb) bbv = atomicAdd(A.bcnt + r % 3, Tb);
-        }
-        const int64_t slot = (int64_t)__shfl_sync(FULL, bsv, 0) + xs - (stay ? 1u : 0u);
-        const int64_t ts = (int64_t)__shfl_sync(FULL, btv, 0) + xt - nt;
-        const int64_t bs = (int64_t)__shfl_sync(FULL, bbv, 0) + xb_ - nb;
+        // lanes 0, 1, 2 issue the three reservations as ONE instruction (one round trip;
+        // from a single lane ptxas aggregates each uniform-address atomic separately)
+        uint32_t *ra = lane == 0 ? A.ucnt + (r + 1) % 3 : (lane == 1 ? A.pcnt + r % 3 : A.bcnt + r % 3);
+        const uint32_t rv = lane == 0 ? Ts : (lane == 1 ? Tt : Tb);
+        const uint32_t rold = atom_add_pred(ra, rv, lane < 3 && rv != 0u);
+        const int64_t slot = (int64_t)__shfl_sync(FULL, rold, 0) + xs - (stay ? 1u : 0u);
+        const int64_t ts = (int64_t)__shfl_sync(FULL, rold, 1) + xt - nt;
+        const int64_t bs = (int64_t)__shfl_sync(FULL, rold, 2) + xb_ - nb;
         if (stay) Un[slot] = h;
         // push tasks of a new colour
         if (nt) {
@@ -1043,16 +1070,6 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
 // bit and one higher neighbour less to wait for.  The push that brings a count to
 // JP_WATCH activates the neighbour (next round's list).  Each stage's loads/atomics
 // are in flight together.
-// 4-B L2 load under a predicate (0xffffffff when !p), no branch
-__device__ __forceinline__ uint32_t ld_cg_pred(const uint32_t *addr, bool p) {
-    uint32_t v = 0xffffffffu;
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q ld.global.cg.u32 %0, [%1];\n\t}"
-                 : "+r"(v)
-                 : "l"(addr), "r"((uint32_t)p)
-                 : "memory");
-    return v;
-}
-
 // returning atomic decrement under a predicate (0 when !p), no branch
 __device__ __forceinline__ uint32_t atom_dec_pred(uint32_t *addr, bool p) {
     uint32_t old = 0u;
