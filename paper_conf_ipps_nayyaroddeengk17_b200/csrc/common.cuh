@@ -157,4 +157,66 @@ __device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t *p) {
     return v;
 }
 
+// Predicated PTX loads/atomics (no branch per element): with `p ? load : default` the
+// compiler branched around each access and, short of registers, consumed its result
+// inside the branch, so K independent accesses ran one after another (~1 us each).
+__device__ __forceinline__ uint32_t ld_cg_pred(const uint32_t *addr, bool p) {  // 0xffffffff if !p
+    uint32_t v = 0xffffffffu;
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q ld.global.cg.u32 %0, [%1];\n\t}"
+                 : "+r"(v)
+                 : "l"(addr), "r"((uint32_t)p)
+                 : "memory");
+    return v;
+}
+
+__device__ __forceinline__ uint4 ld_cg_v4_pred(const uint4 *addr, bool p) {  // {1,0,0,0} if !p
+    uint4 v = make_uint4(1u, 0u, 0u, 0u);
+    asm volatile(
+        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %5, 0;\n\t@q ld.global.cg.v4.u32 {%0, %1, %2, %3}, [%4];\n\t}"
+        : "+r"(v.x), "+r"(v.y), "+r"(v.z), "+r"(v.w)
+        : "l"(addr), "r"((uint32_t)p)
+        : "memory");
+    return v;
+}
+
+__device__ __forceinline__ uint32_t atom_add_pred(uint32_t *addr, uint32_t val, bool p) {  // 0 if !p
+    uint32_t old = 0u;
+    asm volatile(
+        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q atom.global.add.u32 %0, [%1], %3;\n\t}"
+        : "+r"(old)
+        : "l"(addr), "r"((uint32_t)p), "r"(val)
+        : "memory");
+    return old;
+}
+
+// returning atomic decrement under a predicate (0 when !p), no branch
+__device__ __forceinline__ uint32_t atom_dec_pred(uint32_t *addr, bool p) {
+    uint32_t old = 0u;
+    asm volatile(
+        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q atom.global.add.u32 %0, [%1], %3;\n\t}"
+        : "+r"(old)
+        : "l"(addr), "r"((uint32_t)p), "r"(0xffffffffu)
+        : "memory");
+    return old;
+}
+
+// 1-B load under a predicate (dflt when !p), no branch
+__device__ __forceinline__ uint8_t ld_u8_pred(const uint8_t *addr, bool p, uint8_t dflt) {
+    uint32_t v = dflt;
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q ld.global.u8 %0, [%1];\n\t}"
+                 : "+r"(v)
+                 : "l"(addr), "r"((uint32_t)p)
+                 : "memory");
+    return (uint8_t)v;
+}
+
+// read-only 4-B load under a predicate (0 when !p), no branch
+__device__ __forceinline__ uint32_t ld_nc_pred(const uint32_t *addr, bool p) {
+    uint32_t v = 0u;
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q ld.global.nc.u32 %0, [%1];\n\t}"
+                 : "+r"(v)
+                 : "l"(addr), "r"((uint32_t)p));
+    return v;
+}
+
 }  // namespace sym

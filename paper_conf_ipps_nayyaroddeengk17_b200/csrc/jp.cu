@@ -728,38 +728,6 @@ __global__ void k_jpc_scatter(JpArgs A) {
 }
 
 // ---------------------------------------------------------------- rounds
-// Predicated PTX loads/atomics (no branch per element): with `p ? load : default` the
-// compiler branched around each access and, short of registers, consumed its result
-// inside the branch, so K independent accesses ran one after another (~1 us each).
-__device__ __forceinline__ uint32_t ld_cg_pred(const uint32_t *addr, bool p) {  // 0xffffffff if !p
-    uint32_t v = 0xffffffffu;
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q ld.global.cg.u32 %0, [%1];\n\t}"
-                 : "+r"(v)
-                 : "l"(addr), "r"((uint32_t)p)
-                 : "memory");
-    return v;
-}
-
-__device__ __forceinline__ uint4 ld_cg_v4_pred(const uint4 *addr, bool p) {  // {1,0,0,0} if !p
-    uint4 v = make_uint4(1u, 0u, 0u, 0u);
-    asm volatile(
-        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %5, 0;\n\t@q ld.global.cg.v4.u32 {%0, %1, %2, %3}, [%4];\n\t}"
-        : "+r"(v.x), "+r"(v.y), "+r"(v.z), "+r"(v.w)
-        : "l"(addr), "r"((uint32_t)p)
-        : "memory");
-    return v;
-}
-
-__device__ __forceinline__ uint32_t atom_add_pred(uint32_t *addr, uint32_t val, bool p) {  // 0 if !p
-    uint32_t old = 0u;
-    asm volatile(
-        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q atom.global.add.u32 %0, [%1], %3;\n\t}"
-        : "+r"(old)
-        : "l"(addr), "r"((uint32_t)p), "r"(val)
-        : "memory");
-    return old;
-}
-
 __device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *p) {
     uint32_t v;
     asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -1070,17 +1038,6 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
 // bit and one higher neighbour less to wait for.  The push that brings a count to
 // JP_WATCH activates the neighbour (next round's list).  Each stage's loads/atomics
 // are in flight together.
-// returning atomic decrement under a predicate (0 when !p), no branch
-__device__ __forceinline__ uint32_t atom_dec_pred(uint32_t *addr, bool p) {
-    uint32_t old = 0u;
-    asm volatile(
-        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q atom.global.add.u32 %0, [%1], %3;\n\t}"
-        : "+r"(old)
-        : "l"(addr), "r"((uint32_t)p), "r"(0xffffffffu)
-        : "memory");
-    return old;
-}
-
 #ifndef SYM_JP_DIAG
 #define SYM_JP_DIAG 0  // 1: compile the SYM_JP_TRACE=3/4 sub-step timers (they cost registers)
 #endif

@@ -57,8 +57,25 @@ struct MisRoundArgs {
     int ncls;
 };
 
-__device__ __forceinline__ bool mis_in_phase(const MisRoundArgs &A, uint32_t w) {
-    return A.ncls < 0 || (int)((A.nfilter[w >> 5] >> (w & 31)) & 1u) == A.ncls;
+// statuses of neighbours w[u] with want[u] (ST_OUT otherwise -- no effect on the
+// rule), restricted to the phase set: the filter words, then the statuses, each step's
+// loads in flight together
+template <int K>
+__device__ __forceinline__ void mis_gather(const MisRoundArgs &A, const uint32_t (&w)[K], const bool (&want)[K],
+                                           uint8_t (&s)[K]) {
+    bool go[K];
+    if (A.ncls >= 0) {
+        uint32_t fw[K];
+#pragma unroll
+        for (int u = 0; u < K; u++) fw[u] = ld_nc_pred(A.nfilter + (w[u] >> 5), want[u]);
+#pragma unroll
+        for (int u = 0; u < K; u++) go[u] = want[u] && (int)((fw[u] >> (w[u] & 31)) & 1u) == A.ncls;
+    } else {
+#pragma unroll
+        for (int u = 0; u < K; u++) go[u] = want[u];
+    }
+#pragma unroll
+    for (int u = 0; u < K; u++) s[u] = ld_u8_pred(A.st + w[u], go[u], ST_OUT);
 }
 
 // bytes: §8(d) algorithmic = 4 B per column word the kernel loads + 9 B
@@ -77,9 +94,12 @@ __device__ __forceinline__ int mis_scan_small(const MisRoundArgs &A, int64_t b, 
     for (int u = 0; u < MIS_SMALL; u++) w[u] = (b + u < e) ? (uint32_t)__ldcs(A.ci + b + u) : 0u;
     // only higher neighbours can decide v: a lower neighbour turns In only once every
     // higher neighbour of it -- v included -- is Out, so while v is undecided none is In
+    // two batched load steps (predicated, no branch per arc): the phase-filter words of
+    // the higher neighbours, then their statuses
+    bool hi[MIS_SMALL];
 #pragma unroll
-    for (int u = 0; u < MIS_SMALL; u++)
-        s[u] = (b + u < e && vkey(A.k, w[u]) > kv && mis_in_phase(A, w[u])) ? A.st[w[u]] : ST_OUT;
+    for (int u = 0; u < MIS_SMALL; u++) hi[u] = b + u < e && vkey(A.k, w[u]) > kv;
+    mis_gather(A, w, hi, s);
     bool in = false, blk = false;
 #pragma unroll
     for (int u = 0; u < MIS_SMALL; u++) {
@@ -134,14 +154,15 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
                     w[u] = ok[u] ? (uint32_t)__ldcs(A.ci + y) : 0u;
                     lb += ok[u] ? 4 : 0;
                 }
-                bool fin = false, fblk = false;
+                bool fin = false, fblk = false, hi[4];
+                uint8_t sw[4];
+#pragma unroll
+                for (int u = 0; u < 4; u++) hi[u] = ok[u] && vkey(A.k, w[u]) > wk;  // higher neighbours only
+                mis_gather(A, w, hi, sw);
 #pragma unroll
                 for (int u = 0; u < 4; u++) {
-                    if (ok[u] && vkey(A.k, w[u]) > wk && mis_in_phase(A, w[u])) {  // higher neighbours only
-                        uint8_t sw = A.st[w[u]];
-                        fin |= sw == ST_IN;
-                        fblk |= sw == ST_UNDEC;
-                    }
+                    fin |= sw[u] == ST_IN;
+                    fblk |= sw[u] == ST_UNDEC;
                 }
                 if (__any_sync(FULL, fin)) { r = R_OUT; break; }
                 if (__any_sync(FULL, fblk)) { r = R_BLK; break; }
@@ -179,7 +200,8 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
         for (int64_t x = b; x < e; x += 4 * MIS_HUGE_THREADS) {
             bool fin = false, fblk = false;
             uint32_t w[4];
-            bool ok[4];
+            bool ok[4], hi[4];
+            uint8_t sw[4];
 #pragma unroll
             for (int u = 0; u < 4; u++) {
                 int64_t y = x + u * MIS_HUGE_THREADS + threadIdx.x;
@@ -188,12 +210,12 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
                 lb += ok[u] ? 4 : 0;
             }
 #pragma unroll
+            for (int u = 0; u < 4; u++) hi[u] = ok[u] && vkey(A.k, w[u]) > kv;  // higher neighbours only
+            mis_gather(A, w, hi, sw);
+#pragma unroll
             for (int u = 0; u < 4; u++) {
-                if (ok[u] && vkey(A.k, w[u]) > kv && mis_in_phase(A, w[u])) {  // higher neighbours only
-                    uint8_t sw = A.st[w[u]];
-                    fin |= sw == ST_IN;
-                    fblk |= sw == ST_UNDEC;
-                }
+                fin |= sw[u] == ST_IN;
+                fblk |= sw[u] == ST_UNDEC;
             }
             if (__syncthreads_or(fin)) { r = R_OUT; break; }
             if (__syncthreads_or(fblk)) { r = R_BLK; break; }
