@@ -189,13 +189,13 @@ __device__ __forceinline__ uint32_t atom_add_pred(uint32_t *addr, uint32_t val, 
     return old;
 }
 
-// returning atomic decrement under a predicate (0 when !p), no branch
-__device__ __forceinline__ uint32_t atom_dec_pred(uint32_t *addr, bool p) {
-    uint32_t old = 0u;
+// returning 64-bit atomic decrement under a predicate (0 when !p), no branch
+__device__ __forceinline__ uint64_t atom_dec64_pred(unsigned long long *addr, bool p) {
+    unsigned long long old = 0ull;
     asm volatile(
-        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q atom.global.add.u32 %0, [%1], %3;\n\t}"
-        : "+r"(old)
-        : "l"(addr), "r"((uint32_t)p), "r"(0xffffffffu)
+        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q atom.global.add.u64 %0, [%1], %3;\n\t}"
+        : "+l"(old)
+        : "l"(addr), "r"((uint32_t)p), "l"(0xffffffffffffffffull)
         : "memory");
     return old;
 }

@@ -23,9 +23,10 @@
 // their rank in id order; a vertex without any phase arc takes colour 1 at once).  The
 // per-vertex state other vertices touch is one 16-B record in a compact array, so a
 // check or a push touches ONE sector and the hot set (90 MB at R-MAT s24) is mostly
-// L2-resident: hot[h] = {colour (0 = not yet), count = higher neighbours not yet
-// pushed, forbidden colours 1..32, offset of h's words for colours 33..32R in xb[]
-// (R-1 words) | min(R,31) << 27}, R = ceil(cap/32).  meta[h] (32 B, read by h itself) = {R, hdeg, ldeg, watch
+// L2-resident: hot[h] = {colour (0 = not yet), forbidden colours 1..32, count =
+// higher neighbours not yet pushed, offset of h's words for colours 33..32R in xb[]
+// (R-1 words) | min(R,31) << 27}, R = ceil(cap/32) -- count and offset adjacent, so a
+// push's one 64-bit atomic decrements the count and returns the offset.  meta[h] (32 B, read by h itself) = {R, hdeg, ldeg, watch
 // length, blocker position, m at the last failed check, list offset}; lst[off..]
 // = [watch area of JP_WATCH ids if hdeg > JP_WLIST] [higher ids] [lower ids] (compact
 // ids).
@@ -67,6 +68,12 @@ constexpr int JP_LANE_CHECKS = SYM_JP_LANE_CHECKS;  // phase A: entries a lane c
 #ifndef SYM_JP_WLIST
 #define SYM_JP_WLIST 64
 #endif
+#ifndef SYM_JP_LANE_ALL
+#define SYM_JP_LANE_ALL 1
+#endif
+#ifndef SYM_JP_WARP_S2
+#define SYM_JP_WARP_S2 1
+#endif
 #ifndef SYM_JP_PUSH_LANE
 #define SYM_JP_PUSH_LANE 4
 #endif
@@ -93,7 +100,7 @@ struct JpArgs {
     uint32_t *ldeg;      // [n] lower degree (count pass), fill cursor (huge rows)
     uint32_t *arank;     // [2 n/32] per 32 ids: {bitmap of the S vertices with phase arcs,
                          //   exclusive prefix of the popcounts} (rank = compact id)
-    uint4 *hot;          // [n] hot per-vertex state {col, cnt, bm0, xo} (see the header)
+    uint4 *hot;          // [n] hot per-vertex state {col, bm0, cnt, xo} (see the header)
     uint4 *meta;         // [2n] per-vertex own data
     uint32_t *lst;       // watch / higher / lower lists
     uint32_t *xb;        // bitmap words for colours > 32
@@ -532,7 +539,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
             const uint32_t x0 = (uint32_t)(o1 + p1);
             A.meta[2 * h] = make_uint4(R, hd, ld, hd > JP_WLIST ? JP_NOTBUILT : hd);
             A.meta[2 * h + 1] = make_uint4(0u, 0u, (uint32_t)off, (uint32_t)(off >> 32));
-            A.hot[h] = make_uint4(0u, hd, 0u, (x0 & JP_HMASK) | (min(R, JP_R5) << JP_HBITS));
+            A.hot[h] = make_uint4(0u, 0u, hd, (x0 & JP_HMASK) | (min(R, JP_R5) << JP_HBITS));
             for (uint32_t q = 1; q < R; q++) A.xb[x0 + q - 1] = 0u;
             A.hdeg[h] = 0;  // fill cursors of the huge rows
             A.ldeg[h] = 0;
@@ -549,7 +556,7 @@ __device__ __forceinline__ void jp_fixed(const JpArgs &A, int64_t h, uint32_t R,
     const uint32_t c = A.color[w];
     if (c == 0) return;
     const uint32_t q = (c - 1) >> 5, bit = 1u << ((c - 1) & 31);
-    if (q == 0) atomicOr(&A.hot[h].z, bit);
+    if (q == 0) atomicOr(&A.hot[h].y, bit);
     else if (q < R) atomicOr(A.xb + x0 + q - 1, bit);
 }
 
@@ -796,7 +803,7 @@ __device__ __forceinline__ void jp_nb_stage(const JpArgs &A, const uint32_t (&e)
     for (int u = 0; u < N; u++) {
         if (!valid[u]) ok[u] = true;
         else if (s[u].x != 0u) ok[u] = s[u].x != m;
-        else if (q == 0u) ok[u] = (s[u].z >> bit) & 1u;
+        else if (q == 0u) ok[u] = (s[u].y >> bit) & 1u;
         else ok[u] = q >= Rf[u] || ((wd[u] >> bit) & 1u);  // q >= R: m > cap
     }
 }
@@ -841,7 +848,7 @@ __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_i
         } else {
             state = 0;
             const uint4 hs = __ldcg(A.hot + h);
-            const uint32_t z0 = ~hs.z;
+            const uint32_t z0 = ~hs.y;
             if (z0) {
                 m = __ffs(z0);
             } else if (SPARSE) {
@@ -886,7 +893,9 @@ __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_i
     const uint32_t q = (m - 1) >> 5, bit = (m - 1) & 31;
     uint32_t j = (lm == m && pos < wc) ? pos : 0u;  // m unchanged: resume at the last blocker
     // ---- lane: the first JP_LANE_CHECKS entries (all loads of a stage in flight)
-    if (!SPARSE && state == 0) {
+    // (SYM_JP_LANE_ALL = 0: a lane checks its list alone only when the rest of it fits
+    // the lane stage; a longer one goes straight to the warp -- one chain, not two)
+    if (!SPARSE && state == 0 && (SYM_JP_LANE_ALL || wc - j <= (uint32_t)JP_LANE_CHECKS)) {
         uint32_t e[JP_LANE_CHECKS];
         bool valid[JP_LANE_CHECKS], ok[JP_LANE_CHECKS];
 #pragma unroll
@@ -923,7 +932,7 @@ __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_i
         const uint32_t wq = (wm - 1) >> 5, wbit = (wm - 1) & 31;
         int wstate = wj >= wwc ? 1 : 0;
         uint32_t wpos = 0;
-        constexpr int S = SPARSE ? 2 : 1;  // entries per lane per step
+        constexpr int S = (SPARSE || SYM_JP_WARP_S2) ? 2 : 1;  // entries per lane per step
         while (wstate == 0) {
             bool ok[S], valid[S];
             uint32_t eu[S];
@@ -1060,13 +1069,17 @@ __device__ __forceinline__ void jp_push(const JpArgs &A, const uint32_t (&e)[K],
     // (predicated PTX atomics: with `act ? atomicSub(..) : 0` the compiler branched around
     // each atomic and tested its result inside the branch, so the K returning atomics ran
     // one after another -- ~1 us each in the tail)
+    // One 64-bit atomic per target: {count, xo} are adjacent in the hot record, so
+    // adding -1 to the pair decrements the count (never 0 before: no borrow) and
+    // returns the R field and extra-word offset with it -- no separate load.  No colour
+    // filter: a bit in the bitmap of an already coloured vertex is never read (nb_ok
+    // tests its colour first).
 #pragma unroll
-    for (int u = 0; u < K; u++) old[u] = atom_dec_pred(&A.hot[e[u]].y, act[u]);
-    // colours > 32: the R field and extra-word offset (hot.w) of every target, loads in
-    // flight together (predicated PTX again).  No colour filter: a bit in the bitmap of
-    // an already coloured vertex is never read (nb_ok tests its colour first).
-#pragma unroll
-    for (int u = 0; u < K; u++) x[u] = ld_cg_pred(&A.hot[e[u]].w, act[u] && q > 0);
+    for (int u = 0; u < K; u++) {
+        const uint64_t o = atom_dec64_pred(reinterpret_cast<unsigned long long *>(&A.hot[e[u]].z), act[u]);
+        old[u] = (uint32_t)o;
+        x[u] = act[u] && q > 0 ? (uint32_t)(o >> 32) : 0xffffffffu;
+    }
 #if SYM_JP_DIAG
     uint64_t tq1 = 0, tq2 = 0, tq3 = 0;
     if (tr4) {
@@ -1080,7 +1093,7 @@ __device__ __forceinline__ void jp_push(const JpArgs &A, const uint32_t (&e)[K],
     if (q == 0) {
 #pragma unroll
         for (int u = 0; u < K; u++)
-            if (act[u]) atomicOr(&A.hot[e[u]].z, 1u << bit);
+            if (act[u]) atomicOr(&A.hot[e[u]].y, 1u << bit);
     } else {
         uint32_t Rf[K];  // saturated R field (>= 31 words): the full count from meta
 #pragma unroll
