@@ -242,6 +242,16 @@ def roofline(name, v, calls, peak, peak_src, traffic, traffic_src, step_ms=None)
          "ms_per_launch": per_launch_s * 1e3, "launches_per_call": v["launches"] / calls}
     if len(classes) > 1:
         r["classes"] = classes
+    if traffic:
+        # ncu's own view of the same class in the same capture: L2 / DRAM throughput
+        # fractions (time-weighted lts__throughput / dram__throughput) -- the gather-bound
+        # round kernels are judged against the L2 as well as HBM
+        l2 = [(traffic[c]["l2_frac"], traffic[c]["us"]) for c in classes if c in traffic and "l2_frac" in traffic[c]]
+        if l2 and sum(t for _, t in l2) > 0:
+            r["l2_frac_ncu"] = sum(f * t for f, t in l2) / sum(t for _, t in l2)
+        dr = [(traffic[c]["dram_frac"], traffic[c]["us"]) for c in classes if c in traffic and "dram_frac" in traffic[c]]
+        if dr and sum(t for _, t in dr) > 0:
+            r["dram_frac_ncu"] = sum(f * t for f, t in dr) / sum(t for _, t in dr)
     if step_ms:
         r["share_of_step"] = (v["ms"] / calls) / step_ms
     return r

@@ -196,6 +196,7 @@ struct MisWs {
     uint8_t *st = nullptr;
     int32_t *vlist = nullptr;          // class lists (front / back)
     int32_t *fr[2] = {nullptr, nullptr};  // frontier ping-pong
+    int32_t *fp[2] = {nullptr, nullptr};  // resume offsets, parallel to fr
     int64_t *huge = nullptr;           // deferred (v, resume) pairs
     int64_t huge_cap = 0;
     unsigned long long *gmax = nullptr;  // round 0: maxima of rows crossing tiles
@@ -211,6 +212,7 @@ struct MmWs {
     int64_t huge_cap = 0;
     unsigned long long *gmax = nullptr;  // round 0: maxima of rows crossing tiles
     uint32_t *mbits = nullptr;           // matched bitmap
+    int32_t *alt = nullptr;  // second-heaviest believed-live neighbour at the last scan (-1: none)
 };
 
 struct ColorWs {

@@ -155,6 +155,10 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
 __device__ __forceinline__ bool in_set(const uint8_t *inS, uint32_t w) { return inS == nullptr || inS[w] != 0; }
 
 __device__ __forceinline__ uint32_t watch_words(uint32_t hd) { return hd > JP_WLIST ? JP_WATCH : 0u; }
+// list layout at a row's offset: [watch area][higher ids][lower ids]; the area is
+// reserved for every row with more than JP_WLIST S-neighbours (hd + ld) -- a bound the
+// count-free build knows before it has split the row -- and used when hd > JP_WLIST
+__device__ __forceinline__ uint32_t watch_area(uint32_t hd, uint32_t ld) { return hd + ld > JP_WLIST ? JP_WATCH : 0u; }
 
 __device__ __forceinline__ uint64_t meta_off(const uint4 &m1) { return (uint64_t)m1.z | ((uint64_t)m1.w << 32); }
 
@@ -435,7 +439,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_sums(JpArgs A) {
         const int64_t h = base + u * JP_THREADS + threadIdx.x;
         if (h < cnt) {
             const uint32_t hd = A.hdeg[h];
-            sl += watch_words(hd) + hd + A.ldeg[h];
+            sl += watch_area(hd, A.ldeg[h]) + hd + A.ldeg[h];
             sx += jp_words(A, h) - 1u;
         }
     }
@@ -524,7 +528,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
         }
         unsigned long long t0, t1;
         const unsigned long long p0 =
-            block_excl_scan<unsigned long long>(active ? watch_words(hd) + hd + ld : 0ull, sm0, &t0);
+            block_excl_scan<unsigned long long>(active ? watch_area(hd, ld) + hd + ld : 0ull, sm0, &t0);
         const unsigned long long p1 = block_excl_scan<unsigned long long>(active ? R - 1u : 0ull, sm1, &t1);
         // Round 0 can only colour vertices without higher neighbours (nothing is coloured
         // and, without fixed colours -- S given implicitly -- nothing is forbidden), so
@@ -551,6 +555,123 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_place(JpArgs A) {
     }
 }
 
+// ---------------------------------------------------------------- count-free build
+// With S implicit (every vertex of the phase CSR; COLOR-NONE / -Degk / -Rand's first
+// phase) a row's higher + lower neighbours are exactly its phase arcs, so the lists can
+// be placed from the degrees alone and split while they are filled -- higher ids from
+// the front of the row's area, lower ids from the back -- with no counting pass over
+// the arcs.  The counts the fill finds then size the hot records, the bitmap words
+// (true cap) and the first round's lists (k_jpc_place_cf).
+
+__device__ __forceinline__ uint32_t jp_deg(const JpArgs &A, int64_t h) {
+    const int32_t v = A.ov[h];
+    return (uint32_t)(A.rp[v + 1] - A.rp[v]);
+}
+
+// per tile of JP_TILE compact ids: list words (degree + watch area); huge rows' pieces
+__global__ void __launch_bounds__(JP_THREADS) k_jpc_lsums_cf(JpArgs A) {
+    const uint32_t cnt = A.nc[0];
+    const int64_t base = (int64_t)blockIdx.x * JP_TILE;
+    if (base >= cnt) return;
+    unsigned long long sl = 0;
+    for (int u = 0; u < JP_TPT; u++) {
+        const int64_t h = base + u * JP_THREADS + threadIdx.x;
+        const uint32_t d = h < cnt ? jp_deg(A, h) : 0u;
+        sl += watch_area(d, 0u) + d;
+        const uint32_t np = d > (uint32_t)JP_BUDGET ? (d + JP_PIECE - 1) / JP_PIECE : 0u;
+        const int64_t ps = warp_reserve(np, A.huge_cnt);
+        for (uint32_t q = 0; q < np; q++) A.huge[ps + q] = ((int64_t)q << 32) | (uint32_t)h;
+        prof_add(A.prof, 0ull, h < cnt ? 12ull : 0ull);
+        // §8(d) JP (push form): 8 B per phase arc + 12 B per vertex, charged to the rounds
+        prof_add(A.prof_jp, h < cnt ? 8ull * d + 12ull : 0ull, 0ull);
+    }
+    for (int d = 16; d; d >>= 1) sl += __shfl_xor_sync(FULL, sl, d);
+    __shared__ unsigned long long a0;
+    if (threadIdx.x == 0) a0 = 0;
+    __syncthreads();
+    if (lane_id() == 0) atomicAdd(&a0, sl);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        A.tsum[2 * blockIdx.x] = a0;
+        A.tsum[2 * blockIdx.x + 1] = 0;
+    }
+}
+
+// list offsets (meta[2h+1].zw) from the scanned tile sums
+__global__ void __launch_bounds__(JP_THREADS) k_jpc_offs_cf(JpArgs A) {
+    const uint32_t cnt = A.nc[0];
+    const int64_t base = (int64_t)blockIdx.x * JP_TILE;
+    if (base >= cnt) return;
+    __shared__ unsigned long long sm0[8];
+    unsigned long long o0 = A.tsum[2 * blockIdx.x];
+    for (int u = 0; u < JP_TPT; u++) {
+        const int64_t h = base + u * JP_THREADS + threadIdx.x;
+        const uint32_t d = h < cnt ? jp_deg(A, h) : 0u;
+        unsigned long long t0;
+        const unsigned long long p0 = block_excl_scan<unsigned long long>(h < cnt ? watch_area(d, 0u) + d : 0ull, sm0, &t0);
+        if (h < cnt) {
+            const unsigned long long off = o0 + p0;
+            A.meta[2 * h + 1] = make_uint4(0u, 0u, (uint32_t)off, (uint32_t)(off >> 32));
+        }
+        prof_add(A.prof, 0ull, h < cnt ? 28ull : 0ull);
+        o0 += t0;
+    }
+}
+
+// per tile: extra bitmap words of the true cap (hd + 1 bits), once the fill has counted
+__global__ void __launch_bounds__(JP_THREADS) k_jpc_xsums_cf(JpArgs A) {
+    const uint32_t cnt = A.nc[0];
+    const int64_t base = (int64_t)blockIdx.x * JP_TILE;
+    if (base >= cnt) return;
+    unsigned long long sx = 0;
+    for (int u = 0; u < JP_TPT; u++) {
+        const int64_t h = base + u * JP_THREADS + threadIdx.x;
+        if (h < cnt) sx += (A.hdeg[h] + 1u + 31u) / 32u - 1u;
+    }
+    for (int d = 16; d; d >>= 1) sx += __shfl_xor_sync(FULL, sx, d);
+    __shared__ unsigned long long a1;
+    if (threadIdx.x == 0) a1 = 0;
+    __syncthreads();
+    if (lane_id() == 0) atomicAdd(&a1, sx);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        A.tsum[2 * blockIdx.x] = 0;
+        A.tsum[2 * blockIdx.x + 1] = a1;
+    }
+}
+
+// per compact id: meta, hot state, zeroed extra bitmap words, the first round's lists
+// (the list offset is already in meta[2h+1])
+__global__ void __launch_bounds__(JP_THREADS) k_jpc_place_cf(JpArgs A) {
+    const uint32_t cnt = A.nc[0];
+    const int64_t base = (int64_t)blockIdx.x * JP_TILE;
+    if (base >= cnt) return;
+    __shared__ unsigned long long sm1[8];
+    unsigned long long o1 = A.tsum[2 * blockIdx.x + 1];
+    for (int u = 0; u < JP_TPT; u++) {
+        const int64_t h = base + u * JP_THREADS + threadIdx.x;
+        const bool active = h < cnt;
+        uint32_t hd = 0, ld = 0, R = 1;
+        if (active) {
+            hd = A.hdeg[h];
+            ld = A.ldeg[h];
+            R = (hd + 1u + 31u) / 32u;
+        }
+        unsigned long long t1;
+        const unsigned long long p1 = block_excl_scan<unsigned long long>(active ? R - 1u : 0ull, sm1, &t1);
+        const bool ready = active && hd == 0, later = active && hd > 0 && hd <= JP_WATCH;
+        cta_append2x(ready, later, (uint32_t)h, A.ul[0], A.ucnt, A.ul[1], A.ucnt + 1);
+        if (active) {
+            const uint32_t x0 = (uint32_t)(o1 + p1);
+            A.meta[2 * h] = make_uint4(R, hd, ld, hd > JP_WLIST ? JP_NOTBUILT : hd);
+            A.hot[h] = make_uint4(0u, 0u, hd, (x0 & JP_HMASK) | (min(R, JP_R5) << JP_HBITS));
+            for (uint32_t q = 1; q < R; q++) A.xb[x0 + q - 1] = 0u;
+        }
+        prof_add(A.prof, 0ull, active ? 8ull + 40ull + 4ull * (R - 1u) : 0ull);
+        o1 += t1;
+    }
+}
+
 // fixed colour c of a neighbour outside S (COLOR-Rand recolouring) as a forbidden bit
 __device__ __forceinline__ void jp_fixed(const JpArgs &A, int64_t h, uint32_t R, uint32_t x0, uint32_t w) {
     const uint32_t c = A.color[w];
@@ -562,11 +683,14 @@ __device__ __forceinline__ void jp_fixed(const JpArgs &A, int64_t h, uint32_t R,
 
 // fill pass: higher and lower lists (list ids, CSR order); fixed colours of
 // neighbours outside S.  Columns and lists stream (evict-first) so the id map stays
-// in L2 for the gathers.
+// in L2 for the gathers.  CF (count-free build, S implicit): the area of a row is its
+// degree (+ watch area), higher ids fill it from the front and lower ids from the
+// back, and the counts are written out (hdeg / ldeg) for k_jpc_place_cf.
 // 5 CTAs/SM (48 regs, no spills; 59 without the bound -> 4): more rank lookups in flight
 #ifndef SYM_FILL_MINB
 #define SYM_FILL_MINB 5
 #endif
+template <bool CF>
 #if SYM_FILL_MINB > 0
 __global__ void __launch_bounds__(JP_THREADS, SYM_FILL_MINB) k_jpc_fill(JpArgs A) {
 #else
@@ -588,12 +712,20 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
             b = A.rp[v];
             e = A.rp[v + 1];
             kv = jp_okey(A.k, A.okey, A.ord, (uint32_t)v);
-            const uint4 m0 = A.meta[2 * h], m1 = A.meta[2 * h + 1];
-            R = m0.x;
-            x0 = A.hot[h].w & JP_HMASK;
-            hl = meta_off(m1) + watch_words(m0.y);
-            ll = hl + m0.y;
+            if (CF) {
+                const uint4 m1 = A.meta[2 * h + 1];
+                const uint32_t d = (uint32_t)(e - b);
+                hl = meta_off(m1) + watch_area(d, 0u);
+                ll = hl + d;  // lower ids from the back: ll = one past the next slot
+            } else {
+                const uint4 m0 = A.meta[2 * h], m1 = A.meta[2 * h + 1];
+                R = m0.x;
+                x0 = A.hot[h].w & JP_HMASK;
+                hl = meta_off(m1) + watch_area(m0.y, m0.z);
+                ll = hl + m0.y;
+            }
         }
+        const uint64_t hl0 = hl, ll0 = ll;
         if (active && e - b <= JP_SMALL) {  // batches of 4 arcs: their loads in flight together
             for (int64_t xq = b; xq < e; xq += 4) {
                 uint32_t w[4], rk[4];
@@ -605,7 +737,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
                 }
 #pragma unroll
                 for (int u = 0; u < 4; u++) {
-                    sv[u] = ok[u] && in_set(A.inS, w[u]);
+                    sv[u] = ok[u] && (CF || in_set(A.inS, w[u]));
                     rk[u] = sv[u] ? jp_rank(A, w[u]) : 0u;
                 }
 #pragma unroll
@@ -613,8 +745,13 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
                     if (!ok[u]) continue;
                     if (!sv[u]) jp_fixed(A, h, R, x0, w[u]);
                     else if (jp_okey(A.k, A.okey, A.ord, w[u]) > kv) __stcs(A.lst + hl++, rk[u]);
+                    else if (CF) __stcs(A.lst + --ll, rk[u]);
                     else __stcs(A.lst + ll++, rk[u]);
                 }
+            }
+            if (CF) {
+                A.hdeg[h] = (uint32_t)(hl - hl0);
+                A.ldeg[h] = (uint32_t)(ll0 - ll);
             }
         }
         unsigned medm = __ballot_sync(FULL, active && e - b > JP_SMALL && e - b <= JP_BUDGET);
@@ -626,6 +763,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
             const int64_t wh = base + src;
             const uint32_t wR = __shfl_sync(FULL, R, src), wx0 = __shfl_sync(FULL, x0, src);
             uint64_t whl = __shfl_sync(FULL, hl, src), wll = __shfl_sync(FULL, ll, src);
+            const uint64_t whl0 = whl, wll0 = wll;
             const unsigned lt = (1u << lane) - 1u;
             for (int64_t xb0 = wb; xb0 < we; xb0 += 128) {  // 4 steps of 32 arcs in flight
                 uint32_t w[4], rk[4];
@@ -638,20 +776,29 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
 #pragma unroll
                 for (int u = 0; u < 4; u++) {
                     const bool ok = xb0 + u * 32 + lane < we;
-                    const bool sv = ok && in_set(A.inS, w[u]);
+                    const bool sv = ok && (CF || in_set(A.inS, w[u]));
                     up[u] = sv && jp_okey(A.k, A.okey, A.ord, w[u]) > wk;
                     dn[u] = sv && !up[u];
                     rk[u] = sv ? jp_rank(A, w[u]) : 0u;
-                    if (ok && !sv) jp_fixed(A, wh, wR, wx0, w[u]);
+                    if (!CF && ok && !sv) jp_fixed(A, wh, wR, wx0, w[u]);
                 }
 #pragma unroll
                 for (int u = 0; u < 4; u++) {
                     const unsigned mu = __ballot_sync(FULL, up[u]), md = __ballot_sync(FULL, dn[u]);
                     if (up[u]) __stcs(A.lst + whl + __popc(mu & lt), rk[u]);
-                    if (dn[u]) __stcs(A.lst + wll + __popc(md & lt), rk[u]);
+                    if (CF) {
+                        if (dn[u]) __stcs(A.lst + wll - 1 - __popc(md & lt), rk[u]);
+                        wll -= __popc(md);
+                    } else {
+                        if (dn[u]) __stcs(A.lst + wll + __popc(md & lt), rk[u]);
+                        wll += __popc(md);
+                    }
                     whl += __popc(mu);
-                    wll += __popc(md);
                 }
+            }
+            if (CF && lane == 0) {
+                A.hdeg[wh] = (uint32_t)(whl - whl0);
+                A.ldeg[wh] = (uint32_t)(wll0 - wll);
             }
         }
         // algorithmic bytes: the row's columns read + list ids written (huge rows:
@@ -662,7 +809,8 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
 
 // huge rows: one CTA per piece; each warp counts its 512-arc slice (ballots), reserves
 // its positions on the row's two cursors with one atomic each, then writes (the
-// slice is re-read from L2)
+// slice is re-read from L2).  CF: the lower cursor counts from the back of the area.
+template <bool CF>
 __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
     constexpr int SLICE = JP_PIECE / (JP_HUGE_THREADS / 32);
     const uint32_t cnt = *A.huge_cnt;
@@ -677,15 +825,17 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
         const int64_t sb0 = b + j * JP_PIECE + (int64_t)(threadIdx.x >> 5) * SLICE;
         const int64_t se = min(e, sb0 + SLICE);
         const uint64_t kv = jp_okey(A.k, A.okey, A.ord, (uint32_t)v);
-        const uint4 m0 = A.meta[2 * h], m1 = A.meta[2 * h + 1];
-        const uint32_t x0 = A.hot[h].w & JP_HMASK;
-        const uint64_t hl = meta_off(m1) + watch_words(m0.y), ll = hl + m0.y;
+        const uint4 m0 = CF ? make_uint4(0u, 0u, 0u, 0u) : A.meta[2 * h], m1 = A.meta[2 * h + 1];
+        const uint32_t x0 = CF ? 0u : A.hot[h].w & JP_HMASK;
+        const uint32_t d = (uint32_t)(e - b);
+        const uint64_t hl = meta_off(m1) + (CF ? watch_area(d, 0u) : watch_area(m0.y, m0.z));
+        const uint64_t ll = CF ? hl + d : hl + m0.y;  // CF: one past the back of the area
         uint32_t nu = 0, nd = 0;
         for (int64_t x = sb0 + lane; x - lane < se; x += 32) {
             bool up = false, dn = false;
             if (x < se) {
                 const uint32_t w = (uint32_t)__ldg(A.ci + x);
-                if (in_set(A.inS, w)) {
+                if (CF || in_set(A.inS, w)) {
                     up = jp_okey(A.k, A.okey, A.ord, w) > kv;
                     dn = !up;
                 }
@@ -708,17 +858,20 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
 #pragma unroll
             for (int u = 0; u < 4; u++) {
                 const bool ok = xq + u * 32 < se;
-                const bool sv = ok && in_set(A.inS, w[u]);
+                const bool sv = ok && (CF || in_set(A.inS, w[u]));
                 up[u] = sv && jp_okey(A.k, A.okey, A.ord, w[u]) > kv;
                 dn[u] = sv && !up[u];
                 rk[u] = sv ? jp_rank(A, w[u]) : 0u;
-                if (ok && !sv) jp_fixed(A, h, m0.x, x0, w[u]);
+                if (!CF && ok && !sv) jp_fixed(A, h, m0.x, x0, w[u]);
             }
 #pragma unroll
             for (int u = 0; u < 4; u++) {
                 const unsigned mu = __ballot_sync(FULL, up[u]), md = __ballot_sync(FULL, dn[u]);
                 if (up[u]) __stcs(A.lst + hl + pu + __popc(mu & lt), rk[u]);
-                if (dn[u]) __stcs(A.lst + ll + pd + __popc(md & lt), rk[u]);
+                if (dn[u]) {
+                    if (CF) __stcs(A.lst + ll - 1 - (pd + __popc(md & lt)), rk[u]);
+                    else __stcs(A.lst + ll + pd + __popc(md & lt), rk[u]);
+                }
                 pu += __popc(mu);
                 pd += __popc(md);
             }
@@ -892,6 +1045,8 @@ __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_i
     }
     const uint32_t q = (m - 1) >> 5, bit = (m - 1) & 31;
     uint32_t j = (lm == m && pos < wc) ? pos : 0u;  // m unchanged: resume at the last blocker
+    // the list checked: the watch area (hd > JP_WLIST) or the higher list itself
+    const uint64_t coff = off + (hd > JP_WLIST ? 0u : watch_area(hd, ld));
     // ---- lane: the first JP_LANE_CHECKS entries (all loads of a stage in flight)
     // (SYM_JP_LANE_ALL = 0: a lane checks its list alone only when the rest of it fits
     // the lane stage; a longer one goes straight to the warp -- one chain, not two)
@@ -901,7 +1056,7 @@ __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_i
 #pragma unroll
         for (int u = 0; u < JP_LANE_CHECKS; u++) {
             valid[u] = j + u < wc;
-            e[u] = ld_cg_pred(A.lst + off + j + u, valid[u]);
+            e[u] = ld_cg_pred(A.lst + coff + j + u, valid[u]);
         }
         jp_nb_stage<JP_LANE_CHECKS>(A, e, valid, m, q, bit, ok);
 #pragma unroll
@@ -928,7 +1083,7 @@ __device__ __forceinline__ void jp_check(const JpArgs &A, bool act, uint32_t h_i
         need &= need - 1;
         uint32_t wj = __shfl_sync(FULL, j, src);
         const uint32_t wwc = __shfl_sync(FULL, wc, src), wm = __shfl_sync(FULL, m, src);
-        const uint64_t woff = __shfl_sync(FULL, off, src);
+        const uint64_t woff = __shfl_sync(FULL, coff, src);
         const uint32_t wq = (wm - 1) >> 5, wbit = (wm - 1) & 31;
         int wstate = wj >= wwc ? 1 : 0;
         uint32_t wpos = 0;
@@ -1029,7 +1184,7 @@ __device__ __forceinline__ void jp_phase_a(const JpArgs &A, uint32_t r, uint32_t
         if (stay) Un[slot] = h;
         // push tasks of a new colour
         if (nt) {
-            const uint64_t l0 = off + watch_words(hd) + hd;  // the lower list
+            const uint64_t l0 = off + watch_area(hd, ld) + hd;  // the lower list
             for (uint32_t t = 0; t < nt; t++) {
                 const uint64_t s0 = l0 + (uint64_t)t * JP_PUSH;
                 A.task[ts + t] = make_uint4((uint32_t)s0, (uint32_t)(s0 >> 32), min(JP_PUSH, ld - t * JP_PUSH), m);
@@ -1392,6 +1547,39 @@ static int jp_order(const FlowArgs &f) {
 // list.  sync words: [0] barrier arrivals, [1] barrier generation, [4..6] list
 // counts, [8..10] push-task counts, [12..14] build-task counts, [32] error, [33]
 // rounds, [40..41] compact counts.
+// the fill passes (one resident wave of each grid-stride kernel, see mis.cu round_grid)
+template <bool CF>
+static int jp_launch_fill(JpArgs &A, cudaStream_t s) {
+    {
+        int per = 2048 / JP_THREADS;
+#if SYM_ROUND_ONE_WAVE
+        int x = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_jpc_fill<CF>, JP_THREADS, 0) == cudaSuccess && x > 0)
+            per = std::min(per, x);
+#endif
+        k_jpc_fill<CF><<<num_sms() * per, JP_THREADS, 0, s>>>(A);
+    }
+    SYM_LAUNCH_CHECK();
+    {
+        // block-strided pieces: one resident wave (40 regs x 512 threads -> 3 CTAs/SM, not 4)
+        int per = 4;
+#if SYM_ROUND_ONE_WAVE
+        int x = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_jpc_fill_huge<CF>, JP_HUGE_THREADS, 0) == cudaSuccess &&
+            x > 0)
+            per = std::min(per, x);
+#endif
+        k_jpc_fill_huge<CF><<<num_sms() * per, JP_HUGE_THREADS, 0, s>>>(A);
+    }
+    SYM_LAUNCH_CHECK();
+    return SYM_OK;
+}
+
+static bool getenv_flag(const char *name) {
+    const char *e = getenv(name);
+    return e && *e && *e != '0';
+}
+
 static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, const int64_t *rp,
                     const int32_t *ci, const uint8_t *inS, const int32_t *list0, const uint32_t *cnt0,
                     int64_t implicit_n, unsigned long long *rounds_ctr) {
@@ -1455,43 +1643,50 @@ static int jp_build(const FlowArgs &f, ColorWs &w, JpArgs &A, uint32_t *color, c
     SYM_LAUNCH_CHECK();
     k_jpc_assign<<<tiles_w, JP_THREADS, 0, s>>>(A, nwords);
     SYM_LAUNCH_CHECK();
-    k_jpc_count<<<num_sms() * (2048 / JP_THREADS), JP_THREADS, 0, s>>>(A);
-    SYM_LAUNCH_CHECK();
-    k_jpc_count_huge<<<num_sms() * 4, JP_HUGE_THREADS, 0, s>>>(A);
-    SYM_LAUNCH_CHECK();
-    if (tiles_c) {
-        k_jpc_sums<<<tiles_c, JP_THREADS, 0, s>>>(A);
+    // count-free build when S is implicit (every vertex of the phase CSR): the lists are
+    // placed from the degrees and split while filled; otherwise count, place, fill
+    const bool cf = inS == nullptr && list0 == nullptr && !getenv_flag("SYM_JP_COUNTED");
+    if (cf) {
+        SYM_CUDA(cudaMemsetAsync(w.hdeg, 0, sizeof(uint32_t) * (size_t)(n + 1), s));
+        SYM_CUDA(cudaMemsetAsync(w.ldeg, 0, sizeof(uint32_t) * (size_t)(n + 1), s));
+        if (tiles_c) {
+            k_jpc_lsums_cf<<<tiles_c, JP_THREADS, 0, s>>>(A);
+            SYM_LAUNCH_CHECK();
+        }
+        k_jpc_sums_scan<<<1, 1024, 0, s>>>(A, tiles_c);
         SYM_LAUNCH_CHECK();
-    }
-    k_jpc_sums_scan<<<1, 1024, 0, s>>>(A, tiles_c);
-    SYM_LAUNCH_CHECK();
-    if (tiles_c) {
-        k_jpc_place<<<tiles_c, JP_THREADS, 0, s>>>(A);
+        if (tiles_c) {
+            k_jpc_offs_cf<<<tiles_c, JP_THREADS, 0, s>>>(A);
+            SYM_LAUNCH_CHECK();
+        }
+        SYM_TRY(jp_launch_fill<true>(A, s));
+        if (tiles_c) {
+            k_jpc_xsums_cf<<<tiles_c, JP_THREADS, 0, s>>>(A);
+            SYM_LAUNCH_CHECK();
+        }
+        k_jpc_sums_scan<<<1, 1024, 0, s>>>(A, tiles_c);
         SYM_LAUNCH_CHECK();
+        if (tiles_c) {
+            k_jpc_place_cf<<<tiles_c, JP_THREADS, 0, s>>>(A);
+            SYM_LAUNCH_CHECK();
+        }
+    } else {
+        k_jpc_count<<<num_sms() * (2048 / JP_THREADS), JP_THREADS, 0, s>>>(A);
+        SYM_LAUNCH_CHECK();
+        k_jpc_count_huge<<<num_sms() * 4, JP_HUGE_THREADS, 0, s>>>(A);
+        SYM_LAUNCH_CHECK();
+        if (tiles_c) {
+            k_jpc_sums<<<tiles_c, JP_THREADS, 0, s>>>(A);
+            SYM_LAUNCH_CHECK();
+        }
+        k_jpc_sums_scan<<<1, 1024, 0, s>>>(A, tiles_c);
+        SYM_LAUNCH_CHECK();
+        if (tiles_c) {
+            k_jpc_place<<<tiles_c, JP_THREADS, 0, s>>>(A);
+            SYM_LAUNCH_CHECK();
+        }
+        SYM_TRY(jp_launch_fill<false>(A, s));
     }
-    {
-        // one resident wave of the grid-stride fill (see mis.cu round_grid)
-        int per = 2048 / JP_THREADS;
-#if SYM_ROUND_ONE_WAVE
-        int x = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_jpc_fill, JP_THREADS, 0) == cudaSuccess && x > 0)
-            per = std::min(per, x);
-#endif
-        k_jpc_fill<<<num_sms() * per, JP_THREADS, 0, s>>>(A);
-    }
-    SYM_LAUNCH_CHECK();
-    {
-        // block-strided pieces: one resident wave (40 regs x 512 threads -> 3 CTAs/SM, not 4)
-        int per = 4;
-#if SYM_ROUND_ONE_WAVE
-        int x = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, k_jpc_fill_huge, JP_HUGE_THREADS, 0) == cudaSuccess &&
-            x > 0)
-            per = std::min(per, x);
-#endif
-        k_jpc_fill_huge<<<num_sms() * per, JP_HUGE_THREADS, 0, s>>>(A);
-    }
-    SYM_LAUNCH_CHECK();
     prof_end_dev(s, ctr);
     A.prof = nullptr;
     A.prof_jp = nullptr;

@@ -38,6 +38,9 @@ struct MisRoundArgs {
     uint8_t *st;
     const int32_t *in_list;  // nullptr => implicit list [0, implicit_n)
     int in_rev;              // list stored backwards: v = in_list[-1 - i]
+    const int32_t *in_pos;   // nullable: resume offset (from the row start) of in_list[i]
+    int32_t *out_pos;        // nullable: resume offsets of the blocked vertices, parallel to out_list
+    int push_out;            // an In vertex marks its undecided neighbours Out (not in shard mode)
     const uint32_t *in_cnt;
     int64_t implicit_n;
     int32_t *out_list;
@@ -80,37 +83,54 @@ __device__ __forceinline__ void mis_gather(const MisRoundArgs &A, const uint32_t
 
 // bytes: §8(d) algorithmic = 4 B per column word the kernel loads + 9 B
 // per active vertex (row_ptr pair + status); the implementation's own count adds the
-// list entry and status read (5 B more per active vertex) and 1 B per decided status
-// write.  Neighbour-status gathers hit the L2-resident status array: 0 HBM bytes.
-// A short row (<= MIS_SMALL arcs, one sector) is decided by one lane: all column
-// loads, then all status gathers, then the rule (the order of the arcs does not
-// matter: any In neighbour -> Out, else any higher undecided neighbour -> blocked).
-// Column words are streamed with evict-first loads so the gathered status stays in L2.
-__device__ __forceinline__ int mis_scan_small(const MisRoundArgs &A, int64_t b, int64_t e, uint64_t kv,
-                                              unsigned long long &lb) {
-    uint32_t w[MIS_SMALL];
+// list entry, the resume offset and the status read (9 B more per active vertex) and 1 B
+// per decided status write.  Neighbour-status gathers hit the L2-resident status
+// array: 0 HBM bytes.
+// Lane stage: one lane scans the window [x, x + MIS_SMALL) of its row -- all column
+// loads, then all status gathers, then the rule (the order of the arcs does not matter:
+// any In neighbour -> Out, else any higher undecided neighbour -> blocked at the first
+// one).  Column words are streamed with evict-first loads so the gathered status stays
+// in L2.  R_NONE: the window holds neither (the row continues past it, or v is In).
+__device__ __forceinline__ int mis_scan_window(const MisRoundArgs &A, int64_t x, int64_t e, uint64_t kv,
+                                               int64_t &pos, unsigned long long &lb, uint32_t (&w)[MIS_SMALL]) {
     uint8_t s[MIS_SMALL];
 #pragma unroll
-    for (int u = 0; u < MIS_SMALL; u++) w[u] = (b + u < e) ? (uint32_t)__ldcs(A.ci + b + u) : 0u;
+    for (int u = 0; u < MIS_SMALL; u++) w[u] = (x + u < e) ? (uint32_t)__ldcs(A.ci + x + u) : 0u;
     // only higher neighbours can decide v: a lower neighbour turns In only once every
     // higher neighbour of it -- v included -- is Out, so while v is undecided none is In
     // two batched load steps (predicated, no branch per arc): the phase-filter words of
     // the higher neighbours, then their statuses
     bool hi[MIS_SMALL];
 #pragma unroll
-    for (int u = 0; u < MIS_SMALL; u++) hi[u] = b + u < e && vkey(A.k, w[u]) > kv;
+    for (int u = 0; u < MIS_SMALL; u++) hi[u] = x + u < e && vkey(A.k, w[u]) > kv;
     mis_gather(A, w, hi, s);
-    bool in = false, blk = false;
+    bool in = false;
+    int fb = MIS_SMALL;
 #pragma unroll
-    for (int u = 0; u < MIS_SMALL; u++) {
+    for (int u = MIS_SMALL - 1; u >= 0; u--) {
         in |= s[u] == ST_IN;
-        blk |= s[u] == ST_UNDEC;
+        if (s[u] == ST_UNDEC) fb = u;
     }
-    lb += 4 * (unsigned long long)(e - b);
-    return in ? R_OUT : (blk ? R_BLK : R_IN);
+    lb += 4 * (unsigned long long)min(e - x, (int64_t)MIS_SMALL);
+    if (in) return R_OUT;
+    if (fb < MIS_SMALL) {
+        pos = x + fb;
+        return R_BLK;
+    }
+    return R_NONE;
 }
 
+// Resume memo: a blocked vertex records where its scan stopped (the first undecided
+// higher neighbour, or the start of the warp step that found one); every arc before it
+// is a lower neighbour or a final-Out higher one, so the next round resumes there.
+#ifndef SYM_MIS_MINB
+#define SYM_MIS_MINB 5  // 48 regs, 5 CTAs/SM: 1.46 -> 1.39 ms MIS-NONE at R-MAT s24 (62 regs unbounded)
+#endif
+#if SYM_MIS_MINB > 0
+__global__ void __launch_bounds__(MIS_THREADS, SYM_MIS_MINB) k_mis_round(MisRoundArgs A) {
+#else
 __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
+#endif
     const uint32_t cnt = A.in_list ? *A.in_cnt : (uint32_t)A.implicit_n;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         *A.clear_cnt = 0;
@@ -125,25 +145,33 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
         int32_t v = -1;
         if (i < cnt) v = A.in_list ? (A.in_rev ? A.in_list[-1 - i] : A.in_list[i]) : (int32_t)i;
         bool active = v >= 0 && A.st[v] == ST_UNDEC;
-        int64_t b = 0, e = 0;
+        int64_t b = 0, e = 0, x0 = 0;
         uint64_t kv = 0;
         if (active) {
             b = A.rp[v - A.row_base];
             e = A.rp[v - A.row_base + 1];
+            x0 = b + (A.in_pos ? A.in_pos[i] : 0);
             kv = vkey(A.k, (uint32_t)v);
         }
         int res = R_NONE;
-        int64_t resume = 0;
+        int64_t resume = 0, pos = 0;
         unsigned long long lb = 0;  // column words loaded (4 B each)
-        if (active && e - b <= MIS_SMALL) res = mis_scan_small(A, b, e, kv, lb);
-        unsigned longm = __ballot_sync(FULL, active && e - b > MIS_SMALL);
+        // lane stage: the first MIS_SMALL arcs of every row (a long row of an R-MAT graph
+        // is almost always decided or blocked within them)
+        uint32_t wv[MIS_SMALL];
+        if (active) {
+            res = mis_scan_window(A, x0, e, kv, pos, lb, wv);
+            if (res == R_NONE && e - x0 <= MIS_SMALL) res = R_IN;
+        }
+        unsigned longm = __ballot_sync(FULL, active && res == R_NONE);
         while (longm) {
             const int src = __ffs(longm) - 1;
             longm &= longm - 1;
-            const int64_t wb = __shfl_sync(FULL, b, src), we = __shfl_sync(FULL, e, src);
+            const int64_t wb = __shfl_sync(FULL, x0, src) + MIS_SMALL, we = __shfl_sync(FULL, e, src);
             const uint64_t wk = __shfl_sync(FULL, kv, src);
             const int64_t lim = min(we, wb + MIS_BUDGET);
             int r = R_IN;
+            int64_t wpos = 0;
             for (int64_t x = wb; x < lim; x += 128) {
                 uint32_t w[4];
                 bool ok[4];
@@ -165,21 +193,51 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
                     fblk |= sw[u] == ST_UNDEC;
                 }
                 if (__any_sync(FULL, fin)) { r = R_OUT; break; }
-                if (__any_sync(FULL, fblk)) { r = R_BLK; break; }
+                if (__any_sync(FULL, fblk)) { r = R_BLK; wpos = x; break; }
             }
             if (r == R_IN && lim < we) r = R_DEFER;
             if (lane == src) {
                 res = r;
                 resume = lim;
+                pos = wpos;
+            }
+        }
+        // push-Out: a new In vertex marks its undecided neighbours Out (only undecided
+        // ones: INACTIVE vertices are outside the phase), so a blocked vertex waits at
+        // its first undecided higher neighbour and never rescans its row for an In one
+        // (none of those neighbours can turn In meanwhile: each has v above it)
+        if (A.push_out) {
+            const bool lanepush = res == R_IN && x0 == b && e - b <= MIS_SMALL;
+            if (lanepush) {
+                uint8_t sv[MIS_SMALL];
+#pragma unroll
+                for (int u = 0; u < MIS_SMALL; u++) sv[u] = ld_u8_pred(A.st + wv[u], b + u < e, ST_OUT);
+#pragma unroll
+                for (int u = 0; u < MIS_SMALL; u++)
+                    if (sv[u] == ST_UNDEC) A.st[wv[u]] = ST_OUT;
+            }
+            unsigned pm = __ballot_sync(FULL, res == R_IN && !lanepush);
+            while (pm) {
+                const int src = __ffs(pm) - 1;
+                pm &= pm - 1;
+                const int64_t wb = __shfl_sync(FULL, b, src), we = __shfl_sync(FULL, e, src);
+                for (int64_t x = wb + lane; x < we; x += 32) {
+                    const int32_t w = A.ci[x];
+                    if (A.st[w] == ST_UNDEC) A.st[w] = ST_OUT;
+                }
+                prof_add(A.prof, lane == 0 ? 4ull * (we - wb) : 0ull, lane == 0 ? 4ull * (we - wb) : 0ull);  // row re-read
             }
         }
         if (res == R_IN) A.st[v] = ST_IN;
         else if (res == R_OUT) A.st[v] = ST_OUT;
         // §8(d): 4 B per scanned arc + 9 B per active vertex; the implementation also
         // reads the list entry and the status (5 B) and writes decided statuses
-        prof_add(A.prof, lb + (active ? 9 : 0), lb + (active ? 17 : 0) + ((res == R_IN || res == R_OUT) ? 1 : 0));
+        prof_add(A.prof, lb + (active ? 9 : 0), lb + (active ? 18 : 0) + ((res == R_IN || res == R_OUT) ? 1 : 0));
         int64_t slot = warp_append(res == R_BLK, A.out_cnt);
-        if (slot >= 0) A.out_list[slot] = v;
+        if (slot >= 0) {
+            A.out_list[slot] = v;
+            if (A.out_pos) A.out_pos[slot] = (int32_t)(pos - b);
+        }
         int64_t hs = warp_append(res == R_DEFER, A.huge_cnt);
         if (hs >= 0) {
             A.huge[2 * hs] = v;
@@ -196,6 +254,7 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
         const int64_t b = A.huge[2 * h + 1], e = A.rp[v - A.row_base + 1];
         const uint64_t kv = vkey(A.k, (uint32_t)v);
         int r = R_IN;
+        int64_t bpos = b;
         unsigned long long lb = 0;  // column words (the vertex was counted active by k_mis_round)
         for (int64_t x = b; x < e; x += 4 * MIS_HUGE_THREADS) {
             bool fin = false, fblk = false;
@@ -218,7 +277,15 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
                 fblk |= sw[u] == ST_UNDEC;
             }
             if (__syncthreads_or(fin)) { r = R_OUT; break; }
-            if (__syncthreads_or(fblk)) { r = R_BLK; break; }
+            if (__syncthreads_or(fblk)) { r = R_BLK; bpos = x; break; }
+        }
+        if (r == R_IN && A.push_out) {  // push-Out over the whole row (see k_mis_round)
+            const int64_t rb = A.rp[v - A.row_base];
+            for (int64_t x = rb + threadIdx.x; x < e; x += MIS_HUGE_THREADS) {
+                const int32_t w = A.ci[x];
+                if (A.st[w] == ST_UNDEC) A.st[w] = ST_OUT;
+            }
+            prof_add(A.prof, threadIdx.x == 0 ? 4ull * (e - rb) : 0ull, threadIdx.x == 0 ? 4ull * (e - rb) : 0ull);
         }
         if (threadIdx.x == 0) {
             if (r == R_IN) A.st[v] = ST_IN;
@@ -226,6 +293,7 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
             else {
                 uint32_t slot = atomicAdd(A.out_cnt, 1u);
                 A.out_list[slot] = v;
+                if (A.out_pos) A.out_pos[slot] = (int32_t)(bpos - A.rp[v - A.row_base]);
             }
         }
         prof_add(A.prof, lb, lb + (threadIdx.x == 0 ? 9 : 0));  // impl: + row end + status write
@@ -446,6 +514,8 @@ void carve_mis_ws(Arena &a, int64_t n, int64_t nnz, MisWs &w) {
     w.vlist = a.take<int32_t>((size_t)n + 1);
     w.fr[0] = a.take<int32_t>((size_t)n + 1);
     w.fr[1] = a.take<int32_t>((size_t)n + 1);
+    w.fp[0] = a.take<int32_t>((size_t)n + 1);
+    w.fp[1] = a.take<int32_t>((size_t)n + 1);
     w.huge_cap = nnz / MIS_BUDGET + 2;
     w.huge = a.take<int64_t>((size_t)(2 * w.huge_cap));
     w.gmax = a.take<unsigned long long>((size_t)n + 1);
@@ -534,7 +604,7 @@ static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp
     const int batch = 4;  // rounds launched per host poll of the frontier count
     for (;;) {
         for (int b = 0; b < batch && (uint32_t)r < maxr; b++, r++) {  // never past the cap
-            MisRoundArgs A;
+            MisRoundArgs A{};
             A.rp = rp;
             A.ci = ci;
             A.st = st;
@@ -542,13 +612,17 @@ static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp
                 A.in_list = list0;
                 A.in_rev = rev0;
                 A.in_cnt = cnt0;
+                A.in_pos = nullptr;
             } else {
                 A.in_list = w.fr[r & 1];
                 A.in_rev = 0;
                 A.in_cnt = &ctl->ring[r % 3];
+                A.in_pos = w.fp[r & 1];
             }
             A.implicit_n = implicit_n;
             A.out_list = w.fr[(r + 1) & 1];
+            A.out_pos = w.fp[(r + 1) & 1];
+            A.push_out = 1;
             A.out_cnt = &ctl->ring[(r + 1) % 3];
             A.clear_cnt = &ctl->ring[(r + 2) % 3];
             A.huge = w.huge;
@@ -843,7 +917,7 @@ static int mis_sharded_phase(const ShardPlan &P, ShardCtx &x, const sym_params *
         SYM_CUDA(cudaMemsetAsync(x.dcnt(r), 0, 2 * sizeof(uint32_t), s));
         SYM_CUDA(cudaMemsetAsync(x.scratch, 0, 4 * sizeof(uint32_t), s));
         if (local > 0) {
-            MisRoundArgs A;
+            MisRoundArgs A{};
             A.rp = P.rp;
             A.ci = P.ci;
             A.st = st;

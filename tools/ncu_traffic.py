@@ -34,7 +34,9 @@ def main():
     out_csv = os.path.join(ROOT, "gpurun_out", f"{tag}_traffic.csv")
     os.makedirs(os.path.dirname(out_csv), exist_ok=True)
     cmd = ["ncu", "--cache-control", "none", "--clock-control", "none", "--metrics",
-           "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum", "--csv", "--log-file", out_csv,
+           "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum,lts__t_sectors.sum,"
+           "lts__throughput.avg.pct_of_peak_sustained_elapsed,dram__throughput.avg.pct_of_peak_sustained_elapsed",
+           "--csv", "--log-file", out_csv,
            sys.executable, os.path.join(ROOT, "bench.py"), "--profile-only", "--steps", "1", "--warmup", "1"]
     subprocess.run(cmd, check=True, stdout=subprocess.DEVNULL, stderr=subprocess.DEVNULL, timeout=1800)
     rows = [l for l in open(out_csv) if l.startswith('"')]
@@ -57,18 +59,29 @@ def main():
         c = kclass(k["name"])
         if c is None:
             continue
-        a = agg.setdefault(c, {"launches": 0, "dram_bytes": 0.0, "us": 0.0, "kernels": set()})
+        a = agg.setdefault(c, {"launches": 0, "dram_bytes": 0.0, "us": 0.0, "kernels": set(), "l2_sectors": 0.0,
+                               "l2_pct_us": 0.0, "dram_pct_us": 0.0})
         a["launches"] += 1
+        t = k.get("gpu__time_duration.sum", 0.0)
+        a["l2_sectors"] += k.get("lts__t_sectors.sum", 0.0)
+        a["l2_pct_us"] += k.get("lts__throughput.avg.pct_of_peak_sustained_elapsed", 0.0) * t
+        a["dram_pct_us"] += k.get("dram__throughput.avg.pct_of_peak_sustained_elapsed", 0.0) * t
         a["dram_bytes"] += k.get("dram__bytes_read.sum", 0.0) + k.get("dram__bytes_write.sum", 0.0)
         a["us"] += k.get("gpu__time_duration.sum", 0.0)
         a["kernels"].add(k["name"])
     classes = {c: {"launches": a["launches"], "dram_bytes": a["dram_bytes"],
                    "dram_bytes_per_launch": a["dram_bytes"] / a["launches"], "us": a["us"],
+                   "l2_sectors": a["l2_sectors"],
+                   # time-weighted ncu throughput fractions of the class (L2 = lts__throughput, the
+                   # busiest L2 sub-unit; DRAM = dram__throughput)
+                   "l2_frac": a["l2_pct_us"] / a["us"] / 100.0 if a["us"] else 0.0,
+                   "dram_frac": a["dram_pct_us"] / a["us"] / 100.0 if a["us"] else 0.0,
                    "kernels": sorted(a["kernels"])} for c, a in agg.items()}
     res = {"tag": tag, "command": " ".join(cmd[:-7]) + " python bench.py --profile-only --steps 1 --warmup 1",
            "note": "DRAM bytes = dram__bytes_read.sum + dram__bytes_write.sum per kernel class over the measured "
                    "step (the second of two); serialised replay, no cache flush: compare shares and bytes, "
-                   "not absolute times", "classes": classes}
+                   "not absolute times; l2_frac / dram_frac = time-weighted lts__throughput / dram__throughput "
+                   "pct_of_peak_sustained_elapsed", "classes": classes}
     for dst in (os.path.join(ROOT, "profiles", f"{tag}_traffic.json"),
                 os.path.join(ROOT, "gpurun_out", f"{tag}_traffic.json")):
         with open(dst, "w") as f:
