@@ -352,15 +352,29 @@ def main():
         return statistics.median(ts)
 
     def profiled(fn, calls):
-        sb.sym_profile_enable(True)
+        """Per-class profile over `calls` calls: device times from an events-only pass
+        (mode 2: the kernels' byte counters cost time -- MIS rounds ran 2.4x slower with
+        them), byte counts from one counting pass (mode 1), scaled per launch."""
+        sb.sym_profile_enable(1)
         fn()  # the first profiled call allocates the hook's counters
         torch.cuda.synchronize()
         sb.sym_profile_collect()
+        fn()
+        torch.cuda.synchronize()
+        counted = sb.sym_profile_collect()
+        sb.sym_profile_enable(2)
         for _ in range(calls):
             fn()
         torch.cuda.synchronize()
         prof = sb.sym_profile_collect()
         sb.sym_profile_enable(False)
+        for c, v in prof.items():
+            b = counted.get(c)
+            for key in ("alg_bytes", "impl_bytes"):
+                if b is None or b[key] < 0 or b["launches"] <= 0:
+                    v[key] = -1.0
+                else:  # bytes of one counted call, spread over this pass's launches
+                    v[key] = b[key] * calls
         return prof
 
     # ---- per-problem breakdown of the step (events between the calls)

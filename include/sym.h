@@ -290,7 +290,9 @@ int sym_color_sharded(const sym_graph_shard *g, const sym_params *p, sym_comm *c
 
 /* ---- kernel profiling hook (measurement only; off by default) ----
    sym_profile_enable(1) makes every later call record a CUDA event pair on its
-   stream around each hot-kernel launch, grouped by kernel class ("split_degk",
+   stream around each hot-kernel launch (and count bytes on the device; mode 2 records
+   the events only -- the kernels' byte counters cost device time, so timings are taken
+   in mode 2 and byte counts in mode 1; 0 turns the hook off), grouped by kernel class ("split_degk",
    "split_rand", "mis_round", "mis_huge", "mm_round0", "mm_round", "mm_huge",
    "jp_build", "jp_rounds", ...).  sym_profile_collect() synchronises those
    events and returns, per class: launches, summed device milliseconds and two byte

@@ -186,9 +186,11 @@ def sym_color(row_ptr, col_idx, kind="none", param=0, seed=42, decomp=None, stat
                  flags, max_rounds, validate, device)
 
 
-def sym_profile_enable(on: bool = True) -> None:
-    """Record CUDA-event device times per hot-kernel class (measurement hook)."""
-    L.load().sym_profile_enable(1 if on else 0)
+def sym_profile_enable(on=True) -> None:
+    """Record CUDA-event device times per hot-kernel class (measurement hook).
+    True / 1: events and the kernels' device byte counters; 2: events only (timing
+    without the counters' atomics); False / 0: off."""
+    L.load().sym_profile_enable(int(on) if not isinstance(on, bool) else (1 if on else 0))
 
 
 def sym_profile_collect() -> dict:

@@ -241,6 +241,7 @@ static int flow_setup(const sym_graph *g, const sym_params *p, const sym_decomp 
             f.split.rp_x = decomp->row_ptr_x;
             f.split.ci_x = decomp->col_x;
             f.split.nnz_in = decomp->nnz_in;
+            f.split.nnz_x = decomp->nnz_x;
         } else if (g->n > 0) {
             SYM_TRY(run_split(f.g, p->kind, p->param, p->seed, L.sw, L.ctl, L.rp_in, L.ci_in, L.rp_x, L.ci_x,
                               nullptr, s));

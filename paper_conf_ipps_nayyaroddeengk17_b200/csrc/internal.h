@@ -74,6 +74,7 @@ struct Split {
     const int64_t *rp_in = nullptr, *rp_x = nullptr;
     const int32_t *ci_in = nullptr, *ci_x = nullptr;
     int64_t nnz_in = -1;  // known on the host only for a caller-supplied decomposition
+    int64_t nnz_x = -1;
 };
 
 struct Graph {
@@ -83,8 +84,11 @@ struct Graph {
 };
 
 // ------------------------------------------------------------------ decomposition (decompose.cu)
-constexpr int SPLIT_THREADS = 256;
-constexpr int SPLIT_PER_THREAD = 16;
+#ifndef SYM_SPLIT_THREADS
+#define SYM_SPLIT_THREADS 256
+#endif
+constexpr int SPLIT_THREADS = SYM_SPLIT_THREADS;
+constexpr int SPLIT_PER_THREAD = 4096 / SPLIT_THREADS;  // tiles of 4096 arcs
 constexpr int SPLIT_TILE = SPLIT_THREADS * SPLIT_PER_THREAD;  // arcs per tile
 
 // BRIDGE decomposition scratch (bridge.cu; carved only for SYM_DECOMP_BRIDGE)

@@ -34,6 +34,7 @@ struct MmRoundArgs {
     uint32_t *mbits;  // matched bitmap (1 bit per vertex, L2-resident): the liveness gathers
     const int32_t *pick_prev;
     int32_t *pick_cur;
+    int32_t *alt;     // nullable: u's second-heaviest believed-live neighbour at its last scan (-1: none)
     const int32_t *in_list;
     int in_rev;
     const uint32_t *in_cnt;
@@ -59,6 +60,22 @@ struct MmRoundArgs {
 __device__ __forceinline__ bool mm_matched(const uint32_t *mbits, uint32_t v) { return (mbits[v >> 5] >> (v & 31)) & 1u; }
 __device__ __forceinline__ void mm_set_matched(uint32_t *mbits, uint32_t v) { atomicOr(mbits + (v >> 5), 1u << (v & 31)); }
 
+// top-2 of keys offset by one (0 = none; a key's low word is an id < 2^31, so +1 never
+// carries): merge (a1 > a2) with (b1 > b2)
+__device__ __forceinline__ void top2_merge(uint64_t &a1, uint64_t &a2, uint64_t b1, uint64_t b2) {
+    const uint64_t lo = a1 < b1 ? a1 : b1, hi2 = a1 > b1 ? a2 : b2;
+    a1 = a1 > b1 ? a1 : b1;
+    a2 = lo > hi2 ? lo : hi2;
+}
+__device__ __forceinline__ void top2_add(uint64_t &a1, uint64_t &a2, uint64_t k) {
+    if (k > a1) {
+        a2 = a1;
+        a1 = k;
+    } else if (k > a2) {
+        a2 = k;
+    }
+}
+
 __device__ __forceinline__ void mm_row(const MmRoundArgs &A, int32_t u, int64_t &b, int64_t &e, const int32_t *&ci) {
     if (A.dual && ((A.hbits[u >> 5] >> (u & 31)) & 1u)) {
         b = A.rp2[u - A.row_base];
@@ -71,6 +88,9 @@ __device__ __forceinline__ void mm_row(const MmRoundArgs &A, int32_t u, int64_t 
     }
 }
 
+#ifndef SYM_MM_ALT
+#define SYM_MM_ALT 1
+#endif
 // 6 CTAs/SM (<= 40 regs, no spills; 47 without the bound -> 5): more mate gathers in flight
 #ifndef SYM_MM_MINB
 #define SYM_MM_MINB 6
@@ -121,6 +141,18 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
                 // is matching right now: 25 rounds, 5.10 ms)
                 reuse = true;
                 nb += 4;
+            } else if (MATE && p >= 0 && A.alt) {
+                // p is matched: u's second-heaviest neighbour at its last scan, if still
+                // unmatched, is now its heaviest live one (every other heavier neighbour
+                // was already matched then) -- no rescan
+                const int32_t q = A.alt[u];
+                nb += 4;
+                if (q >= 0 && !mm_matched(A.mbits, (uint32_t)q)) {
+                    reuse = true;
+                    p = q;
+                    A.alt[u] = -1;
+                    nb += 8;
+                }
             }
         }
         const bool scan = active && !reuse;
@@ -129,7 +161,7 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
         if (scan) mm_row(A, u, b, e, ci);
         const int64_t d = e - b;
         nb += scan ? 20 : 0;
-        uint64_t best = 0;
+        uint64_t best = 0, sec = 0;  // sec: second-heaviest key + 1 (0 = none)
         bool has = false;
         if (scan && d <= MM_SMALL) {
             // short row by one lane: all column loads (streamed, evict-first so the
@@ -142,13 +174,11 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
 #pragma unroll
             for (int q = 0; q < MM_SMALL; q++) live[q] = (q < d) && (!MATE || !mm_matched(A.mbits, w[q]));
 #pragma unroll
-            for (int q = 0; q < MM_SMALL; q++) {
-                if (live[q]) {
-                    uint64_t kk = ekey(A.k, (uint32_t)u, w[q]);
-                    if (!has || kk > best) best = kk;
-                    has = true;
-                }
-            }
+            uint64_t b1 = 0;
+            for (int q = 0; q < MM_SMALL; q++)
+                if (live[q]) top2_add(b1, sec, ekey(A.k, (uint32_t)u, w[q]) + 1);
+            has = b1 != 0;
+            best = b1 - 1;
         }
         // warp-cooperative argmax for medium rows
         unsigned medm = __ballot_sync(FULL, scan && d > MM_SMALL && d <= MM_BUDGET);
@@ -158,8 +188,7 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
             const int64_t wb = __shfl_sync(FULL, b, src), we = __shfl_sync(FULL, e, src);
             const int32_t wu = __shfl_sync(FULL, u, src);
             const int32_t *wci = (const int32_t *)__shfl_sync(FULL, (unsigned long long)ci, src);
-            uint64_t lb = 0;
-            bool lh = false;
+            uint64_t lb = 0, l2 = 0;  // top-2 keys + 1 (0 = none)
             for (int64_t x = wb; x < we; x += 128) {
                 uint32_t w[4];
                 bool ok[4];
@@ -171,28 +200,24 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
                     colb += ok[q] ? 4 : 0;
                 }
 #pragma unroll
-                for (int q = 0; q < 4; q++) {
-                    if (ok[q] && (!MATE || !mm_matched(A.mbits, w[q]))) {
-                        uint64_t kk = ekey(A.k, (uint32_t)wu, w[q]);
-                        if (!lh || kk > lb) lb = kk;
-                        lh = true;
-                    }
-                }
+                for (int q = 0; q < 4; q++)
+                    if (ok[q] && (!MATE || !mm_matched(A.mbits, w[q]))) top2_add(lb, l2, ekey(A.k, (uint32_t)wu, w[q]) + 1);
             }
 #pragma unroll
             for (int dd = 16; dd; dd >>= 1) {
-                uint64_t o = __shfl_xor_sync(FULL, lb, dd);
-                lb = o > lb ? o : lb;
+                const uint64_t o1 = __shfl_xor_sync(FULL, lb, dd), o2 = __shfl_xor_sync(FULL, l2, dd);
+                top2_merge(lb, l2, o1, o2);
             }
-            bool anyh = __any_sync(FULL, lh);
             if (lane == src) {
-                best = lb;
-                has = anyh;
+                best = lb - 1;
+                has = lb != 0;
+                sec = l2;
             }
         }
         if (reuse) has = true;
         bool defer = scan && d > MM_BUDGET;
         if (active && !defer) A.pick_cur[u] = reuse ? p : (has ? (int32_t)(uint32_t)best : -1);
+        if (A.alt && scan && !defer) A.alt[u] = sec ? (int32_t)(uint32_t)(sec - 1) : -1;
         int64_t slot = warp_append(active && !defer && has, A.out_cnt);
         if (slot >= 0) A.out_list[slot] = u;
         int64_t hs = warp_append(defer, A.huge_cnt);
@@ -202,20 +227,18 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
     }
 }
 
-// rows longer than MM_BUDGET: one CTA per vertex, block argmax
+// rows longer than MM_BUDGET: one CTA per vertex, block top-2 (argmax + the alternate)
 template <bool MATE>
 __global__ void __launch_bounds__(MM_HUGE_THREADS) k_mm_huge(MmRoundArgs A) {
     const uint32_t cnt = *A.huge_cnt;
-    __shared__ unsigned long long s_best[MM_HUGE_THREADS / 32];
-    __shared__ int s_has[MM_HUGE_THREADS / 32];
+    __shared__ unsigned long long s_b1[MM_HUGE_THREADS / 32], s_b2[MM_HUGE_THREADS / 32];
     const int lane = lane_id(), warp = threadIdx.x >> 5;
     for (uint32_t h = blockIdx.x; h < cnt; h += gridDim.x) {
         const int32_t u = A.huge[h];
         int64_t b, e;
         const int32_t *ci;
         mm_row(A, u, b, e, ci);
-        uint64_t lb = 0;
-        bool lh = false;
+        uint64_t l1 = 0, l2 = 0;  // top-2 keys + 1 (0 = none)
         unsigned long long nb = 0;
         for (int64_t x = b; x < e; x += 4 * MM_HUGE_THREADS) {
             uint32_t w[4];
@@ -228,37 +251,26 @@ __global__ void __launch_bounds__(MM_HUGE_THREADS) k_mm_huge(MmRoundArgs A) {
                 nb += ok[q] ? 4 : 0;
             }
 #pragma unroll
-            for (int q = 0; q < 4; q++) {
-                if (ok[q] && (!MATE || !mm_matched(A.mbits, w[q]))) {
-                    uint64_t kk = ekey(A.k, (uint32_t)u, w[q]);
-                    if (!lh || kk > lb) lb = kk;
-                    lh = true;
-                }
-            }
+            for (int q = 0; q < 4; q++)
+                if (ok[q] && (!MATE || !mm_matched(A.mbits, w[q]))) top2_add(l1, l2, ekey(A.k, (uint32_t)u, w[q]) + 1);
         }
 #pragma unroll
         for (int dd = 16; dd; dd >>= 1) {
-            uint64_t o = __shfl_xor_sync(FULL, lb, dd);
-            lb = o > lb ? o : lb;
+            const uint64_t o1 = __shfl_xor_sync(FULL, l1, dd), o2 = __shfl_xor_sync(FULL, l2, dd);
+            top2_merge(l1, l2, o1, o2);
         }
-        bool wh = __any_sync(FULL, lh);
         prof_add(A.prof, nb, nb);
         if (lane == 0) {
-            s_best[warp] = lb;
-            s_has[warp] = wh;
+            s_b1[warp] = l1;
+            s_b2[warp] = l2;
         }
         __syncthreads();
         if (threadIdx.x == 0) {
-            uint64_t bb = 0;
-            bool hh = false;
-            for (int q = 0; q < MM_HUGE_THREADS / 32; q++) {
-                if (s_has[q]) {
-                    bb = (!hh || s_best[q] > bb) ? s_best[q] : bb;
-                    hh = true;
-                }
-            }
-            A.pick_cur[u] = hh ? (int32_t)(uint32_t)bb : -1;
-            if (hh) {
+            uint64_t b1 = 0, b2 = 0;
+            for (int q = 0; q < MM_HUGE_THREADS / 32; q++) top2_merge(b1, b2, s_b1[q], s_b2[q]);
+            A.pick_cur[u] = b1 ? (int32_t)(uint32_t)(b1 - 1) : -1;
+            if (A.alt) A.alt[u] = b2 ? (int32_t)(uint32_t)(b2 - 1) : -1;
+            if (b1) {
                 uint32_t slot = atomicAdd(A.out_cnt, 1u);
                 A.out_list[slot] = u;
             }
@@ -304,6 +316,7 @@ void carve_mm_ws(Arena &a, int64_t n, int64_t nnz, MmWs &w) {
     w.huge = reinterpret_cast<int64_t *>(a.take<int32_t>((size_t)w.huge_cap));
     w.gmax = a.take<unsigned long long>((size_t)n + 1);
     w.mbits = a.take<uint32_t>((size_t)(n + 31) / 32 + 1);
+    w.alt = a.take<int32_t>((size_t)n + 1);
 }
 
 struct MmPhase {
@@ -346,6 +359,9 @@ static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph
     const int full_grid = mm_round_grid();
     int grid = full_grid;
     int r = 0;
+    // no alternates yet (the streaming round 0 finds the heaviest arc only: tracking a
+    // second there cost more than it saved -- 1.7 -> 2.9 ms round 0 at R-MAT s24 MM-NONE)
+    SYM_CUDA(cudaMemsetAsync(w.alt, 0xff, sizeof(int32_t) * (size_t)(f.g.n + 1), s));
     const int batch = 4;  // rounds launched per host poll of the frontier count
     if (ph.first && !ph.dual) {
         // round 0 as one streaming pass: every phase vertex picks its heaviest arc;
@@ -360,7 +376,7 @@ static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph
     }
     for (;;) {
         for (int bb = 0; bb < batch && (uint32_t)r < maxr; bb++, r++) {  // never past the cap
-            MmRoundArgs A;
+            MmRoundArgs A{};
             A.rp = ph.rp;
             A.rp2 = ph.rp2;
             A.ci = ph.ci;
@@ -371,6 +387,7 @@ static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph
             A.mbits = w.mbits;
             A.pick_prev = w.pick[(r + 1) & 1];
             A.pick_cur = w.pick[r & 1];
+            A.alt = SYM_MM_ALT ? w.alt : nullptr;
             if (r == 0) {
                 A.in_list = ph.list0;
                 A.in_rev = ph.rev0;
@@ -595,7 +612,7 @@ static int mm_sharded_phase(const ShardPlan &P, ShardCtx &x, const sym_params *p
         SYM_CUDA(cudaMemsetAsync(x.dcnt(r), 0, 2 * sizeof(uint32_t), s));
         SYM_CUDA(cudaMemsetAsync(x.scratch, 0, 4 * sizeof(uint32_t), s));
         if (local > 0) {
-            MmRoundArgs A;
+            MmRoundArgs A{};
             A.rp = rp;
             A.rp2 = nullptr;
             A.ci = ci;

@@ -19,6 +19,7 @@ struct Rec {
     int slot;  // device byte counter pair slot, or -1
 };
 std::atomic<bool> g_on{false};
+std::atomic<bool> g_bytes{false};  // mode 1: device byte counters too; mode 2: events only
 // device byte counters for launches whose algorithmic bytes depend on the frontier
 // (measurement mode only; the one allocation the library makes, lazily, when
 // profiling is enabled)
@@ -72,7 +73,7 @@ void prof_end(cudaStream_t s, double alg, double impl) {
 }
 
 unsigned long long *prof_counter(cudaStream_t s) {
-    if (!g_on) return nullptr;
+    if (!g_on || !g_bytes) return nullptr;
     std::lock_guard<std::mutex> lk(g_mu);
     if (!g_dev && cudaMalloc(&g_dev, 2 * sizeof(unsigned long long) * DEV_SLOTS) != cudaSuccess) {
         g_dev = nullptr;
@@ -97,6 +98,7 @@ using namespace sym;
 extern "C" int sym_profile_enable(int on) {
     std::lock_guard<std::mutex> lk(g_mu);
     g_on = on != 0;
+    g_bytes = on == 1;
     return SYM_OK;
 }
 

@@ -175,8 +175,8 @@ __global__ void __launch_bounds__(SPLIT_THREADS) k_round0(Round0Args A) {
     // 4. per-row maxima: run-length reduce inside the thread, flush to shared memory
     {
         const uint32_t r_c = (uint32_t)(r_begin > 0 ? r_begin - 1 : 0);  // row carried into the tile
-        int h = carry, cur = -2;
-        unsigned long long m = 0;
+        int h = carry, cur = -2, f_cur = -2;
+        unsigned long long m = 0, f_m = 0;
 #pragma unroll
         for (int q = 0; q < V / 8; q++) {
             int4 hv = *reinterpret_cast<const int4 *>(s_head + j0 + 8 * q);
@@ -187,7 +187,16 @@ __global__ void __launch_bounds__(SPLIT_THREADS) k_round0(Round0Args A) {
                 h = max(h, (int)hh[i]);
                 if (j0 + kx < len) {
                     if (h != cur) {
-                        if (cur != -2) atomicMax(&s_max[cur < 0 ? T : cur], m);
+                        // a run that started inside this thread's arcs and ended before its
+                        // last one is the whole row: a plain store (sm_100 has no 64-bit
+                        // shared atomicMax -- each one is a CAS loop); only the first and
+                        // the last run of a thread can be shared with its neighbours
+                        if (cur >= j0) {
+                            s_max[cur] = m;
+                        } else if (cur != -2) {  // the first run: merged after the loop
+                            f_cur = cur;
+                            f_m = m;
+                        }
                         cur = h;
                         m = 0;
                     }
@@ -197,6 +206,7 @@ __global__ void __launch_bounds__(SPLIT_THREADS) k_round0(Round0Args A) {
                 }
             }
         }
+        if (f_cur != -2) atomicMax(&s_max[f_cur < 0 ? T : f_cur], f_m);
         if (cur != -2) atomicMax(&s_max[cur < 0 ? T : cur], m);
     }
     __syncthreads();
@@ -233,6 +243,10 @@ int phase_arcs(const FlowArgs &f, const int64_t *rp, int64_t *out) {
     }
     if (rp == f.split.rp_in && f.split.nnz_in >= 0) {
         *out = f.split.nnz_in;
+        return SYM_OK;
+    }
+    if (rp == f.split.rp_x && f.split.nnz_x >= 0) {
+        *out = f.split.nnz_x;
         return SYM_OK;
     }
     uint64_t v = 0;
