@@ -17,7 +17,7 @@ timeout 1200 python tools/ncu_traffic.py $TAG > $O/traffic.log 2>&1
 NCU="ncu --set full --import-source on --clock-control none --cache-control none"
 PB="python bench.py --profile-only --steps 1 --warmup 1"
 timeout 900 $NCU -k regex:'^k_jp_rounds$' -s 1 -c 1 -o $O/jp $PB > /dev/null 2>&1
-timeout 900 $NCU -k regex:'^k_jpc_fill$' -s 1 -c 1 -o $O/fill $PB > /dev/null 2>&1
+timeout 900 $NCU -k regex:'^k_jpc_fill' -s 1 -c 1 -o $O/fill $PB > /dev/null 2>&1
 timeout 900 $NCU -k regex:'^k_split' -s 2 -c 2 -o $O/split $PB > /dev/null 2>&1
 timeout 900 $NCU -k regex:'^k_(round0|mm_round)' -s 20 -c 4 -o $O/mm $PB > /dev/null 2>&1
 timeout 900 $NCU -k regex:'^k_mis_round' -s 16 -c 4 -o $O/mis $PB > /dev/null 2>&1
