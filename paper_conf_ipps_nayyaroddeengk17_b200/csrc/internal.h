@@ -84,6 +84,9 @@ struct Graph {
 };
 
 // ------------------------------------------------------------------ decomposition (decompose.cu)
+#ifndef SYM_POLL_BATCH
+#define SYM_POLL_BATCH 4  // MIS / MM rounds launched per host poll of the frontier count
+#endif
 #ifndef SYM_SPLIT_THREADS
 #define SYM_SPLIT_THREADS 256
 #endif

@@ -690,6 +690,9 @@ __device__ __forceinline__ void jp_fixed(const JpArgs &A, int64_t h, uint32_t R,
 #ifndef SYM_FILL_MINB
 #define SYM_FILL_MINB 5
 #endif
+#ifndef SYM_FILL_BATCH
+#define SYM_FILL_BATCH 4  // arcs per batch of a lane's short row
+#endif
 template <bool CF>
 #if SYM_FILL_MINB > 0
 __global__ void __launch_bounds__(JP_THREADS, SYM_FILL_MINB) k_jpc_fill(JpArgs A) {
@@ -726,22 +729,23 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
             }
         }
         const uint64_t hl0 = hl, ll0 = ll;
-        if (active && e - b <= JP_SMALL) {  // batches of 4 arcs: their loads in flight together
-            for (int64_t xq = b; xq < e; xq += 4) {
-                uint32_t w[4], rk[4];
-                bool ok[4], sv[4];
+        if (active && e - b <= JP_SMALL) {  // batches of FB arcs: their loads in flight together
+            constexpr int FB = SYM_FILL_BATCH;
+            for (int64_t xq = b; xq < e; xq += FB) {
+                uint32_t w[FB], rk[FB];
+                bool ok[FB], sv[FB];
 #pragma unroll
-                for (int u = 0; u < 4; u++) {
+                for (int u = 0; u < FB; u++) {
                     ok[u] = xq + u < e;
                     w[u] = ok[u] ? (uint32_t)__ldcs(A.ci + xq + u) : 0u;
                 }
 #pragma unroll
-                for (int u = 0; u < 4; u++) {
+                for (int u = 0; u < FB; u++) {
                     sv[u] = ok[u] && (CF || in_set(A.inS, w[u]));
                     rk[u] = sv[u] ? jp_rank(A, w[u]) : 0u;
                 }
 #pragma unroll
-                for (int u = 0; u < 4; u++) {
+                for (int u = 0; u < FB; u++) {
                     if (!ok[u]) continue;
                     if (!sv[u]) jp_fixed(A, h, R, x0, w[u]);
                     else if (jp_okey(A.k, A.okey, A.ord, w[u]) > kv) __stcs(A.lst + hl++, rk[u]);
@@ -807,9 +811,9 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
     }
 }
 
-// huge rows: one CTA per piece; each warp counts its 512-arc slice (ballots), reserves
-// its positions on the row's two cursors with one atomic each, then writes (the
-// slice is re-read from L2).  CF: the lower cursor counts from the back of the area.
+// huge rows: one CTA per piece; each warp holds its 512-arc slice in registers, counts
+// it (ballots), reserves its positions on the row's two cursors with one atomic each,
+// then writes.  CF: the lower cursor counts from the back of the area.
 template <bool CF>
 __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
     constexpr int SLICE = JP_PIECE / (JP_HUGE_THREADS / 32);
@@ -830,19 +834,30 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
         const uint32_t d = (uint32_t)(e - b);
         const uint64_t hl = meta_off(m1) + (CF ? watch_area(d, 0u) : watch_area(m0.y, m0.z));
         const uint64_t ll = CF ? hl + d : hl + m0.y;  // CF: one past the back of the area
-        uint32_t nu = 0, nd = 0;
-        for (int64_t x = sb0 + lane; x - lane < se; x += 32) {
-            bool up = false, dn = false;
-            if (x < se) {
-                const uint32_t w = (uint32_t)__ldg(A.ci + x);
-                if (CF || in_set(A.inS, w)) {
-                    up = jp_okey(A.k, A.okey, A.ord, w) > kv;
-                    dn = !up;
-                }
-            }
-            nu += __popc(__ballot_sync(FULL, up));
-            nd += __popc(__ballot_sync(FULL, dn));
+        // the warp's slice stays in registers (16 arcs per lane, all loads in flight):
+        // classify, count by ballots, reserve both cursors once, then rank and store
+        static_assert(SLICE == 16 * 32, "slice layout");
+        uint32_t w[16], rk[16];
+        unsigned upm = 0, dnm = 0;
+#pragma unroll
+        for (int i = 0; i < 16; i++) {
+            const int64_t x = sb0 + lane + 32 * i;
+            w[i] = x < se ? (uint32_t)__ldg(A.ci + x) : 0u;
         }
+        uint32_t nu = 0, nd = 0;
+#pragma unroll
+        for (int i = 0; i < 16; i++) {
+            const bool ok = sb0 + lane + 32 * i < se;
+            const bool sv = ok && (CF || in_set(A.inS, w[i]));
+            const bool up = sv && jp_okey(A.k, A.okey, A.ord, w[i]) > kv;
+            upm |= (up ? 1u : 0u) << i;
+            dnm |= (sv && !up ? 1u : 0u) << i;
+            if (!CF && ok && !sv) jp_fixed(A, h, m0.x, x0, w[i]);
+            nu += __popc(__ballot_sync(FULL, up));
+            nd += __popc(__ballot_sync(FULL, sv && !up));
+        }
+#pragma unroll
+        for (int i = 0; i < 16; i++) rk[i] = ((upm | dnm) >> i) & 1u ? jp_rank(A, w[i]) : 0u;
         uint32_t pu = 0, pd = 0;
         if (lane == 0) {
             if (nu) pu = atomicAdd(A.hdeg + h, nu);
@@ -850,31 +865,17 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
         }
         pu = __shfl_sync(FULL, pu, 0);
         pd = __shfl_sync(FULL, pd, 0);
-        for (int64_t xq = sb0 + lane; xq - lane < se; xq += 128) {  // 4 steps of 32 arcs in flight
-            uint32_t w[4], rk[4];
-            bool up[4], dn[4];
 #pragma unroll
-            for (int u = 0; u < 4; u++) w[u] = xq + u * 32 < se ? (uint32_t)__ldg(A.ci + xq + u * 32) : 0u;
-#pragma unroll
-            for (int u = 0; u < 4; u++) {
-                const bool ok = xq + u * 32 < se;
-                const bool sv = ok && (CF || in_set(A.inS, w[u]));
-                up[u] = sv && jp_okey(A.k, A.okey, A.ord, w[u]) > kv;
-                dn[u] = sv && !up[u];
-                rk[u] = sv ? jp_rank(A, w[u]) : 0u;
-                if (!CF && ok && !sv) jp_fixed(A, h, m0.x, x0, w[u]);
+        for (int i = 0; i < 16; i++) {
+            const bool up = (upm >> i) & 1u, dn = (dnm >> i) & 1u;
+            const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
+            if (up) __stcs(A.lst + hl + pu + __popc(mu & lt), rk[i]);
+            if (dn) {
+                if (CF) __stcs(A.lst + ll - 1 - (pd + __popc(md & lt)), rk[i]);
+                else __stcs(A.lst + ll + pd + __popc(md & lt), rk[i]);
             }
-#pragma unroll
-            for (int u = 0; u < 4; u++) {
-                const unsigned mu = __ballot_sync(FULL, up[u]), md = __ballot_sync(FULL, dn[u]);
-                if (up[u]) __stcs(A.lst + hl + pu + __popc(mu & lt), rk[u]);
-                if (dn[u]) {
-                    if (CF) __stcs(A.lst + ll - 1 - (pd + __popc(md & lt)), rk[u]);
-                    else __stcs(A.lst + ll + pd + __popc(md & lt), rk[u]);
-                }
-                pu += __popc(mu);
-                pd += __popc(md);
-            }
+            pu += __popc(mu);
+            pd += __popc(md);
         }
         prof_add(A.prof, 0ull, lane == 0 && se > sb0 ? 8ull * (uint64_t)(se - sb0) : 0ull);
     }

@@ -601,7 +601,7 @@ static int mis_phase(const FlowArgs &f, MisWs &w, uint8_t *st, const int64_t *rp
     const uint32_t maxr = f.p.max_rounds ? f.p.max_rounds : 0xffffffffu;
     int grid = round_grid();
     int r = 0;
-    const int batch = 4;  // rounds launched per host poll of the frontier count
+    const int batch = SYM_POLL_BATCH;  // rounds launched per host poll of the frontier count
     for (;;) {
         for (int b = 0; b < batch && (uint32_t)r < maxr; b++, r++) {  // never past the cap
             MisRoundArgs A{};

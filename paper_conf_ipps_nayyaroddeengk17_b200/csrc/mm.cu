@@ -20,7 +20,10 @@
 
 namespace sym {
 
-constexpr int MM_SMALL = 8;
+#ifndef SYM_MM_SMALL
+#define SYM_MM_SMALL 8
+#endif
+constexpr int MM_SMALL = SYM_MM_SMALL;  // rows up to MM_SMALL arcs are scanned by one lane
 constexpr int MM_BUDGET = 4096;  // rows longer than this go to the CTA kernel
 constexpr int MM_THREADS = 256;
 constexpr int MM_HUGE_THREADS = 512;
@@ -164,19 +167,22 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
         uint64_t best = 0, sec = 0;  // sec: second-heaviest key + 1 (0 = none)
         bool has = false;
         if (scan && d <= MM_SMALL) {
-            // short row by one lane: all column loads (streamed, evict-first so the
-            // gathered mate array stays in L2), then all mate gathers, then the argmax
+            // short row by one lane, in batches of 8: all column loads (streamed,
+            // evict-first so the gathered bitmap stays in L2), then all liveness gathers,
+            // then the top-2
             colb += 4 * (unsigned long long)d;
-            uint32_t w[MM_SMALL];
-            bool live[MM_SMALL];
-#pragma unroll
-            for (int q = 0; q < MM_SMALL; q++) w[q] = (q < d) ? (uint32_t)__ldcs(ci + b + q) : 0u;
-#pragma unroll
-            for (int q = 0; q < MM_SMALL; q++) live[q] = (q < d) && (!MATE || !mm_matched(A.mbits, w[q]));
-#pragma unroll
             uint64_t b1 = 0;
-            for (int q = 0; q < MM_SMALL; q++)
-                if (live[q]) top2_add(b1, sec, ekey(A.k, (uint32_t)u, w[q]) + 1);
+            for (int64_t xq = b; xq < e; xq += 8) {
+                uint32_t w[8];
+                bool live[8];
+#pragma unroll
+                for (int q = 0; q < 8; q++) w[q] = (xq + q < e) ? (uint32_t)__ldcs(ci + xq + q) : 0u;
+#pragma unroll
+                for (int q = 0; q < 8; q++) live[q] = (xq + q < e) && (!MATE || !mm_matched(A.mbits, w[q]));
+#pragma unroll
+                for (int q = 0; q < 8; q++)
+                    if (live[q]) top2_add(b1, sec, ekey(A.k, (uint32_t)u, w[q]) + 1);
+            }
             has = b1 != 0;
             best = b1 - 1;
         }
@@ -362,7 +368,7 @@ static int mm_phase(const FlowArgs &f, MmWs &w, int32_t *mate, const MmPhase &ph
     // no alternates yet (the streaming round 0 finds the heaviest arc only: tracking a
     // second there cost more than it saved -- 1.7 -> 2.9 ms round 0 at R-MAT s24 MM-NONE)
     SYM_CUDA(cudaMemsetAsync(w.alt, 0xff, sizeof(int32_t) * (size_t)(f.g.n + 1), s));
-    const int batch = 4;  // rounds launched per host poll of the frontier count
+    const int batch = SYM_POLL_BATCH;  // rounds launched per host poll of the frontier count
     if (ph.first && !ph.dual) {
         // round 0 as one streaming pass: every phase vertex picks its heaviest arc;
         // the vertices with a pick form round 1's frontier (fr[1], ring[1])

@@ -33,7 +33,7 @@ def main():
     tag = sys.argv[1] if len(sys.argv) > 1 else "run"
     out_csv = os.path.join(ROOT, "gpurun_out", f"{tag}_traffic.csv")
     os.makedirs(os.path.dirname(out_csv), exist_ok=True)
-    cmd = ["ncu", "--cache-control", "none", "--clock-control", "none", "--metrics",
+    cmd = ["ncu", "--cache-control", "none", "--clock-control", "none", "-k", "regex:^k_", "--metrics",
            "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum,lts__t_sectors.sum,"
            "lts__throughput.avg.pct_of_peak_sustained_elapsed,dram__throughput.avg.pct_of_peak_sustained_elapsed",
            "--csv", "--log-file", out_csv,
