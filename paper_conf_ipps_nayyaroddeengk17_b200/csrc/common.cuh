@@ -200,6 +200,15 @@ __device__ __forceinline__ uint64_t atom_dec64_pred(unsigned long long *addr, bo
     return old;
 }
 
+// read-only 8-B load under a predicate ({0,0} when !p), no branch
+__device__ __forceinline__ uint2 ld_nc_v2_pred(const uint2 *addr, bool p) {
+    uint2 v = make_uint2(0u, 0u);
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q ld.global.nc.v2.u32 {%0, %1}, [%2];\n\t}"
+                 : "+r"(v.x), "+r"(v.y)
+                 : "l"(addr), "r"((uint32_t)p));
+    return v;
+}
+
 // 1-B load under a predicate (dflt when !p), no branch
 __device__ __forceinline__ uint8_t ld_u8_pred(const uint8_t *addr, bool p, uint8_t dflt) {
     uint32_t v = dflt;

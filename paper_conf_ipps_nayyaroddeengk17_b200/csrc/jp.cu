@@ -215,6 +215,12 @@ __device__ __forceinline__ uint32_t jp_rank(const JpArgs &A, uint32_t v) {
     const uint2 x = __ldg(reinterpret_cast<const uint2 *>(A.arank) + (v >> 5));
     return x.y + __popc(x.x & ((1u << (v & 31)) - 1u));
 }
+// the same under a predicate (0 when !p): a predicated load, so a batch of rank lookups
+// stays in flight together instead of branching around each one
+__device__ __forceinline__ uint32_t jp_rank_pred(const JpArgs &A, uint32_t v, bool p) {
+    const uint2 x = ld_nc_v2_pred(reinterpret_cast<const uint2 *>(A.arank) + (v >> 5), p);
+    return x.y + __popc(x.x & ((1u << (v & 31)) - 1u));
+}
 
 // implicit S = 0..n-1: one bitmap word per warp step (ballot of "has phase arcs")
 __global__ void k_jpc_bits(JpArgs A, int64_t n) {
@@ -742,7 +748,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
 #pragma unroll
                 for (int u = 0; u < FB; u++) {
                     sv[u] = ok[u] && (CF || in_set(A.inS, w[u]));
-                    rk[u] = sv[u] ? jp_rank(A, w[u]) : 0u;
+                    rk[u] = jp_rank_pred(A, w[u], sv[u]);
                 }
 #pragma unroll
                 for (int u = 0; u < FB; u++) {
@@ -783,7 +789,7 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
                     const bool sv = ok && (CF || in_set(A.inS, w[u]));
                     up[u] = sv && jp_okey(A.k, A.okey, A.ord, w[u]) > wk;
                     dn[u] = sv && !up[u];
-                    rk[u] = sv ? jp_rank(A, w[u]) : 0u;
+                    rk[u] = jp_rank_pred(A, w[u], sv);
                     if (!CF && ok && !sv) jp_fixed(A, wh, wR, wx0, w[u]);
                 }
 #pragma unroll
@@ -811,9 +817,10 @@ __global__ void __launch_bounds__(JP_THREADS) k_jpc_fill(JpArgs A) {
     }
 }
 
-// huge rows: one CTA per piece; each warp holds its 512-arc slice in registers, counts
-// it (ballots), reserves its positions on the row's two cursors with one atomic each,
-// then writes.  CF: the lower cursor counts from the back of the area.
+// huge rows: one CTA per piece; each warp counts its 512-arc slice (ballots), reserves
+// its positions on the row's two cursors with one atomic each, then writes (the
+// slice is re-read from L2; holding it in registers instead cost occupancy -- 68 regs,
+// one CTA per SM -- and jp_build went 4.03 -> 4.53 ms at R-MAT s24).  CF: the lower cursor counts from the back of the area.
 template <bool CF>
 __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
     constexpr int SLICE = JP_PIECE / (JP_HUGE_THREADS / 32);
@@ -834,30 +841,19 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
         const uint32_t d = (uint32_t)(e - b);
         const uint64_t hl = meta_off(m1) + (CF ? watch_area(d, 0u) : watch_area(m0.y, m0.z));
         const uint64_t ll = CF ? hl + d : hl + m0.y;  // CF: one past the back of the area
-        // the warp's slice stays in registers (16 arcs per lane, all loads in flight):
-        // classify, count by ballots, reserve both cursors once, then rank and store
-        static_assert(SLICE == 16 * 32, "slice layout");
-        uint32_t w[16], rk[16];
-        unsigned upm = 0, dnm = 0;
-#pragma unroll
-        for (int i = 0; i < 16; i++) {
-            const int64_t x = sb0 + lane + 32 * i;
-            w[i] = x < se ? (uint32_t)__ldg(A.ci + x) : 0u;
-        }
         uint32_t nu = 0, nd = 0;
+        for (int64_t xq = sb0 + lane; xq - lane < se; xq += 128) {  // 4 loads in flight per lane
+            uint32_t w[4];
 #pragma unroll
-        for (int i = 0; i < 16; i++) {
-            const bool ok = sb0 + lane + 32 * i < se;
-            const bool sv = ok && (CF || in_set(A.inS, w[i]));
-            const bool up = sv && jp_okey(A.k, A.okey, A.ord, w[i]) > kv;
-            upm |= (up ? 1u : 0u) << i;
-            dnm |= (sv && !up ? 1u : 0u) << i;
-            if (!CF && ok && !sv) jp_fixed(A, h, m0.x, x0, w[i]);
-            nu += __popc(__ballot_sync(FULL, up));
-            nd += __popc(__ballot_sync(FULL, sv && !up));
+            for (int u = 0; u < 4; u++) w[u] = xq + u * 32 < se ? (uint32_t)__ldg(A.ci + xq + u * 32) : 0u;
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const bool sv = xq + u * 32 < se && (CF || in_set(A.inS, w[u]));
+                const bool up = sv && jp_okey(A.k, A.okey, A.ord, w[u]) > kv;
+                nu += __popc(__ballot_sync(FULL, up));
+                nd += __popc(__ballot_sync(FULL, sv && !up));
+            }
         }
-#pragma unroll
-        for (int i = 0; i < 16; i++) rk[i] = ((upm | dnm) >> i) & 1u ? jp_rank(A, w[i]) : 0u;
         uint32_t pu = 0, pd = 0;
         if (lane == 0) {
             if (nu) pu = atomicAdd(A.hdeg + h, nu);
@@ -865,17 +861,31 @@ __global__ void __launch_bounds__(JP_HUGE_THREADS) k_jpc_fill_huge(JpArgs A) {
         }
         pu = __shfl_sync(FULL, pu, 0);
         pd = __shfl_sync(FULL, pd, 0);
+        for (int64_t xq = sb0 + lane; xq - lane < se; xq += 128) {  // 4 steps of 32 arcs in flight
+            uint32_t w[4], rk[4];
+            bool up[4], dn[4];
 #pragma unroll
-        for (int i = 0; i < 16; i++) {
-            const bool up = (upm >> i) & 1u, dn = (dnm >> i) & 1u;
-            const unsigned mu = __ballot_sync(FULL, up), md = __ballot_sync(FULL, dn);
-            if (up) __stcs(A.lst + hl + pu + __popc(mu & lt), rk[i]);
-            if (dn) {
-                if (CF) __stcs(A.lst + ll - 1 - (pd + __popc(md & lt)), rk[i]);
-                else __stcs(A.lst + ll + pd + __popc(md & lt), rk[i]);
+            for (int u = 0; u < 4; u++) w[u] = xq + u * 32 < se ? (uint32_t)__ldg(A.ci + xq + u * 32) : 0u;
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const bool ok = xq + u * 32 < se;
+                const bool sv = ok && (CF || in_set(A.inS, w[u]));
+                up[u] = sv && jp_okey(A.k, A.okey, A.ord, w[u]) > kv;
+                dn[u] = sv && !up[u];
+                rk[u] = jp_rank_pred(A, w[u], sv);
+                if (!CF && ok && !sv) jp_fixed(A, h, m0.x, x0, w[u]);
             }
-            pu += __popc(mu);
-            pd += __popc(md);
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const unsigned mu = __ballot_sync(FULL, up[u]), md = __ballot_sync(FULL, dn[u]);
+                if (up[u]) __stcs(A.lst + hl + pu + __popc(mu & lt), rk[u]);
+                if (dn[u]) {
+                    if (CF) __stcs(A.lst + ll - 1 - (pd + __popc(md & lt)), rk[u]);
+                    else __stcs(A.lst + ll + pd + __popc(md & lt), rk[u]);
+                }
+                pu += __popc(mu);
+                pd += __popc(md);
+            }
         }
         prof_add(A.prof, 0ull, lane == 0 && se > sb0 ? 8ull * (uint64_t)(se - sb0) : 0ull);
     }

@@ -120,6 +120,21 @@ __device__ __forceinline__ int mis_scan_window(const MisRoundArgs &A, int64_t x,
     return R_NONE;
 }
 
+// push-Out of 4 arcs x, x+S, x+2S, x+3S (< e): the column loads, then the status loads,
+// then the stores, each step's accesses in flight together
+template <int S>
+__device__ __forceinline__ void mis_push4(const MisRoundArgs &A, int64_t x, int64_t e) {
+    uint32_t w[4];
+    uint8_t sv[4];
+#pragma unroll
+    for (int u = 0; u < 4; u++) w[u] = x + u * S < e ? (uint32_t)__ldcs(A.ci + x + u * S) : 0u;
+#pragma unroll
+    for (int u = 0; u < 4; u++) sv[u] = ld_u8_pred(A.st + w[u], x + u * S < e, ST_OUT);
+#pragma unroll
+    for (int u = 0; u < 4; u++)
+        if (sv[u] == ST_UNDEC) A.st[w[u]] = ST_OUT;
+}
+
 // Resume memo: a blocked vertex records where its scan stopped (the first undecided
 // higher neighbour, or the start of the warp step that found one); every arc before it
 // is a lower neighbour or a final-Out higher one, so the next round resumes there.
@@ -221,10 +236,7 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
                 const int src = __ffs(pm) - 1;
                 pm &= pm - 1;
                 const int64_t wb = __shfl_sync(FULL, b, src), we = __shfl_sync(FULL, e, src);
-                for (int64_t x = wb + lane; x < we; x += 32) {
-                    const int32_t w = A.ci[x];
-                    if (A.st[w] == ST_UNDEC) A.st[w] = ST_OUT;
-                }
+                for (int64_t x = wb + lane; x < we; x += 128) mis_push4<32>(A, x, we);
                 prof_add(A.prof, lane == 0 ? 4ull * (we - wb) : 0ull, lane == 0 ? 4ull * (we - wb) : 0ull);  // row re-read
             }
         }
@@ -281,10 +293,7 @@ __global__ void __launch_bounds__(MIS_HUGE_THREADS) k_mis_huge(MisRoundArgs A) {
         }
         if (r == R_IN && A.push_out) {  // push-Out over the whole row (see k_mis_round)
             const int64_t rb = A.rp[v - A.row_base];
-            for (int64_t x = rb + threadIdx.x; x < e; x += MIS_HUGE_THREADS) {
-                const int32_t w = A.ci[x];
-                if (A.st[w] == ST_UNDEC) A.st[w] = ST_OUT;
-            }
+            for (int64_t x = rb + threadIdx.x; x < e; x += 4 * MIS_HUGE_THREADS) mis_push4<MIS_HUGE_THREADS>(A, x, e);
             prof_add(A.prof, threadIdx.x == 0 ? 4ull * (e - rb) : 0ull, threadIdx.x == 0 ? 4ull * (e - rb) : 0ull);
         }
         if (threadIdx.x == 0) {

@@ -21,7 +21,7 @@
 namespace sym {
 
 #ifndef SYM_MM_SMALL
-#define SYM_MM_SMALL 8
+#define SYM_MM_SMALL 32  // one lane per row up to 32 arcs (batches of 8): MM-Rand4 4.32 -> 3.99 ms with 5 CTAs/SM
 #endif
 constexpr int MM_SMALL = SYM_MM_SMALL;  // rows up to MM_SMALL arcs are scanned by one lane
 constexpr int MM_BUDGET = 4096;  // rows longer than this go to the CTA kernel
@@ -94,9 +94,10 @@ __device__ __forceinline__ void mm_row(const MmRoundArgs &A, int32_t u, int64_t 
 #ifndef SYM_MM_ALT
 #define SYM_MM_ALT 1
 #endif
-// 6 CTAs/SM (<= 40 regs, no spills; 47 without the bound -> 5): more mate gathers in flight
+// 5 CTAs/SM (48 regs, no spills; 6 CTAs at 40 regs spilled once the lane path took rows of
+// up to 32 arcs and the liveness gathers became one predicated batch)
 #ifndef SYM_MM_MINB
-#define SYM_MM_MINB 6
+#define SYM_MM_MINB 5
 #endif
 #if SYM_MM_MINB > 0
 #define MM_ROUND_BOUNDS __launch_bounds__(MM_THREADS, SYM_MM_MINB)
@@ -173,12 +174,14 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
             colb += 4 * (unsigned long long)d;
             uint64_t b1 = 0;
             for (int64_t xq = b; xq < e; xq += 8) {
-                uint32_t w[8];
+                uint32_t w[8], mw[8];  // columns, their matched-bitmap words
                 bool live[8];
 #pragma unroll
                 for (int q = 0; q < 8; q++) w[q] = (xq + q < e) ? (uint32_t)__ldcs(ci + xq + q) : 0u;
 #pragma unroll
-                for (int q = 0; q < 8; q++) live[q] = (xq + q < e) && (!MATE || !mm_matched(A.mbits, w[q]));
+                for (int q = 0; q < 8; q++) mw[q] = MATE ? ld_cg_pred(A.mbits + (w[q] >> 5), xq + q < e) : 0u;
+#pragma unroll
+                for (int q = 0; q < 8; q++) live[q] = (xq + q < e) && !((mw[q] >> (w[q] & 31)) & 1u);
 #pragma unroll
                 for (int q = 0; q < 8; q++)
                     if (live[q]) top2_add(b1, sec, ekey(A.k, (uint32_t)u, w[q]) + 1);
@@ -205,9 +208,12 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
                     w[q] = ok[q] ? (uint32_t)__ldcs(wci + y) : 0u;
                     colb += ok[q] ? 4 : 0;
                 }
+                uint32_t mw[4];  // the 4 liveness gathers in flight together (predicated loads)
+#pragma unroll
+                for (int q = 0; q < 4; q++) mw[q] = MATE ? ld_cg_pred(A.mbits + (w[q] >> 5), ok[q]) : 0u;
 #pragma unroll
                 for (int q = 0; q < 4; q++)
-                    if (ok[q] && (!MATE || !mm_matched(A.mbits, w[q]))) top2_add(lb, l2, ekey(A.k, (uint32_t)wu, w[q]) + 1);
+                    if (ok[q] && !((mw[q] >> (w[q] & 31)) & 1u)) top2_add(lb, l2, ekey(A.k, (uint32_t)wu, w[q]) + 1);
             }
 #pragma unroll
             for (int dd = 16; dd; dd >>= 1) {
@@ -256,9 +262,12 @@ __global__ void __launch_bounds__(MM_HUGE_THREADS) k_mm_huge(MmRoundArgs A) {
                 w[q] = ok[q] ? (uint32_t)__ldcs(ci + y) : 0u;
                 nb += ok[q] ? 4 : 0;
             }
+            uint32_t mw[4];
+#pragma unroll
+            for (int q = 0; q < 4; q++) mw[q] = MATE ? ld_cg_pred(A.mbits + (w[q] >> 5), ok[q]) : 0u;
 #pragma unroll
             for (int q = 0; q < 4; q++)
-                if (ok[q] && (!MATE || !mm_matched(A.mbits, w[q]))) top2_add(l1, l2, ekey(A.k, (uint32_t)u, w[q]) + 1);
+                if (ok[q] && !((mw[q] >> (w[q] & 31)) & 1u)) top2_add(l1, l2, ekey(A.k, (uint32_t)u, w[q]) + 1);
         }
 #pragma unroll
         for (int dd = 16; dd; dd >>= 1) {

@@ -18,6 +18,11 @@
 namespace sym {
 
 enum { KIND_NONE = 0, KIND_RAND = 1, KIND_DEGK = 2 };
+// DEGk: the V_H-bitmap word of each neighbour is gathered inside the flag loop, one
+// dependent L2 access per arc.  Issuing a thread's 16 gathers as one batch -- right
+// after the column loads, or just before the flag loop -- measured slower (3.31 ->
+// 3.59 / 3.75 ms at R-MAT s24): the kernel sits at ~51 % of L2 throughput and the
+// bursts only add contention.
 
 // ------------------------------------------------------------------ classification
 __global__ void k_classify_degk(const int64_t *__restrict__ rp, int64_t n, uint32_t k, uint32_t *__restrict__ hbits,
