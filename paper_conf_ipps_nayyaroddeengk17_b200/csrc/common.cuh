@@ -200,6 +200,16 @@ __device__ __forceinline__ uint64_t atom_dec64_pred(unsigned long long *addr, bo
     return old;
 }
 
+// streaming (evict-first) 4-B load under a predicate (0 when !p), no branch
+__device__ __forceinline__ uint32_t ld_cs_pred(const uint32_t *addr, bool p) {
+    uint32_t v = 0u;
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q ld.global.cs.u32 %0, [%1];\n\t}"
+                 : "+r"(v)
+                 : "l"(addr), "r"((uint32_t)p)
+                 : "memory");
+    return v;
+}
+
 // read-only 8-B load under a predicate ({0,0} when !p), no branch
 __device__ __forceinline__ uint2 ld_nc_v2_pred(const uint2 *addr, bool p) {
     uint2 v = make_uint2(0u, 0u);

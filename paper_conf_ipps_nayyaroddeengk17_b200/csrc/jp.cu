@@ -1240,11 +1240,16 @@ __device__ __forceinline__ void jp_push(const JpArgs &A, const uint32_t (&e)[K],
     // returns the R field and extra-word offset with it -- no separate load.  No colour
     // filter: a bit in the bitmap of an already coloured vertex is never read (nb_ok
     // tests its colour first).
+    // all K atomics first, their results read only afterwards (with the select in the
+    // same loop ptxas consumed each result before issuing the next atomic: ~14 % of the
+    // rounds kernel's stall samples sat on those selects)
+    uint64_t o[K];
+#pragma unroll
+    for (int u = 0; u < K; u++) o[u] = atom_dec64_pred(reinterpret_cast<unsigned long long *>(&A.hot[e[u]].z), act[u]);
 #pragma unroll
     for (int u = 0; u < K; u++) {
-        const uint64_t o = atom_dec64_pred(reinterpret_cast<unsigned long long *>(&A.hot[e[u]].z), act[u]);
-        old[u] = (uint32_t)o;
-        x[u] = act[u] && q > 0 ? (uint32_t)(o >> 32) : 0xffffffffu;
+        old[u] = (uint32_t)o[u];
+        x[u] = act[u] && q > 0 ? (uint32_t)(o[u] >> 32) : 0xffffffffu;
     }
 #if SYM_JP_DIAG
     uint64_t tq1 = 0, tq2 = 0, tq3 = 0;
@@ -1367,7 +1372,7 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, uint32_t
             for (int u = 0; u < JP_PUSH_LANE; u++) {
                 const uint32_t j = first + u * stride;
                 act[u] = j < wn;
-                e[u] = act[u] ? __ldcs(A.lst + ws + j) : 0u;
+                e[u] = ld_cs_pred(A.lst + ws + j, act[u]);
             }
             jp_push<JP_PUSH_LANE>(A, e, act, q, bit, JpNextList(A, r),
                                   SYM_JP_DIAG && tr && A.trace2 == 4 ? A.trace + r : nullptr);
@@ -1385,9 +1390,9 @@ __device__ __forceinline__ void jp_phase_b(const JpArgs &A, uint32_t r, uint32_t
         constexpr int K = JP_BUILD / 32;
         uint32_t e[K], c[K];
 #pragma unroll
-        for (int u = 0; u < K; u++) e[u] = j0 + u * 32 + lane < j1 ? __ldcs(A.lst + hl + j0 + u * 32 + lane) : 0u;
+        for (int u = 0; u < K; u++) e[u] = ld_cs_pred(A.lst + hl + j0 + u * 32 + lane, j0 + u * 32 + lane < j1);
 #pragma unroll
-        for (int u = 0; u < K; u++) c[u] = j0 + u * 32 + lane < j1 ? __ldcg(&A.hot[e[u]].x) : 1u;
+        for (int u = 0; u < K; u++) c[u] = ld_cg_pred(&A.hot[e[u]].x, j0 + u * 32 + lane < j1);  // != 0 when out of range
         unsigned mk[K];
         uint32_t tot = 0;
 #pragma unroll
