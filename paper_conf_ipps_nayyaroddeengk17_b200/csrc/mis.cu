@@ -321,6 +321,34 @@ __global__ void k_mis_kill_cross(const int64_t *__restrict__ rp_x, const int32_t
     }
 }
 
+// MIS-Deg2 classification fused with the trivial part of phase L: V_H -> back of vlist
+// (undecided); a V_L vertex without G_L arcs is its own component of G_L, so it is in
+// I_L at once and every neighbour of it (all in V_H: it has no G_L arcs) leaves the
+// remaining graph (the fix-up of P:288 for it); the other V_L vertices -> front of vlist
+// for phase L.  Status must be all undecided on entry.
+__global__ void k_mis_degk_classify(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci,
+                                    const int64_t *__restrict__ rp_in, int64_t n, uint32_t k, uint8_t *st,
+                                    int32_t *vlist, uint32_t *cnt_front, uint32_t *cnt_back) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
+        const int64_t v = base + threadIdx.x;
+        bool h = false, lo = false;
+        if (v < n) {
+            const int64_t b = rp[v], e = rp[v + 1];
+            h = e - b > (int64_t)k;
+            if (!h) {
+                if (rp_in[v + 1] == rp_in[v]) {  // isolated in G_L
+                    st[v] = ST_IN;
+                    for (int64_t x = b; x < e; x++) st[ci[x]] = ST_OUT;  // <= k arcs, all to V_H
+                } else {
+                    lo = true;
+                }
+            }
+        }
+        cta_append2(lo, h, (int32_t)v, n, vlist, cnt_front, cnt_back);
+    }
+}
+
 // MIS-Rand: classify by cross degree: interior (front list, UNDEC) / boundary B
 // (back list, INACTIVE during phase A)
 __global__ void k_mis_classify_cross(const int64_t *__restrict__ rp_x, int64_t n, uint8_t *st, int32_t *vlist,
@@ -689,7 +717,9 @@ int run_mis(const FlowArgs &f, MisWs &w, uint8_t *st) {
         // lists V_L (front) and V_H (back); status all undecided
         SYM_CUDA(cudaMemsetAsync(st, ST_UNDEC, (size_t)g.n, s));
         SYM_CUDA(cudaMemsetAsync(&ctl->cnt_front, 0, 2 * sizeof(uint32_t), s));
-        SYM_TRY(launch_classify_degk(g, f.p.param, f.hbits, w.vlist, ctl, s));
+        k_mis_degk_classify<<<num_sms() * 8, 256, 0, s>>>(g.rp, g.ci, f.split.rp_in, g.n, f.p.param, st, w.vlist,
+                                                          &ctl->cnt_front, &ctl->cnt_back);
+        SYM_LAUNCH_CHECK();
         // phase L: I_L = MIS(G_L) on the intra CSR restricted to V_L (tiny: the rows
         // of V_H in the same CSR are not in this phase, so no streaming round 0)
         SYM_TRY(mis_phase(f, w, st, f.split.rp_in, f.split.ci_in, w.vlist, 0, &ctl->cnt_front, 0, 0, false));

@@ -133,7 +133,8 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
                 A.pick_cur[u] = -1;
                 active = false;
                 nb += 4;
-            } else if (A.mate[u] >= 0) {  // defensive: never re-pick a matched vertex
+            } else if (mm_matched(A.mbits, (uint32_t)u)) {  // defensive: never re-pick a matched vertex
+                // (the matched bitmap, 2 MB and L2-resident, not the 67 MB mate array)
                 A.pick_cur[u] = -1;
                 active = false;
             } else if (MATE && p >= 0 && !mm_matched(A.mbits, (uint32_t)p)) {
