@@ -1,4 +1,6 @@
-O=gpurun_out/r2q
+# Quick GPU check: build, one bench line, the GPU tests (without scale 27).
+#   gpurun -- bash tools/gpu_quick.sh <tag>
+O=gpurun_out/${1:-quick}
 mkdir -p $O
 python -m paper_conf_ipps_nayyaroddeengk17_b200.build > $O/build.log 2>&1
 python -c "import oracle; oracle.build()" >> $O/build.log 2>&1
