@@ -68,3 +68,52 @@ class ConcurrentStep:
         main.wait_stream(self.sA)
         main.wait_stream(self.sB)
         return I, C, M
+
+
+class OverlapStep:
+    """The latency-bound prefix of the step on two streams, the colouring alone:
+
+        stream A: DEG2 decomposition -> MIS-Deg2
+        stream B: RAND4 decomposition -> MM-Rand4        (a second host thread)
+        then, after both:  COLOR-Deg2 on the caller's stream
+
+    The MIS/MM round kernels leave most of the GPU idle (dependent gathers: DRAM 14 %,
+    L2 26-28 % busy) and the two splits have different bottlenecks (L2 for DEGk, issue
+    for RAND), so the two chains interleave; the JP rounds kernel, which holds every
+    SM's register file, runs alone (co-running with it was slower, see ConcurrentStep).
+    Every call is the public API; results are bit-identical to the calls in order."""
+
+    def __init__(self, device, seed: int, k: int = 2, p: int = 4):
+        self.dev = torch.device(device)
+        self.seed, self.k, self.p = seed, k, p
+        self.sA = torch.cuda.Stream(self.dev)
+        self.sB = torch.cuda.Stream(self.dev)
+        self.pool = cf.ThreadPoolExecutor(1)
+
+    def __call__(self, rp: torch.Tensor, ci: torch.Tensor):
+        """-> (in_set, color, mate) of MIS-Deg{k}, COLOR-Deg{k}, MM-Rand{p} on (rp, ci)."""
+        seed, k, p = self.seed, self.k, self.p
+        main = torch.cuda.current_stream(self.dev)
+        self.sA.wait_stream(main)
+        self.sB.wait_stream(main)
+
+        def side():
+            with torch.cuda.device(self.dev), torch.cuda.stream(self.sB):
+                dR = sym_decompose(rp, ci, "rand", p, seed)
+                return sym_mm(rp, ci, "rand", p, seed, decomp=dR)
+
+        fut = self.pool.submit(side)
+        with torch.cuda.stream(self.sA):
+            dD = sym_decompose(rp, ci, "degk", k, seed)
+            I = sym_mis(rp, ci, "degk", k, seed, decomp=dD)
+        M = fut.result()
+        for t in (rp, ci):
+            t.record_stream(self.sA)
+            t.record_stream(self.sB)
+        for t in (dD.row_ptr_in, dD.col_in, dD.row_ptr_x, dD.col_x, I):
+            t.record_stream(self.sA)
+        M.record_stream(self.sB)
+        main.wait_stream(self.sA)
+        main.wait_stream(self.sB)
+        C = sym_color(rp, ci, "degk", k, seed, decomp=dD)
+        return I, C, M
