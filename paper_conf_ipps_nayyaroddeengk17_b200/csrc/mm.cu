@@ -24,7 +24,13 @@ namespace sym {
 #define SYM_MM_SMALL 32  // one lane per row up to 32 arcs (batches of 8): MM-Rand4 4.32 -> 3.99 ms with 5 CTAs/SM
 #endif
 constexpr int MM_SMALL = SYM_MM_SMALL;  // rows up to MM_SMALL arcs are scanned by one lane
-constexpr int MM_BUDGET = 4096;  // rows longer than this go to the CTA kernel
+#ifndef SYM_MM_WSTEP
+#define SYM_MM_WSTEP 4
+#endif
+#ifndef SYM_MM_BUDGET
+#define SYM_MM_BUDGET 1024  // 4096 -> 1024: MM-Rand4 3.95 -> 3.89 ms (a 4096-arc row was 32 serial warp steps)
+#endif
+constexpr int MM_BUDGET = SYM_MM_BUDGET;  // rows longer than this go to the CTA kernel
 constexpr int MM_THREADS = 256;
 constexpr int MM_HUGE_THREADS = 512;
 
@@ -199,21 +205,22 @@ __global__ void MM_ROUND_BOUNDS k_mm_round(MmRoundArgs A) {
             const int32_t wu = __shfl_sync(FULL, u, src);
             const int32_t *wci = (const int32_t *)__shfl_sync(FULL, (unsigned long long)ci, src);
             uint64_t lb = 0, l2 = 0;  // top-2 keys + 1 (0 = none)
-            for (int64_t x = wb; x < we; x += 128) {
-                uint32_t w[4];
-                bool ok[4];
+            constexpr int WS = SYM_MM_WSTEP;  // arcs per lane per warp step, all loads in flight
+            for (int64_t x = wb; x < we; x += 32 * WS) {
+                uint32_t w[WS];
+                bool ok[WS];
 #pragma unroll
-                for (int q = 0; q < 4; q++) {
+                for (int q = 0; q < WS; q++) {
                     int64_t y = x + q * 32 + lane;
                     ok[q] = y < we;
                     w[q] = ok[q] ? (uint32_t)__ldcs(wci + y) : 0u;
                     colb += ok[q] ? 4 : 0;
                 }
-                uint32_t mw[4];  // the 4 liveness gathers in flight together (predicated loads)
+                uint32_t mw[WS];  // the liveness gathers in flight together (predicated loads)
 #pragma unroll
-                for (int q = 0; q < 4; q++) mw[q] = MATE ? ld_cg_pred(A.mbits + (w[q] >> 5), ok[q]) : 0u;
+                for (int q = 0; q < WS; q++) mw[q] = MATE ? ld_cg_pred(A.mbits + (w[q] >> 5), ok[q]) : 0u;
 #pragma unroll
-                for (int q = 0; q < 4; q++)
+                for (int q = 0; q < WS; q++)
                     if (ok[q] && !((mw[q] >> (w[q] & 31)) & 1u)) top2_add(lb, l2, ekey(A.k, (uint32_t)wu, w[q]) + 1);
             }
 #pragma unroll
