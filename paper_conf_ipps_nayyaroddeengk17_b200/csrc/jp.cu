@@ -54,7 +54,10 @@ constexpr int JP_HUGE_THREADS = 512;
 #define SYM_JP_SMALL 32
 #endif
 constexpr int JP_SMALL = SYM_JP_SMALL;  // build: rows <= JP_SMALL arcs are handled by one lane
-constexpr int JP_BUDGET = 4096;  // build: rows > JP_BUDGET arcs are split into pieces
+#ifndef SYM_JP_BUDGET
+#define SYM_JP_BUDGET 4096
+#endif
+constexpr int JP_BUDGET = SYM_JP_BUDGET;  // build: rows > JP_BUDGET arcs are split into pieces
 constexpr int JP_PIECE = 8192;   // arcs per CTA piece of a huge row in the build passes
 constexpr int JP_TILE = 2048;    // build: compact ids per scan tile (JP_THREADS x 8)
 constexpr int JP_TPT = JP_TILE / JP_THREADS;

@@ -26,7 +26,10 @@
 namespace sym {
 
 constexpr int MIS_SMALL = 8;
-constexpr int MIS_BUDGET = 4096;
+#ifndef SYM_MIS_BUDGET
+#define SYM_MIS_BUDGET 4096
+#endif
+constexpr int MIS_BUDGET = SYM_MIS_BUDGET;
 constexpr int MIS_THREADS = 256;
 constexpr int MIS_HUGE_THREADS = 512;
 

@@ -1,5 +1,5 @@
-"""The two-stream concurrent step (schedule.ConcurrentStep) equals the sequential calls
-bit for bit, and both equal the oracle on a small graph."""
+"""The two-stream steps (schedule.ConcurrentStep, schedule.OverlapStep) equal the
+sequential calls bit for bit, and both equal the oracle on a small graph."""
 import pytest
 import torch
 
@@ -19,13 +19,14 @@ def _seq(sb, rp, ci, seed):
 
 
 @pytest.mark.parametrize("scale", [12, 18])
-def test_concurrent_step_equals_sequential(scale):
+@pytest.mark.parametrize("kind", ["concurrent", "overlap"])
+def test_concurrent_step_equals_sequential(scale, kind):
     import paper_conf_ipps_nayyaroddeengk17_b200 as sb
-    from paper_conf_ipps_nayyaroddeengk17_b200.schedule import ConcurrentStep
+    from paper_conf_ipps_nayyaroddeengk17_b200.schedule import ConcurrentStep, OverlapStep
     dev = torch.device("cuda", 0)
     rp, ci = graphgen.rmat(scale, 8, seed=3, device=dev)
     ref = _seq(sb, rp, ci, 42)
-    step = ConcurrentStep(dev, 42)
+    step = (ConcurrentStep if kind == "concurrent" else OverlapStep)(dev, 42)
     for _ in range(3):
         got = step(rp, ci)
         torch.cuda.synchronize()
