@@ -13,12 +13,19 @@
 // MIS (Blelloch et al. [6]).  Neighbours marked INACTIVE are not
 // in the current phase and are ignored.
 //
+// Push-Out: a vertex that turns IN marks its undecided phase neighbours OUT at once, so
+// a blocked vertex only waits at its first undecided higher neighbour and resumes there
+// next round (resume memo, out_pos parallel to the frontier list).
+//
 // Load balance for power-law rows (R-MAT: max degree ~4e5 at scale 24):
-//   rows <= MIS_SMALL arcs  : one lane scans serially with early exit;
-//   longer rows             : the warp scans 4x32 arcs per step (ballot early exit)
+//   every row               : one lane checks the window of MIS_SMALL arcs at its resume
+//                             position (all loads in flight); most rows block or decide there;
+//   rows past their window  : the warp scans 4x32 arcs per step (ballot early exit)
 //                             for up to MIS_BUDGET arcs;
 //   rows still undecided    : deferred (v, resume offset) to k_mis_huge, where a
 //                             whole CTA scans the rest with __syncthreads_or exits.
+// MIS-Deg2's classification (k_mis_degk_classify) decides the V_L vertices without G_L
+// arcs directly (In, and their V_H neighbours Out).
 #include <algorithm>
 
 #include "internal.h"

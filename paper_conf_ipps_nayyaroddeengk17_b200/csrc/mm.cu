@@ -15,7 +15,12 @@
 // Round 0 of the first phase specialises away the mate gathers (nothing is matched
 // yet): a pure streaming pass over col_idx with the edge hash computed on the fly.
 // A vertex whose previous pick is still unmatched keeps it without rescanning its row
-// (the live set only shrinks and the keys are fixed, so it is still the heaviest).
+// (the live set only shrinks and the keys are fixed, so it is still the heaviest); if
+// the pick is matched but the second-heaviest neighbour of the last scan (alt) is
+// not, that one is now the heaviest -- again no rescan.  Liveness is one bit of the
+// matched bitmap (2 MB at s24, L2-resident), gathered in predicated batches.
+// Rows: one lane up to MM_SMALL arcs (batches of 8), a warp up to MM_BUDGET, a CTA
+// beyond (k_mm_huge).
 #include "internal.h"
 
 namespace sym {
