@@ -28,8 +28,10 @@
 // (R-1 words) | min(R,31) << 27}, R = ceil(cap/32) -- count and offset adjacent, so a
 // push's one 64-bit atomic decrements the count and returns the offset.  meta[h] (32 B, read by h itself) = {R, hdeg, ldeg, watch
 // length, blocker position, m at the last failed check, list offset}; lst[off..]
-// = [watch area of JP_WATCH ids if hdeg > JP_WLIST] [higher ids] [lower ids] (compact
-// ids).
+// = [watch area of JP_WATCH ids if hdeg + ldeg > JP_WLIST (used if hdeg > JP_WLIST)]
+// [higher ids] [lower ids] (compact ids).  With S implicit the build is count-free: a
+// row's area is sized from its degree, higher ids are filled from the front and lower
+// ids from the back, and the counts found by the fill size the records afterwards.
 // A round: phase A -- every vertex whose count is <= JP_WATCH checks its watch list
 // (the higher neighbours still uncoloured when it was built; a list of <= JP_WLIST
 // higher neighbours is its own watch list), resuming at the last blocker when m is
