@@ -148,6 +148,9 @@ __device__ __forceinline__ void mis_push4(const MisRoundArgs &A, int64_t x, int6
 // Resume memo: a blocked vertex records where its scan stopped (the first undecided
 // higher neighbour, or the start of the warp step that found one); every arc before it
 // is a lower neighbour or a final-Out higher one, so the next round resumes there.
+#ifndef SYM_MIS_LANE_ITERS
+#define SYM_MIS_LANE_ITERS 2  // MIS-Deg2 1.13 -> 1.06 ms (MIS-NONE unchanged; 4 windows: slower)
+#endif
 #ifndef SYM_MIS_MINB
 #define SYM_MIS_MINB 5  // 48 regs, 5 CTAs/SM: 1.46 -> 1.39 ms MIS-NONE at R-MAT s24 (62 regs unbounded)
 #endif
@@ -184,15 +187,21 @@ __global__ void __launch_bounds__(MIS_THREADS) k_mis_round(MisRoundArgs A) {
         // lane stage: the first MIS_SMALL arcs of every row (a long row of an R-MAT graph
         // is almost always decided or blocked within them)
         uint32_t wv[MIS_SMALL];
+        int64_t xw = x0 + MIS_SMALL;  // where the warp stage starts
         if (active) {
             res = mis_scan_window(A, x0, e, kv, pos, lb, wv);
-            if (res == R_NONE && e - x0 <= MIS_SMALL) res = R_IN;
+            // (SYM_MIS_LANE_ITERS > 1: more lane windows before the warp stage)
+            for (int it = 1; it < SYM_MIS_LANE_ITERS && res == R_NONE && xw < e; it++, xw += MIS_SMALL) {
+                uint32_t wt[MIS_SMALL];
+                res = mis_scan_window(A, xw, e, kv, pos, lb, wt);
+            }
+            if (res == R_NONE && xw >= e) res = R_IN;
         }
         unsigned longm = __ballot_sync(FULL, active && res == R_NONE);
         while (longm) {
             const int src = __ffs(longm) - 1;
             longm &= longm - 1;
-            const int64_t wb = __shfl_sync(FULL, x0, src) + MIS_SMALL, we = __shfl_sync(FULL, e, src);
+            const int64_t wb = __shfl_sync(FULL, xw, src), we = __shfl_sync(FULL, e, src);
             const uint64_t wk = __shfl_sync(FULL, kv, src);
             const int64_t lim = min(we, wb + MIS_BUDGET);
             int r = R_IN;
