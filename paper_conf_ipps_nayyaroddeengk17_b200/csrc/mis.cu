@@ -32,7 +32,10 @@
 
 namespace sym {
 
-constexpr int MIS_SMALL = 8;
+#ifndef SYM_MIS_SMALL
+#define SYM_MIS_SMALL 8
+#endif
+constexpr int MIS_SMALL = SYM_MIS_SMALL;  // arcs per lane window
 #ifndef SYM_MIS_BUDGET
 #define SYM_MIS_BUDGET 4096
 #endif
