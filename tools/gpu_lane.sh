@@ -1,2 +1,2 @@
-O=gpurun_out/r2zw; mkdir -p $O
-bash tools/ab.sh r2zw "mis_none mis_deg2 mm_none mm_rand4 color_deg2" "" "-DSYM_MIS_SMALL=16 -DSYM_MIS_LANE_ITERS=1" "-DSYM_JP_SMALL=64" "-DSYM_JP_SMALL=16" "-DSYM_MM_SMALL=64"
+O=gpurun_out/r2zx; mkdir -p $O
+bash tools/ab.sh r2zx "split_degk split_rand4 mm_none mm_rand4" "" "-DSYM_SPLIT_THREADS=512" "-DSYM_SPLIT_THREADS=128"
